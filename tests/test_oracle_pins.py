@@ -1,0 +1,195 @@
+"""Pins of the CPU oracle against what the paper and the mathematics fix
+(DESIGN.md "Oracle pins").  CPU only."""
+import json
+import os
+import random
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from oracle.belady import belady_loads, belady_loads_one, brute_force_opt, dsets_of
+from conftest import GOLDEN
+from validate import validate
+
+
+def _golden(name):
+    with open(os.path.join(GOLDEN, name)) as f:
+        return json.load(f)
+
+
+def _unit(inst):
+    """Unit sizes / unit task time: capacity in data counts, delta = tau = 1 tick
+    with a 1e9 B/s bus."""
+    M = int(inst.mem_capacity // int(inst.data_size[0]))
+    return inst.with_(data_size=np.ones(inst.n, dtype=np.uint64), mem_capacity=M,
+                      default_task_ns=1, task_ns=None)
+
+
+def _check(inst, r, W=0, bus=oracle.DEFAULT_BUS_BPS, complete=True):
+    return validate(inst, r.serve_gpu, r.serve_task, r.events, r.task_start, r.task_end,
+                    W=W, bus_bps=bus, complete=complete)
+
+
+# ---------------------------------------------------------------- P1 (paper)
+def test_p1_fig1_paper_schedule_belady_11_loads():
+    g = _golden("fig1_paper_schedule.json")
+    ds = dsets_of(gen.fig1())
+    per = [belady_loads_one(o, ds, g["M"]) for o in g["sigma"]]
+    assert per == g["per_gpu_loads_by_hand"]
+    assert sum(per) == g["paper_total_loads"] == 11
+
+
+# ---------------------------------------------------------------- P2 (hand)
+@pytest.mark.parametrize("flags", [oracle.F_FALLBACK2, 0])
+def test_p2_fig1_darts_luf_hand_trace(flags):
+    g = _golden("fig1_darts_luf_hand.json")
+    inst = gen.fig1(K=g["K"], M=g["M"])
+    r = oracle.run(inst, bus_bps=10 ** 9, flags=flags)
+    assert [list(map(int, o)) for o in r.orders()] == g["orders"]
+    loads = [[int(e["gpu"]), int(e["data"])] for e in r.events if e["op"] == 0]
+    evs = [[int(e["gpu"]), int(e["data"])] for e in r.events if e["op"] == 1]
+    assert loads == g["loads_in_event_order"]
+    assert evs == g["evictions_in_event_order"]
+    assert (r.n_loads, r.n_evictions, r.makespan) == (g["n_loads"], g["n_evictions"], g["makespan"])
+    if flags:
+        assert r.n_fallback2 == g["n_fallback2"]
+    _check(inst, r, bus=10 ** 9)
+
+
+# ---------------------------------------------------------------- H0
+def test_h0_2d_N2_equals_brute_force():
+    g = _golden("h0_2d_N2.json")
+    inst = _unit(gen.matmul2d(2, M=2, K=1))
+    r = oracle.run(inst, bus_bps=10 ** 9)
+    assert list(map(int, r.orders()[0])) == g["order"]
+    assert r.n_loads == g["n_loads"]
+    assert brute_force_opt(dsets_of(inst), 2) == g["brute_force_opt"] == r.n_loads
+
+
+# ---------------------------------------------------------------- P3 / H1
+def test_p3_h1_config1_hand_trace():
+    g = _golden("h1_2d_N10_M6.json")
+    inst = _unit(gen.matmul2d(10, M=6, K=1))
+    r = oracle.run(inst, bus_bps=10 ** 9)
+    name = lambda d: f"A{d}" if d < 10 else f"B{d - 10}"
+    seq = [name(int(e["data"])) for e in r.events if e["op"] == 0]
+    assert seq == g["load_sequence"]
+    assert r.n_loads == g["n_loads"] and r.n_evictions == g["n_evictions"]
+    assert r.n_scans == g["n_scans"] and r.n_fallback2 == g["n_fallback2"]
+    assert r.n_fallback_first == g["n_fallback_first"]
+    assert r.n_idle_requests == g["n_idle_requests"]
+    assert r.n_served - r.n_scans == g["pops"]
+    assert r.makespan == 43 * 1 + 100 * 1
+    _check(inst, r, bus=10 ** 9)
+
+
+def test_config1_real_units_makespan_closed_form():
+    """K=1, W=0: the GPU requests at the end of its task and the bus is idle
+    then, so makespan = sum of transfer times + sum of task times exactly."""
+    inst = gen.config_instances("C1")[0]
+    r = oracle.run(inst)
+    d = -(-gen.DATUM_2D_BYTES * 10 ** 9 // gen.DEFAULT_BUS_BPS)
+    assert d == 1_228_800
+    assert r.n_loads == 43
+    assert r.makespan == 43 * d + 100 * gen.TAU_2D_NS
+    assert r.bytes_loaded == 43 * gen.DATUM_2D_BYTES
+    _check(inst, r)
+
+
+# ---------------------------------------------------------------- P4
+def _small_instances():
+    out = [gen.matmul2d(6, M=4, K=1), gen.matmul2d(7, M=5, K=2, order="random", seed=3),
+           gen.matmul3d(4, M=6, K=2), gen.matmul3d(3, M=9, K=3, with_c=True),
+           gen.cholesky(6, M=5, K=2), gen.random_shared(300, 64, 3, M=8, K=3, seed=7),
+           gen.random_shared(200, 32, 2, M=3, K=1, seed=9),
+           gen.matmul2d(20, M=6, K=4, keep_frac=0.1, seed=5)]
+    return out
+
+
+@pytest.mark.parametrize("idx", range(8))
+def test_p4_ample_memory_each_datum_loaded_once(idx):
+    inst = _small_instances()[idx]
+    big = inst.with_(mem_capacity=int(inst.data_size.sum()))
+    r = oracle.run(big)
+    _check(big, r)
+    used = np.unique(inst.task_data)
+    loads = [(int(e["gpu"]), int(e["data"])) for e in r.events if e["op"] == 0]
+    assert len(loads) == len(set(loads)), "a GPU loaded a datum twice with ample memory"
+    assert r.n_evictions == 0
+    if inst.K == 1:
+        assert r.n_loads == len(used)
+        assert r.bytes_loaded == int(inst.data_size[used].sum())
+
+
+@pytest.mark.parametrize("N", [3, 5, 8])
+def test_p4_2d_memory_2N_loads_2N(N):
+    inst = gen.matmul2d(N, M=2 * N, K=1)
+    r = oracle.run(inst)
+    assert r.n_loads == 2 * N and r.n_evictions == 0
+
+
+# ---------------------------------------------------------------- P5
+@pytest.mark.parametrize("idx", range(8))
+@pytest.mark.parametrize("W", [0, 1])
+def test_p5_invariants(idx, W):
+    inst = _small_instances()[idx]
+    if W == 1:
+        inst = inst.with_(mem_capacity=int(inst.mem_capacity) + int(inst.data_size.max()) * 3)
+    r = oracle.run(inst, W=W)
+    chk = _check(inst, r, W=W)
+    assert chk["n_loads"] == r.n_loads and chk["n_evictions"] == r.n_evictions
+    assert chk["bytes_loaded"] == r.bytes_loaded and chk["makespan"] == r.makespan
+    assert r.n_belady == 0  # unreachable with the capacity check (reading R7)
+    assert sum(len(o) for o in r.orders()) == inst.m
+
+
+def test_p5_heterogeneous_sizes():
+    rng = np.random.default_rng(4)
+    base = gen.random_shared(400, 64, 3, M=8, K=3, seed=11)
+    sizes = rng.integers(1, 5, size=64).astype(np.uint64) * 1_000_000
+    inst = base.with_(data_size=sizes, mem_capacity=int(sizes.max()) * 7)
+    r = oracle.run(inst)
+    _check(inst, r)
+
+
+def test_prefix_is_prefix_of_full_run():
+    inst = gen.random_shared(500, 64, 3, M=6, K=4, seed=5)
+    full = oracle.run(inst)
+    pre = oracle.run(inst, max_served=123)
+    assert pre.n_served == 123
+    assert np.array_equal(pre.serve_task, full.serve_task[:123])
+    assert np.array_equal(pre.events, full.events[:len(pre.events)])
+    _check(inst, pre, complete=False)
+
+
+# ---------------------------------------------------------------- P6
+def _tiny(seed, m, n, K, M):
+    rnd = random.Random(seed)
+    rows = [sorted(rnd.sample(range(n), rnd.choice([1, 2, 2, 3]))) for _ in range(m)]
+    tp = np.zeros(m + 1, np.int64)
+    tp[1:] = np.cumsum([len(r) for r in rows])
+    td = np.array([d for r in rows for d in r], np.int32)
+    return gen.Instance(f"tiny{seed}", tp, td, np.ones(n, np.uint64), None, 1, M, K)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_p6_brute_force_k1(seed):
+    inst = _tiny(seed, m=6 + seed % 2, n=5, K=1, M=3)
+    r = oracle.run(inst, bus_bps=10 ** 9)
+    ds = dsets_of(inst)
+    opt = brute_force_opt(ds, 3)
+    bel = belady_loads(r.orders(), ds, 3)
+    assert opt <= bel <= r.n_loads
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_p6_brute_force_k2(seed):
+    inst = _tiny(100 + seed, m=5, n=5, K=2, M=3)
+    r = oracle.run(inst, bus_bps=10 ** 9)
+    ds = dsets_of(inst)
+    opt = brute_force_opt(ds, 3, K=2)
+    bel = belady_loads(r.orders(), ds, 3)
+    assert opt <= bel <= r.n_loads
+    _check(inst, r, bus=10 ** 9)
