@@ -1,0 +1,168 @@
+/*
+ * dts.h -- C ABI of libdts: B200-native (sm_100a) DARTS+LUF memory-aware task
+ * scheduling simulator.
+ *
+ * Method: Gonthier, Marchal, Thibault, "Memory-Aware Scheduling of Tasks
+ * Sharing Data on Multiple GPUs with Dynamic Runtime Systems", IPDPS 2022.
+ * Citations are to /root/reference/PAPER.md lines (section / algorithm).
+ *
+ * Problem (§III): m independent tasks T and n data D form a
+ * bipartite graph; D(T) is the set of inputs of T.  K GPUs each hold at most
+ * `mem_capacity_bytes` of data (M data when sizes are uniform).  A schedule
+ * assigns each task to one GPU and orders it; before a task runs, its missing
+ * inputs are loaded over a shared bus (Fig. 2), after evictions if needed
+ * (PAPER.md:285-295).  The library computes the DARTS+LUF schedule:
+ *   - DARTS data selection, Algorithm 5, with the
+ *     "3inputs" fallback of §V-E, flag DTS_F_FALLBACK2;
+ *   - LUF eviction, Algorithm 6;
+ * deterministically (lowest-id tie-breaks, readings R1-R27 of DESIGN.md), and
+ * returns the per-GPU task order sigma(k,i), the load/evict trace V(k,i), the
+ * bytes transferred (Obj. 2) and the modelled makespan.
+ *
+ * Every step runs in CUDA kernels on one B200; there is no CPU fallback: a
+ * missing or unusable GPU is reported as DTS_E_CUDA.
+ *
+ * Conventions
+ *   - All ids are 0-based int32.  All times are integer nanoseconds.
+ *   - Every function returns a dts_status; nothing aborts.  On error,
+ *     dts_last_error() returns a thread-local message.
+ *   - Ownership: dts_instance_create COPIES the caller's arrays (the caller
+ *     keeps ownership of them).  Result views belong to the instance and stay
+ *     valid until the next dts_run on it or dts_instance_destroy.
+ *   - Thread safety: distinct instances may be used from distinct threads;
+ *     one instance must not be used concurrently.
+ */
+#ifndef DTS_H
+#define DTS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct dts_instance dts_instance; /* opaque, owned by the library */
+
+typedef enum {
+    DTS_OK = 0,
+    DTS_E_INVAL = -1,       /* malformed argument (pointer, range, monotonicity) */
+    DTS_E_CAPACITY = -2,    /* capacity < (W+1) * max_T sum_{D in D(T)} size(D) */
+    DTS_E_NOMEM = -3,       /* host or device allocation failed */
+    DTS_E_CUDA = -4,        /* CUDA error, no device, or device is not sm_100 */
+    DTS_E_STATE = -5,       /* call out of order (e.g. dts_result before dts_run) */
+    DTS_E_UNSUPPORTED = -6  /* outside the packed-state limits (see dts_instance_create) */
+} dts_status;
+
+typedef enum {
+    DTS_POLICY_DARTS_LUF = 1 /* Alg. 5 + Alg. 6 */
+} dts_policy;
+
+enum {
+    /* "3inputs" fallback when no datum frees a task: load the datum that
+     * makes the most tasks one load away.  Default ON. */
+    DTS_F_FALLBACK2 = 1u << 0
+};
+
+typedef struct {
+    uint32_t flags;           /* DTS_F_* ; default DTS_F_FALLBACK2 */
+    uint32_t lookahead_W;     /* taskBuffer depth beyond the served task;
+                                 0 (default, the formal model of §III) -- others: UNSUPPORTED */
+    uint64_t bus_bytes_per_s; /* shared host->GPU bus bandwidth; default 12e9 (reading R9) */
+    int32_t device;           /* CUDA device ordinal; default 0 */
+    int32_t n_ctas;           /* CTAs cooperating on one instance; 0 = automatic */
+    int64_t max_served;       /* stop after this many served tasks (prefix runs); -1 = all */
+    void *cuda_stream;        /* cudaStream_t to enqueue on; NULL = the legacy default stream */
+} dts_run_opts;
+
+/* Fill *opts with the defaults above. */
+void dts_run_opts_default(dts_run_opts *opts);
+
+/* One entry of the load/evict trace.  32 bytes, naturally aligned.
+ *   op 0 = LOAD : datum `data` crosses the shared bus to GPU `gpu` during
+ *                 [t_ns, t_end_ns) (FIFO bus);
+ *   op 1 = EVICT: datum `data` leaves GPU `gpu` memory at t_ns = t_end_ns
+ *                 (Alg. 6 l.9);
+ * `task` is the task whose service triggered the event (the task of step i
+ * in V(k,i) / D(T_sigma(k,i))). */
+typedef struct {
+    int64_t t_ns, t_end_ns;
+    int32_t gpu, data, task;
+    uint8_t op;
+    uint8_t pad[3];
+} dts_event;
+
+/* Create an instance from a task->data CSR.
+ *   n_tasks, n_data : m >= 0, n >= 0; n < 2^24.
+ *   task_ptr  [m+1] : host, task_ptr[0] = 0, non-decreasing.
+ *   task_data [task_ptr[m]] : host, ids in [0, n).  Duplicates inside a row
+ *                     are removed (D(T) is a set); at most
+ *                     127 distinct inputs per task (else DTS_E_UNSUPPORTED).
+ *   data_size [n]   : host, bytes, each > 0 (uniform sizes = the paper's
+ *                     model; heterogeneous sizes = the extension of
+ *                     PAPER.md:449-451, reading R11).
+ *   task_ns   [m]   : host, task durations (>= 0) or NULL => default_task_ns.
+ *   mem_capacity_bytes : per simulated GPU.
+ *   K               : simulated GPUs, 1 <= K <= 64.
+ *   out             : receives the new instance; destroy with dts_instance_destroy.
+ * Host-only: validates and copies; no device work happens until dts_run. */
+dts_status dts_instance_create(int32_t n_tasks, int32_t n_data, const int64_t *task_ptr,
+                               const int32_t *task_data, const uint64_t *data_size,
+                               const int64_t *task_ns, int64_t default_task_ns,
+                               uint64_t mem_capacity_bytes, int32_t K, dts_instance **out);
+
+/* Optional: pre-stage the instance's raw CSR on `device` (H2D on `cuda_stream`),
+ * so that a later dts_run starts with its inputs resident in HBM. */
+dts_status dts_instance_upload(dts_instance *inst, int32_t device, void *cuda_stream);
+
+/* Run the policy.  Enqueues on opts->cuda_stream: (upload if needed) -> CSR
+ * build (sort/dedup rows, data->task transpose) -> state init -> the device-
+ * resident decision loop -> result assembly.  Returns after enqueueing; the
+ * results stay on the device until dts_result (which synchronises).
+ * opts may be NULL (defaults).  DTS_E_CAPACITY if the capacity cannot hold
+ * (W+1) tasks' inputs (this keeps Alg. 6 l.4's first branch non-empty). */
+dts_status dts_run(dts_instance *inst, dts_policy policy, const dts_run_opts *opts);
+
+typedef struct {
+    int32_t K, n_tasks;
+    const int64_t *gpu_task_ptr;   /* [K+1] offsets into gpu_task_ids                      */
+    const int32_t *gpu_task_ids;   /* [n_served] sigma(k, .) for each k, in processing order */
+    const int32_t *serve_gpu;      /* [n_served] GPU of the i-th served request (event order) */
+    const int32_t *serve_task;     /* [n_served] task of the i-th served request              */
+    const int64_t *task_start_ns;  /* [n_tasks], -1 if not served (prefix runs)               */
+    const int64_t *task_end_ns;    /* [n_tasks]                                               */
+    int64_t n_events;
+    const dts_event *events;       /* [n_events] load/evict trace in event order              */
+    uint64_t bytes_loaded;         /* sum of sizes of the LOAD events (Obj. 2 in bytes)       */
+    int64_t n_loads, n_evictions;
+    int64_t makespan_ns;           /* max task end                                            */
+    double makespan_s;
+    int64_t n_served;              /* served requests = decisions (reading R21)              */
+    int64_t n_scans;               /* requests that found plannedTasks_k empty and got a task */
+    int64_t n_fallback2, n_fallback_first, n_belady, n_idle_requests;
+    uint64_t alg_bytes;            /* algorithmic HBM bytes of the decision loop  */
+    uint64_t scan_alg_bytes;       /* ... of which in the per-scan pass                       */
+    float loop_ms;                 /* device time of the decision-loop kernel (CUDA events)  */
+    float total_ms;                /* device time of the whole run (CSR build..assembly)     */
+} dts_result_view;
+
+/* Synchronise on the run's stream, copy the results to host (once) and fill *out. */
+dts_status dts_result(dts_instance *inst, dts_result_view *out);
+
+/* Sweep (BASELINE config 5): run every instance of insts[0..n) on ONE device
+ * with one CTA per instance in a single batched launch of the same loop
+ * (no communication between instances).  opts->device selects the device.
+ * Results are read per instance with dts_result. */
+dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy,
+                         const dts_run_opts *opts);
+
+void dts_instance_destroy(dts_instance *inst);
+const char *dts_status_str(dts_status s);
+const char *dts_last_error(void);
+
+/* ABI version: (major << 16) | minor. */
+uint32_t dts_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DTS_H */

@@ -1,0 +1,25 @@
+"""B200-native (sm_100a) DARTS+LUF memory-aware task scheduling simulator.
+
+The compute path is ``lib/libdts.so`` (hand-written CUDA, C ABI in
+``include/dts.h``); this package is its thin Python binding.  No CPU
+fallback: without the library or a B200 the calls raise ``DtsError``.
+"""
+from .dts import (  # noqa: F401
+    DTS_F_FALLBACK2,
+    DTS_POLICY_DARTS_LUF,
+    EVENT_DTYPE,
+    EXPORTED,
+    LIB_PATH,
+    DtsError,
+    Instance,
+    Result,
+    dts_instance_create,
+    dts_instance_upload,
+    dts_result,
+    dts_run,
+    dts_run_opts_default,
+    dts_sweep_run,
+    dts_version,
+    load_library,
+    schedule,
+)

@@ -1,0 +1,529 @@
+// dts_api.cu -- the C ABI of libdts (include/dts.h): validation, device memory,
+// stream orchestration and result transfer.  Host code never computes any part
+// of the schedule: it validates and copies inputs, launches the kernels of
+// dts_csr.cu / dts_loop.cu, and copies results back.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "dts.h"
+#include "dts_csr.cuh"
+#include "dts_internal.cuh"
+#include "dts_loop.cuh"
+
+namespace {
+
+thread_local std::string g_err;
+
+dts_status fail(dts_status s, const std::string &msg) {
+    g_err = msg;
+    return s;
+}
+
+dts_status cuda_fail(cudaError_t e, const char *where) {
+    g_err = std::string(where) + ": " + cudaGetErrorString(e);
+    return DTS_E_CUDA;
+}
+
+#define CK(expr, where)                          \
+    do {                                         \
+        cudaError_t _e = (expr);                 \
+        if (_e != cudaSuccess) return cuda_fail(_e, where); \
+    } while (0)
+
+int bits_for(uint64_t v) {  // bits needed to represent v (>= 1)
+    int b = 1;
+    while (b < 64 && (v >> b) != 0) b++;
+    return b;
+}
+
+struct Arena {
+    char *base = nullptr;
+    size_t size = 0;
+    size_t used = 0;
+    template <typename T>
+    T *take(size_t count) {
+        size_t bytes = (sizeof(T) * count + 255) & ~size_t(255);
+        T *p = reinterpret_cast<T *>(base + used);
+        used += bytes;
+        return p;
+    }
+};
+
+}  // namespace
+
+struct dts_instance {
+    int32_t m = 0, n = 0, K = 1;
+    int64_t E_raw = 0;
+    uint64_t cap = 0;
+    int64_t default_ns = 0;
+    std::vector<int64_t> task_ptr;
+    std::vector<int32_t> task_data;
+    std::vector<uint64_t> size;
+    std::vector<int64_t> task_ns;
+    bool has_tau = false;
+    int32_t max_deg_ub = 0;
+    uint64_t max_row_bytes = 0;
+    uint64_t min_size = 1;
+    int32_t res_cap = 1;
+    int32_t m_pad = 0;
+
+    // device side
+    int device = -1;
+    Arena ar;
+    size_t arena_bytes = 0;
+    bool uploaded = false;
+    int64_t *d_raw_ptr = nullptr;
+    int32_t *d_raw_dat = nullptr;
+    uint64_t *d_size = nullptr;
+    int64_t *d_tau = nullptr;
+    int64_t *d_delta = nullptr;
+    int64_t **d_delta_ptr = nullptr;
+    void *d_csr_scratch = nullptr;
+    int *d_work = nullptr;
+    dts::Inst h_inst{};
+    dts::Inst *d_inst = nullptr;
+    cudaStream_t stream = nullptr;
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+
+    // run state / results
+    bool ran = false;
+    bool have_host = false;
+    dts::Out out{};
+    std::vector<int64_t> r_gpu_ptr;
+    std::vector<int32_t> r_gpu_ids, r_serve_gpu, r_serve_task;
+    std::vector<int64_t> r_tstart, r_tend;
+    std::vector<dts_event> r_events;
+    float loop_ms = 0.f, total_ms = 0.f;
+
+    ~dts_instance() {
+        if (device >= 0) {
+            int cur = 0;
+            cudaGetDevice(&cur);
+            cudaSetDevice(device);
+            if (ar.base) cudaFree(ar.base);
+            for (auto &e : ev)
+                if (e) cudaEventDestroy(e);
+            cudaSetDevice(cur);
+        }
+    }
+};
+
+extern "C" {
+
+void dts_run_opts_default(dts_run_opts *o) {
+    if (!o) return;
+    std::memset(o, 0, sizeof *o);
+    o->flags = DTS_F_FALLBACK2;
+    o->lookahead_W = 0;
+    o->bus_bytes_per_s = 12000000000ull;
+    o->device = 0;
+    o->n_ctas = 0;
+    o->max_served = -1;
+    o->cuda_stream = nullptr;
+}
+
+const char *dts_status_str(dts_status s) {
+    switch (s) {
+        case DTS_OK: return "DTS_OK";
+        case DTS_E_INVAL: return "DTS_E_INVAL";
+        case DTS_E_CAPACITY: return "DTS_E_CAPACITY";
+        case DTS_E_NOMEM: return "DTS_E_NOMEM";
+        case DTS_E_CUDA: return "DTS_E_CUDA";
+        case DTS_E_STATE: return "DTS_E_STATE";
+        case DTS_E_UNSUPPORTED: return "DTS_E_UNSUPPORTED";
+    }
+    return "DTS_E_UNKNOWN";
+}
+
+const char *dts_last_error(void) { return g_err.c_str(); }
+
+uint32_t dts_version(void) { return (1u << 16) | 0u; }
+
+dts_status dts_instance_create(int32_t n_tasks, int32_t n_data, const int64_t *task_ptr,
+                               const int32_t *task_data, const uint64_t *data_size,
+                               const int64_t *task_ns, int64_t default_task_ns,
+                               uint64_t mem_capacity_bytes, int32_t K, dts_instance **out) {
+    if (!out) return fail(DTS_E_INVAL, "out is NULL");
+    *out = nullptr;
+    if (n_tasks < 0 || n_data < 0) return fail(DTS_E_INVAL, "negative size");
+    if (K < 1) return fail(DTS_E_INVAL, "K < 1");
+    if (K > dts::MAX_K) return fail(DTS_E_UNSUPPORTED, "K > 64");
+    if (n_data >= (1 << 24)) return fail(DTS_E_UNSUPPORTED, "n_data >= 2^24 (packed xor field)");
+    if (!task_ptr) return fail(DTS_E_INVAL, "task_ptr is NULL");
+    if (n_data > 0 && !data_size) return fail(DTS_E_INVAL, "data_size is NULL");
+    if (task_ptr[0] != 0) return fail(DTS_E_INVAL, "task_ptr[0] != 0");
+    const int64_t E = task_ptr[n_tasks];
+    if (E > 0 && !task_data) return fail(DTS_E_INVAL, "task_data is NULL");
+    if (default_task_ns < 0) return fail(DTS_E_INVAL, "default_task_ns < 0");
+    if (E >= (int64_t)INT32_MAX) return fail(DTS_E_UNSUPPORTED, "too many edges");
+    dts_instance *I = new (std::nothrow) dts_instance();
+    if (!I) return fail(DTS_E_NOMEM, "host allocation");
+    try {
+        I->m = n_tasks;
+        I->n = n_data;
+        I->K = K;
+        I->E_raw = E;
+        I->cap = mem_capacity_bytes;
+        I->default_ns = default_task_ns;
+        I->task_ptr.assign(task_ptr, task_ptr + (size_t)n_tasks + 1);
+        if (E > 0) I->task_data.assign(task_data, task_data + E);
+        if (n_data > 0) I->size.assign(data_size, data_size + n_data);
+        if (task_ns) {
+            I->task_ns.assign(task_ns, task_ns + n_tasks);
+            I->has_tau = true;
+        }
+    } catch (...) {
+        delete I;
+        return fail(DTS_E_NOMEM, "host allocation");
+    }
+    // validation (input checking only; the schedule is computed on the device)
+    uint64_t min_size = UINT64_MAX;
+    for (int32_t D = 0; D < n_data; D++) {
+        if (I->size[D] == 0) {
+            delete I;
+            return fail(DTS_E_INVAL, "data_size[" + std::to_string(D) + "] == 0");
+        }
+        min_size = std::min(min_size, I->size[D]);
+    }
+    if (n_data == 0) min_size = 1;
+    std::vector<int32_t> occ((size_t)n_data + 1, 0);
+    int32_t scratch[dts::MAX_ROW];
+    for (int32_t T = 0; T < n_tasks; T++) {
+        int64_t b = I->task_ptr[T], e = I->task_ptr[T + 1];
+        if (e < b) {
+            delete I;
+            return fail(DTS_E_INVAL, "task_ptr not monotone at " + std::to_string(T));
+        }
+        if (e - b > dts::MAX_ROW) {
+            delete I;
+            return fail(DTS_E_UNSUPPORTED, "task " + std::to_string(T) + " has > 127 inputs");
+        }
+        if (I->has_tau && I->task_ns[T] < 0) {
+            delete I;
+            return fail(DTS_E_INVAL, "task_ns < 0");
+        }
+        int q = 0;
+        uint64_t bytes = 0;
+        for (int64_t i = b; i < e; i++) {
+            int32_t D = I->task_data[i];
+            if (D < 0 || D >= n_data) {
+                delete I;
+                return fail(DTS_E_INVAL, "task_data id out of range at edge " + std::to_string(i));
+            }
+            bool dup = false;
+            for (int j = 0; j < q; j++) dup |= (scratch[j] == D);
+            if (!dup) {
+                scratch[q++] = D;
+                bytes += I->size[D];
+                occ[D]++;
+            }
+        }
+        I->max_row_bytes = std::max(I->max_row_bytes, bytes);
+    }
+    int32_t md = 1;
+    for (int32_t D = 0; D < n_data; D++) md = std::max(md, occ[D]);
+    I->max_deg_ub = md;
+    I->min_size = min_size;
+    uint64_t rc = mem_capacity_bytes / min_size;
+    I->res_cap = (int32_t)std::max<uint64_t>(1, std::min<uint64_t>(rc, (uint64_t)std::max(n_data, 1)));
+    I->m_pad = (n_tasks + 3) & ~3;
+    int hb = bits_for((uint64_t)md), idb = bits_for(n_data > 0 ? (uint64_t)(n_data - 1) : 0);
+    if (2 * hb + idb > 63) {
+        delete I;
+        return fail(DTS_E_UNSUPPORTED, "argmax key does not fit 64 bits");
+    }
+    *out = I;
+    return DTS_OK;
+}
+
+void dts_instance_destroy(dts_instance *inst) { delete inst; }
+
+}  // extern "C"
+
+namespace {
+
+dts_status check_device(int device) {
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0) return fail(DTS_E_CUDA, "no CUDA device (libdts has no CPU path)");
+    if (device < 0 || device >= ndev) return fail(DTS_E_INVAL, "device ordinal out of range");
+    cudaDeviceProp p;
+    CK(cudaGetDeviceProperties(&p, device), "cudaGetDeviceProperties");
+    if (p.major != 10) return fail(DTS_E_CUDA, "libdts is built for sm_100a (B200); device is sm_" +
+                                                   std::to_string(p.major) + std::to_string(p.minor));
+    return DTS_OK;
+}
+
+dts_status ensure_device(dts_instance *I, int device) {
+    if (I->device == device && I->ar.base) return DTS_OK;
+    if (I->device >= 0 && I->ar.base) {
+        cudaSetDevice(I->device);
+        cudaFree(I->ar.base);
+        for (auto &e : I->ev)
+            if (e) cudaEventDestroy(e);
+        I->ar = Arena{};
+        I->uploaded = false;
+    }
+    dts_status s = check_device(device);
+    if (s != DTS_OK) return s;
+    CK(cudaSetDevice(device), "cudaSetDevice");
+    const size_t m = (size_t)I->m, n = (size_t)I->n, K = (size_t)I->K, E = (size_t)I->E_raw;
+    const size_t mp = (size_t)I->m_pad;
+    const size_t ev_cap = 2 * E + 16;
+    const size_t plan_cap = (size_t)I->max_deg_ub + 1;
+    const size_t res_cap = (size_t)I->res_cap + 1;
+    size_t need = 0;
+    auto add = [&](size_t bytes) { need += (bytes + 255) & ~size_t(255); };
+    add(8 * (m + 1)); add(4 * (E + 1)); add(8 * (n + 1)); add(8 * (m + 1));        // raw
+    add(8 * (m + 1)); add(4 * (E + 1)); add(8 * (n + 1)); add(4 * (E + 1));        // CSR
+    add(8 * (n + 1)); add(8);                                                      // delta
+    add(4 * K * mp + 16); add(4 * (n + 1)); add(4 * (n + 1)); add(4 * K * (n + 1)); // s u hist np
+    add(4 * K * res_cap); add(4 * K * (n + 1)); add(4 * K * plan_cap);            // residency, plans
+    add(sizeof(dts::Ctrl)); add(sizeof(dts::Out));
+    add(4 * (m + 1)); add(4 * (m + 1)); add(8 * (m + 1)); add(8 * (m + 1));        // serve, times
+    add(sizeof(dts_event) * ev_cap); add(8 * (K + 1)); add(4 * (m + 1));
+    add(sizeof(dts::Inst)); add(64);
+    add(dts::csr_scratch_bytes(I->m, I->n, I->E_raw));
+    char *base = nullptr;
+    cudaError_t e = cudaMalloc(&base, need);
+    if (e != cudaSuccess) return fail(DTS_E_NOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    I->ar.base = base;
+    I->ar.size = need;
+    I->ar.used = 0;
+    I->device = device;
+    for (auto &ev : I->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
+
+    Arena &A = I->ar;
+    dts::Inst &h = I->h_inst;
+    std::memset(&h, 0, sizeof h);
+    I->d_raw_ptr = A.take<int64_t>(m + 1);
+    I->d_raw_dat = A.take<int32_t>(E + 1);
+    I->d_size = A.take<uint64_t>(n + 1);
+    I->d_tau = A.take<int64_t>(m + 1);
+    h.tptr = A.take<int64_t>(m + 1);
+    h.tdat = A.take<int32_t>(E + 1);
+    h.dptr = A.take<int64_t>(n + 1);
+    h.ddat = A.take<int32_t>(E + 1);
+    I->d_delta = A.take<int64_t>(n + 1);
+    I->d_delta_ptr = A.take<int64_t *>(1);
+    h.s = A.take<uint32_t>(K * mp + 4);
+    h.u = A.take<int32_t>(n + 1);
+    h.hist = A.take<int32_t>(n + 1);
+    h.np = A.take<int32_t>(K * (n + 1));
+    h.res_list = A.take<int32_t>(K * res_cap);
+    h.res_pos = A.take<int32_t>(K * (n + 1));
+    h.planned = A.take<int32_t>(K * plan_cap);
+    h.ctrl = A.take<dts::Ctrl>(1);
+    h.out = A.take<dts::Out>(1);
+    h.serve_gpu = A.take<int32_t>(m + 1);
+    h.serve_task = A.take<int32_t>(m + 1);
+    h.tstart = A.take<int64_t>(m + 1);
+    h.tend = A.take<int64_t>(m + 1);
+    h.events = A.take<dts_event>(ev_cap);
+    h.gpu_task_ptr = A.take<int64_t>(K + 1);
+    h.gpu_task_ids = A.take<int32_t>(m + 1);
+    I->d_inst = A.take<dts::Inst>(1);
+    I->d_work = A.take<int>(16);
+    I->d_csr_scratch = A.take<char>(dts::csr_scratch_bytes(I->m, I->n, I->E_raw));
+    if (A.used > A.size) return fail(DTS_E_NOMEM, "arena overflow (internal)");
+
+    h.m = I->m;
+    h.n = I->n;
+    h.K = I->K;
+    h.m_pad = I->m_pad;
+    h.cap = I->cap;
+    h.plan_cap = (int32_t)plan_cap;
+    h.res_cap = (int32_t)res_cap;
+    h.id_bits = bits_for(I->n > 0 ? (uint64_t)(I->n - 1) : 0);
+    h.u_bits = bits_for((uint64_t)I->max_deg_ub);
+    h.E = I->E_raw;
+    h.size = I->d_size;
+    h.delta = I->d_delta;
+    h.tau = I->has_tau ? I->d_tau : nullptr;
+    h.default_tau = I->default_ns;
+    h.ev_cap = (int64_t)ev_cap;
+    return DTS_OK;
+}
+
+dts_status upload(dts_instance *I, cudaStream_t st) {
+    if (I->uploaded) return DTS_OK;
+    CK(cudaMemcpyAsync(I->d_raw_ptr, I->task_ptr.data(), 8 * ((size_t)I->m + 1), cudaMemcpyHostToDevice, st),
+       "H2D task_ptr");
+    if (I->E_raw > 0)
+        CK(cudaMemcpyAsync(I->d_raw_dat, I->task_data.data(), 4 * (size_t)I->E_raw, cudaMemcpyHostToDevice, st),
+           "H2D task_data");
+    if (I->n > 0)
+        CK(cudaMemcpyAsync(I->d_size, I->size.data(), 8 * (size_t)I->n, cudaMemcpyHostToDevice, st),
+           "H2D data_size");
+    if (I->has_tau && I->m > 0)
+        CK(cudaMemcpyAsync(I->d_tau, I->task_ns.data(), 8 * (size_t)I->m, cudaMemcpyHostToDevice, st),
+           "H2D task_ns");
+    CK(cudaMemcpyAsync(I->d_delta_ptr, &I->d_delta, sizeof(int64_t *), cudaMemcpyHostToDevice, st),
+       "H2D delta ptr");
+    I->uploaded = true;
+    return DTS_OK;
+}
+
+dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_opts *o) {
+    if (policy != DTS_POLICY_DARTS_LUF) return fail(DTS_E_UNSUPPORTED, "policy");
+    if (o->flags & ~(uint32_t)DTS_F_FALLBACK2) return fail(DTS_E_UNSUPPORTED, "unknown flags");
+    if (o->lookahead_W != 0) return fail(DTS_E_UNSUPPORTED, "lookahead_W != 0 (NEXT)");
+    if (o->bus_bytes_per_s == 0) return fail(DTS_E_INVAL, "bus_bytes_per_s == 0");
+    if (o->n_ctas < 0) return fail(DTS_E_INVAL, "n_ctas < 0");
+    unsigned __int128 need = (unsigned __int128)(o->lookahead_W + 1) * I->max_row_bytes;
+    if ((unsigned __int128)I->cap < need)
+        return fail(DTS_E_CAPACITY, "mem_capacity_bytes < (W+1) * max_T size(D(T))");
+    return DTS_OK;
+}
+
+int env_int(const char *name, int dflt) {
+    const char *v = std::getenv(name);
+    return v ? std::atoi(v) : dflt;
+}
+
+}  // namespace
+
+extern "C" {
+
+dts_status dts_instance_upload(dts_instance *I, int32_t device, void *cuda_stream) {
+    if (!I) return fail(DTS_E_INVAL, "instance is NULL");
+    dts_status s = ensure_device(I, device);
+    if (s != DTS_OK) return s;
+    cudaStream_t st = (cudaStream_t)cuda_stream;
+    return upload(I, st);
+}
+
+dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts) {
+    if (!I) return fail(DTS_E_INVAL, "instance is NULL");
+    dts_run_opts o;
+    if (opts) o = *opts;
+    else dts_run_opts_default(&o);
+    dts_status s = check_opts(I, policy, &o);
+    if (s != DTS_OK) return s;
+    s = ensure_device(I, o.device);
+    if (s != DTS_OK) return s;
+    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    cudaStream_t st = (cudaStream_t)o.cuda_stream;
+    I->stream = st;
+    I->ran = false;
+    I->have_host = false;
+    s = upload(I, st);
+    if (s != DTS_OK) return s;
+
+    dts::Inst &h = I->h_inst;
+    h.W = (int32_t)o.lookahead_W;
+    h.flags = o.flags;
+    h.max_served = o.max_served;
+
+    int nsm = 0;
+    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
+    int G = o.n_ctas;
+    if (G == 0) {
+        int64_t want = ((int64_t)I->m + 16383) / 16384;
+        G = (int)std::max<int64_t>(1, std::min<int64_t>(want, nsm));
+    }
+    int block = env_int("DTS_BLOCK", 512);
+    int smem_hist_cap = (G == 1 && I->n <= 32768) ? std::max(I->n, 1) : 0;
+    if (G > 1) {
+        int per = dts::loop_max_blocks_per_sm(block, 0);
+        if (per * nsm < G) return fail(DTS_E_UNSUPPORTED, "n_ctas exceeds co-resident CTAs");
+    }
+
+    CK(cudaEventRecord(I->ev[0], st), "event");
+    CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
+                      (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, I->d_csr_scratch, st),
+       "build_csr");
+    CK(cudaMemcpyAsync(I->d_inst, &h, sizeof h, cudaMemcpyHostToDevice, st), "H2D inst");
+    int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n);
+    CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, I->d_delta_ptr, work, st), "init");
+    CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
+    CK(cudaEventRecord(I->ev[1], st), "event");
+    CK(dts::launch_loop(I->d_inst, 1, G, block, 1, I->d_work, smem_hist_cap, st), "loop");
+    CK(cudaEventRecord(I->ev[2], st), "event");
+    CK(dts::launch_assemble(I->d_inst, 1, st), "assemble");
+    CK(cudaEventRecord(I->ev[3], st), "event");
+    I->ran = true;
+    return DTS_OK;
+}
+
+dts_status dts_result(dts_instance *I, dts_result_view *v) {
+    if (!I || !v) return fail(DTS_E_INVAL, "NULL argument");
+    if (!I->ran) return fail(DTS_E_STATE, "dts_result before dts_run");
+    if (!I->have_host) {
+        CK(cudaSetDevice(I->device), "cudaSetDevice");
+        CK(cudaEventSynchronize(I->ev[3]), "run");
+        CK(cudaMemcpy(&I->out, I->h_inst.out, sizeof I->out, cudaMemcpyDeviceToHost), "D2H out");
+        if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim (Belady branch)");
+        const dts::Inst &h = I->h_inst;
+        size_t ns = (size_t)I->out.n_served, ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);
+        size_t m = (size_t)I->m;
+        I->r_gpu_ptr.resize((size_t)I->K + 1);
+        I->r_gpu_ids.resize(ns);
+        I->r_serve_gpu.resize(ns);
+        I->r_serve_task.resize(ns);
+        I->r_tstart.resize(m);
+        I->r_tend.resize(m);
+        I->r_events.resize(ne);
+        CK(cudaMemcpy(I->r_gpu_ptr.data(), h.gpu_task_ptr, 8 * ((size_t)I->K + 1), cudaMemcpyDeviceToHost), "D2H");
+        if (ns) {
+            CK(cudaMemcpy(I->r_gpu_ids.data(), h.gpu_task_ids, 4 * ns, cudaMemcpyDeviceToHost), "D2H");
+            CK(cudaMemcpy(I->r_serve_gpu.data(), h.serve_gpu, 4 * ns, cudaMemcpyDeviceToHost), "D2H");
+            CK(cudaMemcpy(I->r_serve_task.data(), h.serve_task, 4 * ns, cudaMemcpyDeviceToHost), "D2H");
+        }
+        if (m) {
+            CK(cudaMemcpy(I->r_tstart.data(), h.tstart, 8 * m, cudaMemcpyDeviceToHost), "D2H");
+            CK(cudaMemcpy(I->r_tend.data(), h.tend, 8 * m, cudaMemcpyDeviceToHost), "D2H");
+        }
+        if (ne) CK(cudaMemcpy(I->r_events.data(), h.events, sizeof(dts_event) * ne, cudaMemcpyDeviceToHost), "D2H");
+        CK(cudaEventElapsedTime(&I->loop_ms, I->ev[1], I->ev[2]), "elapsed");
+        CK(cudaEventElapsedTime(&I->total_ms, I->ev[0], I->ev[3]), "elapsed");
+        I->have_host = true;
+    }
+    std::memset(v, 0, sizeof *v);
+    v->K = I->K;
+    v->n_tasks = I->m;
+    v->gpu_task_ptr = I->r_gpu_ptr.data();
+    v->gpu_task_ids = I->r_gpu_ids.data();
+    v->serve_gpu = I->r_serve_gpu.data();
+    v->serve_task = I->r_serve_task.data();
+    v->task_start_ns = I->r_tstart.data();
+    v->task_end_ns = I->r_tend.data();
+    v->n_events = (int64_t)I->r_events.size();
+    v->events = I->r_events.data();
+    v->bytes_loaded = I->out.bytes_loaded;
+    v->n_loads = I->out.n_loads;
+    v->n_evictions = I->out.n_evictions;
+    v->makespan_ns = I->out.makespan;
+    v->makespan_s = (double)I->out.makespan * 1e-9;
+    v->n_served = I->out.n_served;
+    v->n_scans = I->out.n_scans;
+    v->n_fallback2 = I->out.n_fallback2;
+    v->n_fallback_first = I->out.n_fallback_first;
+    v->n_belady = I->out.n_belady;
+    v->n_idle_requests = I->out.n_idle;
+    v->alg_bytes = I->out.alg_bytes;
+    v->scan_alg_bytes = I->out.scan_alg_bytes;
+    v->loop_ms = I->loop_ms;
+    v->total_ms = I->total_ms;
+    return DTS_OK;
+}
+
+dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy,
+                         const dts_run_opts *opts) {
+    (void)insts;
+    (void)n;
+    (void)policy;
+    (void)opts;
+    return fail(DTS_E_UNSUPPORTED, "dts_sweep_run: not built yet");
+}
+
+}  // extern "C"

@@ -1,0 +1,16 @@
+// dts_loop.cuh -- launchers of the decision loop (see dts_loop.cu).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "dts_internal.cuh"
+
+namespace dts {
+cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t *const *d_deltas,
+                        int64_t work, cudaStream_t st);
+cudaError_t launch_loop(const Inst *d_insts, int n_inst, int G, int block, int grid,
+                        int *work_counter, int smem_hist_cap, cudaStream_t st);
+cudaError_t launch_assemble(const Inst *d_insts, int n_inst, cudaStream_t st);
+int loop_max_blocks_per_sm(int block, int smem_hist_cap);
+}  // namespace dts

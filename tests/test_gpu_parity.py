@@ -1,0 +1,169 @@
+"""GPU parity: libdts (sm_100a kernels, through the C ABI) vs the plain CPU
+oracle, element by element, bit-exact (integer schedule, reading R22).
+Needs a B200."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+import paper_conf_ipps_gonthiermt22_b200 as dts
+from conftest import GOLDEN
+from digest import digest
+from parity import assert_parity
+from validate import validate
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_gpu():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    dts.load_library()
+
+
+def _unit(inst):
+    M = int(inst.mem_capacity // int(inst.data_size[0]))
+    return inst.with_(data_size=np.ones(inst.n, dtype=np.uint64), mem_capacity=M,
+                      default_task_ns=1, task_ns=None)
+
+
+def _both(inst, bus=oracle.DEFAULT_BUS_BPS, n_ctas=0, flags=1, max_served=-1):
+    g = dts.schedule(inst, bus_bps=bus, n_ctas=n_ctas, flags=flags, max_served=max_served)
+    o = oracle.run(inst, bus_bps=bus, flags=flags, max_served=max_served)
+    return g, o
+
+
+# ------------------------------------------------------------ hand traces
+@pytest.mark.parametrize("flags", [1, 0])
+def test_fig1(flags):
+    inst = gen.fig1()
+    g, o = _both(inst, bus=10 ** 9, flags=flags)
+    assert_parity(g, o)
+    gold = json.load(open(os.path.join(GOLDEN, "fig1_darts_luf_hand.json")))
+    assert [list(map(int, x)) for x in g.orders()] == gold["orders"]
+    assert g.n_loads == 11 and g.makespan == 12
+
+
+def test_h1_config1_unit():
+    inst = _unit(gen.matmul2d(10, M=6, K=1))
+    g, o = _both(inst, bus=10 ** 9)
+    assert_parity(g, o)
+    assert g.n_loads == 43 and g.n_evictions == 37
+
+
+def test_config1():
+    inst = gen.config_instances("C1")[0]
+    g, o = _both(inst)
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("idx", range(20))
+def test_config2(idx):
+    inst = gen.config_instances("C2")[idx]
+    g, o = _both(inst)
+    assert_parity(g, o)
+
+
+# ------------------------------------------------------------ varied shapes
+def _shapes():
+    return [gen.matmul2d(6, M=4, K=1), gen.matmul2d(7, M=5, K=2, order="random", seed=3),
+            gen.matmul3d(4, M=6, K=2), gen.matmul3d(3, M=9, K=3, with_c=True),
+            gen.cholesky(6, M=5, K=2), gen.random_shared(300, 64, 3, M=8, K=3, seed=7),
+            gen.random_shared(200, 32, 2, M=3, K=1, seed=9),
+            gen.matmul2d(20, M=6, K=4, keep_frac=0.1, seed=5),
+            gen.random_shared(5000, 256, 3, M=20, K=8, seed=1),
+            gen.cholesky(20, M=30, K=4), gen.matmul3d(10, M=25, K=4),
+            gen.matmul2d(30, M=12, K=3, order="random", seed=8)]
+
+
+@pytest.mark.parametrize("idx", range(12))
+@pytest.mark.parametrize("n_ctas", [1, 3, 16])
+def test_shapes_group_sizes(idx, n_ctas):
+    inst = _shapes()[idx]
+    g, o = _both(inst, n_ctas=n_ctas)
+    assert_parity(g, o)
+    validate(inst, g.serve_gpu, g.serve_task, g.events, g.task_start, g.task_end)
+
+
+def test_heterogeneous_sizes():
+    rng = np.random.default_rng(4)
+    base = gen.random_shared(2000, 128, 3, M=8, K=4, seed=11)
+    sizes = rng.integers(1, 5, size=128).astype(np.uint64) * 1_000_000
+    inst = base.with_(data_size=sizes, mem_capacity=int(sizes.max()) * 9)
+    for G in (1, 4):
+        g, o = _both(inst, n_ctas=G)
+        assert_parity(g, o)
+
+
+def test_ample_memory_and_duplicates():
+    inst = gen.random_shared(3000, 128, 3, M=8, K=2, seed=2)
+    # duplicated ids inside rows are removed (D(T) is a set, R27)
+    td = inst.task_data.copy()
+    td[1::3] = td[0::3]
+    dup = inst.with_(task_data=td)
+    g, o = _both(dup)
+    assert_parity(g, o)
+    big = inst.with_(mem_capacity=int(inst.data_size.sum()))
+    g, o = _both(big, n_ctas=4)
+    assert_parity(g, o)
+    assert g.n_evictions == 0
+
+
+def test_empty_and_degenerate():
+    # tasks without inputs, an unused datum, a single task
+    tp = np.array([0, 0, 2, 2, 3], np.int64)
+    td = np.array([0, 2, 2], np.int32)
+    inst = gen.Instance("degen", tp, td, np.ones(4, np.uint64), None, 5, 2, 2)
+    g, o = _both(inst, bus=10 ** 9)
+    assert_parity(g, o)
+    one = gen.Instance("one", np.array([0, 1], np.int64), np.array([0], np.int32),
+                       np.ones(1, np.uint64), None, 3, 1, 3)
+    g, o = _both(one, bus=10 ** 9)
+    assert_parity(g, o)
+    empty = gen.Instance("empty", np.array([0], np.int64), np.zeros(0, np.int32),
+                         np.ones(2, np.uint64), None, 3, 1, 2)
+    g = dts.schedule(empty)
+    assert g.n_served == 0 and len(g.events) == 0
+
+
+def test_ragged_tail_sizes():
+    # m not a multiple of 4 (uint4 scan tail) and of the CTA size
+    for m in (1, 2, 3, 5, 4097, 10001):
+        inst = gen.random_shared(m, 64, 3, M=6, K=2, seed=m)
+        g, o = _both(inst, n_ctas=2)
+        assert_parity(g, o)
+
+
+# ------------------------------------------------------------ larger configs
+def test_config3():
+    inst = gen.config_instances("C3")[0]
+    g, o = _both(inst)
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("cfg", ["C4a", "C4b"])
+def test_config4_prefix(cfg):
+    """Full-size config 4 in the bench's launch configuration, prefix of 1,500
+    served requests (the plain oracle costs O(E) per scan)."""
+    inst = gen.config_instances(cfg)[0]
+    g, o = _both(inst, max_served=1500)
+    assert_parity(g, o, complete=False)
+
+
+@pytest.mark.parametrize("cfg", ["C4a", "C4b"])
+def test_config4_full_digest(cfg):
+    path = os.path.join(GOLDEN, f"digests_{cfg}.json")
+    if not os.path.exists(path):
+        pytest.skip("golden digest not produced yet (tests/golden/make_digests.py)")
+    gold = json.load(open(path))
+    inst = gen.config_instances(cfg)[0]
+    g = dts.schedule(inst)
+    for k in ("n_served", "n_loads", "n_evictions", "n_scans", "n_fallback2", "n_fallback_first",
+              "bytes_loaded", "makespan"):
+        assert getattr(g, k) == gold[k], k
+    assert digest(g.serve_gpu, g.serve_task, g.task_start, g.task_end, g.events) == gold["sha256"]
