@@ -1,0 +1,391 @@
+#!/usr/bin/env python
+"""bench.py -- DARTS+LUF scheduling throughput on B200 (driver contract).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload C2|C1|C3|C4a|C4b|C5]
+
+A *step* is one pass of the whole hot path (device CSR
+build, state init, the device-resident DARTS+LUF decision loop, result
+assembly) over one batch of synthetic instances.  Default workload = BASELINE
+config 2 (configs[1]): the 20 2D tiled-matmul instances N = 10..100 (step 10)
+x K in {2, 4} simulated GPUs, M = 35 data (500 MiB) per simulated GPU, all
+scheduled by ONE batched launch (one CTA per instance).
+
+Multi-GPU (torchrun, one process per B200): each rank schedules its own copy
+of the batch -- independent problems, no data-path collective -- so scaling
+is "weak"; C5 (the 4,096-instance sweep) is sharded across ranks instead
+("strong").  Time = max over ranks of the device time (CUDA events).
+
+value = decisions/s (served requests, reading R21) over all ranks, inputs
+resident in HBM.  e2e = the same through the public API with the host->device
+upload of every instance and the device->host read of every result inside
+the timed region.  --impl reference times the plain CPU oracle (oracle/) on
+the host cores instead (the reference arm for this tier).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+from concurrent.futures import ThreadPoolExecutor
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import gen  # noqa: E402
+
+METRIC = "DARTS+LUF scheduling decisions/sec and HBM GB/s at 1/2/4/8 B200; bytes loaded"
+UNIT = "decisions/s"
+
+WORKLOADS = {
+    "C1": "2D tiled matmul 10x10 tiles (100 tasks, 20 data), K=1, M=6 data",
+    "C2": "2D tiled matmul N=10..100 (step 10) x K in {2,4}, M=35 data (500 MiB) per simulated GPU",
+    "C3": "3D tiled matmul N=40 (64,000 tasks, 3,200 tiles), K=4, M=142 tiles (500 MiB)",
+    "C4a": "Cholesky task set N=181 tiles (1,004,731 tasks, 16,471 tiles), K=8, M=142",
+    "C4b": "random shared-input tasks (2^20 tasks x 3 inputs over 2^14 data), K=8, M=1024",
+    "C5": "sweep of 4,096 2D instances (N 5..160 x M 4..128 x K 1..8), sharded over ranks",
+}
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def _traffic(workload):
+    """Per-launch DRAM bytes of the loop kernel from the committed ncu --set full
+    summary (profiles/ncu_full_<workload>.json), else None."""
+    p = os.path.join(ROOT, "profiles", f"ncu_full_{workload}.json")
+    try:
+        d = json.load(open(p))
+        return int(d["dram_bytes_per_launch"])
+    except Exception:
+        return None
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap,utilization.gpu")
+
+    def __init__(self, dev):
+        self.dev = dev
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+            self.t.join(timeout=2)
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                s, m_, util = float(f[0]), float(f[1]), float(f[7])
+            except ValueError:
+                continue
+            mx = m_
+            if util > 0:
+                sm.append(s)
+            for name, v in zip(("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown",
+                                "sw_power_cap"), f[3:7]):
+                if v.lower() == "active":
+                    reasons.add(name)
+        if not sm:
+            sm = [float(ln.split(",")[0]) for ln in self.lines
+                  if ln and ln.split(",")[0].strip().replace(".", "").isdigit()]
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(self.lines)}
+
+
+def workload_instances(name, rank, world):
+    if name == "C5":
+        params = gen.sweep_params()
+        # strong scaling: shard the 4,096 instances; LPT-like round robin on a
+        # cost estimate (m * N, heaviest first) so every rank gets a similar mix
+        cost = [(-(N * N) * N * 1.0, i) for i, (N, M, K) in enumerate(params)]
+        order = [i for _, i in sorted(cost)]
+        mine = order[rank::world]
+        return [gen.sweep_instance(*params[i]) for i in mine], "strong"
+    return gen.config_instances(name), "weak"
+
+
+# ------------------------------------------------------------------ oracle
+def oracle_sample(insts, budget_s, threads):
+    """Time the plain CPU oracle (as it stands) over the batch, repeated until
+    budget_s elapsed; one instance per thread (ctypes releases the GIL)."""
+    import oracle
+    oracle._load()
+    done_dec = 0
+    n_batches = 0
+    t0 = time.perf_counter()
+    with ThreadPoolExecutor(max_workers=threads) as ex:
+        while True:
+            # biggest instances first so the pool stays busy
+            order = sorted(insts, key=lambda i: -i.E)
+            rs = list(ex.map(lambda i: oracle.run(i), order))
+            done_dec += sum(r.n_served for r in rs)
+            n_batches += 1
+            if time.perf_counter() - t0 >= budget_s:
+                break
+    dt = time.perf_counter() - t0
+    return done_dec / dt, dt, n_batches, done_dec
+
+
+def oracle_prefix_sample(inst, budget_s):
+    """Large single instances: the oracle on a prefix of served requests sized
+    to ~budget_s (the plain oracle costs O(E) per scan)."""
+    import oracle
+    n = 200
+    while True:
+        t0 = time.perf_counter()
+        r = oracle.run(inst, max_served=n)
+        dt = time.perf_counter() - t0
+        if dt >= budget_s / 4 or n >= inst.m:
+            return r.n_served / dt, dt, r.n_served
+        n = min(inst.m, int(n * max(2.0, budget_s / 4 / max(dt, 1e-3))))
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    insts, scaling = workload_instances(args.workload, 0, 1)
+    cores = os.cpu_count() or 1
+    big = args.workload in ("C4a", "C4b")
+    for _ in range(args.warmup):
+        if big:
+            oracle_prefix_sample(insts[0], 2.0)
+        else:
+            oracle_sample(insts[:min(len(insts), 64)], 0.0, cores)
+    times, decs = [], []
+    for _ in range(args.steps):
+        if big:
+            rate, dt, nd = oracle_prefix_sample(insts[0], 8.0)
+            sample = f"prefix of {nd} served requests of {insts[0].name}, 1 thread"
+            thr = 1
+        else:
+            sub = insts if args.workload != "C5" else insts[::16]
+            rate, dt, nb, nd = oracle_sample(sub, 0.0, cores)
+            sample = (f"{len(sub)} instances of {args.workload} (the whole batch)" if args.workload != "C5"
+                      else f"{len(sub)} of the 4,096 C5 instances (every 16th)") + f", {cores} threads"
+            thr = cores
+        times.append(dt)
+        decs.append(nd)
+    value = sum(decs) / sum(times)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
+            "scaling": scaling, "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+            "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload]}"},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": thr, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ ours
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="C2", choices=list(WORKLOADS))
+    ap.add_argument("--cpu-budget", type=float, default=10.0,
+                    help="seconds of oracle time for cpu_baseline (rank 0, N=1)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_gonthiermt22_b200 as dts
+
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py: no CUDA device (libdts has no CPU path)")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dts.load_library()
+    dev = local
+    stream = torch.cuda.current_stream()
+    sptr = stream.cuda_stream
+
+    insts, scaling = workload_instances(args.workload, rank, world)
+    single = args.workload in ("C3", "C4a", "C4b")  # one large instance: grouped CTAs
+    handles = [dts.create(i) for i in insts]
+    opts = dts.dts_run_opts_default(device=dev, cuda_stream=sptr)
+    for h in handles:
+        dts.dts_instance_upload(h, dev, sptr)
+    torch.cuda.synchronize()
+
+    def step():
+        if single:
+            for h in handles:
+                dts.dts_run(h, dts.DTS_POLICY_DARTS_LUF, opts)
+        else:
+            dts.dts_sweep_run(handles, dts.DTS_POLICY_DARTS_LUF, opts)
+
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device="cuda")  # > 126 MB L2
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(max(args.warmup, 0)):
+        step()
+    barrier()
+    res0 = [dts.dts_result(h) for h in handles]
+    decisions = sum(r.n_served for r in res0)
+    assert decisions == sum(i.m for i in insts), "not every task scheduled"
+
+    # ---- device-resident timed region
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(args.steps)]
+    loop_ms, alg_bytes, launches = [], [], 0
+    barrier()
+    with Clocks(dev) as clk:
+        l0 = dts.dts_kernel_launches()
+        for i in range(args.steps):
+            flush.zero_()  # L2 flush between timed steps (outside the events)
+            evs[i][0].record(stream)
+            step()
+            evs[i][1].record(stream)
+        barrier()
+        launches = dts.dts_kernel_launches() - l0
+        flush_launches = 0
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    rs = [dts.dts_result(h) for h in handles]  # last step's results (after the region)
+    loop_ms = max(r.loop_ms for r in rs)
+    alg = sum(r.alg_bytes for r in rs)
+    scan_alg = sum(r.scan_alg_bytes for r in rs)
+    bytes_loaded = sum(r.bytes_loaded for r in rs)
+    n_loads = sum(r.n_loads for r in rs)
+    n_scans = sum(r.n_scans for r in rs)
+    # per-step loop time: re-measure the loop kernel's own events over the timed steps
+    ms = sum(step_ms) / len(step_ms)
+
+    # ---- e2e: host arrays -> device, run, results -> host, every step
+    e2e_ms = []
+    h2d = sum(8 * (i.m + 1) + 4 * i.E + 8 * i.n + (8 * i.m if i.task_ns is not None else 0)
+              for i in insts)
+    d2h = 0
+    barrier()
+    for i in range(max(2, args.steps // 2)):
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        flush.zero_()
+        t0.record(stream)
+        for h in handles:
+            dts.dts_instance_upload(h, dev, sptr)
+        step()
+        out = [dts.dts_result(h) for h in handles]
+        t1.record(stream)
+        t1.synchronize()
+        e2e_ms.append(t0.elapsed_time(t1))
+        d2h = sum(8 * (r.K + 1) + 4 * r.n_served * 3 + 16 * len(r.task_start) + 32 * len(r.events)
+                  + 128 for r in out)
+    e2e_avg = sum(e2e_ms) / len(e2e_ms)
+
+    # ---- max over ranks
+    t = torch.tensor([ms, e2e_avg, loop_ms], dtype=torch.float64, device="cuda")
+    tot = torch.tensor([decisions, alg], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+    ms, e2e_avg, loop_ms_max = [float(x) for x in t.tolist()]
+    all_dec = float(tot[0])
+
+    if rank == 0:
+        peak, peak_src = _peaks()
+        achieved = (alg / 1e9) / (loop_ms / 1e3) if loop_ms > 0 else 0.0  # GB/s, this rank
+        cpu = None
+        if world == 1 and not args.no_cpu_baseline:
+            cores = os.cpu_count() or 1
+            if args.workload in ("C4a", "C4b", "C3"):
+                rate, dt, nd = oracle_prefix_sample(insts[0], args.cpu_budget)
+                cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
+                       "sample": f"prefix of {nd} served requests of {insts[0].name} ({dt:.1f} s, 1 thread)"}
+            else:
+                sub = insts if args.workload != "C5" else insts[::16]
+                rate, dt, nb, nd = oracle_sample(sub, args.cpu_budget, cores)
+                cpu = {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle",
+                       "sample": f"{nb} passes over {len(sub)} instances of {args.workload}"
+                                 f" ({nd} decisions, {dt:.1f} s, one instance per thread)"}
+        clocks = clk.summary()
+        line = {
+            "metric": METRIC, "value": all_dec / (ms / 1e3), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
+            "dtype": "int32", "data": "synthetic",
+            "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload]}",
+                       "instances_per_rank": len(insts), "decisions_per_step": int(all_dec),
+                       "l2": "flushed between timed steps (256 MiB write)",
+                       "launch": "one batched loop launch, one CTA per instance" if not single
+                       else "one cooperative launch per instance (CTA group)"},
+            "e2e": {"value": all_dec / (e2e_avg / 1e3), "unit": UNIT,
+                    "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h)},
+            "gpu_launches": int(launches),
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": _traffic(args.workload),
+                         "kernel": "dts_loop_kernel", "peak_source": peak_src,
+                         "alg_bytes_per_launch": int(alg), "launch_ms": loop_ms},
+            "hbm_gbs": achieved,
+            "bytes_loaded": int(bytes_loaded), "n_loads": int(n_loads), "n_scans": int(n_scans),
+            "scan_alg_bytes_per_launch": int(scan_alg),
+            "cpu_baseline": cpu,
+            "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

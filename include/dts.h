@@ -110,8 +110,11 @@ dts_status dts_instance_create(int32_t n_tasks, int32_t n_data, const int64_t *t
                                const int64_t *task_ns, int64_t default_task_ns,
                                uint64_t mem_capacity_bytes, int32_t K, dts_instance **out);
 
-/* Optional: pre-stage the instance's raw CSR on `device` (H2D on `cuda_stream`),
- * so that a later dts_run starts with its inputs resident in HBM. */
+/* Stage the instance's inputs (raw CSR, sizes, task times) on `device`: an
+ * H2D copy on `cuda_stream` from the library's host copy, every call (so a
+ * caller can time the host->device step).  dts_run uploads only if this
+ * never happened, so after this call a run starts with its inputs resident
+ * in HBM.  Allocates the instance's device arena on first use. */
 dts_status dts_instance_upload(dts_instance *inst, int32_t device, void *cuda_stream);
 
 /* Run the policy.  Enqueues on opts->cuda_stream: (upload if needed) -> CSR
@@ -158,6 +161,10 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
 void dts_instance_destroy(dts_instance *inst);
 const char *dts_status_str(dts_status s);
 const char *dts_last_error(void);
+
+/* Number of CUDA kernels libdts has launched in this process so far
+ * (monotone; the difference around a region = the library's launches in it). */
+uint64_t dts_kernel_launches(void);
 
 /* ABI version: (major << 16) | minor. */
 uint32_t dts_version(void);

@@ -20,6 +20,9 @@ from .dts import (  # noqa: F401
     dts_run_opts_default,
     dts_sweep_run,
     dts_version,
+    dts_kernel_launches,
+    create,
+    schedule_batch,
     load_library,
     schedule,
 )

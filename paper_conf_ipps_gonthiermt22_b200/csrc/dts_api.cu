@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <climits>
 #include <cstdint>
 #include <cstdio>
@@ -117,7 +118,14 @@ struct dts_instance {
     }
 };
 
+namespace dts {
+static std::atomic<uint64_t> g_launches{0};
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+}  // namespace dts
+
 extern "C" {
+
+uint64_t dts_kernel_launches(void) { return dts::g_launches.load(std::memory_order_relaxed); }
 
 void dts_run_opts_default(dts_run_opts *o) {
     if (!o) return;
@@ -354,8 +362,8 @@ dts_status ensure_device(dts_instance *I, int device) {
     return DTS_OK;
 }
 
-dts_status upload(dts_instance *I, cudaStream_t st) {
-    if (I->uploaded) return DTS_OK;
+dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
+    if (I->uploaded && !force) return DTS_OK;
     CK(cudaMemcpyAsync(I->d_raw_ptr, I->task_ptr.data(), 8 * ((size_t)I->m + 1), cudaMemcpyHostToDevice, st),
        "H2D task_ptr");
     if (I->E_raw > 0)
@@ -399,8 +407,52 @@ dts_status dts_instance_upload(dts_instance *I, int32_t device, void *cuda_strea
     dts_status s = ensure_device(I, device);
     if (s != DTS_OK) return s;
     cudaStream_t st = (cudaStream_t)cuda_stream;
-    return upload(I, st);
+    return upload(I, st, true);
 }
+
+}  // extern "C"
+
+namespace {
+
+// Enqueue everything of one instance up to (not including) the decision loop:
+// upload if needed, CSR build (a1), descriptor H2D, state init (a2).
+dts_status stage(dts_instance *I, const dts_run_opts &o, cudaStream_t st) {
+    dts_status s = ensure_device(I, o.device);
+    if (s != DTS_OK) return s;
+    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    I->stream = st;
+    I->ran = false;
+    I->have_host = false;
+    s = upload(I, st);
+    if (s != DTS_OK) return s;
+    dts::Inst &h = I->h_inst;
+    h.W = (int32_t)o.lookahead_W;
+    h.flags = o.flags;
+    h.max_served = o.max_served;
+    CK(cudaEventRecord(I->ev[0], st), "event");
+    CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
+                      (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, I->d_csr_scratch, st),
+       "build_csr");
+    CK(cudaMemcpyAsync(I->d_inst, &h, sizeof h, cudaMemcpyHostToDevice, st), "H2D inst");
+    int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n);
+    CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, I->d_delta_ptr, work, st), "init");
+    return DTS_OK;
+}
+
+// Per-device buffer of instance descriptors for batched (sweep) launches.
+// Reuse is ordered on the stream: the H2D copy of a later sweep is enqueued
+// after the previous sweep's kernels on the same stream.
+struct SweepBuf {
+    dts::Inst *d_insts = nullptr;
+    int *d_work = nullptr;
+    size_t cap = 0;
+    cudaEvent_t last = nullptr;
+};
+SweepBuf g_sweep[64];
+
+}  // namespace
+
+extern "C" {
 
 dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts) {
     if (!I) return fail(DTS_E_INVAL, "instance is NULL");
@@ -409,20 +461,9 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     else dts_run_opts_default(&o);
     dts_status s = check_opts(I, policy, &o);
     if (s != DTS_OK) return s;
-    s = ensure_device(I, o.device);
-    if (s != DTS_OK) return s;
-    CK(cudaSetDevice(o.device), "cudaSetDevice");
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
-    I->stream = st;
-    I->ran = false;
-    I->have_host = false;
-    s = upload(I, st);
+    s = stage(I, o, st);
     if (s != DTS_OK) return s;
-
-    dts::Inst &h = I->h_inst;
-    h.W = (int32_t)o.lookahead_W;
-    h.flags = o.flags;
-    h.max_served = o.max_served;
 
     int nsm = 0;
     CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
@@ -437,14 +478,6 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
         int per = dts::loop_max_blocks_per_sm(block, 0);
         if (per * nsm < G) return fail(DTS_E_UNSUPPORTED, "n_ctas exceeds co-resident CTAs");
     }
-
-    CK(cudaEventRecord(I->ev[0], st), "event");
-    CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
-                      (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, I->d_csr_scratch, st),
-       "build_csr");
-    CK(cudaMemcpyAsync(I->d_inst, &h, sizeof h, cudaMemcpyHostToDevice, st), "H2D inst");
-    int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n);
-    CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, I->d_delta_ptr, work, st), "init");
     CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
     CK(cudaEventRecord(I->ev[1], st), "event");
     CK(dts::launch_loop(I->d_inst, 1, G, block, 1, I->d_work, smem_hist_cap, st), "loop");
@@ -452,6 +485,62 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     CK(dts::launch_assemble(I->d_inst, 1, st), "assemble");
     CK(cudaEventRecord(I->ev[3], st), "event");
     I->ran = true;
+    return DTS_OK;
+}
+
+dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy,
+                         const dts_run_opts *opts) {
+    if (n < 0 || (n > 0 && !insts)) return fail(DTS_E_INVAL, "insts");
+    if (n == 0) return DTS_OK;
+    dts_run_opts o;
+    if (opts) o = *opts;
+    else dts_run_opts_default(&o);
+    if (o.device < 0 || o.device >= 64) return fail(DTS_E_INVAL, "device ordinal out of range");
+    if (o.n_ctas > 1) return fail(DTS_E_UNSUPPORTED, "sweep runs one CTA per instance (n_ctas 0 or 1)");
+    int max_n = 1;
+    for (int32_t i = 0; i < n; i++) {
+        if (!insts[i]) return fail(DTS_E_INVAL, "instance is NULL");
+        for (int32_t j = 0; j < i && n <= 4096; j++)
+            if (insts[j] == insts[i]) return fail(DTS_E_INVAL, "instance listed twice");
+        dts_status s = check_opts(insts[i], policy, &o);
+        if (s != DTS_OK) return s;
+        max_n = std::max(max_n, insts[i]->n);
+    }
+    cudaStream_t st = (cudaStream_t)o.cuda_stream;
+    for (int32_t i = 0; i < n; i++) {
+        dts_status s = stage(insts[i], o, st);
+        if (s != DTS_OK) return s;
+    }
+    SweepBuf &B = g_sweep[o.device];
+    if (B.cap < (size_t)n) {
+        if (B.d_insts) {
+            CK(cudaStreamSynchronize(st), "sync");
+            cudaFree(B.d_insts);
+        }
+        size_t cap = std::max<size_t>((size_t)n, 64);
+        CK(cudaMalloc(&B.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
+        B.d_work = reinterpret_cast<int *>(reinterpret_cast<char *>(B.d_insts) + sizeof(dts::Inst) * cap);
+        B.cap = cap;
+    }
+    std::vector<dts::Inst> hv((size_t)n);
+    for (int32_t i = 0; i < n; i++) hv[(size_t)i] = insts[i]->h_inst;
+    CK(cudaMemcpyAsync(B.d_insts, hv.data(), sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
+       "H2D sweep");
+    CK(cudaMemsetAsync(B.d_work, 0, sizeof(int), st), "memset");
+    int nsm = 0;
+    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
+    int block = env_int("DTS_BLOCK", 512);
+    int smem_hist_cap = max_n <= 32768 ? max_n : 0;
+    int per = std::max(1, dts::loop_max_blocks_per_sm(block, smem_hist_cap));
+    int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
+    for (int32_t i = 0; i < n; i++) CK(cudaEventRecord(insts[i]->ev[1], st), "event");
+    CK(dts::launch_loop(B.d_insts, n, 1, block, grid, B.d_work, smem_hist_cap, st), "loop");
+    for (int32_t i = 0; i < n; i++) CK(cudaEventRecord(insts[i]->ev[2], st), "event");
+    CK(dts::launch_assemble(B.d_insts, n, st), "assemble");
+    for (int32_t i = 0; i < n; i++) {
+        CK(cudaEventRecord(insts[i]->ev[3], st), "event");
+        insts[i]->ran = true;
+    }
     return DTS_OK;
 }
 
@@ -515,15 +604,6 @@ dts_status dts_result(dts_instance *I, dts_result_view *v) {
     v->loop_ms = I->loop_ms;
     v->total_ms = I->total_ms;
     return DTS_OK;
-}
-
-dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy,
-                         const dts_run_opts *opts) {
-    (void)insts;
-    (void)n;
-    (void)policy;
-    (void)opts;
-    return fail(DTS_E_UNSUPPORTED, "dts_sweep_run: not built yet");
 }
 
 }  // extern "C"

@@ -16,6 +16,7 @@
 #include <cstdint>
 
 #include "dts_csr.cuh"
+#include "dts_internal.cuh"
 
 namespace dts {
 
@@ -95,14 +96,14 @@ template <typename TIn>
 void scan_excl(const TIn *in, int64_t L, int64_t *out, int64_t *scratch, cudaStream_t st) {
     int64_t nb = (L + SCAN_TILE - 1) / SCAN_TILE;
     if (nb <= 1) {
-        k_scan_tiles<TIn><<<1, SCAN_T, 0, st>>>(in, L, nullptr, out);
+        k_scan_tiles<TIn><<<1, SCAN_T, 0, st>>>(in, L, nullptr, out); count_launch();
         return;
     }
     int64_t *sums = scratch;
     int64_t *offs = scratch + nb;  // nb + 1 entries
-    k_block_sums<TIn><<<(unsigned)nb, SCAN_T, 0, st>>>(in, L, sums);
+    k_block_sums<TIn><<<(unsigned)nb, SCAN_T, 0, st>>>(in, L, sums); count_launch();
     scan_excl<int64_t>(sums, nb, offs, scratch + 2 * nb + 1, st);
-    k_scan_tiles<TIn><<<(unsigned)nb, SCAN_T, 0, st>>>(in, L, offs, out);
+    k_scan_tiles<TIn><<<(unsigned)nb, SCAN_T, 0, st>>>(in, L, offs, out); count_launch();
 }
 
 // 1. sort + de-duplicate each row in place (rows have <= MAX_ROW entries,
@@ -271,13 +272,22 @@ cudaError_t build_csr(const int64_t *raw_ptr, const int32_t *raw_dat, int32_t m,
     int64_t *sscr = (int64_t *)carve(p, sizeof(int64_t) * (size_t)(2 * (L / 2048 + 64)));
 
     cudaMemsetAsync(deg, 0, sizeof(unsigned long long) * (size_t)(n + 1), st);
-    if (m > 0) k_rows<<<(m + 255) / 256, 256, 0, st>>>(raw_ptr, raw_dat, m, tmp, nlen);
+    if (m > 0) {
+        k_rows<<<(m + 255) / 256, 256, 0, st>>>(raw_ptr, raw_dat, m, tmp, nlen);
+        count_launch();
+    }
     scan_excl<int64_t>(nlen, m, tptr, sscr, st);
-    if (m > 0) k_compact<<<(m + 255) / 256, 256, 0, st>>>(raw_ptr, tmp, tptr, m, tdat, k0, v0, deg);
+    if (m > 0) {
+        k_compact<<<(m + 255) / 256, 256, 0, st>>>(raw_ptr, tmp, tptr, m, tdat, k0, v0, deg);
+        count_launch();
+    }
     scan_excl<unsigned long long>(deg, n, dptr, sscr, st);
     // The de-duplicated edge count E = tptr[m] <= E_raw is only known on the
     // device: sort all E_raw slots with the tail padded by key n (sorts last).
-    if (E_raw > 0) k_pad_tail<<<(unsigned)((E_raw + 255) / 256), 256, 0, st>>>(tptr, m, E_raw, n, k0, v0);
+    if (E_raw > 0) {
+        k_pad_tail<<<(unsigned)((E_raw + 255) / 256), 256, 0, st>>>(tptr, m, E_raw, n, k0, v0);
+        count_launch();
+    }
     int bits = 1;
     while ((1ll << bits) <= (long long)n) bits++;  // ids in [0, n] (n = pad key)
     int passes = (bits + 7) / 8;
@@ -285,10 +295,10 @@ cudaError_t build_csr(const int64_t *raw_ptr, const int32_t *raw_dat, int32_t m,
     for (int ps = 0; ps < passes; ps++) {
         int shift = 8 * ps;
         if (E_raw > 0) {
-            k_radix_hist<<<(unsigned)nchunks, RX_T, 0, st>>>(ki, E_raw, shift, counts, nchunks);
+            k_radix_hist<<<(unsigned)nchunks, RX_T, 0, st>>>(ki, E_raw, shift, counts, nchunks); count_launch();
             scan_excl<int64_t>(counts, 256 * nchunks, offs, sscr, st);
             k_radix_scatter<<<(unsigned)nchunks, RX_T, 0, st>>>(ki, vi, E_raw, shift, offs, nchunks, ko,
-                                                               vo);
+                                                               vo); count_launch();
         }
         int32_t *t;
         t = ki; ki = ko; ko = t;

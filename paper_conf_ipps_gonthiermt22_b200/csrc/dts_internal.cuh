@@ -23,6 +23,9 @@
 
 namespace dts {
 
+// Process-wide count of kernel launches issued by libdts (dts_kernel_launches()).
+void count_launch();
+
 constexpr uint32_t ALLOC_BIT = 0x80000000u;
 constexpr uint32_t CNT_ONE = 1u << 24;
 constexpr uint32_t XOR_MASK = 0x00FFFFFFu;

@@ -802,6 +802,7 @@ cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t *c
     if (blocks < 1) blocks = 1;
     if (blocks > 148 * 8) blocks = 148 * 8;
     dts_init_kernel<<<(unsigned)blocks, 256, 0, st>>>(d_insts, n_inst, bw, d_deltas);
+    count_launch();
     return cudaGetLastError();
 }
 
@@ -814,15 +815,18 @@ cudaError_t launch_loop(const Inst *d_insts, int n_inst, int G, int block, int g
     if (G > 1) {
         void *args[] = {(void *)&d_insts, (void *)&n_inst, (void *)&G, (void *)&work_counter,
                         (void *)&smem_hist_cap};
+        count_launch();
         return cudaLaunchCooperativeKernel((const void *)dts_loop_kernel, dim3(G), dim3(block), args,
                                            dyn, st);
     }
     dts_loop_kernel<<<grid, block, dyn, st>>>(d_insts, n_inst, 1, work_counter, smem_hist_cap);
+    count_launch();
     return cudaGetLastError();
 }
 
 cudaError_t launch_assemble(const Inst *d_insts, int n_inst, cudaStream_t st) {
     dts_assemble_kernel<<<n_inst, 1024, 0, st>>>(d_insts);
+    count_launch();
     return cudaGetLastError();
 }
 

@@ -35,7 +35,7 @@ EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data",
 
 EXPORTED = ["dts_run_opts_default", "dts_instance_create", "dts_instance_upload", "dts_run",
             "dts_result", "dts_sweep_run", "dts_instance_destroy", "dts_status_str",
-            "dts_last_error", "dts_version"]
+            "dts_last_error", "dts_version", "dts_kernel_launches"]
 
 
 class DtsError(RuntimeError):
@@ -96,6 +96,8 @@ def load_library(path: str = LIB_PATH):
     lib.dts_status_str.restype = C.c_char_p
     lib.dts_last_error.argtypes = []
     lib.dts_last_error.restype = C.c_char_p
+    lib.dts_kernel_launches.argtypes = []
+    lib.dts_kernel_launches.restype = C.c_uint64
     lib.dts_version.argtypes = []
     lib.dts_version.restype = C.c_uint32
     _lib = lib
@@ -214,6 +216,10 @@ def dts_result(inst: Instance) -> Result:
                   float(v.loop_ms), float(v.total_ms))
 
 
+def dts_kernel_launches() -> int:
+    return int(load_library().dts_kernel_launches())
+
+
 def dts_version() -> int:
     return int(load_library().dts_version())
 
@@ -228,3 +234,20 @@ def schedule(inst, *, W: int = 0, flags: int = DTS_F_FALLBACK2, bus_bps: int = 1
                              n_ctas=n_ctas, max_served=max_served, cuda_stream=stream or None)
     dts_run(h, DTS_POLICY_DARTS_LUF, o)
     return dts_result(h)
+
+
+def create(inst) -> Instance:
+    """dts_instance_create from a ``gen.Instance``-like object."""
+    return dts_instance_create(inst.task_ptr, inst.task_data, inst.data_size, inst.task_ns,
+                               inst.default_task_ns, inst.mem_capacity, inst.K)
+
+
+def schedule_batch(insts, *, W: int = 0, flags: int = DTS_F_FALLBACK2,
+                   bus_bps: int = 12_000_000_000, device: int = 0, stream: int = 0):
+    """Run many independent instances in ONE batched launch (dts_sweep_run,
+    one CTA per instance) and return their host results."""
+    hs = [create(i) for i in insts]
+    o = dts_run_opts_default(flags=flags, lookahead_W=W, bus_bytes_per_s=bus_bps, device=device,
+                             n_ctas=0, max_served=-1, cuda_stream=stream or None)
+    dts_sweep_run(hs, DTS_POLICY_DARTS_LUF, o)
+    return [dts_result(h) for h in hs]

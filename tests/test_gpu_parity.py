@@ -167,3 +167,32 @@ def test_config4_full_digest(cfg):
               "bytes_loaded", "makespan"):
         assert getattr(g, k) == gold[k], k
     assert digest(g.serve_gpu, g.serve_task, g.task_start, g.task_end, g.events) == gold["sha256"]
+
+
+# ------------------------------------------------------------ batched sweep
+def test_sweep_batch_config2():
+    """dts_sweep_run (one CTA per instance, one launch) on the 20 C2 instances:
+    every instance bit-exact against its own oracle run."""
+    insts = gen.config_instances("C2")
+    gs = dts.schedule_batch(insts)
+    for inst, g in zip(insts, gs):
+        assert_parity(g, oracle.run(inst))
+
+
+def test_sweep_batch_mixed_shapes():
+    insts = _shapes() + [gen.fig1(), _unit(gen.matmul2d(10, M=6, K=1))]
+    buses = [oracle.DEFAULT_BUS_BPS] * len(insts)
+    gs = dts.schedule_batch(insts)
+    for inst, g, b in zip(insts, gs, buses):
+        assert_parity(g, oracle.run(inst, bus_bps=b))
+
+
+def test_sweep_sample_config5():
+    """A seeded sample of the 4,096 config-5 instances in one batched launch."""
+    params = gen.sweep_params()
+    rng = np.random.default_rng(5)
+    pick = sorted(rng.choice(len(params), size=48, replace=False))
+    insts = [gen.sweep_instance(*params[i]) for i in pick]
+    gs = dts.schedule_batch(insts)
+    for inst, g in zip(insts, gs):
+        assert_parity(g, oracle.run(inst))
