@@ -60,7 +60,12 @@ typedef enum {
 enum {
     /* "3inputs" fallback when no datum frees a task: load the datum that
      * makes the most tasks one load away.  Default ON. */
-    DTS_F_FALLBACK2 = 1u << 0
+    DTS_F_FALLBACK2 = 1u << 0,
+    /* Debug / parity mode: at every scan, recompute the
+     * scores n_k(D), n2_k(D), u(D) and every task's missing count from their
+     * definitions (a full pass over all tasks) and count disagreements with
+     * the incremental state in dts_result_view.n_verify_err.  Slow. */
+    DTS_F_VERIFY = 1u << 1
 };
 
 typedef struct {
@@ -69,7 +74,12 @@ typedef struct {
                                  0 (default, the formal model of §III) -- others: UNSUPPORTED */
     uint64_t bus_bytes_per_s; /* shared host->GPU bus bandwidth; default 12e9 (reading R9) */
     int32_t device;           /* CUDA device ordinal; default 0 */
-    int32_t n_ctas;           /* CTAs cooperating on one instance; 0 = automatic */
+    int32_t block_threads;    /* threads of the ONE CTA that runs an instance: a multiple of
+                                 32 in [32, 512]; 0 = automatic */
+    int32_t smem_budget;      /* bytes of shared memory per CTA for state placement
+                                 (DESIGN.md "Data layout"); 0 = automatic (all that fits);
+                                 -1 = none (every array in its global home) */
+    int32_t pad;
     int64_t max_served;       /* stop after this many served tasks (prefix runs); -1 = all */
     void *cuda_stream;        /* cudaStream_t to enqueue on; NULL = the legacy default stream */
 } dts_run_opts;
@@ -142,19 +152,25 @@ typedef struct {
     int64_t n_served;              /* served requests = decisions (reading R21)              */
     int64_t n_scans;               /* requests that found plannedTasks_k empty and got a task */
     int64_t n_fallback2, n_fallback_first, n_belady, n_idle_requests;
+    int64_t n_verify_err;          /* DTS_F_VERIFY: disagreements found (0 = consistent)       */
     uint64_t alg_bytes;            /* algorithmic HBM bytes of the decision loop  */
     uint64_t scan_alg_bytes;       /* ... of which in the per-scan pass                       */
     float loop_ms;                 /* device time of the decision-loop kernel (CUDA events)  */
     float total_ms;                /* device time of the whole run (CSR build..assembly)     */
+    int64_t prof_cycles[8];        /* diagnostics: SM cycles of the loop per phase (pop, argmax,
+                                      plan, serve-with-loads, LUF, evict, load-update, other) */
 } dts_result_view;
 
 /* Synchronise on the run's stream, copy the results to host (once) and fill *out. */
 dts_status dts_result(dts_instance *inst, dts_result_view *out);
 
-/* Sweep (BASELINE config 5): run every instance of insts[0..n) on ONE device
- * with one CTA per instance in a single batched launch of the same loop
- * (no communication between instances).  opts->device selects the device.
- * Results are read per instance with dts_result. */
+/* Sweep (BASELINE config 5) / batch: run every instance of insts[0..n) on
+ * ONE device (opts->device) in a single batched launch of the decision loop,
+ * one CTA per instance, CTAs pulling instances from a device counter (no
+ * communication between instances).  Each instance gets the same options.
+ * Results are read per instance with dts_result.  An instance must not
+ * appear twice.  Multi-GPU sweeps shard the list across processes (one per
+ * GPU, bench.py) -- nothing crosses devices. */
 dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy,
                          const dts_run_opts *opts);
 

@@ -87,7 +87,8 @@ struct dts_instance {
     uint64_t *d_size = nullptr;
     int64_t *d_tau = nullptr;
     int64_t *d_delta = nullptr;
-    int64_t **d_delta_ptr = nullptr;
+    dts::Inst *h_pinned = nullptr;   // pinned staging copy of the descriptor (async H2D)
+    cudaEvent_t ev_desc = nullptr;   // the last H2D copy out of h_pinned
     void *d_csr_scratch = nullptr;
     int *d_work = nullptr;
     dts::Inst h_inst{};
@@ -113,8 +114,10 @@ struct dts_instance {
             if (ar.base) cudaFree(ar.base);
             for (auto &e : ev)
                 if (e) cudaEventDestroy(e);
+            if (ev_desc) cudaEventDestroy(ev_desc);
             cudaSetDevice(cur);
         }
+        if (h_pinned) cudaFreeHost(h_pinned);
     }
 };
 
@@ -134,7 +137,8 @@ void dts_run_opts_default(dts_run_opts *o) {
     o->lookahead_W = 0;
     o->bus_bytes_per_s = 12000000000ull;
     o->device = 0;
-    o->n_ctas = 0;
+    o->block_threads = 0;
+    o->smem_budget = 0;
     o->max_served = -1;
     o->cuda_stream = nullptr;
 }
@@ -154,7 +158,7 @@ const char *dts_status_str(dts_status s) {
 
 const char *dts_last_error(void) { return g_err.c_str(); }
 
-uint32_t dts_version(void) { return (1u << 16) | 0u; }
+uint32_t dts_version(void) { return (1u << 16) | 1u; }
 
 dts_status dts_instance_create(int32_t n_tasks, int32_t n_data, const int64_t *task_ptr,
                                const int32_t *task_data, const uint64_t *data_size,
@@ -271,6 +275,7 @@ dts_status check_device(int device) {
     return DTS_OK;
 }
 
+
 dts_status ensure_device(dts_instance *I, int device) {
     if (I->device == device && I->ar.base) return DTS_OK;
     if (I->device >= 0 && I->ar.base) {
@@ -278,6 +283,8 @@ dts_status ensure_device(dts_instance *I, int device) {
         cudaFree(I->ar.base);
         for (auto &e : I->ev)
             if (e) cudaEventDestroy(e);
+        if (I->ev_desc) cudaEventDestroy(I->ev_desc);
+        I->ev_desc = nullptr;
         I->ar = Arena{};
         I->uploaded = false;
     }
@@ -289,15 +296,18 @@ dts_status ensure_device(dts_instance *I, int device) {
     const size_t ev_cap = 2 * E + 16;
     const size_t plan_cap = (size_t)I->max_deg_ub + 1;
     const size_t res_cap = (size_t)I->res_cap + 1;
+    const size_t nw = (n + 31) / 32 + 1;
     size_t need = 0;
     auto add = [&](size_t bytes) { need += (bytes + 255) & ~size_t(255); };
-    add(8 * (m + 1)); add(4 * (E + 1)); add(8 * (n + 1)); add(8 * (m + 1));        // raw
-    add(8 * (m + 1)); add(4 * (E + 1)); add(8 * (n + 1)); add(4 * (E + 1));        // CSR
-    add(8 * (n + 1)); add(8);                                                      // delta
-    add(4 * K * mp + 16); add(4 * (n + 1)); add(4 * (n + 1)); add(4 * K * (n + 1)); // s u hist np
-    add(4 * K * res_cap); add(4 * K * (n + 1)); add(4 * K * plan_cap);            // residency, plans
-    add(sizeof(dts::Ctrl)); add(sizeof(dts::Out));
-    add(4 * (m + 1)); add(4 * (m + 1)); add(8 * (m + 1)); add(8 * (m + 1));        // serve, times
+    add(8 * (m + 1)); add(4 * (E + 1)); add(8 * (n + 1)); add(8 * (m + 1));          // raw inputs
+    add(8 * (m + 1)); add(4 * (E + 1)); add(8 * (n + 1)); add(4 * (E + 1));          // CSR
+    add(16 * (E + 1));                                                               // edge records
+    add(8 * (n + 1)); add(8);                                                        // delta
+    add(4 * K * mp + 16); add(4 * (n + 1)); add(4 * K * (n + 1)); add(4 * K * (n + 1));  // s u h h2
+    add(4 * K * (n + 1)); add(4 * K * nw); add(4 * K * res_cap);                     // np resb res_list
+    add(16 * K * plan_cap); add(8 * K * plan_cap); add(4 * (3 * n + 1));              // plan tau vhist
+    add(sizeof(dts::Out));
+    add(4 * (m + 1)); add(4 * (m + 1)); add(8 * (m + 1)); add(8 * (m + 1));          // serve, times
     add(sizeof(dts_event) * ev_cap); add(8 * (K + 1)); add(4 * (m + 1));
     add(sizeof(dts::Inst)); add(64);
     add(dts::csr_scratch_bytes(I->m, I->n, I->E_raw));
@@ -309,6 +319,8 @@ dts_status ensure_device(dts_instance *I, int device) {
     I->ar.used = 0;
     I->device = device;
     for (auto &ev : I->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
+    CK(cudaEventCreateWithFlags(&I->ev_desc, cudaEventDisableTiming), "cudaEventCreate");
+    if (!I->h_pinned) CK(cudaMallocHost(&I->h_pinned, sizeof(dts::Inst)), "cudaMallocHost");
 
     Arena &A = I->ar;
     dts::Inst &h = I->h_inst;
@@ -321,16 +333,18 @@ dts_status ensure_device(dts_instance *I, int device) {
     h.tdat = A.take<int32_t>(E + 1);
     h.dptr = A.take<int64_t>(n + 1);
     h.ddat = A.take<int32_t>(E + 1);
+    h.dedge = A.take<int4>(E + 1);
     I->d_delta = A.take<int64_t>(n + 1);
-    I->d_delta_ptr = A.take<int64_t *>(1);
     h.s = A.take<uint32_t>(K * mp + 4);
     h.u = A.take<int32_t>(n + 1);
-    h.hist = A.take<int32_t>(n + 1);
+    h.h = A.take<int32_t>(K * (n + 1));
+    h.h2 = A.take<int32_t>(K * (n + 1));
     h.np = A.take<int32_t>(K * (n + 1));
+    h.resb = A.take<uint32_t>(K * nw);
     h.res_list = A.take<int32_t>(K * res_cap);
-    h.res_pos = A.take<int32_t>(K * (n + 1));
-    h.planned = A.take<int32_t>(K * plan_cap);
-    h.ctrl = A.take<dts::Ctrl>(1);
+    h.plan = A.take<int4>(K * plan_cap);
+    h.plan_tau = A.take<int64_t>(K * plan_cap);
+    h.vhist = A.take<int32_t>(3 * n + 1);
     h.out = A.take<dts::Out>(1);
     h.serve_gpu = A.take<int32_t>(m + 1);
     h.serve_task = A.take<int32_t>(m + 1);
@@ -351,6 +365,7 @@ dts_status ensure_device(dts_instance *I, int device) {
     h.cap = I->cap;
     h.plan_cap = (int32_t)plan_cap;
     h.res_cap = (int32_t)res_cap;
+    h.nw = (int32_t)nw;
     h.id_bits = bits_for(I->n > 0 ? (uint64_t)(I->n - 1) : 0);
     h.u_bits = bits_for((uint64_t)I->max_deg_ub);
     h.E = I->E_raw;
@@ -375,28 +390,126 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
     if (I->has_tau && I->m > 0)
         CK(cudaMemcpyAsync(I->d_tau, I->task_ns.data(), 8 * (size_t)I->m, cudaMemcpyHostToDevice, st),
            "H2D task_ns");
-    CK(cudaMemcpyAsync(I->d_delta_ptr, &I->d_delta, sizeof(int64_t *), cudaMemcpyHostToDevice, st),
-       "H2D delta ptr");
     I->uploaded = true;
     return DTS_OK;
 }
 
 dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_opts *o) {
     if (policy != DTS_POLICY_DARTS_LUF) return fail(DTS_E_UNSUPPORTED, "policy");
-    if (o->flags & ~(uint32_t)DTS_F_FALLBACK2) return fail(DTS_E_UNSUPPORTED, "unknown flags");
+    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY)) return fail(DTS_E_UNSUPPORTED, "unknown flags");
     if (o->lookahead_W != 0) return fail(DTS_E_UNSUPPORTED, "lookahead_W != 0 (NEXT)");
     if (o->bus_bytes_per_s == 0) return fail(DTS_E_INVAL, "bus_bytes_per_s == 0");
-    if (o->n_ctas < 0) return fail(DTS_E_INVAL, "n_ctas < 0");
+    if (o->block_threads != 0 && (o->block_threads < 32 || o->block_threads > 512 || o->block_threads % 32))
+        return fail(DTS_E_INVAL, "block_threads must be 0 or a multiple of 32 in [32, 512]");
+    if (o->smem_budget < -1) return fail(DTS_E_INVAL, "smem_budget < -1");
     unsigned __int128 need = (unsigned __int128)(o->lookahead_W + 1) * I->max_row_bytes;
     if ((unsigned __int128)I->cap < need)
         return fail(DTS_E_CAPACITY, "mem_capacity_bytes < (W+1) * max_T size(D(T))");
     return DTS_OK;
 }
 
+// Shared-memory placement of one instance's state:
+// greedy, most latency-critical array first, each either fully in the CTA's
+// dynamic shared memory or in its global home.  Returns the bytes used.
+int place_smem(dts::Inst &h, bool has_tau, int budget) {
+    const int64_t K = h.K, n = h.n;
+    int used = 0;
+    auto put = [&](int32_t &so, int64_t bytes) {
+        bytes = (bytes + 15) & ~int64_t(15);
+        if (budget > 0 && used + bytes <= budget) {
+            so = used;
+            used += (int)bytes;
+        } else {
+            so = -1;
+        }
+    };
+    put(h.so_resb, 4 * K * h.nw);
+    put(h.so_plan, 16 * K * h.plan_cap);
+    if (has_tau) put(h.so_plan_tau, 8 * K * h.plan_cap);
+    else h.so_plan_tau = -1;
+    put(h.so_res_list, 4 * K * h.res_cap);
+    put(h.so_u, 4 * n);
+    put(h.so_h, 4 * K * n);
+    put(h.so_h2, 4 * K * n);
+    put(h.so_np, 4 * K * n);
+    put(h.so_s, 4 * K * (int64_t)h.m_pad);  // last: the largest, worth it only when it fits
+    h.smem_bytes = used;
+    return used;
+}
+
+int max_dyn_smem(int device) {
+    static int cache[64] = {0};
+    if (device >= 0 && device < 64 && cache[device] > 0) return cache[device];
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+    int st = dts::loop_static_smem();
+    if (st < 0) st = 16384;
+    const int r = std::max(0, optin - st - 1024);
+    if (device >= 0 && device < 64) cache[device] = r;
+    return r;
+}
+
+// Threads of the CTA: enough to cover a data segment (deg(D)) in one pass
+// and the score argmax in <= 8 entries per thread, within [64, 512].
+int auto_block(const dts_instance *I) {
+    int b = 64;
+    while (b < 512 && (b * 8 < I->n || b < I->max_deg_ub)) b *= 2;
+    return b;
+}
+
 int env_int(const char *name, int dflt) {
     const char *v = std::getenv(name);
     return v ? std::atoi(v) : dflt;
 }
+
+// Enqueue everything of one instance up to (not including) the decision loop:
+// upload if needed, CSR build (a1), state init (a2), descriptor H2D.
+dts_status stage(dts_instance *I, const dts_run_opts &o, int budget, cudaStream_t st,
+                 bool copy_desc = true) {
+    dts_status s = ensure_device(I, o.device);
+    if (s != DTS_OK) return s;
+    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    I->stream = st;
+    I->ran = false;
+    I->have_host = false;
+    s = upload(I, st);
+    if (s != DTS_OK) return s;
+    dts::Inst &h = I->h_inst;
+    h.W = (int32_t)o.lookahead_W;
+    h.flags = o.flags;
+    h.max_served = o.max_served;
+    place_smem(h, I->has_tau, budget);
+    CK(cudaEventRecord(I->ev[0], st), "event");
+    CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
+                      (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, (int4 *)h.dedge,
+                      I->d_csr_scratch, st),
+       "build_csr");
+    if (!copy_desc) return DTS_OK;
+    // descriptor H2D from pinned memory (a pageable copy would serialise the host)
+    CK(cudaEventSynchronize(I->ev_desc), "desc event");
+    *I->h_pinned = h;
+    CK(cudaMemcpyAsync(I->d_inst, I->h_pinned, sizeof h, cudaMemcpyHostToDevice, st), "H2D inst");
+    CK(cudaEventRecord(I->ev_desc, st), "event");
+    return DTS_OK;
+}
+
+int budget_of(const dts_run_opts &o) {
+    if (o.smem_budget < 0) return 0;
+    const int mx = max_dyn_smem(o.device);
+    return o.smem_budget == 0 ? mx : std::min(o.smem_budget, mx);
+}
+
+// Per-device buffer of instance descriptors for batched (sweep) launches.
+// Reuse is ordered on the stream: the H2D copy of a later sweep is enqueued
+// after the previous sweep's kernels on the same stream.
+struct SweepBuf {
+    dts::Inst *d_insts = nullptr;
+    dts::Inst *h_insts = nullptr;  // pinned staging
+    int *d_work = nullptr;
+    size_t cap = 0;
+    cudaEvent_t copied = nullptr;   // the last H2D copy out of h_insts
+};
+SweepBuf g_sweep[64];
 
 }  // namespace
 
@@ -410,50 +523,6 @@ dts_status dts_instance_upload(dts_instance *I, int32_t device, void *cuda_strea
     return upload(I, st, true);
 }
 
-}  // extern "C"
-
-namespace {
-
-// Enqueue everything of one instance up to (not including) the decision loop:
-// upload if needed, CSR build (a1), descriptor H2D, state init (a2).
-dts_status stage(dts_instance *I, const dts_run_opts &o, cudaStream_t st) {
-    dts_status s = ensure_device(I, o.device);
-    if (s != DTS_OK) return s;
-    CK(cudaSetDevice(o.device), "cudaSetDevice");
-    I->stream = st;
-    I->ran = false;
-    I->have_host = false;
-    s = upload(I, st);
-    if (s != DTS_OK) return s;
-    dts::Inst &h = I->h_inst;
-    h.W = (int32_t)o.lookahead_W;
-    h.flags = o.flags;
-    h.max_served = o.max_served;
-    CK(cudaEventRecord(I->ev[0], st), "event");
-    CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
-                      (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, I->d_csr_scratch, st),
-       "build_csr");
-    CK(cudaMemcpyAsync(I->d_inst, &h, sizeof h, cudaMemcpyHostToDevice, st), "H2D inst");
-    int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n);
-    CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, I->d_delta_ptr, work, st), "init");
-    return DTS_OK;
-}
-
-// Per-device buffer of instance descriptors for batched (sweep) launches.
-// Reuse is ordered on the stream: the H2D copy of a later sweep is enqueued
-// after the previous sweep's kernels on the same stream.
-struct SweepBuf {
-    dts::Inst *d_insts = nullptr;
-    int *d_work = nullptr;
-    size_t cap = 0;
-    cudaEvent_t last = nullptr;
-};
-SweepBuf g_sweep[64];
-
-}  // namespace
-
-extern "C" {
-
 dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts) {
     if (!I) return fail(DTS_E_INVAL, "instance is NULL");
     dts_run_opts o;
@@ -461,28 +530,19 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     else dts_run_opts_default(&o);
     dts_status s = check_opts(I, policy, &o);
     if (s != DTS_OK) return s;
-    cudaStream_t st = (cudaStream_t)o.cuda_stream;
-    s = stage(I, o, st);
+    s = check_device(o.device);
     if (s != DTS_OK) return s;
-
-    int nsm = 0;
-    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
-    int G = o.n_ctas;
-    if (G == 0) {
-        int64_t want = ((int64_t)I->m + 16383) / 16384;
-        G = (int)std::max<int64_t>(1, std::min<int64_t>(want, nsm));
-    }
-    int block = env_int("DTS_BLOCK", 512);
-    int smem_hist_cap = (G == 1 && I->n <= 32768) ? std::max(I->n, 1) : 0;
-    if (G > 1) {
-        int per = dts::loop_max_blocks_per_sm(block, 0);
-        if (per * nsm < G) return fail(DTS_E_UNSUPPORTED, "n_ctas exceeds co-resident CTAs");
-    }
+    cudaStream_t st = (cudaStream_t)o.cuda_stream;
+    const int budget = budget_of(o);
+    s = stage(I, o, budget, st);
+    if (s != DTS_OK) return s;
+    const int block = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", auto_block(I));
+    const int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n * I->K);
+    CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
     CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
     CK(cudaEventRecord(I->ev[1], st), "event");
-    CK(dts::launch_loop(I->d_inst, 1, G, block, 1, I->d_work, smem_hist_cap, st), "loop");
+    CK(dts::launch_loop(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");
     CK(cudaEventRecord(I->ev[2], st), "event");
-    CK(dts::launch_assemble(I->d_inst, 1, st), "assemble");
     CK(cudaEventRecord(I->ev[3], st), "event");
     I->ran = true;
     return DTS_OK;
@@ -495,49 +555,60 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     dts_run_opts o;
     if (opts) o = *opts;
     else dts_run_opts_default(&o);
-    if (o.device < 0 || o.device >= 64) return fail(DTS_E_INVAL, "device ordinal out of range");
-    if (o.n_ctas > 1) return fail(DTS_E_UNSUPPORTED, "sweep runs one CTA per instance (n_ctas 0 or 1)");
-    int max_n = 1;
+    dts_status s = check_device(o.device);
+    if (s != DTS_OK) return s;
+    int block = 32;
+    int64_t work = 1;
+    std::vector<dts_instance *> seen(insts, insts + n);
+    std::sort(seen.begin(), seen.end());
+    if (std::adjacent_find(seen.begin(), seen.end()) != seen.end())
+        return fail(DTS_E_INVAL, "instance listed twice");
     for (int32_t i = 0; i < n; i++) {
         if (!insts[i]) return fail(DTS_E_INVAL, "instance is NULL");
-        for (int32_t j = 0; j < i && n <= 4096; j++)
-            if (insts[j] == insts[i]) return fail(DTS_E_INVAL, "instance listed twice");
-        dts_status s = check_opts(insts[i], policy, &o);
+        s = check_opts(insts[i], policy, &o);
         if (s != DTS_OK) return s;
-        max_n = std::max(max_n, insts[i]->n);
+        block = std::max(block, auto_block(insts[i]));
+        work = std::max<int64_t>(work, std::max<int64_t>(insts[i]->m_pad, (int64_t)insts[i]->n * insts[i]->K));
     }
+    if (o.block_threads) block = o.block_threads;
+    else block = env_int("DTS_BLOCK", block);
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
+    const int budget = budget_of(o);
+    int smem = 0;
     for (int32_t i = 0; i < n; i++) {
-        dts_status s = stage(insts[i], o, st);
+        s = stage(insts[i], o, budget, st, false);
         if (s != DTS_OK) return s;
+        smem = std::max(smem, insts[i]->h_inst.smem_bytes);
     }
     SweepBuf &B = g_sweep[o.device];
+    if (!B.copied) CK(cudaEventCreateWithFlags(&B.copied, cudaEventDisableTiming), "cudaEventCreate");
+    CK(cudaEventSynchronize(B.copied), "sweep event");
     if (B.cap < (size_t)n) {
         if (B.d_insts) {
-            CK(cudaStreamSynchronize(st), "sync");
+            CK(cudaDeviceSynchronize(), "sync");
             cudaFree(B.d_insts);
+            cudaFreeHost(B.h_insts);
         }
         size_t cap = std::max<size_t>((size_t)n, 64);
         CK(cudaMalloc(&B.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
-        B.d_work = reinterpret_cast<int *>(reinterpret_cast<char *>(B.d_insts) + sizeof(dts::Inst) * cap);
+        CK(cudaMallocHost(&B.h_insts, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
+        B.d_work = reinterpret_cast<int *>(B.d_insts + cap);
         B.cap = cap;
     }
-    std::vector<dts::Inst> hv((size_t)n);
-    for (int32_t i = 0; i < n; i++) hv[(size_t)i] = insts[i]->h_inst;
-    CK(cudaMemcpyAsync(B.d_insts, hv.data(), sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
+    for (int32_t i = 0; i < n; i++) B.h_insts[i] = insts[i]->h_inst;
+    CK(cudaMemcpyAsync(B.d_insts, B.h_insts, sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
        "H2D sweep");
+    CK(cudaEventRecord(B.copied, st), "event");
     CK(cudaMemsetAsync(B.d_work, 0, sizeof(int), st), "memset");
+    CK(dts::launch_init(B.d_insts, n, o.bus_bytes_per_s, work, st), "init");
     int nsm = 0;
     CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
-    int block = env_int("DTS_BLOCK", 512);
-    int smem_hist_cap = max_n <= 32768 ? max_n : 0;
-    int per = std::max(1, dts::loop_max_blocks_per_sm(block, smem_hist_cap));
-    int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
+    const int per = std::max(1, dts::loop_max_blocks_per_sm(block, smem));
+    const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
     for (int32_t i = 0; i < n; i++) CK(cudaEventRecord(insts[i]->ev[1], st), "event");
-    CK(dts::launch_loop(B.d_insts, n, 1, block, grid, B.d_work, smem_hist_cap, st), "loop");
-    for (int32_t i = 0; i < n; i++) CK(cudaEventRecord(insts[i]->ev[2], st), "event");
-    CK(dts::launch_assemble(B.d_insts, n, st), "assemble");
+    CK(dts::launch_loop(B.d_insts, n, block, grid, B.d_work, smem, st), "loop");
     for (int32_t i = 0; i < n; i++) {
+        CK(cudaEventRecord(insts[i]->ev[2], st), "event");
         CK(cudaEventRecord(insts[i]->ev[3], st), "event");
         insts[i]->ran = true;
     }
@@ -599,8 +670,10 @@ dts_status dts_result(dts_instance *I, dts_result_view *v) {
     v->n_fallback_first = I->out.n_fallback_first;
     v->n_belady = I->out.n_belady;
     v->n_idle_requests = I->out.n_idle;
+    v->n_verify_err = I->out.n_verify_err;
     v->alg_bytes = I->out.alg_bytes;
     v->scan_alg_bytes = I->out.scan_alg_bytes;
+    for (int i = 0; i < 8; i++) v->prof_cycles[i] = I->out.prof[i];
     v->loop_ms = I->loop_ms;
     v->total_ms = I->total_ms;
     return DTS_OK;

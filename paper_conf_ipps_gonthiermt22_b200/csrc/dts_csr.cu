@@ -227,6 +227,34 @@ __global__ void k_radix_scatter(const int32_t *__restrict__ kin, const int32_t *
     }
 }
 
+// 6. edge records: for edge i of datum D's segment, {T, T's other inputs, |D(T)|}.
+__global__ void k_edges(const int64_t *__restrict__ tptr, const int32_t *__restrict__ tdat,
+                        const int64_t *__restrict__ dptr, const int32_t *__restrict__ ddat, int32_t n,
+                        int64_t E_raw, int4 *__restrict__ dedge) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= E_raw || i >= dptr[n]) return;
+    int32_t lo = 0, hi = n - 1;  // D = the segment containing i: dptr[D] <= i < dptr[D+1]
+    while (lo < hi) {
+        const int32_t mid = (lo + hi + 1) >> 1;
+        if (dptr[mid] <= i) lo = mid;
+        else hi = mid - 1;
+    }
+    const int32_t D = lo, T = ddat[i];
+    const int64_t rb = tptr[T], re = tptr[T + 1];
+    int4 e;
+    e.x = T;
+    e.y = -1;
+    e.z = -1;
+    e.w = (int32_t)(re - rb);
+    for (int64_t j = rb; j < re; j++) {
+        const int32_t o = tdat[j];
+        if (o == D) continue;
+        if (e.y < 0) e.y = o;
+        else if (e.z < 0) e.z = o;
+    }
+    dedge[i] = e;
+}
+
 }  // namespace
 
 size_t csr_scratch_bytes(int32_t m, int32_t n, int64_t E_raw) {
@@ -253,7 +281,7 @@ static inline char *carve(char *&p, size_t bytes) {
 
 cudaError_t build_csr(const int64_t *raw_ptr, const int32_t *raw_dat, int32_t m, int32_t n,
                       int64_t E_raw, int64_t *tptr, int32_t *tdat, int64_t *dptr, int32_t *ddat,
-                      void *scratch, cudaStream_t st) {
+                      int4 *dedge, void *scratch, cudaStream_t st) {
     char *p = (char *)scratch;
     int32_t *tmp = (int32_t *)carve(p, sizeof(int32_t) * (size_t)(E_raw + 4));
     int64_t *nlen = (int64_t *)carve(p, sizeof(int64_t) * (size_t)(m + 4));
@@ -305,6 +333,10 @@ cudaError_t build_csr(const int64_t *raw_ptr, const int32_t *raw_dat, int32_t m,
         t = vi; vi = vo; vo = t;
     }
     if (E_raw > 0) cudaMemcpyAsync(ddat, vi, sizeof(int32_t) * (size_t)E_raw, cudaMemcpyDeviceToDevice, st);
+    if (E_raw > 0 && dedge) {
+        k_edges<<<(unsigned)((E_raw + 255) / 256), 256, 0, st>>>(tptr, tdat, dptr, ddat, n, E_raw, dedge);
+        count_launch();
+    }
     return cudaGetLastError();
 }
 

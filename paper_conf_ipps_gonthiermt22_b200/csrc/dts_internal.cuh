@@ -1,21 +1,31 @@
 // dts_internal.cuh -- device-side data layout of libdts (sm_100a).
 //
-// Layout in HBM, per instance:
-//   CSR (built on device, §8(a) a1):  tptr[m+1] int64, tdat[E] int32 (rows sorted,
-//       de-duplicated), dptr[n+1] int64, ddat[E] int32 (each data segment in
-//       ascending task id).
-//   s[K][m_pad] uint32 -- per (simulated GPU k, task T) packed state
+// One CTA runs one instance's whole schedule.  Layout
+// per instance; arrays marked [S/G] live in the
+// CTA's shared memory when the host's placement (Inst::so_*) fits them in the
+// budget, else in their global (HBM/L2) home:
+//
+//   CSR (built on device, §8(a) a1):  tptr[m+1] int64, tdat[E] int32 (rows
+//       sorted, de-duplicated), dptr[n+1] int64, ddat[E] int32 (each data
+//       segment in ascending task id), dedge[E] int4 = ddat's edge records
+//       {T, other inputs of T, |D(T)|} so a segment walk needs no row lookup [G]
+//   s[K][m_pad] uint32 -- per (simulated GPU k, task T) packed state    [S/G]
 //       bit 31      : T allocated (left the shared pool of unprocessed tasks, R2)
 //       bits 24..30 : cnt_k(T) = |D(T) \ R_k|   (<= 127)
 //       bits  0..23 : x_k(T)   = XOR of the ids in D(T) \ R_k   (n < 2^24)
-//     so (s >> 24) == 1  <=>  T unallocated and exactly one input missing, and
-//     then x_k(T) IS that missing datum: "tasks that depend only on D and data
-//     already loaded" (Alg. 5 l.5) need no rescan.
-//   u[n] int32   -- #unallocated tasks using D (Alg. 5 l.9 secondary key, R23)
-//   hist[n] int32 -- per-scan score n_k(D) (zero between scans)
-//   np[K][n] int32 -- #tasks of plannedTasks_k using D (Alg. 6 l.3)
-//   res_list[K][res_cap], res_pos[K][n] -- resident set of each simulated GPU
-//   planned[K][plan_cap] -- plannedTasks_k in ascending id (-1 = removed by LUF)
+//     so a task with cnt 1 NAMES its one missing datum: x_k(T).
+//   h[K][n]  int32 -- n_k(D)  = #unallocated T with cnt_k(T)=1, x_k(T)=D: the
+//       DARTS score of Alg. 5 l.4-5, kept incrementally [S/G]
+//   h2[K][n] int32 -- n2_k(D) = #unallocated T with cnt_k(T)=2, D missing:
+//       the "3inputs" score, kept incrementally      [S/G]
+//   u[n]     int32 -- #unallocated tasks using D (secondary key, R23)     [S/G]
+//   np[K][n] int32 -- #tasks of plannedTasks_k using D (Alg. 6 l.3)       [S/G]
+//   resb[K][nw] uint32 -- residency bitmap of each simulated GPU          [S/G]
+//   res_list[K][res_cap] int32 -- resident data of each GPU (LUF scan)    [S/G]
+//   plan[K][plan_cap] int4 -- plannedTasks_k in ascending id: {T, D0, D1, D2}
+//       (T = -1: removed by LUF; D(T) cached when |D(T)| <= 3, D2 = -2 when
+//       the row is longer)                                           [S/G]
+//   plan_tau[K][plan_cap] int64 -- their durations (per-task times only)  [S/G]
 #pragma once
 #include <cstdint>
 
@@ -31,60 +41,55 @@ constexpr uint32_t CNT_ONE = 1u << 24;
 constexpr uint32_t XOR_MASK = 0x00FFFFFFu;
 constexpr int MAX_K = 64;
 constexpr int MAX_ROW = 127;
-
-enum Cmd : int { CMD_NONE = 0, CMD_SCAN = 1, CMD_FSCAN = 2, CMD_DONE = 3 };
-
-// Per-instance control block (global memory, zeroed by the init kernel).
-struct Ctrl {
-    unsigned bar_count;
-    unsigned bar_gen;
-    int cmd;
-    int cmd_k;
-    unsigned long long best_key;  // argmax over D of packed (score, u, ~id), atomicMax
-    int min_avail;                // lowest unallocated task id (fallback, Alg. 5 l.13)
-    int error;
-};
+constexpr int ROW_LONG = -2;  // plan entry: |D(T)| > 3, read the row from the CSR
 
 // Scalar results written by the decision loop.
 struct Out {
     int64_t n_events, n_served, n_loads, n_evictions, n_scans, n_fallback2, n_fallback_first,
-        n_belady, n_idle;
+        n_belady, n_idle, n_verify_err;
     uint64_t bytes_loaded;
     int64_t makespan;
     uint64_t alg_bytes, scan_alg_bytes;
     int32_t error;
     int32_t pad;
+    int64_t prof[8];  // SM cycles seen by thread 0 per phase (see PROF_* in dts_loop.cu)
 };
 
-// Device descriptor of one instance (passed by pointer to the loop kernel).
+// Device descriptor of one instance.
 struct Inst {
     int32_t m, n, K, W;
     uint32_t flags;
-    int32_t m_pad;       // m rounded up to a multiple of 4 (uint4 scans); pad words = ALLOC_BIT
+    int32_t m_pad;       // m rounded up to a multiple of 4; pad words = ALLOC_BIT
     int64_t max_served;  // -1 = run to completion
     uint64_t cap;        // bytes per simulated GPU
     int32_t plan_cap;    // >= max_D deg(D)
     int32_t res_cap;     // >= max resident data per GPU
     int32_t id_bits, u_bits;
+    int32_t nw;          // 32-bit words per residency bitmap row
+    int32_t pad0;
     int64_t E;
     // CSR (device)
     const int64_t *tptr;
     const int32_t *tdat;
     const int64_t *dptr;
     const int32_t *ddat;
+    const int4 *dedge;     // [E] edge records of the data->task CSR: {T, o1, o2, |D(T)|},
+                           // o1/o2 = T's other inputs (-1 if none; first two if |D(T)| > 3)
     const uint64_t *size;
     const int64_t *delta;  // ceil(size * 1e9 / bw) ns (reading R9)
     const int64_t *tau;    // [m] or nullptr
     int64_t default_tau;
-    // state
+    // state: global homes
     uint32_t *s;
-    int32_t *u;
-    int32_t *hist;
-    int32_t *np;
+    int32_t *u, *h, *h2, *np;
+    uint32_t *resb;
     int32_t *res_list;
-    int32_t *res_pos;
-    int32_t *planned;
-    Ctrl *ctrl;
+    int4 *plan;
+    int64_t *plan_tau;
+    int32_t *vhist;  // DTS_F_VERIFY scratch [3 n]
+    // shared-memory placement: byte offset in the CTA's dynamic smem, -1 = global home
+    int32_t so_u, so_h, so_h2, so_np, so_resb, so_res_list, so_plan, so_plan_tau, so_s;
+    int32_t smem_bytes;
     // outputs
     int32_t *serve_gpu;
     int32_t *serve_task;

@@ -1,23 +1,31 @@
 // dts_loop.cu -- the device-resident DARTS+LUF decision loop (§8(a) a2-a8).
 //
-// One launch runs a whole schedule.  A "group" of G CTAs cooperates on one
-// instance (G = 1 for small instances and for the batched sweep, G = #SMs for
-// the 1M-task configs).  Warp 0 of the group's CTA 0 -- the LEADER -- owns the
-// sequential part of the method (event order, plannedTasks pops, LUF, loads,
-// evictions, the bus/time model, the trace).  When a request finds
-// plannedTasks_k empty (Alg. 5 l.3), the leader hands one data-parallel pass to
-// the whole group:
+// ONE CTA runs ONE instance's whole schedule in a single launch (a batched
+// launch runs many instances: each CTA pulls the next instance from a device
+// counter).  The method is a chain of sequential decisions (PAPER.md:697-730:
+// each request depends on every earlier load, eviction and allocation), so the
+// kernel is built for per-decision LATENCY: thread 0 owns the scalar state
+// (event order, pops, the bus/time model, the trace) in shared memory, and
+// the whole CTA joins only for the data-parallel steps:
 //
-//   SCAN(k)  : for every task T, if (s_k[T] >> 24) == 1 then hist[x_k(T)] += 1
-//              -- n_k(D) of Alg. 5 l.4-5 for every D at once
-//   FSCAN(k) : tasks with two missing inputs add 1 to both (3inputs,
-//              PAPER.md:1823-1834) + the lowest unallocated id (Alg. 5 l.13)
-//   ARGMAX   : each CTA reduces its slice of D to the packed key
-//              (score, u(D), ~D) -- ties -> more unprocessed uses, then lower
-//              id (Alg. 5 l.6-9, R1/R23) -- and one atomicMax per CTA.
+//   score    : n_k(D) = #unallocated tasks whose only missing input is D
+//              (Alg. 5 l.4-5) is kept INCREMENTALLY in
+//              h[k][D]: every residency change walks the datum's data->task
+//              segment and moves each touched task between the cnt==1 / cnt==2
+//              buckets.  A scan is then a block argmax over D of the packed key
+//              (n(D), u(D), ~D): more unprocessed uses, then lower id, on ties
+//              (Alg. 5 l.6-9, readings R1/R23) -- O(n), not O(m).
+//   3inputs  : the same with h2[k][D] (tasks with two missing inputs, both
+//              credited) when no datum frees a task.
+//   plan     : ordered compaction of Dopt's segment -> plannedTasks_k (Alg. 5 l.10)
+//   LUF      : block min over the resident data of (np(D), D) among those the
+//              taskBuffer does not use (Alg. 6).
+//   residency: segment update of the packed (cnt, xor) state + score buckets.
 //
-// Group barriers: __syncthreads when G == 1, else a sense-reversing barrier on
-// a global counter (the launch is cooperative, so all G CTAs are resident).
+// Pops (Alg. 5 l.1-2) -- most requests -- are served by thread 0 alone with no
+// barrier and no global read: a planned task has all its inputs resident
+// (its inputs were resident or Dopt when planned; LUF drops planned tasks whose
+// inputs it evicts, Alg. 6 l.8), so serving it is pure time-model arithmetic.
 #include <cuda_runtime.h>
 
 #include <climits>
@@ -32,69 +40,52 @@ namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
 
-struct LState {  // leader-only state, in CTA 0's shared memory
+enum Cmd : int { CMD_SCAN = 1, CMD_DONE = 2 };
+
+// Per-phase cycle accounting by thread 0 (diagnostics, dts_result_view.prof_cycles).
+enum Prof : int { P_POP = 0, P_ARGMAX, P_PLAN, P_LOADS, P_LUF, P_EVICT, P_SEG, P_OTHER };
+#define PROF_T0(var) const long long var = (threadIdx.x == 0) ? clock64() : 0
+#define PROF_ADD(L, slot, var) \
+    do {                       \
+        if (threadIdx.x == 0) (L).prof[slot] += clock64() - (var); \
+    } while (0)
+
+struct Lead {  // leader scalars + broadcast slots (static shared memory)
     int64_t req[MAX_K];
     int64_t gpu_free[MAX_K];
     uint64_t used[MAX_K];
     int32_t plan_head[MAX_K], plan_end[MAX_K], plan_live[MAX_K];
     int32_t res_cnt[MAX_K];
-    int32_t last_task[MAX_K];
     int32_t idle[MAX_K];
     int64_t bus_free;
-    int64_t n_events, n_served, n_loads, n_evictions, n_scans, n_fb2, n_fbf, n_belady, n_idle;
-    uint64_t bytes_loaded;
+    int64_t n_events, n_served, n_loads, n_evictions, n_scans, n_fb2, n_fbf, n_belady, n_idle,
+        n_verr;
+    uint64_t bytes_loaded, alg_bytes, scan_alg_bytes;
     int64_t makespan;
-    uint64_t alg_bytes, scan_alg_bytes;
-    int32_t n_avail;
-    int32_t pending;  // CMD_SCAN / CMD_FSCAN awaiting its result, or CMD_NONE
-    int32_t pend_k;
-    int64_t pend_t;
-    int32_t row[MAX_ROW + 1];  // D(T) of the task being served
-    int32_t row_len;
+    int32_t n_avail, avail_lo;
     int32_t error;
+    int32_t cmd, k, T, vslot, row_len;
+    int64_t t, ready;
+    int32_t row[MAX_ROW + 1];
+    unsigned long long red64[32];
+    int32_t red32[32];
+    int32_t wcnt[32];
+    long long prof[8];
 };
 
-__device__ __forceinline__ int ldcg_i32(const int32_t *p) { return __ldcg(p); }
-__device__ __forceinline__ uint32_t ldcg_u32(const uint32_t *p) { return __ldcg(p); }
+// Per-instance views: shared-memory arrays where placed, else global homes.
+struct View {
+    uint32_t *s;
+    int32_t *u, *h, *h2, *np;
+    uint32_t *resb;
+    int32_t *res_list;
+    int4 *plan;
+    int64_t *plan_tau;
+};
 
-__device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long *p) {
-    return *(const volatile unsigned long long *)p;
-}
-
-// ------------------------------------------------------------ group barrier
-__device__ __forceinline__ void group_sync(Ctrl *c, int G) {
-    __syncthreads();
-    if (G > 1) {
-        if (threadIdx.x == 0) {
-            volatile unsigned *vgen = &c->bar_gen;
-            unsigned gen = *vgen;
-            __threadfence();
-            unsigned arrived = atomicAdd(&c->bar_count, 1u);
-            if (arrived == (unsigned)G - 1) {
-                c->bar_count = 0;
-                __threadfence();
-                atomicAdd(&c->bar_gen, 1u);
-            } else {
-                while (*vgen == gen) __nanosleep(32);
-            }
-            __threadfence();
-        }
-        __syncthreads();
-    }
-}
-
-// ------------------------------------------------------------ warp helpers
 __device__ __forceinline__ int warp_sum(int v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
-    return v;
-}
-__device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        unsigned long long t = __shfl_xor_sync(FULL, v, o);
-        v = t < v ? t : v;
-    }
     return v;
 }
 __device__ __forceinline__ unsigned long long warp_max_u64(unsigned long long v) {
@@ -105,78 +96,195 @@ __device__ __forceinline__ unsigned long long warp_max_u64(unsigned long long v)
     }
     return v;
 }
-__device__ __forceinline__ int warp_min_i32(int v) {
+__device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long v) {
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v = min(v, __shfl_xor_sync(FULL, v, o));
+    for (int o = 16; o > 0; o >>= 1) {
+        unsigned long long t = __shfl_xor_sync(FULL, v, o);
+        v = t < v ? t : v;
+    }
     return v;
 }
 
-__device__ __forceinline__ bool row_contains(const Inst &I, int32_t T, int32_t D) {
-    int64_t b = __ldg(&I.tptr[T]), e = __ldg(&I.tptr[T + 1]);
-    for (int64_t i = b; i < e; i++)
-        if (__ldg(&I.tdat[i]) == D) return true;
-    return false;
+// Block reductions (every thread calls; the result is returned to every thread).
+__device__ unsigned long long block_max_u64(Lead &L, unsigned long long v) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    v = warp_max_u64(v);
+    __syncthreads();
+    if (lane == 0) L.red64[w] = v;
+    __syncthreads();
+    unsigned long long r = 0ull;
+    for (int i = 0; i < nw; i++) r = L.red64[i] > r ? L.red64[i] : r;
+    return r;
+}
+__device__ unsigned long long block_min_u64(Lead &L, unsigned long long v) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    v = warp_min_u64(v);
+    __syncthreads();
+    if (lane == 0) L.red64[w] = v;
+    __syncthreads();
+    unsigned long long r = ~0ull;
+    for (int i = 0; i < nw; i++) r = L.red64[i] < r ? L.red64[i] : r;
+    return r;
+}
+__device__ int block_sum(Lead &L, int v) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    v = warp_sum(v);
+    __syncthreads();
+    if (lane == 0) L.red32[w] = v;
+    __syncthreads();
+    int r = 0;
+    for (int i = 0; i < nw; i++) r += L.red32[i];
+    return r;
+}
+
+__device__ __forceinline__ bool resident(const Inst &I, const View &V, int k, int32_t D) {
+    return (V.resb[(size_t)k * I.nw + (D >> 5)] >> (D & 31)) & 1u;
 }
 
 __device__ __forceinline__ int64_t tau_of(const Inst &I, int32_t T) {
     return I.tau ? __ldg(&I.tau[T]) : I.default_tau;
 }
 
-// a2: residency update of GPU k's packed state along D's data->task segment.
-// load: cnt -= 1, x ^= D ; evict: cnt += 1, x ^= D.  Each task appears once in
-// the segment, so plain read-modify-write (no atomics) is race-free.
-__device__ void seg_update(const Inst &I, int k, int32_t D, bool load, int lane) {
-    const int64_t b = __ldg(&I.dptr[D]), e = __ldg(&I.dptr[D + 1]);
-    uint32_t *sk = I.s + (size_t)k * I.m_pad;
-    for (int64_t i = b + lane; i < e; i += 128) {
-        int32_t T[4];
-        uint32_t w[4];
+// D(T) as carried by an edge record / plan entry: the full row when
+// len <= 3 (r0..r2, -1 = absent), else only len (rows are read from the CSR).
+struct Row {
+    int32_t r0, r1, r2, len;
+};
+
+__device__ __forceinline__ Row row_of_task(const Inst &I, int32_t T) {
+    const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+    Row r;
+    r.len = (int32_t)(re - rb);
+    r.r0 = r.len > 0 ? __ldg(&I.tdat[rb]) : -1;
+    r.r1 = r.len > 1 ? __ldg(&I.tdat[rb + 1]) : -1;
+    r.r2 = r.len > 2 ? __ldg(&I.tdat[rb + 2]) : -1;
+    return r;
+}
+
+// The (first two) inputs of T not resident on GPU k, skipping `skip`.
+__device__ __forceinline__ void missing_pair(const Inst &I, const View &V, int k, int32_t T, Row r,
+                                             int32_t skip, int32_t &a, int32_t &b) {
+    a = -1;
+    b = -1;
+    if (r.len <= 3) {
+        const int32_t c[3] = {r.r0, r.r1, r.r2};
 #pragma unroll
-        for (int j = 0; j < 4; j++) {
-            int64_t ii = i + 32 * j;
-            T[j] = ii < e ? __ldg(&I.ddat[ii]) : -1;
+        for (int i = 0; i < 3; i++) {
+            const int32_t D = c[i];
+            if (D < 0 || D == skip || resident(I, V, k, D)) continue;
+            if (a < 0) a = D;
+            else b = D;
         }
+        return;
+    }
+    const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+    for (int64_t i = rb; i < re; i++) {
+        const int32_t D = __ldg(&I.tdat[i]);
+        if (D == skip || resident(I, V, k, D)) continue;
+        if (a < 0) a = D;
+        else if (b < 0) b = D;
+    }
+}
+
+// T leaves (sign = -1) or re-enters (sign = +1) the shared pool of unallocated
+// tasks (R2, R4): the ALLOC bit in all K state copies, the score buckets of
+// every GPU on which T has one or two missing inputs, u(D) for its inputs,
+// and np_k(D) when it enters / leaves plannedTasks_k (plan_k >= 0).  Called by
+// ONE thread per task; the touched words of s are T's own.  The K state words
+// are loaded together (one round trip), then updated.
+__device__ void pool_move(const Inst &I, const View &V, int32_t T, Row r, int sign, int plan_k) {
+    for (int j0 = 0; j0 < I.K; j0 += 8) {
+        uint32_t w[8];
 #pragma unroll
-        for (int j = 0; j < 4; j++) w[j] = T[j] >= 0 ? ldcg_u32(&sk[T[j]]) : 0u;
+        for (int jj = 0; jj < 8; jj++)
+            if (j0 + jj < I.K) w[jj] = V.s[(size_t)(j0 + jj) * I.m_pad + T];
 #pragma unroll
-        for (int j = 0; j < 4; j++)
-            if (T[j] >= 0) sk[T[j]] = (load ? (w[j] - CNT_ONE) : (w[j] + CNT_ONE)) ^ (uint32_t)D;
+        for (int jj = 0; jj < 8; jj++) {
+            const int j = j0 + jj;
+            if (j >= I.K) break;
+            V.s[(size_t)j * I.m_pad + T] = sign < 0 ? (w[jj] | ALLOC_BIT) : (w[jj] & ~ALLOC_BIT);
+            const uint32_t c = (w[jj] >> 24) & 0x7fu;
+            if (c == 1u) {
+                atomicAdd(&V.h[(size_t)j * I.n + (w[jj] & XOR_MASK)], sign);
+            } else if (c == 2u) {
+                int32_t a, b;
+                missing_pair(I, V, j, T, r, -1, a, b);
+                atomicAdd(&V.h2[(size_t)j * I.n + a], sign);
+                atomicAdd(&V.h2[(size_t)j * I.n + b], sign);
+            }
+        }
+    }
+    if (r.len <= 3) {
+        const int32_t c[3] = {r.r0, r.r1, r.r2};
+#pragma unroll
+        for (int i = 0; i < 3; i++) {
+            if (c[i] < 0) continue;
+            atomicAdd(&V.u[c[i]], sign);
+            if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.n + c[i]], -sign);
+        }
+        return;
+    }
+    const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+    for (int64_t i = rb; i < re; i++) {
+        const int32_t D = __ldg(&I.tdat[i]);
+        atomicAdd(&V.u[D], sign);
+        if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.n + D], -sign);
     }
 }
 
-// Mark T allocated (it leaves the shared pool, R2): ALLOC bit in all K state
-// copies, u(D) -= 1 for its inputs, np_k(D) += 1 if it enters plannedTasks_k.
-// Called by ONE lane per task.
-__device__ void allocate_task(const Inst &I, int k, int32_t T, bool planned) {
-    for (int j = 0; j < I.K; j++) {
-        uint32_t *p = I.s + (size_t)j * I.m_pad + T;
-        *p = ldcg_u32(p) | ALLOC_BIT;
-    }
-    int64_t b = __ldg(&I.tptr[T]), e = __ldg(&I.tptr[T + 1]);
-    for (int64_t i = b; i < e; i++) {
-        int32_t D = __ldg(&I.tdat[i]);
-        atomicSub(&I.u[D], 1);
-        if (planned) atomicAdd(&I.np[(size_t)k * I.n + D], 1);
+// a2: datum D becomes resident (load) / leaves (evict) on GPU k.  Walk D's
+// data->task segment (edge records: the task and its other inputs in one 16 B
+// load): cnt_k(T) -/+= 1, x_k(T) ^= D, and move every unallocated task between
+// the score buckets h (cnt 1) and h2 (cnt 2).  The residency bit of D is
+// already updated.  Each task appears once in the segment, so the state words
+// are plain read-modify-writes; the buckets are atomics.
+__device__ void seg_update(const Inst &I, const View &V, int k, int32_t D, bool load) {
+    const int64_t b = __ldg(&I.dptr[D]), e = __ldg(&I.dptr[D + 1]);
+    uint32_t *sk = V.s + (size_t)k * I.m_pad;
+    int32_t *hk = V.h + (size_t)k * I.n;
+    int32_t *h2k = V.h2 + (size_t)k * I.n;
+    for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
+        const int4 ed = __ldg(&I.dedge[i]);
+        const int32_t T = ed.x;
+        const uint32_t w = sk[T];
+        sk[T] = (load ? (w - CNT_ONE) : (w + CNT_ONE)) ^ (uint32_t)D;
+        if (w & ALLOC_BIT) continue;
+        const uint32_t c = (w >> 24) & 0x7fu;
+        const int32_t x = (int32_t)(w & XOR_MASK);
+        if (load) {
+            if (c == 1u) {  // 1 -> 0: no longer scores for D
+                atomicSub(&hk[D], 1);
+            } else if (c == 2u) {  // 2 -> 1: now freed by its other missing datum
+                const int32_t o = x ^ D;
+                atomicSub(&h2k[D], 1);
+                atomicSub(&h2k[o], 1);
+                atomicAdd(&hk[o], 1);
+            } else if (c == 3u) {  // 3 -> 2: one load away from two data
+                int32_t a2 = ed.y, b2 = ed.z;  // |D(T)| = 3: both others miss
+                if (ed.w > 3) missing_pair(I, V, k, T, Row{-1, -1, -1, ed.w}, -1, a2, b2);
+                atomicAdd(&h2k[a2], 1);
+                atomicAdd(&h2k[b2], 1);
+            }
+        } else {
+            if (c == 0u) {  // 0 -> 1
+                atomicAdd(&hk[D], 1);
+            } else if (c == 1u) {  // 1 -> 2: missing {x, D}
+                atomicSub(&hk[x], 1);
+                atomicAdd(&h2k[x], 1);
+                atomicAdd(&h2k[D], 1);
+            } else if (c == 2u) {  // 2 -> 3
+                int32_t a2 = ed.y, b2 = ed.z;  // |D(T)| = 3: both others missed
+                if (ed.w > 3) missing_pair(I, V, k, T, Row{-1, -1, -1, ed.w}, D, a2, b2);
+                atomicSub(&h2k[a2], 1);
+                atomicSub(&h2k[b2], 1);
+            }
+        }
     }
 }
 
-// Inverse of allocate_task for a planned task removed by LUF (Alg. 6 l.8, R4).
-__device__ void unallocate_task(const Inst &I, int k, int32_t T) {
-    for (int j = 0; j < I.K; j++) {
-        uint32_t *p = I.s + (size_t)j * I.m_pad + T;
-        *p = ldcg_u32(p) & ~ALLOC_BIT;
-    }
-    int64_t b = __ldg(&I.tptr[T]), e = __ldg(&I.tptr[T + 1]);
-    for (int64_t i = b; i < e; i++) {
-        int32_t D = __ldg(&I.tdat[i]);
-        atomicAdd(&I.u[D], 1);
-        atomicSub(&I.np[(size_t)k * I.n + D], 1);
-    }
-}
-
-__device__ __forceinline__ void push_event(const Inst &I, LState &L, uint8_t op, int k, int32_t D,
+__device__ __forceinline__ void push_event(const Inst &I, Lead &L, uint8_t op, int k, int32_t D,
                                            int32_t T, int64_t t, int64_t te) {
-    int64_t i = L.n_events;
+    const int64_t i = L.n_events;
     if (i < I.ev_cap) {
         dts_event ev;
         ev.t_ns = t;
@@ -191,495 +299,751 @@ __device__ __forceinline__ void push_event(const Inst &I, LState &L, uint8_t op,
     L.n_events = i + 1;
 }
 
-// ------------------------------------------------------------ LUF (Alg. 6)
-// Among the data in GPU k's memory not used by the taskBuffer (nb(D) = 0,
-// l.4-5), the one with the fewest uses in plannedTasks_k (np), lowest id on ties.
-__device__ int32_t luf_victim(const Inst &I, LState &L, int k, int lane) {
-    const int cnt = L.res_cnt[k];
-    const int32_t *rl = I.res_list + (size_t)k * I.res_cap;
-    unsigned long long best = ~0ull;
-    for (int i = lane; i < cnt; i += 32) {
-        int32_t D = ldcg_i32(&rl[i]);
-        bool in_buf = false;
-        for (int r = 0; r < L.row_len; r++) in_buf |= (L.row[r] == D);
-        if (in_buf) continue;  // nb(D) > 0
-        unsigned long long key =
-            ((unsigned long long)(uint32_t)ldcg_i32(&I.np[(size_t)k * I.n + D]) << 32) | (uint32_t)D;
-        best = key < best ? key : best;
-    }
-    best = warp_min_u64(best);
-    if (best == ~0ull) return -1;  // Belady branch (l.7): unreachable with the capacity check
-    return (int32_t)(best & 0xffffffffu);
+// Thread 0: record the service of T on k (time model of PAPER.md:276-342, R7, R9).
+__device__ __forceinline__ void finish_serve(const Inst &I, Lead &L, int k, int32_t T, int64_t ready,
+                                             int64_t tau) {
+    const int64_t start = ready > L.gpu_free[k] ? ready : L.gpu_free[k];
+    const int64_t end = start + tau;
+    L.gpu_free[k] = end;
+    I.tstart[T] = start;
+    I.tend[T] = end;
+    if (end > L.makespan) L.makespan = end;
+    I.serve_gpu[L.n_served] = k;
+    I.serve_task[L.n_served] = T;
+    L.n_served++;
+    L.req[k] = (I.W == 0) ? end : start;  // R7
+    L.alg_bytes += 24;
 }
 
-__device__ void evict(const Inst &I, LState &L, int k, int32_t V, int32_t Tserved, int64_t t,
-                      int lane) {
-    // Alg. 6 l.8: planned tasks that use V return to the shared pool (R4)
-    int nret = 0;
-    int32_t *pl = I.planned + (size_t)k * I.plan_cap;
-    for (int i = L.plan_head[k] + lane; i < L.plan_end[k]; i += 32) {
-        int32_t T2 = ldcg_i32(&pl[i]);
-        if (T2 >= 0 && row_contains(I, T2, V)) {
-            pl[i] = -1;
-            unallocate_task(I, k, T2);
-            nret++;
+// Thread 0: pop the smallest planned task of k (Alg. 5 l.2 / l.11, R3); it
+// leaves plannedTasks_k (np_k(D) -= 1 for its inputs).  Returns T and its tau.
+__device__ int32_t pop_planned(const Inst &I, const View &V, Lead &L, int k, int64_t *tau) {
+    const int4 *pl = V.plan + (size_t)k * I.plan_cap;
+    int h = L.plan_head[k];
+    int4 e = pl[h];
+    while (e.x < 0) e = pl[++h];
+    L.plan_head[k] = h + 1;
+    L.plan_live[k]--;
+    int32_t *npk = V.np + (size_t)k * I.n;
+    if (e.w != ROW_LONG) {
+        if (e.y >= 0) atomicSub(&npk[e.y], 1);
+        if (e.z >= 0) atomicSub(&npk[e.z], 1);
+        if (e.w >= 0) atomicSub(&npk[e.w], 1);
+    } else {
+        const int64_t rb = __ldg(&I.tptr[e.x]), re = __ldg(&I.tptr[e.x + 1]);
+        for (int64_t i = rb; i < re; i++) atomicSub(&npk[__ldg(&I.tdat[i])], 1);
+    }
+    *tau = V.plan_tau ? V.plan_tau[(size_t)k * I.plan_cap + h] : I.default_tau;
+    // D(T) for serve_loads, ascending (R10), straight from the entry when cached
+    if (e.w != ROW_LONG) {
+        int32_t a = e.y, b = e.z, c = e.w;  // -1 = absent; sort descending, count
+        if (a < b) { const int32_t t = a; a = b; b = t; }
+        if (b < c) { const int32_t t = b; b = c; c = t; }
+        if (a < b) { const int32_t t = a; a = b; b = t; }
+        const int len = (a >= 0) + (b >= 0) + (c >= 0);
+        L.row_len = len;
+        if (len == 3) { L.row[0] = c; L.row[1] = b; L.row[2] = a; }
+        else if (len == 2) { L.row[0] = b; L.row[1] = a; }
+        else if (len == 1) { L.row[0] = a; }
+    } else {
+        L.row_len = -1;
+    }
+    return e.x;
+}
+
+// Thread 0: serve every request that finds plannedTasks_k non-empty (Alg. 5
+// l.1-2) until one finds it empty (returns that k; L.k, L.t set) or the run
+// ends (-1).  No other thread, no barrier, no global read: the popped task's
+// inputs are resident, so serving it is time-model arithmetic.
+// np_k is NOT maintained here: LUF on GPU k only runs while k serves the first
+// task of a new plan (or a fallback task, with no plan), and every scan resets
+// np_k (reset_plan), so the pops of an old plan never reach a LUF decision.
+// The per-GPU scalars live in registers (KR >= K, compile-time) so a pop is a
+// short dependent chain; outputs go out with plain global stores.
+template <int KR>
+__device__ int pop_run(const Inst &I, const View &V, Lead &L) {
+    const int K = I.K, W = I.W, pcap = I.plan_cap;
+    const int64_t maxs = I.max_served, dtau = I.default_tau;
+    int32_t *const sg = I.serve_gpu;
+    int32_t *const stk = I.serve_task;
+    int64_t *const tst = I.tstart;
+    int64_t *const ten = I.tend;
+    int64_t rq[KR], gf[KR];
+    int hd[KR], lv[KR];
+    bool act[KR];
+#pragma unroll
+    for (int j = 0; j < KR; j++) {
+        act[j] = j < K && !L.idle[j];
+        rq[j] = j < K ? L.req[j] : 0;
+        gf[j] = j < K ? L.gpu_free[j] : 0;
+        hd[j] = j < K ? L.plan_head[j] : 0;
+        lv[j] = j < K ? L.plan_live[j] : 0;
+    }
+    int64_t ns = L.n_served, mk = L.makespan, pops = 0;
+    int ret = -1;
+    while (maxs < 0 || ns < maxs) {
+        // the earliest (req, k) and the runner-up among non-idle GPUs (R8)
+        int k = -1, k2 = -1;
+        int64_t t1 = 0, t2 = 0;
+#pragma unroll
+        for (int j = 0; j < KR; j++) {
+            if (!act[j]) continue;
+            const int64_t r = rq[j];
+            if (k < 0 || r < t1) {
+                k2 = k;
+                t2 = t1;
+                k = j;
+                t1 = r;
+            } else if (k2 < 0 || r < t2) {
+                k2 = j;
+                t2 = r;
+            }
+        }
+        if (k < 0) break;
+        int live = 0, h = 0;
+        int64_t gfree = 0;
+#pragma unroll
+        for (int j = 0; j < KR; j++)
+            if (j == k) {
+                live = lv[j];
+                h = hd[j];
+                gfree = gf[j];
+            }
+        if (live == 0) {
+            ret = k;
+            L.k = k;
+            L.t = t1;
+            break;
+        }
+        int64_t req = t1;
+        const int4 *pl = V.plan + (size_t)k * pcap;
+        const int64_t *pt = V.plan_tau ? V.plan_tau + (size_t)k * pcap : nullptr;
+        while (true) {
+            int T = pl[h].x;
+            while (T < 0) T = pl[++h].x;
+            const int64_t tau = pt ? pt[h] : dtau;
+            h++;
+            live--;
+            const int64_t start = req > gfree ? req : gfree;
+            const int64_t end = start + tau;
+            gfree = end;
+            __stcg(&tst[T], start);
+            __stcg(&ten[T], end);
+            mk = end > mk ? end : mk;
+            __stcg(&sg[ns], k);
+            __stcg(&stk[ns], T);
+            ns++;
+            pops++;
+            req = (W == 0) ? end : start;  // R7
+            if (live == 0 || (maxs >= 0 && ns >= maxs)) break;
+            if (k2 >= 0 && (req > t2 || (req == t2 && k2 < k))) break;  // another GPU is next
+        }
+#pragma unroll
+        for (int j = 0; j < KR; j++)
+            if (j == k) {
+                lv[j] = live;
+                hd[j] = h;
+                gf[j] = gfree;
+                rq[j] = req;
+            }
+    }
+#pragma unroll
+    for (int j = 0; j < KR; j++)
+        if (j < K) {
+            L.req[j] = rq[j];
+            L.gpu_free[j] = gf[j];
+            L.plan_head[j] = hd[j];
+            L.plan_live[j] = lv[j];
+        }
+    L.n_served = ns;
+    L.makespan = mk;
+    L.alg_bytes += 24ull * (uint64_t)pops;
+    return ret;
+}
+
+// pop_run for K > 8: the same, with the per-GPU scalars left in shared memory.
+__device__ int pop_run_smem(const Inst &I, const View &V, Lead &L) {
+    const int K = I.K, W = I.W, pcap = I.plan_cap;
+    const int64_t maxs = I.max_served, dtau = I.default_tau;
+    int32_t *const sg = I.serve_gpu;
+    int32_t *const stk = I.serve_task;
+    int64_t *const tst = I.tstart;
+    int64_t *const ten = I.tend;
+    int64_t ns = L.n_served, mk = L.makespan, pops = 0;
+    int ret = -1;
+    while (maxs < 0 || ns < maxs) {
+        int k = -1, k2 = -1;
+        int64_t t1 = 0, t2 = 0;
+        for (int j = 0; j < K; j++) {
+            if (L.idle[j]) continue;
+            const int64_t r = L.req[j];
+            if (k < 0 || r < t1) {
+                k2 = k;
+                t2 = t1;
+                k = j;
+                t1 = r;
+            } else if (k2 < 0 || r < t2) {
+                k2 = j;
+                t2 = r;
+            }
+        }
+        if (k < 0) break;
+        int live = L.plan_live[k];
+        if (live == 0) {
+            ret = k;
+            L.k = k;
+            L.t = t1;
+            break;
+        }
+        int h = L.plan_head[k];
+        int64_t req = t1, gfree = L.gpu_free[k];
+        const int4 *pl = V.plan + (size_t)k * pcap;
+        const int64_t *pt = V.plan_tau ? V.plan_tau + (size_t)k * pcap : nullptr;
+        while (true) {
+            int T = pl[h].x;
+            while (T < 0) T = pl[++h].x;
+            const int64_t tau = pt ? pt[h] : dtau;
+            h++;
+            live--;
+            const int64_t start = req > gfree ? req : gfree;
+            const int64_t end = start + tau;
+            gfree = end;
+            __stcg(&tst[T], start);
+            __stcg(&ten[T], end);
+            mk = end > mk ? end : mk;
+            __stcg(&sg[ns], k);
+            __stcg(&stk[ns], T);
+            ns++;
+            pops++;
+            req = (W == 0) ? end : start;  // R7
+            if (live == 0 || (maxs >= 0 && ns >= maxs)) break;
+            if (k2 >= 0 && (req > t2 || (req == t2 && k2 < k))) break;
+        }
+        L.plan_head[k] = h;
+        L.plan_live[k] = live;
+        L.req[k] = req;
+        L.gpu_free[k] = gfree;
+    }
+    L.n_served = ns;
+    L.makespan = mk;
+    L.alg_bytes += 24ull * (uint64_t)pops;
+    return ret;
+}
+
+// CTA-wide, at every scan of GPU k: plannedTasks_k is empty (all popped or
+// removed); clear np_k for every datum its last plan touched, so that np_k
+// counts exactly the plan this scan creates (Alg. 6 l.3).
+__device__ void reset_plan(const Inst &I, const View &V, Lead &L, int k) {
+    const int4 *pl = V.plan + (size_t)k * I.plan_cap;
+    int32_t *npk = V.np + (size_t)k * I.n;
+    const int pe = L.plan_end[k];
+    for (int i = threadIdx.x; i < pe; i += blockDim.x) {
+        const int4 e = pl[i];
+        if (e.w != ROW_LONG) {
+            if (e.y >= 0) npk[e.y] = 0;
+            if (e.z >= 0) npk[e.z] = 0;
+            if (e.w >= 0) npk[e.w] = 0;
+        } else {
+            const int T = e.x >= 0 ? e.x : -1;
+            if (T >= 0) {
+                const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+                for (int64_t j = rb; j < re; j++) npk[__ldg(&I.tdat[j])] = 0;
+            }
         }
     }
-    nret = warp_sum(nret);
-    // l.9: evict V
-    if (lane == 0) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        L.plan_head[k] = 0;
+        L.plan_end[k] = 0;
+        L.plan_live[k] = 0;
+    }
+    __syncthreads();
+}
+
+__device__ __forceinline__ Row row_of_entry(int4 e) {
+    if (e.w == ROW_LONG) return Row{-1, -1, -1, 4};
+    return Row{e.y, e.z, e.w, (e.y >= 0) + (e.z >= 0) + (e.w >= 0)};
+}
+
+__device__ __forceinline__ bool entry_uses(const Inst &I, int4 e, int32_t D) {
+    if (e.y == D || e.z == D) return true;
+    if (e.w != ROW_LONG) return e.w == D;
+    const int64_t rb = __ldg(&I.tptr[e.x]), re = __ldg(&I.tptr[e.x + 1]);
+    for (int64_t i = rb; i < re; i++)
+        if (__ldg(&I.tdat[i]) == D) return true;
+    return false;
+}
+
+// LUF (Alg. 6): among the data in GPU k's memory that the taskBuffer does not
+// use (nb(D) = 0, l.4-5; the taskBuffer = the task being served for W = 0),
+// the one with the fewest uses in plannedTasks_k, lowest id on ties (R1).
+// Block-wide; returns V (or -1: the Belady branch, unreachable, R7) and sets
+// L.vslot to its index in res_list.
+__device__ int32_t luf_victim(const Inst &I, const View &V, Lead &L, int k) {
+    const int cnt = L.res_cnt[k];
+    const int32_t *rl = V.res_list + (size_t)k * I.res_cap;
+    const int32_t *npk = V.np + (size_t)k * I.n;
+    unsigned long long best = ~0ull;
+    for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
+        const int32_t D = rl[i];
+        bool in_buf = false;
+        for (int r = 0; r < L.row_len; r++) in_buf |= (L.row[r] == D);
+        if (in_buf) continue;
+        const unsigned long long key =
+            ((unsigned long long)(uint32_t)npk[D] << 32) | (unsigned long long)(uint32_t)D;
+        best = key < best ? key : best;
+    }
+    best = block_min_u64(L, best);
+    if (best == ~0ull) return -1;
+    const int32_t Vd = (int32_t)(best & 0xffffffffull);
+    for (int i = threadIdx.x; i < cnt; i += blockDim.x)
+        if (rl[i] == Vd) L.vslot = i;
+    __syncthreads();
+    return Vd;
+}
+
+// Alg. 6 l.8-9: planned tasks of k that use V return to the shared pool (R4,
+// idle GPUs wake at t, R18); then V leaves GPU k's memory.  Block-wide.
+__device__ void evict(const Inst &I, const View &V, Lead &L, int k, int32_t Vd, int32_t Tserved,
+                      int64_t t) {
+    int4 *pl = V.plan + (size_t)k * I.plan_cap;
+    int nret = 0;
+    unsigned long long tmin = ~0ull;
+    const int ph = L.plan_head[k], pe = L.plan_end[k];
+    for (int i = ph + threadIdx.x; i < pe; i += blockDim.x) {
+        const int4 e = pl[i];
+        if (e.x >= 0 && entry_uses(I, e, Vd)) {
+            pl[i].x = -1;
+            pool_move(I, V, e.x, row_of_entry(e), +1, k);
+            nret++;
+            tmin = (unsigned long long)e.x < tmin ? (unsigned long long)e.x : tmin;
+        }
+    }
+    nret = block_sum(L, nret);
+    tmin = block_min_u64(L, tmin);
+    if (threadIdx.x == 0) {
         if (nret > 0) {
             L.plan_live[k] -= nret;
             L.n_avail += nret;
-            for (int j = 0; j < I.K; j++)  // wake idle GPUs (R18)
+            if ((int)tmin < L.avail_lo) L.avail_lo = (int)tmin;
+            for (int j = 0; j < I.K; j++)  // R18
                 if (L.idle[j]) {
                     L.idle[j] = 0;
                     L.req[j] = t;
                 }
         }
-        int32_t *rl = I.res_list + (size_t)k * I.res_cap;
-        int32_t *rp = I.res_pos + (size_t)k * I.n;
-        int p = rp[V];
-        int last = L.res_cnt[k] - 1;
-        int32_t Dl = rl[last];
-        rl[p] = Dl;
-        rp[Dl] = p;
-        rp[V] = -1;
+        int32_t *rl = V.res_list + (size_t)k * I.res_cap;
+        const int last = L.res_cnt[k] - 1;
+        rl[L.vslot] = rl[last];
         L.res_cnt[k] = last;
-        L.used[k] -= __ldg(&I.size[V]);
+        V.resb[(size_t)k * I.nw + (Vd >> 5)] &= ~(1u << (Vd & 31));
+        L.used[k] -= __ldg(&I.size[Vd]);
         L.n_evictions++;
-        push_event(I, L, 1, k, V, Tserved, t, t);
-        int64_t deg = __ldg(&I.dptr[V + 1]) - __ldg(&I.dptr[V]);
-        L.alg_bytes += 12ull * (uint64_t)deg + 16ull * (uint64_t)nret * (uint64_t)I.K;
+        push_event(I, L, 1, k, Vd, Tserved, t, t);
+        const int64_t deg = __ldg(&I.dptr[Vd + 1]) - __ldg(&I.dptr[Vd]);
+        L.alg_bytes += 12ull * (uint64_t)deg + (uint64_t)nret * (8ull * I.K + 32ull);
     }
-    __syncwarp();
-    seg_update(I, k, V, false, lane);
-    __syncwarp();
+    __syncthreads();
+    seg_update(I, V, k, Vd, false);
+    __syncthreads();
 }
 
-// Serve T on GPU k at request time t: evict V(k,i), load the missing inputs in
-// ascending id (R10), process; shared FIFO bus (R9).
-__device__ void serve(const Inst &I, LState &L, int k, int32_t T, int64_t t, int lane) {
-    const int64_t b = __ldg(&I.tptr[T]), e = __ldg(&I.tptr[T + 1]);
-    const int len = (int)(e - b);
-    for (int r = lane; r < len; r += 32) L.row[r] = __ldg(&I.tdat[b + r]);
-    if (lane == 0) L.row_len = len;
-    __syncwarp();
-    int64_t ready = t;
-    const int32_t *rp = I.res_pos + (size_t)k * I.n;
+// Serve T on GPU k at time t with loads: evict V(k,i), load the missing inputs
+// in ascending id (R10), process; shared FIFO bus (R9).
+// Block-wide.  L.row holds D(T).
+__device__ void serve_loads(const Inst &I, const View &V, Lead &L, int k, int32_t T, int64_t t) {
+    if (threadIdx.x == 0) L.ready = t;
+    __syncthreads();
+    const int len = L.row_len;
     for (int r = 0; r < len; r++) {
+        // every thread reads the shared state before thread 0 may change it
         const int32_t D = L.row[r];
-        if (ldcg_i32(&rp[D]) >= 0) continue;  // resident
+        const bool res = resident(I, V, k, D);
+        __syncthreads();
+        if (res) continue;
         const uint64_t sz = __ldg(&I.size[D]);
-        while (L.used[k] + sz > I.cap) {  // R11: repeat LUF until D fits
-            int32_t V = luf_victim(I, L, k, lane);
-            if (V < 0) {
-                if (lane == 0) L.error = 1;
-                __syncwarp();
+        while (true) {  // R11: LUF until D fits
+            const bool full = L.used[k] + sz > I.cap;
+            __syncthreads();
+            if (!full) break;
+            PROF_T0(p_luf);
+            const int32_t Vd = luf_victim(I, V, L, k);
+            PROF_ADD(L, P_LUF, p_luf);
+            if (Vd < 0) {
+                if (threadIdx.x == 0) L.error = 1;
+                __syncthreads();
                 return;
             }
-            evict(I, L, k, V, T, t, lane);
+            PROF_T0(p_ev);
+            evict(I, V, L, k, Vd, T, t);
+            PROF_ADD(L, P_EVICT, p_ev);
         }
-        if (lane == 0) {
-            int32_t *rl = I.res_list + (size_t)k * I.res_cap;
-            int c = L.res_cnt[k];
-            rl[c] = D;
-            I.res_pos[(size_t)k * I.n + D] = c;
-            L.res_cnt[k] = c + 1;
+        if (threadIdx.x == 0) {
+            int32_t *rl = V.res_list + (size_t)k * I.res_cap;
+            rl[L.res_cnt[k]++] = D;
+            V.resb[(size_t)k * I.nw + (D >> 5)] |= 1u << (D & 31);
             L.used[k] += sz;
-            int64_t st = L.bus_free > t ? L.bus_free : t;
-            int64_t en = st + __ldg(&I.delta[D]);
+            const int64_t st = L.bus_free > t ? L.bus_free : t;
+            const int64_t en = st + __ldg(&I.delta[D]);
             L.bus_free = en;
+            if (en > L.ready) L.ready = en;
             L.n_loads++;
             L.bytes_loaded += sz;
             push_event(I, L, 0, k, D, T, st, en);
-            int64_t deg = __ldg(&I.dptr[D + 1]) - __ldg(&I.dptr[D]);
+            const int64_t deg = __ldg(&I.dptr[D + 1]) - __ldg(&I.dptr[D]);
             L.alg_bytes += 12ull * (uint64_t)deg;
         }
-        __syncwarp();
-        ready = max(ready, L.bus_free);  // this load's end == bus_free now
-        seg_update(I, k, D, true, lane);
-        __syncwarp();
+        __syncthreads();
+        PROF_T0(p_seg);
+        seg_update(I, V, k, D, true);
+        __syncthreads();
+        PROF_ADD(L, P_SEG, p_seg);
     }
-    if (lane == 0) {
-        int64_t start = ready > L.gpu_free[k] ? ready : L.gpu_free[k];
-        int64_t end = start + tau_of(I, T);
-        L.gpu_free[k] = end;
-        I.tstart[T] = start;
-        I.tend[T] = end;
-        if (end > L.makespan) L.makespan = end;
-        I.serve_gpu[L.n_served] = k;
-        I.serve_task[L.n_served] = T;
-        L.n_served++;
-        L.last_task[k] = T;
-        L.req[k] = (I.W == 0) ? end : start;  // R7
-    }
-    __syncwarp();
+    if (threadIdx.x == 0) finish_serve(I, L, k, T, L.ready, tau_of(I, T));
+    __syncthreads();
 }
 
-// Pop the smallest planned task of GPU k (Alg. 5 l.2 / l.11, R3).
-__device__ int32_t pop_planned(const Inst &I, LState &L, int k, int lane) {
-    const int32_t *pl = I.planned + (size_t)k * I.plan_cap;
-    int h = L.plan_head[k];
-    int32_t T = -1;
-    while (true) {  // skip entries removed by LUF, 32 at a time
-        int i = h + lane;
-        int32_t v = i < L.plan_end[k] ? ldcg_i32(&pl[i]) : -1;
-        unsigned msk = __ballot_sync(FULL, v >= 0);
-        if (msk) {
-            int f = __ffs(msk) - 1;
-            T = __shfl_sync(FULL, v, f);
-            h += f + 1;
-            break;
-        }
-        h += 32;
-    }
-    // it leaves plannedTasks_k: np_k(D) -= 1 for its inputs
-    int64_t b = __ldg(&I.tptr[T]), e = __ldg(&I.tptr[T + 1]);
-    for (int64_t i = b + lane; i < e; i += 32) atomicSub(&I.np[(size_t)k * I.n + __ldg(&I.tdat[i])], 1);
-    __syncwarp();
-    if (lane == 0) {
-        L.plan_head[k] = h;
-        L.plan_live[k]--;
-    }
-    __syncwarp();
-    return T;
-}
-
-// Alg. 5 l.10: plannedTasks_k <- unallocated tasks depending only on Dopt and
-// data in memory = tasks of Dopt's segment with (s_k >> 24) == 1, in
-// ascending id (ordered warp compaction).
-__device__ void plan(const Inst &I, LState &L, int k, int32_t Dopt, int lane) {
-    const int64_t b = __ldg(&I.dptr[Dopt]), e = __ldg(&I.dptr[Dopt + 1]);
-    const uint32_t *sk = I.s + (size_t)k * I.m_pad;
-    int32_t *pl = I.planned + (size_t)k * I.plan_cap;
-    const unsigned lt = (1u << lane) - 1u;
-    int w = 0;
-    for (int64_t base = b; base < e; base += 32) {
-        int64_t i = base + lane;
-        int32_t T = -1;
-        bool sel = false;
-        if (i < e) {
-            T = __ldg(&I.ddat[i]);
-            sel = (ldcg_u32(&sk[T]) >> 24) == 1u;
-        }
-        unsigned msk = __ballot_sync(FULL, sel);
-        if (sel) {
-            pl[w + __popc(msk & lt)] = T;
-            allocate_task(I, k, T, true);
-        }
-        w += __popc(msk);
-    }
-    __syncwarp();
-    if (lane == 0) {
-        L.plan_head[k] = 0;
-        L.plan_end[k] = w;
-        L.plan_live[k] = w;
-        L.n_avail -= w;
-        int64_t segl = e - b;
-        L.alg_bytes += 8ull * (uint64_t)segl + (uint64_t)w * (4ull * I.K + 16ull);
-    }
-    __syncwarp();
-}
-
-// The leader's sequential event loop (R8).  Returns the command for the group.
-__device__ int leader_run(const Inst &I, LState &L, int lane) {
-    Ctrl *C = I.ctrl;
-    if (L.pending == CMD_SCAN) {
-        const int k = L.pend_k;
-        const int64_t t = L.pend_t;
-        unsigned long long key = ld_volatile_u64(&C->best_key);
-        __syncwarp();
-        if (lane == 0) C->best_key = 0ull;
-        if (key != 0ull) {  // Alg. 5 l.7: nmax > 0
-            const int32_t idmask = (int32_t)((1u << I.id_bits) - 1u);
-            const int32_t Dopt = idmask - (int32_t)(key & (unsigned long long)idmask);
-            plan(I, L, k, Dopt, lane);
-            int32_t T = pop_planned(I, L, k, lane);
-            if (lane == 0) {
-                L.n_scans++;
-                L.pending = CMD_NONE;
-            }
-            __syncwarp();
-            serve(I, L, k, T, t, lane);
-        } else {
-            if (lane == 0) L.pending = CMD_FSCAN;
-            __syncwarp();
-            if (lane == 0) {
-                C->cmd = CMD_FSCAN;
-                C->cmd_k = k;
-                L.scan_alg_bytes += 4ull * (uint64_t)L.n_avail;
-                L.alg_bytes += 4ull * (uint64_t)L.n_avail + 8ull * (uint64_t)I.n;
-            }
-            __syncwarp();
-            return CMD_FSCAN;
-        }
-    } else if (L.pending == CMD_FSCAN) {
-        const int k = L.pend_k;
-        const int64_t t = L.pend_t;
-        unsigned long long key = ld_volatile_u64(&C->best_key);
-        int minav = *(volatile int *)&C->min_avail;
-        __syncwarp();
-        if (lane == 0) {
-            C->best_key = 0ull;
-            C->min_avail = INT_MAX;
-            L.pending = CMD_NONE;
-        }
-        __syncwarp();
-        int32_t T = -1;
-        if (key != 0ull) {  // 3inputs: lowest-id task of D2 with two missing inputs
-            const int32_t idmask = (int32_t)((1u << I.id_bits) - 1u);
-            const int32_t D2 = idmask - (int32_t)(key & (unsigned long long)idmask);
-            const int64_t b = __ldg(&I.dptr[D2]), e = __ldg(&I.dptr[D2 + 1]);
-            const uint32_t *sk = I.s + (size_t)k * I.m_pad;
-            for (int64_t base = b; base < e && T < 0; base += 32) {
-                int64_t i = base + lane;
-                int32_t Tc = i < e ? __ldg(&I.ddat[i]) : -1;
-                bool ok = Tc >= 0 && (ldcg_u32(&sk[Tc]) >> 24) == 2u;
-                unsigned msk = __ballot_sync(FULL, ok);
-                if (msk) T = __shfl_sync(FULL, Tc, __ffs(msk) - 1);
-            }
-            if (lane == 0) L.n_fb2++;
-        } else if (minav != INT_MAX) {  // Alg. 5 l.13, reading R5
-            T = minav;
-            if (lane == 0) L.n_fbf++;
-        }
-        if (T >= 0) {
-            if (lane == 0) {
-                allocate_task(I, k, T, false);
-                L.n_avail--;
-                L.n_scans++;
-            }
-            __syncwarp();
-            serve(I, L, k, T, t, lane);
-        } else {
-            if (lane == 0) {
-                L.idle[k] = 1;
-                L.n_idle++;
-            }
-            __syncwarp();
-        }
-    }
-    // event loop
-    while (true) {
-        if (L.error) break;
-        if (I.max_served >= 0 && L.n_served >= I.max_served) break;
-        // next request: smallest (req_k, k) over non-idle GPUs (R8)
-        int kk = -1;
-        int64_t tb = 0;
-        for (int j = lane; j < I.K; j += 32) {
-            if (L.idle[j]) continue;
-            int64_t r = L.req[j];
-            if (kk < 0 || r < tb) {
-                kk = j;
-                tb = r;
-            }
-        }
-        // warp argmin on (req, k)
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            int ok = __shfl_xor_sync(FULL, kk, o);
-            int64_t ot = __shfl_xor_sync(FULL, tb, o);
-            if (ok >= 0 && (kk < 0 || ot < tb || (ot == tb && ok < kk))) {
-                kk = ok;
-                tb = ot;
-            }
-        }
-        if (kk < 0) break;  // every GPU idle
-        const int k = kk;
-        const int64_t t = tb;
-        if (L.plan_live[k] > 0) {  // Alg. 5 l.1-2
-            int32_t T = pop_planned(I, L, k, lane);
-            serve(I, L, k, T, t, lane);
-            continue;
-        }
-        // Alg. 5 l.4: scan dataNotInMem_k -- needs the whole group
-        if (lane == 0) {
-            L.pending = CMD_SCAN;
-            L.pend_k = k;
-            L.pend_t = t;
-            C->cmd = CMD_SCAN;
-            C->cmd_k = k;
-            L.scan_alg_bytes += 4ull * (uint64_t)L.n_avail + 8ull * (uint64_t)I.n;
-            L.alg_bytes += 4ull * (uint64_t)L.n_avail + 8ull * (uint64_t)I.n;
-        }
-        __syncwarp();
-        return CMD_SCAN;
-    }
-    if (lane == 0) C->cmd = CMD_DONE;
-    __syncwarp();
-    return CMD_DONE;
-}
-
-// ------------------------------------------------------------ group phases
-__device__ __forceinline__ void count_one(int32_t *hist, bool smem_hist, uint32_t w) {
-    if ((w >> 24) == 1u) atomicAdd(&hist[w & XOR_MASK], 1);
-    (void)smem_hist;
-}
-
-// SCAN(k): n_k(D) for all D in one pass over the packed state (4 B / task).
-__device__ void scan_phase(const Inst &I, int k, int32_t *hist, bool smem_hist, int cta, int G) {
-    const uint4 *sv = reinterpret_cast<const uint4 *>(I.s + (size_t)k * I.m_pad);
-    const int64_t nv = I.m_pad >> 2;
-    const int64_t stride = (int64_t)G * blockDim.x;
-    int64_t v = (int64_t)cta * blockDim.x + threadIdx.x;
-    for (; v + stride < nv; v += 2 * stride) {
-        uint4 a = __ldcg(&sv[v]);
-        uint4 c = __ldcg(&sv[v + stride]);
-        count_one(hist, smem_hist, a.x);
-        count_one(hist, smem_hist, a.y);
-        count_one(hist, smem_hist, a.z);
-        count_one(hist, smem_hist, a.w);
-        count_one(hist, smem_hist, c.x);
-        count_one(hist, smem_hist, c.y);
-        count_one(hist, smem_hist, c.z);
-        count_one(hist, smem_hist, c.w);
-    }
-    if (v < nv) {
-        uint4 a = __ldcg(&sv[v]);
-        count_one(hist, smem_hist, a.x);
-        count_one(hist, smem_hist, a.y);
-        count_one(hist, smem_hist, a.z);
-        count_one(hist, smem_hist, a.w);
-    }
-}
-
-// FSCAN(k): n2_k(D) (tasks with exactly two missing inputs, both credited) and
-// the lowest unallocated task id.
-__device__ void fscan_phase(const Inst &I, int k, int32_t *hist, int cta, int G, int *sh_min) {
-    const uint32_t *sk = I.s + (size_t)k * I.m_pad;
-    const int32_t *rp = I.res_pos + (size_t)k * I.n;
-    const bool fb2 = (I.flags & DTS_F_FALLBACK2) != 0;
-    const int64_t stride = (int64_t)G * blockDim.x;
-    int mn = INT_MAX;
-    for (int64_t T = (int64_t)cta * blockDim.x + threadIdx.x; T < I.m; T += stride) {
-        uint32_t w = __ldcg(&sk[T]);
-        if (w & ALLOC_BIT) continue;
-        mn = min(mn, (int)T);
-        if (fb2 && (w >> 24) == 2u) {
-            int64_t b = __ldg(&I.tptr[T]), e = __ldg(&I.tptr[T + 1]);
-            for (int64_t i = b; i < e; i++) {
-                int32_t D = __ldg(&I.tdat[i]);
-                if (__ldcg(&rp[D]) < 0) atomicAdd(&hist[D], 1);
-            }
-        }
-    }
-    mn = warp_min_i32(mn);
-    if ((threadIdx.x & 31) == 0 && mn != INT_MAX) atomicMin(sh_min, mn);
-}
-
-// ARGMAX over this CTA's slice of D of (score, u, ~id); resets the histogram.
-__device__ void argmax_phase(const Inst &I, int32_t *hist, bool smem_hist, int cta, int G,
-                             unsigned long long *sh_key) {
-    const int64_t n = I.n;
-    const int64_t lo = n * cta / G, hi = n * (cta + 1) / G;
+// Block argmax over D of (score[D], u[D], ~D) with score[D] > 0 (Alg. 5
+// l.6-9).  A datum with a positive score is never resident (its tasks miss it).
+__device__ int32_t score_argmax(const Inst &I, const View &V, Lead &L, const int32_t *score) {
     const unsigned ib = (unsigned)I.id_bits, ub = (unsigned)I.u_bits;
     const unsigned long long idmask = (1ull << ib) - 1ull;
     unsigned long long best = 0ull;
-    for (int64_t D = lo + threadIdx.x; D < hi; D += blockDim.x) {
-        int32_t h = smem_hist ? hist[D] : __ldcg(&hist[D]);
-        if (h > 0) {
-            hist[D] = 0;
-            unsigned long long uu = (unsigned long long)(uint32_t)__ldcg(&I.u[D]);
-            unsigned long long key = ((unsigned long long)(uint32_t)h << (ub + ib)) | (uu << ib) |
-                                     (idmask - (unsigned long long)D);
+    for (int D = threadIdx.x; D < I.n; D += blockDim.x) {
+        const int32_t sc = score[D];
+        if (sc > 0) {
+            const unsigned long long key = ((unsigned long long)(uint32_t)sc << (ub + ib)) |
+                                           ((unsigned long long)(uint32_t)V.u[D] << ib) |
+                                           (idmask - (unsigned long long)D);
             best = key > best ? key : best;
         }
     }
-    best = warp_max_u64(best);
-    if ((threadIdx.x & 31) == 0 && best) atomicMax(sh_key, best);
+    best = block_max_u64(L, best);
+    if (best == 0ull) return -1;
+    return (int32_t)(idmask - (best & idmask));
+}
+
+// Alg. 5 l.10: plannedTasks_k <- unallocated tasks of Dopt's segment with one
+// missing input (= Dopt), ascending id (ordered block compaction).  Block-wide.
+__device__ void plan(const Inst &I, const View &V, Lead &L, int k, int32_t Dopt) {
+    const int64_t b = __ldg(&I.dptr[Dopt]), e = __ldg(&I.dptr[Dopt + 1]);
+    const uint32_t *sk = V.s + (size_t)k * I.m_pad;
+    int4 *pl = V.plan + (size_t)k * I.plan_cap;
+    int64_t *pt = V.plan_tau ? V.plan_tau + (size_t)k * I.plan_cap : nullptr;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    int base_out = 0;
+    for (int64_t base = b; base < e; base += blockDim.x) {
+        const int64_t i = base + threadIdx.x;
+        int32_t T = -1;
+        bool sel = false;
+        int4 ed = make_int4(-1, -1, -1, 0);
+        if (i < e) {
+            ed = __ldg(&I.dedge[i]);
+            T = ed.x;
+            sel = (sk[T] >> 24) == 1u;
+        }
+        const unsigned msk = __ballot_sync(FULL, sel);
+        if (lane == 0) L.wcnt[w] = __popc(msk);
+        __syncthreads();
+        int off = base_out, tot = 0;
+        for (int j = 0; j < nw; j++) {
+            const int c = L.wcnt[j];
+            if (j < w) off += c;
+            tot += c;
+        }
+        if (sel) {
+            const int pos = off + __popc(msk & lt);
+            const Row r = ed.w > 3 ? Row{-1, -1, -1, ed.w} : Row{Dopt, ed.y, ed.z, ed.w};
+            pl[pos] = make_int4(T, Dopt, ed.y, ed.w > 3 ? ROW_LONG : ed.z);
+            if (pt) pt[pos] = tau_of(I, T);
+            pool_move(I, V, T, r, -1, k);
+        }
+        base_out += tot;
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+        L.plan_head[k] = 0;
+        L.plan_end[k] = base_out;
+        L.plan_live[k] = base_out;
+        L.n_avail -= base_out;
+        L.alg_bytes += 8ull * (uint64_t)(e - b) + (uint64_t)base_out * (8ull * I.K + 48ull);
+    }
+    __syncthreads();
+}
+
+// 3inputs: the lowest-id unallocated task of D2's segment with two missing inputs.
+__device__ int32_t first_cnt2(const Inst &I, const View &V, Lead &L, int k, int32_t D2) {
+    const int64_t b = __ldg(&I.dptr[D2]), e = __ldg(&I.dptr[D2 + 1]);
+    const uint32_t *sk = V.s + (size_t)k * I.m_pad;
+    for (int64_t base = b; base < e; base += blockDim.x) {
+        const int64_t i = base + threadIdx.x;
+        unsigned long long c = ~0ull;
+        if (i < e) {
+            const int32_t T = __ldg(&I.dedge[i]).x;
+            if ((sk[T] >> 24) == 2u) c = (unsigned long long)T;
+        }
+        c = block_min_u64(L, c);
+        if (c != ~0ull) return (int32_t)c;
+    }
+    return -1;
+}
+
+// Alg. 5 l.13 (R5): the lowest-id unallocated task, scanning up from avail_lo.
+__device__ int32_t first_avail(const Inst &I, const View &V, Lead &L) {
+    for (int64_t base = L.avail_lo; base < I.m; base += blockDim.x) {
+        const int64_t T = base + threadIdx.x;
+        unsigned long long c = ~0ull;
+        if (T < I.m && !(V.s[T] & ALLOC_BIT)) c = (unsigned long long)T;
+        c = block_min_u64(L, c);
+        if (c != ~0ull) return (int32_t)c;
+    }
+    return -1;
+}
+
+// DTS_F_VERIFY (P9): recompute n_k(D), n2_k(D), u(D) and cnt_k(T) from their
+// definitions -- the full non-incremental pass of Alg. 5 l.4-5 -- and count
+// mismatches against the incremental state.
+__device__ void verify_scores(const Inst &I, const View &V, Lead &L, int k) {
+    int32_t *vh = I.vhist, *vh2 = I.vhist + I.n, *vu = I.vhist + 2 * I.n;
+    for (int D = threadIdx.x; D < 3 * I.n; D += blockDim.x) vh[D] = 0;
+    __syncthreads();
+    const uint32_t *sk = V.s + (size_t)k * I.m_pad;
+    int bad = 0;
+    for (int T = threadIdx.x; T < I.m; T += blockDim.x) {
+        const uint32_t w = sk[T];
+        const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+        int c = 0;
+        uint32_t x = 0;
+        for (int64_t i = rb; i < re; i++) {
+            const int32_t D = __ldg(&I.tdat[i]);
+            if (!resident(I, V, k, D)) c++, x ^= (uint32_t)D;
+        }
+        bad += (c != (int)((w >> 24) & 0x7fu)) || (x != (w & XOR_MASK));
+        if (w & ALLOC_BIT) continue;
+        for (int64_t i = rb; i < re; i++) {
+            const int32_t D = __ldg(&I.tdat[i]);
+            atomicAdd(&vu[D], 1);
+            if (c == 2 && !resident(I, V, k, D)) atomicAdd(&vh2[D], 1);
+        }
+        if (c == 1) atomicAdd(&vh[x], 1);
+    }
+    __syncthreads();
+    for (int D = threadIdx.x; D < I.n; D += blockDim.x)
+        bad += (__ldcg(&vh[D]) != V.h[(size_t)k * I.n + D]) +
+               (__ldcg(&vh2[D]) != V.h2[(size_t)k * I.n + D]) + (__ldcg(&vu[D]) != V.u[D]);
+    bad = block_sum(L, bad);
+    if (threadIdx.x == 0) L.n_verr += bad;
+    __syncthreads();
+}
+
+// a8: sigma(k, .) for every k -- stable partition of the service sequence by GPU.
+__device__ void assemble(const Inst &I, int64_t ns) {
+    __shared__ unsigned long long off[MAX_K];
+    __shared__ int tot[MAX_K];
+    __shared__ int wk[32][MAX_K];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    for (int k = threadIdx.x; k < MAX_K; k += blockDim.x) off[k] = 0;
+    __syncthreads();
+    for (int64_t i = threadIdx.x; i < ns; i += blockDim.x) atomicAdd(&off[I.serve_gpu[i]], 1ull);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned long long run = 0;
+        for (int k = 0; k < I.K; k++) {
+            const unsigned long long c = off[k];
+            I.gpu_task_ptr[k] = (int64_t)run;
+            off[k] = run;
+            run += c;
+        }
+        I.gpu_task_ptr[I.K] = (int64_t)run;
+    }
+    __syncthreads();
+    for (int64_t base = 0; base < ns; base += blockDim.x) {
+        for (int j = threadIdx.x; j < nw * MAX_K; j += blockDim.x) wk[j / MAX_K][j % MAX_K] = 0;
+        __syncthreads();
+        const int64_t i = base + threadIdx.x;
+        const int k = i < ns ? I.serve_gpu[i] : -1;
+        const unsigned peers = __match_any_sync(FULL, k);
+        if (k >= 0 && lane == __ffs(peers) - 1) wk[w][k] = __popc(peers);
+        __syncthreads();
+        for (int kk = threadIdx.x; kk < I.K; kk += blockDim.x) {  // exclusive prefix over warps
+            int run = 0;
+            for (int ww = 0; ww < nw; ww++) {
+                const int c = wk[ww][kk];
+                wk[ww][kk] = run;
+                run += c;
+            }
+            tot[kk] = run;
+        }
+        __syncthreads();
+        if (k >= 0) I.gpu_task_ids[off[k] + wk[w][k] + __popc(peers & lt)] = I.serve_task[i];
+        __syncthreads();
+        for (int kk = threadIdx.x; kk < I.K; kk += blockDim.x) off[kk] += tot[kk];
+        __syncthreads();
+    }
 }
 
 }  // namespace
 
-// One group of gridDim.x / n_groups ... : when G > 1 the grid IS the group
-// (n_inst == 1, cooperative launch); when G == 1 each CTA pulls instances from
-// a device-side work counter (batched sweep).
-__global__ void __launch_bounds__(1024, 1)
-    dts_loop_kernel(const Inst *__restrict__ insts, int n_inst, int G, int *work_counter,
-                    int smem_hist_cap) {
-    extern __shared__ int32_t dyn_smem[];
-    __shared__ LState L;
+// One CTA per instance; instances pulled from *work_counter.
+__global__ void __launch_bounds__(512, 1)
+    dts_cta_kernel(const Inst *__restrict__ insts, int n_inst, int *work_counter) {
+    extern __shared__ __align__(16) unsigned char dsm[];
+    __shared__ Lead L;
+    __shared__ Inst SI;  // this CTA's instance descriptor, read at smem latency
     __shared__ int sh_inst;
-    __shared__ unsigned long long sh_key;
-    __shared__ int sh_min;
-    __shared__ int sh_cmd, sh_k;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int cta = (G > 1) ? (int)blockIdx.x : 0;
+    const int tid = threadIdx.x;
 
     while (true) {
-        if (threadIdx.x == 0) sh_inst = (G > 1) ? (blockIdx.x == 0 ? 0 : 0) : atomicAdd(work_counter, 1);
+        if (tid == 0) sh_inst = atomicAdd(work_counter, 1);
         __syncthreads();
         const int ii = sh_inst;
-        if (G == 1 && ii >= n_inst) break;
-        const Inst I = insts[ii];
-        Ctrl *C = I.ctrl;
-        const bool smem_hist = (G == 1) && (I.n <= smem_hist_cap);
-        int32_t *hist = smem_hist ? dyn_smem : I.hist;
-        if (smem_hist)
-            for (int D = threadIdx.x; D < I.n; D += blockDim.x) hist[D] = 0;
-        const bool leader_cta = (cta == 0);
-        if (leader_cta && threadIdx.x == 0) {
+        if (ii >= n_inst) break;
+        if (tid == 0) SI = insts[ii];
+        __syncthreads();
+        const Inst &I = SI;
+        View V;
+        V.s = I.so_s >= 0 ? (uint32_t *)(dsm + I.so_s) : I.s;
+        V.u = I.so_u >= 0 ? (int32_t *)(dsm + I.so_u) : I.u;
+        V.h = I.so_h >= 0 ? (int32_t *)(dsm + I.so_h) : I.h;
+        V.h2 = I.so_h2 >= 0 ? (int32_t *)(dsm + I.so_h2) : I.h2;
+        V.np = I.so_np >= 0 ? (int32_t *)(dsm + I.so_np) : I.np;
+        V.resb = I.so_resb >= 0 ? (uint32_t *)(dsm + I.so_resb) : I.resb;
+        V.res_list = I.so_res_list >= 0 ? (int32_t *)(dsm + I.so_res_list) : I.res_list;
+        V.plan = I.so_plan >= 0 ? (int4 *)(dsm + I.so_plan) : I.plan;
+        V.plan_tau = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
+
+        // ---- CTA-local copies of the initial state (global homes were
+        //      initialised by dts_init_kernel)
+        const int n = I.n, K = I.K;
+        if (I.so_s >= 0) {
+            const uint4 *src = reinterpret_cast<const uint4 *>(I.s);
+            uint4 *dst = reinterpret_cast<uint4 *>(V.s);
+            for (int i = tid; i < (K * I.m_pad) / 4; i += blockDim.x) dst[i] = __ldcg(&src[i]);
+        }
+        if (I.so_u >= 0)
+            for (int D = tid; D < n; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
+        if (I.so_h >= 0)
+            for (int i = tid; i < K * n; i += blockDim.x) V.h[i] = __ldcg(&I.h[i]);
+        if (I.so_h2 >= 0)
+            for (int i = tid; i < K * n; i += blockDim.x) V.h2[i] = __ldcg(&I.h2[i]);
+        if (I.so_np >= 0)
+            for (int i = tid; i < K * n; i += blockDim.x) V.np[i] = 0;
+        if (I.so_resb >= 0)
+            for (int i = tid; i < K * I.nw; i += blockDim.x) V.resb[i] = 0u;
+        if (tid == 0) {
             for (int k = 0; k < MAX_K; k++) {
                 L.req[k] = 0;
                 L.gpu_free[k] = 0;
                 L.used[k] = 0;
                 L.plan_head[k] = L.plan_end[k] = L.plan_live[k] = 0;
                 L.res_cnt[k] = 0;
-                L.last_task[k] = -1;
                 L.idle[k] = 0;
             }
             L.bus_free = 0;
             L.n_events = L.n_served = L.n_loads = L.n_evictions = L.n_scans = L.n_fb2 = L.n_fbf =
-                L.n_belady = L.n_idle = 0;
-            L.bytes_loaded = 0;
+                L.n_belady = L.n_idle = L.n_verr = 0;
+            L.bytes_loaded = L.alg_bytes = L.scan_alg_bytes = 0;
             L.makespan = 0;
-            L.alg_bytes = L.scan_alg_bytes = 0;
             L.n_avail = I.m;
-            L.pending = CMD_NONE;
+            L.avail_lo = 0;
             L.error = 0;
             L.row_len = 0;
+            for (int i = 0; i < 8; i++) L.prof[i] = 0;
         }
         __syncthreads();
+
+        // ---- the decision loop
         while (true) {
-            if (leader_cta) {
-                if (warp == 0) {
-                    int cmd = leader_run(I, L, lane);
-                    if (lane == 0) {
-                        sh_cmd = cmd;
-                        sh_k = L.pend_k;
+            PROF_T0(p_pop);
+            if (tid == 0) {
+                // Pops need no other thread: serve them here until a request
+                // finds plannedTasks_k empty (Alg. 5 l.3) or the run ends.
+                int cmd = CMD_DONE;
+                if (!L.error) {
+                    const int r = I.K <= 4 ? pop_run<4>(I, V, L)
+                                           : (I.K <= 8 ? pop_run<8>(I, V, L) : pop_run_smem(I, V, L));
+                    if (r >= 0) cmd = CMD_SCAN;
+                }
+                L.cmd = cmd;
+            }
+            PROF_ADD(L, P_POP, p_pop);
+            __syncthreads();
+            if (L.cmd == CMD_DONE) break;
+            const int k = L.k;
+            const int64_t t = L.t;
+            reset_plan(I, V, L, k);
+            if (I.flags & DTS_F_VERIFY) verify_scores(I, V, L, k);
+            // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
+            int32_t T = -1;
+            PROF_T0(p_am);
+            const int32_t Dopt = score_argmax(I, V, L, V.h + (size_t)k * n);
+            PROF_ADD(L, P_ARGMAX, p_am);
+            PROF_T0(p_pl);
+            if (tid == 0) {
+                L.scan_alg_bytes += 8ull * (uint64_t)n;
+                L.alg_bytes += 8ull * (uint64_t)n;
+            }
+            if (Dopt >= 0) {
+                plan(I, V, L, k, Dopt);
+                if (tid == 0) {
+                    int64_t tau;
+                    L.T = pop_planned(I, V, L, k, &tau);
+                    L.n_scans++;
+                }
+                __syncthreads();
+                T = L.T;
+                PROF_ADD(L, P_PLAN, p_pl);
+            } else {
+                if (I.flags & DTS_F_FALLBACK2) {
+                    const int32_t D2 = score_argmax(I, V, L, V.h2 + (size_t)k * n);
+                    if (D2 >= 0) {
+                        T = first_cnt2(I, V, L, k, D2);
+                        if (tid == 0) L.n_fb2++;
                     }
                 }
+                if (T < 0 && L.n_avail > 0) {
+                    T = first_avail(I, V, L);
+                    if (tid == 0) {
+                        L.n_fbf++;
+                        L.avail_lo = T;
+                    }
+                }
+                if (T >= 0) {
+                    if (tid == 0) {
+                        L.row_len = -1;
+                        pool_move(I, V, T, row_of_task(I, T), -1, -1);
+                        L.n_avail--;
+                        L.n_scans++;
+                    }
+                } else if (tid == 0) {
+                    L.idle[k] = 1;
+                    L.n_idle++;
+                }
+                __syncthreads();
+                PROF_ADD(L, P_OTHER, p_pl);
+                if (T < 0) continue;
             }
-            group_sync(C, G);
-            int cmd, k;
-            if (leader_cta) {
-                cmd = sh_cmd;
-                k = sh_k;
-            } else {
-                cmd = *(volatile int *)&C->cmd;
-                k = *(volatile int *)&C->cmd_k;
-            }
-            if (cmd == CMD_DONE) break;
-            if (threadIdx.x == 0) {
-                sh_key = 0ull;
-                sh_min = INT_MAX;
+            // serve T with its loads (block-wide); D(T) from the CSR unless cached
+            const bool need_row = L.row_len < 0;
+            __syncthreads();
+            if (need_row && tid < 32) {
+                const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+                for (int r = tid; r < (int)(re - rb); r += 32) L.row[r] = __ldg(&I.tdat[rb + r]);
+                if (tid == 0) L.row_len = (int)(re - rb);
             }
             __syncthreads();
-            if (cmd == CMD_SCAN)
-                scan_phase(I, k, hist, smem_hist, cta, G);
-            else
-                fscan_phase(I, k, hist, cta, G, &sh_min);
-            __syncthreads();
-            if (threadIdx.x == 0 && sh_min != INT_MAX) atomicMin(&C->min_avail, sh_min);
-            group_sync(C, G);
-            argmax_phase(I, hist, smem_hist, cta, G, &sh_key);
-            __syncthreads();
-            if (threadIdx.x == 0 && sh_key) atomicMax(&C->best_key, sh_key);
-            group_sync(C, G);
+            PROF_T0(p_ld);
+            serve_loads(I, V, L, k, T, t);
+            PROF_ADD(L, P_LOADS, p_ld);
+            if (L.error) break;
         }
-        // write back the scalars
-        if (leader_cta && threadIdx.x == 0) {
+        __syncthreads();
+
+        // ---- a8: per-GPU orders, scalars
+        assemble(I, L.n_served);
+        if (tid == 0) {
             Out *o = I.out;
             o->n_events = L.n_events;
             o->n_served = L.n_served;
@@ -690,31 +1054,32 @@ __global__ void __launch_bounds__(1024, 1)
             o->n_fallback_first = L.n_fbf;
             o->n_belady = L.n_belady;
             o->n_idle = L.n_idle;
+            o->n_verify_err = L.n_verr;
             o->bytes_loaded = L.bytes_loaded;
             o->makespan = L.makespan;
             o->alg_bytes = L.alg_bytes;
             o->scan_alg_bytes = L.scan_alg_bytes;
             o->error = L.error;
+            for (int i = 0; i < 8; i++) o->prof[i] = L.prof[i];
         }
-        if (G > 1) break;
         __syncthreads();
     }
 }
 
 // ---------------------------------------------------------------- init (a2)
-// s_k(T) = (|D(T)| << 24) | XOR D(T) for every k (nothing resident), pad words
-// allocated; u(D) = deg(D); empty histograms / plans / residency; delta(D).
-__global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint64_t bw,
-                                int64_t *const *__restrict__ deltas) {
+// Global homes: s_k(T) = (|D(T)| << 24) | XOR D(T) for every k (nothing
+// resident), pad words allocated; u(D) = deg(D); h_k(D) / h2_k(D) = the tasks
+// of D's segment with 1 / 2 inputs (all missing); np = 0; delta(D); times -1.
+__global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint64_t bw) {
     for (int ii = 0; ii < n_inst; ii++) {
         const Inst I = insts[ii];
-        int64_t *delta = deltas[ii];
+        int64_t *delta = const_cast<int64_t *>(I.delta);
         const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
         const int64_t str = (int64_t)gridDim.x * blockDim.x;
         for (int64_t T = tid; T < I.m_pad; T += str) {
             uint32_t w = ALLOC_BIT;
             if (T < I.m) {
-                int64_t b = I.tptr[T], e = I.tptr[T + 1];
+                const int64_t b = I.tptr[T], e = I.tptr[T + 1];
                 uint32_t x = 0;
                 for (int64_t i = b; i < e; i++) x ^= (uint32_t)I.tdat[i];
                 w = ((uint32_t)(e - b) << 24) | x;
@@ -724,119 +1089,59 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
             for (int k = 0; k < I.K; k++) I.s[(size_t)k * I.m_pad + T] = w;
         }
         for (int64_t D = tid; D < I.n; D += str) {
-            I.u[D] = (int32_t)(I.dptr[D + 1] - I.dptr[D]);
-            I.hist[D] = 0;
+            const int64_t b = I.dptr[D], e = I.dptr[D + 1];
+            int32_t c1 = 0, c2 = 0;
+            for (int64_t i = b; i < e; i++) {
+                const int32_t T = I.ddat[i];
+                const int64_t len = I.tptr[T + 1] - I.tptr[T];
+                c1 += (len == 1);
+                c2 += (len == 2);
+            }
+            I.u[D] = (int32_t)(e - b);
             unsigned __int128 num = (unsigned __int128)I.size[D] * 1000000000ull + (bw - 1);
             delta[D] = (int64_t)(num / bw);
             for (int k = 0; k < I.K; k++) {
+                I.h[(size_t)k * I.n + D] = c1;
+                I.h2[(size_t)k * I.n + D] = c2;
                 I.np[(size_t)k * I.n + D] = 0;
-                I.res_pos[(size_t)k * I.n + D] = -1;
             }
         }
-        if (tid == 0) {
-            Ctrl *c = I.ctrl;
-            c->bar_count = 0;
-            c->bar_gen = 0;
-            c->cmd = CMD_NONE;
-            c->cmd_k = 0;
-            c->best_key = 0ull;
-            c->min_avail = INT_MAX;
-            c->error = 0;
-        }
-    }
-}
-
-// ---------------------------------------------------------- assembly (a8)
-// sigma(k, .) for every k: stable partition of the service sequence by GPU.
-__global__ void __launch_bounds__(1024) dts_assemble_kernel(const Inst *__restrict__ insts) {
-    const Inst I = insts[blockIdx.x];
-    __shared__ unsigned long long cnt[MAX_K];
-    __shared__ long long off[MAX_K];
-    __shared__ int wcount[32][MAX_K];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    const unsigned lt = (1u << lane) - 1u;
-    const int64_t ns = I.out->n_served;
-    for (int k = threadIdx.x; k < MAX_K; k += blockDim.x) cnt[k] = 0;
-    __syncthreads();
-    for (int64_t i = threadIdx.x; i < ns; i += blockDim.x) atomicAdd(&cnt[I.serve_gpu[i]], 1ull);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        long long run = 0;
-        for (int k = 0; k < I.K; k++) {
-            I.gpu_task_ptr[k] = run;
-            off[k] = run;
-            run += cnt[k];
-        }
-        I.gpu_task_ptr[I.K] = run;
-    }
-    __syncthreads();
-    for (int64_t base = 0; base < ns; base += blockDim.x) {
-        for (int j = threadIdx.x; j < nw * MAX_K; j += blockDim.x) wcount[j / MAX_K][j % MAX_K] = 0;
-        __syncthreads();
-        const int64_t i = base + threadIdx.x;
-        const int k = i < ns ? I.serve_gpu[i] : -1;
-        const unsigned peers = __match_any_sync(FULL, k);
-        if (k >= 0 && lane == __ffs(peers) - 1) wcount[w][k] = __popc(peers);
-        __syncthreads();
-        if (threadIdx.x < I.K) {
-            long long run = off[threadIdx.x];
-            for (int ww = 0; ww < nw; ww++) {
-                int t = wcount[ww][threadIdx.x];
-                wcount[ww][threadIdx.x] = (int)(run - off[threadIdx.x]);
-                run += t;
-            }
-            cnt[threadIdx.x] = run;  // new running offset, published after the scatter
-        }
-        __syncthreads();
-        if (k >= 0) I.gpu_task_ids[off[k] + wcount[w][k] + __popc(peers & lt)] = I.serve_task[i];
-        __syncthreads();
-        if (threadIdx.x < I.K) off[threadIdx.x] = cnt[threadIdx.x];
-        __syncthreads();
+        for (int64_t i = tid; i < (int64_t)I.K * I.nw; i += str) I.resb[i] = 0u;
     }
 }
 
 // ---------------------------------------------------------------- launchers
-cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t *const *d_deltas,
-                        int64_t work, cudaStream_t st) {
+cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t work, cudaStream_t st) {
     int64_t blocks = (work + 255) / 256;
     if (blocks < 1) blocks = 1;
     if (blocks > 148 * 8) blocks = 148 * 8;
-    dts_init_kernel<<<(unsigned)blocks, 256, 0, st>>>(d_insts, n_inst, bw, d_deltas);
+    dts_init_kernel<<<(unsigned)blocks, 256, 0, st>>>(d_insts, n_inst, bw);
     count_launch();
     return cudaGetLastError();
 }
 
-cudaError_t launch_loop(const Inst *d_insts, int n_inst, int G, int block, int grid,
-                        int *work_counter, int smem_hist_cap, cudaStream_t st) {
-    size_t dyn = (G == 1) ? sizeof(int32_t) * (size_t)smem_hist_cap : 0;
-    cudaError_t e = cudaFuncSetAttribute(dts_loop_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)dyn);
+cudaError_t launch_loop(const Inst *d_insts, int n_inst, int block, int grid, int *work_counter,
+                        int smem_bytes, cudaStream_t st) {
+    cudaError_t e = cudaFuncSetAttribute(dts_cta_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         smem_bytes);
     if (e != cudaSuccess) return e;
-    if (G > 1) {
-        void *args[] = {(void *)&d_insts, (void *)&n_inst, (void *)&G, (void *)&work_counter,
-                        (void *)&smem_hist_cap};
-        count_launch();
-        return cudaLaunchCooperativeKernel((const void *)dts_loop_kernel, dim3(G), dim3(block), args,
-                                           dyn, st);
-    }
-    dts_loop_kernel<<<grid, block, dyn, st>>>(d_insts, n_inst, 1, work_counter, smem_hist_cap);
+    dts_cta_kernel<<<grid, block, smem_bytes, st>>>(d_insts, n_inst, work_counter);
     count_launch();
     return cudaGetLastError();
 }
 
-cudaError_t launch_assemble(const Inst *d_insts, int n_inst, cudaStream_t st) {
-    dts_assemble_kernel<<<n_inst, 1024, 0, st>>>(d_insts);
-    count_launch();
-    return cudaGetLastError();
-}
-
-int loop_max_blocks_per_sm(int block, int smem_hist_cap) {
+int loop_max_blocks_per_sm(int block, int smem_bytes) {
     int nb = 0;
-    size_t dyn = sizeof(int32_t) * (size_t)smem_hist_cap;
-    cudaFuncSetAttribute(dts_loop_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, dts_loop_kernel, block, dyn) != cudaSuccess)
+    cudaFuncSetAttribute(dts_cta_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, dts_cta_kernel, block, smem_bytes) != cudaSuccess)
         return 0;
     return nb;
+}
+
+int loop_static_smem() {
+    cudaFuncAttributes a;
+    if (cudaFuncGetAttributes(&a, dts_cta_kernel) != cudaSuccess) return -1;
+    return (int)a.sharedSizeBytes;
 }
 
 }  // namespace dts

@@ -7,10 +7,10 @@
 #include "dts_internal.cuh"
 
 namespace dts {
-cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t *const *d_deltas,
-                        int64_t work, cudaStream_t st);
-cudaError_t launch_loop(const Inst *d_insts, int n_inst, int G, int block, int grid,
-                        int *work_counter, int smem_hist_cap, cudaStream_t st);
-cudaError_t launch_assemble(const Inst *d_insts, int n_inst, cudaStream_t st);
-int loop_max_blocks_per_sm(int block, int smem_hist_cap);
+cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t work, cudaStream_t st);
+// One CTA per instance (grid CTAs pull instances from *work_counter).
+cudaError_t launch_loop(const Inst *d_insts, int n_inst, int block, int grid, int *work_counter,
+                        int smem_bytes, cudaStream_t st);
+int loop_max_blocks_per_sm(int block, int smem_bytes);
+int loop_static_smem();
 }  // namespace dts

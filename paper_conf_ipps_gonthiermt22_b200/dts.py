@@ -29,6 +29,7 @@ DTS_E_STATE = -5
 DTS_E_UNSUPPORTED = -6
 DTS_POLICY_DARTS_LUF = 1
 DTS_F_FALLBACK2 = 1
+DTS_F_VERIFY = 2
 
 EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data", "<i4"),
                         ("task", "<i4"), ("op", "u1"), ("pad", "u1", (3,))])
@@ -46,7 +47,8 @@ class DtsError(RuntimeError):
 
 class dts_run_opts(C.Structure):
     _fields_ = [("flags", C.c_uint32), ("lookahead_W", C.c_uint32),
-                ("bus_bytes_per_s", C.c_uint64), ("device", C.c_int32), ("n_ctas", C.c_int32),
+                ("bus_bytes_per_s", C.c_uint64), ("device", C.c_int32),
+                ("block_threads", C.c_int32), ("smem_budget", C.c_int32), ("pad", C.c_int32),
                 ("max_served", C.c_int64), ("cuda_stream", C.c_void_p)]
 
 
@@ -60,8 +62,10 @@ class dts_result_view(C.Structure):
                 ("makespan_ns", C.c_int64), ("makespan_s", C.c_double),
                 ("n_served", C.c_int64), ("n_scans", C.c_int64), ("n_fallback2", C.c_int64),
                 ("n_fallback_first", C.c_int64), ("n_belady", C.c_int64),
-                ("n_idle_requests", C.c_int64), ("alg_bytes", C.c_uint64),
-                ("scan_alg_bytes", C.c_uint64), ("loop_ms", C.c_float), ("total_ms", C.c_float)]
+                ("n_idle_requests", C.c_int64), ("n_verify_err", C.c_int64),
+                ("alg_bytes", C.c_uint64),
+                ("scan_alg_bytes", C.c_uint64), ("loop_ms", C.c_float), ("total_ms", C.c_float),
+                ("prof_cycles", C.c_int64 * 8)]
 
 
 _lib = None
@@ -185,10 +189,12 @@ class Result:
     n_fallback_first: int
     n_belady: int
     n_idle_requests: int
+    n_verify_err: int
     alg_bytes: int
     scan_alg_bytes: int
     loop_ms: float
     total_ms: float
+    prof_cycles: tuple = ()
 
     def orders(self):
         p = self.gpu_task_ptr
@@ -212,8 +218,9 @@ def dts_result(inst: Instance) -> Result:
                   _arr(v.events, v.n_events, EVENT_DTYPE), int(v.bytes_loaded), int(v.n_loads),
                   int(v.n_evictions), int(v.makespan_ns), float(v.makespan_s), ns, int(v.n_scans),
                   int(v.n_fallback2), int(v.n_fallback_first), int(v.n_belady),
-                  int(v.n_idle_requests), int(v.alg_bytes), int(v.scan_alg_bytes),
-                  float(v.loop_ms), float(v.total_ms))
+                  int(v.n_idle_requests), int(v.n_verify_err), int(v.alg_bytes),
+                  int(v.scan_alg_bytes),
+                  float(v.loop_ms), float(v.total_ms), tuple(int(x) for x in v.prof_cycles))
 
 
 def dts_kernel_launches() -> int:
@@ -225,13 +232,15 @@ def dts_version() -> int:
 
 
 def schedule(inst, *, W: int = 0, flags: int = DTS_F_FALLBACK2, bus_bps: int = 12_000_000_000,
-             device: int = 0, n_ctas: int = 0, max_served: int = -1, stream: int = 0) -> Result:
+             device: int = 0, block_threads: int = 0, smem_budget: int = 0,
+             max_served: int = -1, stream: int = 0) -> Result:
     """One call: create the instance from host arrays (a ``gen.Instance``-like
     object), run DARTS+LUF on the GPU, return the host result."""
     h = dts_instance_create(inst.task_ptr, inst.task_data, inst.data_size, inst.task_ns,
                             inst.default_task_ns, inst.mem_capacity, inst.K)
     o = dts_run_opts_default(flags=flags, lookahead_W=W, bus_bytes_per_s=bus_bps, device=device,
-                             n_ctas=n_ctas, max_served=max_served, cuda_stream=stream or None)
+                             block_threads=block_threads, smem_budget=smem_budget,
+                             max_served=max_served, cuda_stream=stream or None)
     dts_run(h, DTS_POLICY_DARTS_LUF, o)
     return dts_result(h)
 
@@ -243,11 +252,13 @@ def create(inst) -> Instance:
 
 
 def schedule_batch(insts, *, W: int = 0, flags: int = DTS_F_FALLBACK2,
-                   bus_bps: int = 12_000_000_000, device: int = 0, stream: int = 0):
+                   bus_bps: int = 12_000_000_000, device: int = 0, block_threads: int = 0,
+                   smem_budget: int = 0, stream: int = 0):
     """Run many independent instances in ONE batched launch (dts_sweep_run,
     one CTA per instance) and return their host results."""
     hs = [create(i) for i in insts]
     o = dts_run_opts_default(flags=flags, lookahead_W=W, bus_bytes_per_s=bus_bps, device=device,
-                             n_ctas=0, max_served=-1, cuda_stream=stream or None)
+                             block_threads=block_threads, smem_budget=smem_budget,
+                             max_served=-1, cuda_stream=stream or None)
     dts_sweep_run(hs, DTS_POLICY_DARTS_LUF, o)
     return [dts_result(h) for h in hs]

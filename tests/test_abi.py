@@ -31,7 +31,7 @@ def test_library_exports_every_declared_symbol():
 
 def test_struct_layouts():
     assert dts.EVENT_DTYPE.itemsize == 32
-    assert C.sizeof(B.dts_run_opts) == 40
+    assert C.sizeof(B.dts_run_opts) == 48
     assert dts.dts_version() >> 16 == 1
 
 

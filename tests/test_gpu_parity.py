@@ -32,8 +32,9 @@ def _unit(inst):
                       default_task_ns=1, task_ns=None)
 
 
-def _both(inst, bus=oracle.DEFAULT_BUS_BPS, n_ctas=0, flags=1, max_served=-1):
-    g = dts.schedule(inst, bus_bps=bus, n_ctas=n_ctas, flags=flags, max_served=max_served)
+def _both(inst, bus=oracle.DEFAULT_BUS_BPS, block=0, smem=0, flags=1, max_served=-1):
+    g = dts.schedule(inst, bus_bps=bus, block_threads=block, smem_budget=smem, flags=flags,
+                     max_served=max_served)
     o = oracle.run(inst, bus_bps=bus, flags=flags, max_served=max_served)
     return g, o
 
@@ -81,11 +82,13 @@ def _shapes():
             gen.matmul2d(30, M=12, K=3, order="random", seed=8)]
 
 
+# block sizes x shared-memory placements: 0 = all that fits, -1 = every array
+# in its global home, 3000 B = a partial placement
 @pytest.mark.parametrize("idx", range(12))
-@pytest.mark.parametrize("n_ctas", [1, 3, 16])
-def test_shapes_group_sizes(idx, n_ctas):
+@pytest.mark.parametrize("block,smem", [(0, 0), (32, 0), (512, 0), (64, -1), (128, 3000)])
+def test_shapes_block_and_placement(idx, block, smem):
     inst = _shapes()[idx]
-    g, o = _both(inst, n_ctas=n_ctas)
+    g, o = _both(inst, block=block, smem=smem)
     assert_parity(g, o)
     validate(inst, g.serve_gpu, g.serve_task, g.events, g.task_start, g.task_end)
 
@@ -95,8 +98,8 @@ def test_heterogeneous_sizes():
     base = gen.random_shared(2000, 128, 3, M=8, K=4, seed=11)
     sizes = rng.integers(1, 5, size=128).astype(np.uint64) * 1_000_000
     inst = base.with_(data_size=sizes, mem_capacity=int(sizes.max()) * 9)
-    for G in (1, 4):
-        g, o = _both(inst, n_ctas=G)
+    for smem in (0, -1):
+        g, o = _both(inst, smem=smem)
         assert_parity(g, o)
 
 
@@ -109,7 +112,7 @@ def test_ample_memory_and_duplicates():
     g, o = _both(dup)
     assert_parity(g, o)
     big = inst.with_(mem_capacity=int(inst.data_size.sum()))
-    g, o = _both(big, n_ctas=4)
+    g, o = _both(big, smem=-1)
     assert_parity(g, o)
     assert g.n_evictions == 0
 
@@ -135,8 +138,34 @@ def test_ragged_tail_sizes():
     # m not a multiple of 4 (uint4 scan tail) and of the CTA size
     for m in (1, 2, 3, 5, 4097, 10001):
         inst = gen.random_shared(m, 64, 3, M=6, K=2, seed=m)
-        g, o = _both(inst, n_ctas=2)
+        g, o = _both(inst, block=64)
         assert_parity(g, o)
+
+
+@pytest.mark.parametrize("idx", [0, 2, 4, 5, 6, 8, 9])
+@pytest.mark.parametrize("smem", [0, -1])
+def test_verify_incremental_scores(idx, smem):
+    """P9: at every scan the incremental scores n_k(D), n2_k(D), u(D) and every
+    task's (cnt, xor) equal a from-scratch recomputation."""
+    inst = _shapes()[idx]
+    g = dts.schedule(inst, flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_VERIFY, smem_budget=smem)
+    assert g.n_verify_err == 0
+    assert_parity(g, oracle.run(inst))
+
+
+def test_long_rows():
+    """Tasks with more than 3 inputs (the plan entry caches 3) and 1-input tasks."""
+    rng = np.random.default_rng(12)
+    rows = [sorted(rng.choice(40, size=int(rng.integers(1, 7)), replace=False)) for _ in range(600)]
+    tp = np.zeros(601, np.int64)
+    tp[1:] = np.cumsum([len(r) for r in rows])
+    td = np.concatenate(rows).astype(np.int32)
+    inst = gen.Instance("long", tp, td, np.ones(40, np.uint64), None, 3, 9, 3)
+    for smem in (0, -1):
+        g = dts.schedule(inst, bus_bps=10 ** 9, smem_budget=smem,
+                         flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_VERIFY)
+        assert g.n_verify_err == 0
+        assert_parity(g, oracle.run(inst, bus_bps=10 ** 9))
 
 
 # ------------------------------------------------------------ larger configs
@@ -196,3 +225,14 @@ def test_sweep_sample_config5():
     gs = dts.schedule_batch(insts)
     for inst, g in zip(insts, gs):
         assert_parity(g, oracle.run(inst))
+
+
+@pytest.mark.parametrize("K", [5, 9, 16, 64])
+def test_many_simulated_gpus(K):
+    """K beyond the register-resident pop path (K <= 8) and up to MAX_K = 64."""
+    inst = gen.random_shared(6000, 512, 3, M=24, K=K, seed=K)
+    g, o = _both(inst)
+    assert_parity(g, o)
+    inst2 = gen.matmul2d(40, M=10, K=K)
+    g, o = _both(inst2, smem=-1)
+    assert_parity(g, o)
