@@ -297,14 +297,15 @@ dts_status ensure_device(dts_instance *I, int device) {
     const size_t plan_cap = (size_t)I->max_deg_ub + 1;
     const size_t res_cap = (size_t)I->res_cap + 1;
     const size_t nw = (n + 31) / 32 + 1;
+    const size_t nstr = (n + 3) & ~size_t(3);
     size_t need = 0;
     auto add = [&](size_t bytes) { need += (bytes + 255) & ~size_t(255); };
     add(8 * (m + 1)); add(4 * (E + 1)); add(8 * (n + 1)); add(8 * (m + 1));          // raw inputs
     add(8 * (m + 1)); add(4 * (E + 1)); add(8 * (n + 1)); add(4 * (E + 1));          // CSR
     add(16 * (E + 1));                                                               // edge records
     add(8 * (n + 1)); add(8);                                                        // delta
-    add(4 * K * mp + 16); add(4 * (n + 1)); add(4 * K * (n + 1)); add(4 * K * (n + 1));  // s u h h2
-    add(4 * K * (n + 1)); add(4 * K * nw); add(4 * K * res_cap);                     // np resb res_list
+    add(4 * K * mp + 16); add(4 * (nstr + 4)); add(4 * K * (nstr + 4)); add(4 * K * (nstr + 4));  // s u h h2
+    add(4 * K * (nstr + 4)); add(4 * K * nw); add(4 * K * res_cap);                  // np resb res_list
     add(16 * K * plan_cap); add(8 * K * plan_cap); add(4 * (3 * n + 1));              // plan tau vhist
     add(sizeof(dts::Out));
     add(4 * (m + 1)); add(4 * (m + 1)); add(8 * (m + 1)); add(8 * (m + 1));          // serve, times
@@ -336,10 +337,10 @@ dts_status ensure_device(dts_instance *I, int device) {
     h.dedge = A.take<int4>(E + 1);
     I->d_delta = A.take<int64_t>(n + 1);
     h.s = A.take<uint32_t>(K * mp + 4);
-    h.u = A.take<int32_t>(n + 1);
-    h.h = A.take<int32_t>(K * (n + 1));
-    h.h2 = A.take<int32_t>(K * (n + 1));
-    h.np = A.take<int32_t>(K * (n + 1));
+    h.u = A.take<int32_t>(nstr + 4);
+    h.h = A.take<int32_t>(K * (nstr + 4));
+    h.h2 = A.take<int32_t>(K * (nstr + 4));
+    h.np = A.take<int32_t>(K * (nstr + 4));
     h.resb = A.take<uint32_t>(K * nw);
     h.res_list = A.take<int32_t>(K * res_cap);
     h.plan = A.take<int4>(K * plan_cap);
@@ -366,8 +367,10 @@ dts_status ensure_device(dts_instance *I, int device) {
     h.plan_cap = (int32_t)plan_cap;
     h.res_cap = (int32_t)res_cap;
     h.nw = (int32_t)nw;
+    h.nstr = (int32_t)nstr;
     h.id_bits = bits_for(I->n > 0 ? (uint64_t)(I->n - 1) : 0);
     h.u_bits = bits_for((uint64_t)I->max_deg_ub);
+    h.key32 = I->max_deg_ub < 32768 ? 1 : 0;  // n(D), n2(D), u(D) <= deg(D)
     h.E = I->E_raw;
     h.size = I->d_size;
     h.delta = I->d_delta;
@@ -424,14 +427,15 @@ int place_smem(dts::Inst &h, bool has_tau, int budget) {
         }
     };
     put(h.so_resb, 4 * K * h.nw);
+    put(h.so_dptr, 4 * (n + 1));
     put(h.so_plan, 16 * K * h.plan_cap);
     if (has_tau) put(h.so_plan_tau, 8 * K * h.plan_cap);
     else h.so_plan_tau = -1;
     put(h.so_res_list, 4 * K * h.res_cap);
-    put(h.so_u, 4 * n);
-    put(h.so_h, 4 * K * n);
-    put(h.so_h2, 4 * K * n);
-    put(h.so_np, 4 * K * n);
+    put(h.so_u, 4 * (int64_t)h.nstr);
+    put(h.so_h, 4 * K * (int64_t)h.nstr);
+    put(h.so_h2, 4 * K * (int64_t)h.nstr);
+    put(h.so_np, 4 * K * (int64_t)h.nstr);
     put(h.so_s, 4 * K * (int64_t)h.m_pad);  // last: the largest, worth it only when it fits
     h.smem_bytes = used;
     return used;
@@ -478,6 +482,13 @@ dts_status stage(dts_instance *I, const dts_run_opts &o, int budget, cudaStream_
     h.W = (int32_t)o.lookahead_W;
     h.flags = o.flags;
     h.max_served = o.max_served;
+    h.size0 = 0;
+    h.delta0 = 0;
+    if (I->n > 0 && std::all_of(I->size.begin(), I->size.end(), [&](uint64_t x) { return x == I->size[0]; })) {
+        h.size0 = I->size[0];
+        const unsigned __int128 num = (unsigned __int128)h.size0 * 1000000000u + (o.bus_bytes_per_s - 1);
+        h.delta0 = (int64_t)(num / o.bus_bytes_per_s);  // ceil, reading R9 (same as dts_init_kernel)
+    }
     place_smem(h, I->has_tau, budget);
     CK(cudaEventRecord(I->ev[0], st), "event");
     CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
@@ -537,7 +548,7 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     s = stage(I, o, budget, st);
     if (s != DTS_OK) return s;
     const int block = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", auto_block(I));
-    const int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n * I->K);
+    const int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n + 4);
     CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
     CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
     CK(cudaEventRecord(I->ev[1], st), "event");

@@ -14,12 +14,12 @@
 //       bits 24..30 : cnt_k(T) = |D(T) \ R_k|   (<= 127)
 //       bits  0..23 : x_k(T)   = XOR of the ids in D(T) \ R_k   (n < 2^24)
 //     so a task with cnt 1 NAMES its one missing datum: x_k(T).
-//   h[K][n]  int32 -- n_k(D)  = #unallocated T with cnt_k(T)=1, x_k(T)=D: the
+//   h[K][nstr] int32 -- n_k(D)  = #unallocated T with cnt_k(T)=1, x_k(T)=D: the
 //       DARTS score of Alg. 5 l.4-5, kept incrementally [S/G]
-//   h2[K][n] int32 -- n2_k(D) = #unallocated T with cnt_k(T)=2, D missing:
+//   h2[K][nstr] int32 -- n2_k(D) = #unallocated T with cnt_k(T)=2, D missing:
 //       the "3inputs" score, kept incrementally      [S/G]
-//   u[n]     int32 -- #unallocated tasks using D (secondary key, R23)     [S/G]
-//   np[K][n] int32 -- #tasks of plannedTasks_k using D (Alg. 6 l.3)       [S/G]
+//   u[nstr]  int32 -- #unallocated tasks using D (secondary key, R23)     [S/G]
+//   np[K][nstr] int32 -- #tasks of plannedTasks_k using D (Alg. 6 l.3)       [S/G]
 //   resb[K][nw] uint32 -- residency bitmap of each simulated GPU          [S/G]
 //   res_list[K][res_cap] int32 -- resident data of each GPU (LUF scan)    [S/G]
 //   plan[K][plan_cap] int4 -- plannedTasks_k in ascending id: {T, D0, D1, D2}
@@ -65,8 +65,10 @@ struct Inst {
     int32_t plan_cap;    // >= max_D deg(D)
     int32_t res_cap;     // >= max resident data per GPU
     int32_t id_bits, u_bits;
-    int32_t nw;          // 32-bit words per residency bitmap row
+    int32_t key32;       // scores and u(D) < 2^15: 32-bit argmax keys (score << 16 | u)
     int32_t pad0;
+    int32_t nw;          // 32-bit words per residency bitmap row
+    int32_t nstr;        // row stride of h, h2, np (and length of u): n rounded up to 4
     int64_t E;
     // CSR (device)
     const int64_t *tptr;
@@ -77,6 +79,8 @@ struct Inst {
                            // o1/o2 = T's other inputs (-1 if none; first two if |D(T)| > 3)
     const uint64_t *size;
     const int64_t *delta;  // ceil(size * 1e9 / bw) ns (reading R9)
+    uint64_t size0;        // != 0: every datum has this size (then delta0 = its bus time)
+    int64_t delta0;
     const int64_t *tau;    // [m] or nullptr
     int64_t default_tau;
     // state: global homes
@@ -88,8 +92,9 @@ struct Inst {
     int64_t *plan_tau;
     int32_t *vhist;  // DTS_F_VERIFY scratch [3 n]
     // shared-memory placement: byte offset in the CTA's dynamic smem, -1 = global home
-    int32_t so_u, so_h, so_h2, so_np, so_resb, so_res_list, so_plan, so_plan_tau, so_s;
+    int32_t so_u, so_h, so_h2, so_np, so_resb, so_res_list, so_plan, so_plan_tau, so_s, so_dptr;
     int32_t smem_bytes;
+    int32_t pad1;
     // outputs
     int32_t *serve_gpu;
     int32_t *serve_task;

@@ -68,9 +68,12 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     int64_t t, ready;
     int32_t row[MAX_ROW + 1];
     unsigned long long red64[32];
+    unsigned long long red64b[32];
     int32_t red32[32];
     int32_t wcnt[32];
     long long prof[8];
+    int64_t bstart[MAX_K], bS[MAX_K];  // pop batch: first start / next scan time per GPU
+    int32_t bcnt[MAX_K], boff[MAX_K + 1];
 };
 
 // Per-instance views: shared-memory arrays where placed, else global homes.
@@ -80,7 +83,8 @@ struct View {
     uint32_t *resb;
     int32_t *res_list;
     int4 *plan;
-    int64_t *plan_tau;
+    int64_t *plan_cum;  // inclusive prefix sums of the planned tasks' tau (per-task times only)
+    int32_t *dptr32;    // shared-memory copy of dptr, or nullptr
 };
 
 __device__ __forceinline__ int warp_sum(int v) {
@@ -105,40 +109,56 @@ __device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long v)
     return v;
 }
 
-// Block reductions (every thread calls; the result is returned to every thread).
+// Block reductions (every thread calls; the result is returned to every
+// thread): warp shuffle, one barrier-protected exchange, warp shuffle again.
 __device__ unsigned long long block_max_u64(Lead &L, unsigned long long v) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     v = warp_max_u64(v);
+    if (nw == 1) return v;
     __syncthreads();
     if (lane == 0) L.red64[w] = v;
     __syncthreads();
-    unsigned long long r = 0ull;
-    for (int i = 0; i < nw; i++) r = L.red64[i] > r ? L.red64[i] : r;
-    return r;
+    return warp_max_u64(lane < nw ? L.red64[lane] : 0ull);
 }
 __device__ unsigned long long block_min_u64(Lead &L, unsigned long long v) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     v = warp_min_u64(v);
+    if (nw == 1) return v;
     __syncthreads();
     if (lane == 0) L.red64[w] = v;
     __syncthreads();
-    unsigned long long r = ~0ull;
-    for (int i = 0; i < nw; i++) r = L.red64[i] < r ? L.red64[i] : r;
-    return r;
+    return warp_min_u64(lane < nw ? L.red64[lane] : ~0ull);
 }
 __device__ int block_sum(Lead &L, int v) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     v = warp_sum(v);
+    if (nw == 1) return v;
     __syncthreads();
     if (lane == 0) L.red32[w] = v;
     __syncthreads();
-    int r = 0;
-    for (int i = 0; i < nw; i++) r += L.red32[i];
-    return r;
+    return warp_sum(lane < nw ? L.red32[lane] : 0);
 }
 
 __device__ __forceinline__ bool resident(const Inst &I, const View &V, int k, int32_t D) {
     return (V.resb[(size_t)k * I.nw + (D >> 5)] >> (D & 31)) & 1u;
+}
+
+// Data->task segment bounds of D (int32 copy in shared memory when placed).
+__device__ __forceinline__ void seg_of(const Inst &I, const View &V, int32_t D, int64_t &b, int64_t &e) {
+    if (V.dptr32) {
+        b = V.dptr32[D];
+        e = V.dptr32[D + 1];
+    } else {
+        b = __ldg(&I.dptr[D]);
+        e = __ldg(&I.dptr[D + 1]);
+    }
+}
+// Size and bus time of D: scalars when all sizes are equal (the paper's model).
+__device__ __forceinline__ uint64_t size_of(const Inst &I, int32_t D) {
+    return I.size0 ? I.size0 : __ldg(&I.size[D]);
+}
+__device__ __forceinline__ int64_t delta_of(const Inst &I, int32_t D) {
+    return I.size0 ? I.delta0 : __ldg(&I.delta[D]);
 }
 
 __device__ __forceinline__ int64_t tau_of(const Inst &I, int32_t T) {
@@ -205,12 +225,12 @@ __device__ void pool_move(const Inst &I, const View &V, int32_t T, Row r, int si
             V.s[(size_t)j * I.m_pad + T] = sign < 0 ? (w[jj] | ALLOC_BIT) : (w[jj] & ~ALLOC_BIT);
             const uint32_t c = (w[jj] >> 24) & 0x7fu;
             if (c == 1u) {
-                atomicAdd(&V.h[(size_t)j * I.n + (w[jj] & XOR_MASK)], sign);
+                atomicAdd(&V.h[(size_t)j * I.nstr + (w[jj] & XOR_MASK)], sign);
             } else if (c == 2u) {
                 int32_t a, b;
                 missing_pair(I, V, j, T, r, -1, a, b);
-                atomicAdd(&V.h2[(size_t)j * I.n + a], sign);
-                atomicAdd(&V.h2[(size_t)j * I.n + b], sign);
+                atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+                atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
             }
         }
     }
@@ -220,7 +240,7 @@ __device__ void pool_move(const Inst &I, const View &V, int32_t T, Row r, int si
         for (int i = 0; i < 3; i++) {
             if (c[i] < 0) continue;
             atomicAdd(&V.u[c[i]], sign);
-            if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.n + c[i]], -sign);
+            if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[i]], -sign);
         }
         return;
     }
@@ -228,7 +248,7 @@ __device__ void pool_move(const Inst &I, const View &V, int32_t T, Row r, int si
     for (int64_t i = rb; i < re; i++) {
         const int32_t D = __ldg(&I.tdat[i]);
         atomicAdd(&V.u[D], sign);
-        if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.n + D], -sign);
+        if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + D], -sign);
     }
 }
 
@@ -239,10 +259,11 @@ __device__ void pool_move(const Inst &I, const View &V, int32_t T, Row r, int si
 // already updated.  Each task appears once in the segment, so the state words
 // are plain read-modify-writes; the buckets are atomics.
 __device__ void seg_update(const Inst &I, const View &V, int k, int32_t D, bool load) {
-    const int64_t b = __ldg(&I.dptr[D]), e = __ldg(&I.dptr[D + 1]);
+    int64_t b, e;
+    seg_of(I, V, D, b, e);
     uint32_t *sk = V.s + (size_t)k * I.m_pad;
-    int32_t *hk = V.h + (size_t)k * I.n;
-    int32_t *h2k = V.h2 + (size_t)k * I.n;
+    int32_t *hk = V.h + (size_t)k * I.nstr;
+    int32_t *h2k = V.h2 + (size_t)k * I.nstr;
     for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
         const int4 ed = __ldg(&I.dedge[i]);
         const int32_t T = ed.x;
@@ -324,7 +345,7 @@ __device__ int32_t pop_planned(const Inst &I, const View &V, Lead &L, int k, int
     while (e.x < 0) e = pl[++h];
     L.plan_head[k] = h + 1;
     L.plan_live[k]--;
-    int32_t *npk = V.np + (size_t)k * I.n;
+    int32_t *npk = V.np + (size_t)k * I.nstr;
     if (e.w != ROW_LONG) {
         if (e.y >= 0) atomicSub(&npk[e.y], 1);
         if (e.z >= 0) atomicSub(&npk[e.z], 1);
@@ -333,7 +354,12 @@ __device__ int32_t pop_planned(const Inst &I, const View &V, Lead &L, int k, int
         const int64_t rb = __ldg(&I.tptr[e.x]), re = __ldg(&I.tptr[e.x + 1]);
         for (int64_t i = rb; i < re; i++) atomicSub(&npk[__ldg(&I.tdat[i])], 1);
     }
-    *tau = V.plan_tau ? V.plan_tau[(size_t)k * I.plan_cap + h] : I.default_tau;
+    if (V.plan_cum) {
+        const int64_t *pc = V.plan_cum + (size_t)k * I.plan_cap;
+        *tau = pc[h] - (h > 0 ? pc[h - 1] : 0);
+    } else {
+        *tau = I.default_tau;
+    }
     // D(T) for serve_loads, ascending (R10), straight from the entry when cached
     if (e.w != ROW_LONG) {
         int32_t a = e.y, b = e.z, c = e.w;  // -1 = absent; sort descending, count
@@ -351,118 +377,14 @@ __device__ int32_t pop_planned(const Inst &I, const View &V, Lead &L, int k, int
     return e.x;
 }
 
-// Thread 0: serve every request that finds plannedTasks_k non-empty (Alg. 5
-// l.1-2) until one finds it empty (returns that k; L.k, L.t set) or the run
-// ends (-1).  No other thread, no barrier, no global read: the popped task's
-// inputs are resident, so serving it is time-model arithmetic.
-// np_k is NOT maintained here: LUF on GPU k only runs while k serves the first
-// task of a new plan (or a fallback task, with no plan), and every scan resets
-// np_k (reset_plan), so the pops of an old plan never reach a LUF decision.
-// The per-GPU scalars live in registers (KR >= K, compile-time) so a pop is a
-// short dependent chain; outputs go out with plain global stores.
-template <int KR>
-__device__ int pop_run(const Inst &I, const View &V, Lead &L) {
-    const int K = I.K, W = I.W, pcap = I.plan_cap;
-    const int64_t maxs = I.max_served, dtau = I.default_tau;
-    int32_t *const sg = I.serve_gpu;
-    int32_t *const stk = I.serve_task;
-    int64_t *const tst = I.tstart;
-    int64_t *const ten = I.tend;
-    int64_t rq[KR], gf[KR];
-    int hd[KR], lv[KR];
-    bool act[KR];
-#pragma unroll
-    for (int j = 0; j < KR; j++) {
-        act[j] = j < K && !L.idle[j];
-        rq[j] = j < K ? L.req[j] : 0;
-        gf[j] = j < K ? L.gpu_free[j] : 0;
-        hd[j] = j < K ? L.plan_head[j] : 0;
-        lv[j] = j < K ? L.plan_live[j] : 0;
-    }
-    int64_t ns = L.n_served, mk = L.makespan, pops = 0;
-    int ret = -1;
-    while (maxs < 0 || ns < maxs) {
-        // the earliest (req, k) and the runner-up among non-idle GPUs (R8)
-        int k = -1, k2 = -1;
-        int64_t t1 = 0, t2 = 0;
-#pragma unroll
-        for (int j = 0; j < KR; j++) {
-            if (!act[j]) continue;
-            const int64_t r = rq[j];
-            if (k < 0 || r < t1) {
-                k2 = k;
-                t2 = t1;
-                k = j;
-                t1 = r;
-            } else if (k2 < 0 || r < t2) {
-                k2 = j;
-                t2 = r;
-            }
-        }
-        if (k < 0) break;
-        int live = 0, h = 0;
-        int64_t gfree = 0;
-#pragma unroll
-        for (int j = 0; j < KR; j++)
-            if (j == k) {
-                live = lv[j];
-                h = hd[j];
-                gfree = gf[j];
-            }
-        if (live == 0) {
-            ret = k;
-            L.k = k;
-            L.t = t1;
-            break;
-        }
-        int64_t req = t1;
-        const int4 *pl = V.plan + (size_t)k * pcap;
-        const int64_t *pt = V.plan_tau ? V.plan_tau + (size_t)k * pcap : nullptr;
-        while (true) {
-            int T = pl[h].x;
-            while (T < 0) T = pl[++h].x;
-            const int64_t tau = pt ? pt[h] : dtau;
-            h++;
-            live--;
-            const int64_t start = req > gfree ? req : gfree;
-            const int64_t end = start + tau;
-            gfree = end;
-            __stcg(&tst[T], start);
-            __stcg(&ten[T], end);
-            mk = end > mk ? end : mk;
-            __stcg(&sg[ns], k);
-            __stcg(&stk[ns], T);
-            ns++;
-            pops++;
-            req = (W == 0) ? end : start;  // R7
-            if (live == 0 || (maxs >= 0 && ns >= maxs)) break;
-            if (k2 >= 0 && (req > t2 || (req == t2 && k2 < k))) break;  // another GPU is next
-        }
-#pragma unroll
-        for (int j = 0; j < KR; j++)
-            if (j == k) {
-                lv[j] = live;
-                hd[j] = h;
-                gf[j] = gfree;
-                rq[j] = req;
-            }
-    }
-#pragma unroll
-    for (int j = 0; j < KR; j++)
-        if (j < K) {
-            L.req[j] = rq[j];
-            L.gpu_free[j] = gf[j];
-            L.plan_head[j] = hd[j];
-            L.plan_live[j] = lv[j];
-        }
-    L.n_served = ns;
-    L.makespan = mk;
-    L.alg_bytes += 24ull * (uint64_t)pops;
-    return ret;
-}
-
-// pop_run for K > 8: the same, with the per-GPU scalars left in shared memory.
-__device__ int pop_run_smem(const Inst &I, const View &V, Lead &L) {
+// Thread 0, sequential pops (used for prefix runs, max_served >= 0): serve
+// every request that finds plannedTasks_k non-empty (Alg. 5 l.1-2) until one
+// finds it empty (returns that k; L.k, L.t set) or the run ends (-1).  The
+// popped task's inputs are resident (LUF drops planned tasks whose inputs it
+// evicts, Alg. 6 l.8), so serving it is time-model arithmetic.
+// np_k is not maintained by pops: LUF on GPU k only runs while k serves the
+// first task of a new plan (or a fallback task), and every scan resets np_k.
+__device__ int pop_run_seq(const Inst &I, const View &V, Lead &L) {
     const int K = I.K, W = I.W, pcap = I.plan_cap;
     const int64_t maxs = I.max_served, dtau = I.default_tau;
     int32_t *const sg = I.serve_gpu;
@@ -498,11 +420,10 @@ __device__ int pop_run_smem(const Inst &I, const View &V, Lead &L) {
         int h = L.plan_head[k];
         int64_t req = t1, gfree = L.gpu_free[k];
         const int4 *pl = V.plan + (size_t)k * pcap;
-        const int64_t *pt = V.plan_tau ? V.plan_tau + (size_t)k * pcap : nullptr;
+        const int64_t *pc = V.plan_cum ? V.plan_cum + (size_t)k * pcap : nullptr;
         while (true) {
-            int T = pl[h].x;
-            while (T < 0) T = pl[++h].x;
-            const int64_t tau = pt ? pt[h] : dtau;
+            const int T = pl[h].x;
+            const int64_t tau = pc ? pc[h] - (h > 0 ? pc[h - 1] : 0) : dtau;
             h++;
             live--;
             const int64_t start = req > gfree ? req : gfree;
@@ -530,12 +451,205 @@ __device__ int pop_run_smem(const Inst &I, const View &V, Lead &L) {
     return ret;
 }
 
+
+// a[lo..hi) := base + inclusive prefix sums of a[lo..hi).  Block-wide.
+__device__ void block_incl_scan(Lead &L, int64_t *a, int lo, int hi, int64_t base) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    int64_t carry = base;
+    for (int c = lo; c < hi; c += blockDim.x) {
+        const int i = c + threadIdx.x;
+        int64_t v = i < hi ? a[i] : 0;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int64_t t = __shfl_up_sync(FULL, v, o);
+            if (lane >= o) v += t;
+        }
+        __syncthreads();
+        if (lane == 31) L.red64[w] = (unsigned long long)v;
+        __syncthreads();
+        int64_t off = 0, tot = 0;
+        for (int j = 0; j < nw; j++) {
+            const int64_t x = (int64_t)L.red64[j];
+            if (j < w) off += x;
+            tot += x;
+        }
+        if (i < hi) a[i] = carry + off + v;
+        carry += tot;
+    }
+    __syncthreads();
+}
+
+// After LUF removed planned tasks of k (T = -1), close the holes: ordered
+// compaction of [head, end) so the live entries are contiguous (pop_batch
+// indexes them directly), and rebuild their tau prefix sums.  Block-wide.
+__device__ void compact_plan(const Inst &I, const View &V, Lead &L, int k) {
+    int4 *pl = V.plan + (size_t)k * I.plan_cap;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    const int ph = L.plan_head[k], pe = L.plan_end[k];
+    int out = ph;
+    for (int c = ph; c < pe; c += blockDim.x) {
+        const int i = c + threadIdx.x;
+        const int4 e = i < pe ? pl[i] : make_int4(-1, -1, -1, -1);
+        const bool keep = e.x >= 0;
+        const unsigned msk = __ballot_sync(FULL, keep);
+        if (lane == 0) L.wcnt[w] = __popc(msk);
+        __syncthreads();  // every read of this chunk happened (writes go below its start)
+        int off = out, tot = 0;
+        for (int j = 0; j < nw; j++) {
+            const int x = L.wcnt[j];
+            if (j < w) off += x;
+            tot += x;
+        }
+        if (keep) pl[off + __popc(msk & lt)] = e;
+        out += tot;
+        __syncthreads();
+    }
+    if (V.plan_cum) {
+        int64_t *pc = V.plan_cum + (size_t)k * I.plan_cap;
+        for (int i = ph + threadIdx.x; i < out; i += blockDim.x) pc[i] = tau_of(I, pl[i].x);
+        __syncthreads();
+        block_incl_scan(L, pc, ph, out, ph > 0 ? pc[ph - 1] : 0);
+    }
+    if (threadIdx.x == 0) L.plan_end[k] = out;
+    __syncthreads();
+}
+
+// Sum of tau over the first c live planned tasks of GPU j (from its head).
+__device__ __forceinline__ int64_t plan_span(const Inst &I, const View &V, const Lead &L, int j, int c) {
+    if (c <= 0) return 0;
+    if (!V.plan_cum) return (int64_t)c * I.default_tau;
+    const int64_t *pc = V.plan_cum + (size_t)j * I.plan_cap;
+    const int h = L.plan_head[j];
+    return pc[h + c - 1] - (h > 0 ? pc[h - 1] : 0);
+}
+
+// Request time of the i-th pop of GPU j in this batch (W = 0: the GPU asks
+// again when its task ends, R7).
+__device__ __forceinline__ int64_t pop_req(const Inst &I, const View &V, const Lead &L, int j, int i) {
+    return i == 0 ? L.req[j] : L.bstart[j] + plan_span(I, V, L, j, i);
+}
+
+// #{ i < c : (req_{j,i}, j) < (r, k) } -- the pops of GPU j that precede the
+// event (r, k) in the (time, GPU id) order of requests (R8); binary search.
+__device__ __forceinline__ int pops_before(const Inst &I, const View &V, const Lead &L, int j, int c,
+                                           int64_t r, int k) {
+    int lo = 0, hi = c;  // answer in [lo, hi]
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        const int64_t rm = pop_req(I, V, L, j, mid);
+        if (rm < r || (rm == r && j < k)) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// Every request that finds plannedTasks_k non-empty (Alg. 5 l.1-2) up to the
+// next one that finds it empty, served at once by the whole CTA.  Between two
+// scans nothing but pops happens, and a pop only moves time: the popped
+// task's inputs are resident (LUF drops planned tasks whose inputs it evicts,
+// Alg. 6 l.8) and np_k is rebuilt at every scan of k (reset_plan), so each
+// GPU's request times are prefix sums of its planned tasks' tau (PAPER.md:
+// 276-342, W = 0).  The next scan is the earliest (request after the last pop,
+// k) (R8); every pop before it is placed in the global service order by
+// merge ranks.  Sets L.cmd (CMD_SCAN with L.k, L.t, or CMD_DONE).
+__device__ void pop_batch(const Inst &I, const View &V, Lead &L) {
+    const int K = I.K;
+    for (int j = threadIdx.x; j < K; j += blockDim.x) {
+        const int live = L.plan_end[j] - L.plan_head[j];
+        const int64_t start0 = L.req[j] > L.gpu_free[j] ? L.req[j] : L.gpu_free[j];
+        L.bstart[j] = start0;
+        L.bS[j] = L.idle[j] ? INT64_MAX : (live == 0 ? L.req[j] : start0 + plan_span(I, V, L, j, live));
+    }
+    __syncthreads();
+    if (threadIdx.x < 32) {  // k* = argmin (S_j, j) over non-idle GPUs
+        int kb = -1;
+        int64_t sb = INT64_MAX;
+        for (int j = threadIdx.x; j < K; j += 32)
+            if (!L.idle[j] && (kb < 0 || L.bS[j] < sb)) {
+                kb = j;
+                sb = L.bS[j];
+            }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            const int ko = __shfl_xor_sync(FULL, kb, o);
+            const int64_t so = __shfl_xor_sync(FULL, sb, o);
+            if (ko >= 0 && (kb < 0 || so < sb || (so == sb && ko < kb))) {
+                kb = ko;
+                sb = so;
+            }
+        }
+        if (threadIdx.x == 0) {
+            L.k = kb;
+            L.t = sb;
+            L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
+        }
+    }
+    __syncthreads();
+    const int ks = L.k;
+    const int64_t ts = L.t;
+    if (ks < 0) return;
+    for (int j = threadIdx.x; j < K; j += blockDim.x) {
+        const int live = L.plan_end[j] - L.plan_head[j];
+        L.bcnt[j] = L.idle[j] ? 0 : (j == ks ? live : pops_before(I, V, L, j, live, ts, ks));
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int run = 0;
+        for (int j = 0; j < K; j++) {
+            L.boff[j] = run;
+            run += L.bcnt[j];
+        }
+        L.boff[K] = run;
+    }
+    __syncthreads();
+    const int P = L.boff[K];
+    const int64_t ns = L.n_served;
+    int64_t mk = 0;
+    int32_t *const sg = I.serve_gpu;
+    int32_t *const stk = I.serve_task;
+    for (int p = threadIdx.x; p < P; p += blockDim.x) {
+        int j = 0;
+        while (L.boff[j + 1] <= p) j++;
+        const int i = p - L.boff[j];
+        const int64_t r = pop_req(I, V, L, j, i);
+        const int64_t start = i == 0 ? L.bstart[j] : r;
+        const int64_t end = L.bstart[j] + plan_span(I, V, L, j, i + 1);
+        const int T = V.plan[(size_t)j * I.plan_cap + L.plan_head[j] + i].x;
+        int64_t pos = ns + i;
+        for (int j2 = 0; j2 < K; j2++)
+            if (j2 != j && L.bcnt[j2] > 0) pos += pops_before(I, V, L, j2, L.bcnt[j2], r, j);
+        __stcg(&I.tstart[T], start);
+        __stcg(&I.tend[T], end);
+        __stcg(&sg[pos], j);
+        __stcg(&stk[pos], T);
+        mk = end > mk ? end : mk;
+    }
+    mk = (int64_t)block_max_u64(L, (unsigned long long)mk);
+    for (int j = threadIdx.x; j < K; j += blockDim.x) {
+        const int c = L.bcnt[j];
+        if (c > 0) {
+            const int64_t end = L.bstart[j] + plan_span(I, V, L, j, c);
+            L.req[j] = end;  // W = 0 (R7)
+            L.gpu_free[j] = end;
+            L.plan_head[j] += c;
+            L.plan_live[j] -= c;
+        }
+    }
+    if (threadIdx.x == 0) {
+        L.n_served = ns + P;
+        if (mk > L.makespan) L.makespan = mk;
+        L.alg_bytes += 24ull * (uint64_t)P;
+    }
+    __syncthreads();
+}
+
 // CTA-wide, at every scan of GPU k: plannedTasks_k is empty (all popped or
 // removed); clear np_k for every datum its last plan touched, so that np_k
 // counts exactly the plan this scan creates (Alg. 6 l.3).
 __device__ void reset_plan(const Inst &I, const View &V, Lead &L, int k) {
     const int4 *pl = V.plan + (size_t)k * I.plan_cap;
-    int32_t *npk = V.np + (size_t)k * I.n;
+    int32_t *npk = V.np + (size_t)k * I.nstr;
     const int pe = L.plan_end[k];
     for (int i = threadIdx.x; i < pe; i += blockDim.x) {
         const int4 e = pl[i];
@@ -582,7 +696,7 @@ __device__ __forceinline__ bool entry_uses(const Inst &I, int4 e, int32_t D) {
 __device__ int32_t luf_victim(const Inst &I, const View &V, Lead &L, int k) {
     const int cnt = L.res_cnt[k];
     const int32_t *rl = V.res_list + (size_t)k * I.res_cap;
-    const int32_t *npk = V.np + (size_t)k * I.n;
+    const int32_t *npk = V.np + (size_t)k * I.nstr;
     unsigned long long best = ~0ull;
     for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
         const int32_t D = rl[i];
@@ -637,13 +751,15 @@ __device__ void evict(const Inst &I, const View &V, Lead &L, int k, int32_t Vd, 
         rl[L.vslot] = rl[last];
         L.res_cnt[k] = last;
         V.resb[(size_t)k * I.nw + (Vd >> 5)] &= ~(1u << (Vd & 31));
-        L.used[k] -= __ldg(&I.size[Vd]);
+        L.used[k] -= size_of(I, Vd);
         L.n_evictions++;
         push_event(I, L, 1, k, Vd, Tserved, t, t);
-        const int64_t deg = __ldg(&I.dptr[Vd + 1]) - __ldg(&I.dptr[Vd]);
-        L.alg_bytes += 12ull * (uint64_t)deg + (uint64_t)nret * (8ull * I.K + 32ull);
+        int64_t sb, se;
+        seg_of(I, V, Vd, sb, se);
+        L.alg_bytes += 20ull * (uint64_t)(se - sb) + (uint64_t)nret * (8ull * I.K + 32ull);
     }
     __syncthreads();
+    if (nret > 0) compact_plan(I, V, L, k);
     seg_update(I, V, k, Vd, false);
     __syncthreads();
 }
@@ -661,7 +777,7 @@ __device__ void serve_loads(const Inst &I, const View &V, Lead &L, int k, int32_
         const bool res = resident(I, V, k, D);
         __syncthreads();
         if (res) continue;
-        const uint64_t sz = __ldg(&I.size[D]);
+        const uint64_t sz = size_of(I, D);
         while (true) {  // R11: LUF until D fits
             const bool full = L.used[k] + sz > I.cap;
             __syncthreads();
@@ -684,14 +800,15 @@ __device__ void serve_loads(const Inst &I, const View &V, Lead &L, int k, int32_
             V.resb[(size_t)k * I.nw + (D >> 5)] |= 1u << (D & 31);
             L.used[k] += sz;
             const int64_t st = L.bus_free > t ? L.bus_free : t;
-            const int64_t en = st + __ldg(&I.delta[D]);
+            const int64_t en = st + delta_of(I, D);
             L.bus_free = en;
             if (en > L.ready) L.ready = en;
             L.n_loads++;
             L.bytes_loaded += sz;
             push_event(I, L, 0, k, D, T, st, en);
-            const int64_t deg = __ldg(&I.dptr[D + 1]) - __ldg(&I.dptr[D]);
-            L.alg_bytes += 12ull * (uint64_t)deg;
+            int64_t sb, se;
+            seg_of(I, V, D, sb, se);
+            L.alg_bytes += 20ull * (uint64_t)(se - sb);
         }
         __syncthreads();
         PROF_T0(p_seg);
@@ -703,33 +820,88 @@ __device__ void serve_loads(const Inst &I, const View &V, Lead &L, int k, int32_
     __syncthreads();
 }
 
-// Block argmax over D of (score[D], u[D], ~D) with score[D] > 0 (Alg. 5
-// l.6-9).  A datum with a positive score is never resident (its tasks miss it).
+// Alg. 5 l.6-9 (and the 3inputs fallback): block argmax
+// over D of (score[D], u(D), -D) among data with a positive score -- more
+// freed tasks, then more unprocessed uses, then the lower id (R1, R23, R24).
+// A datum with a positive score is never resident (its tasks miss it), so no
+// residency test is needed.  Rows are padded to nstr (multiple of 4, pad
+// scores 0): 16-byte loads, UN vectors in flight per array and thread.
+// Fast path (score, u < 2^15, checked on the host: I.key32): the pair packs
+// into one 32-bit key score << 16 | u, and since each thread visits D in
+// increasing order a strict '>' keeps the lowest id among equal keys; the
+// 64-bit (key, ~D) is formed once per thread for the block reduction.
 __device__ int32_t score_argmax(const Inst &I, const View &V, Lead &L, const int32_t *score) {
-    const unsigned ib = (unsigned)I.id_bits, ub = (unsigned)I.u_bits;
+    const unsigned ib = (unsigned)I.id_bits;
     const unsigned long long idmask = (1ull << ib) - 1ull;
+    const int4 *h4 = reinterpret_cast<const int4 *>(score);
+    const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
+    const int nv = I.nstr >> 2;
+    constexpr int UN = 4;
     unsigned long long best = 0ull;
-    for (int D = threadIdx.x; D < I.n; D += blockDim.x) {
-        const int32_t sc = score[D];
-        if (sc > 0) {
-            const unsigned long long key = ((unsigned long long)(uint32_t)sc << (ub + ib)) |
-                                           ((unsigned long long)(uint32_t)V.u[D] << ib) |
-                                           (idmask - (unsigned long long)D);
-            best = key > best ? key : best;
+    if (I.key32) {
+        uint32_t bk = 0u;
+        int32_t bd = 0;
+        for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
+            int4 hv[UN], uv[UN];
+#pragma unroll
+            for (int q = 0; q < UN; q++) {
+                const int v = v0 + q * blockDim.x;
+                hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
+                uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
+            }
+#pragma unroll
+            for (int q = 0; q < UN; q++) {
+                const int D = 4 * (v0 + q * blockDim.x);
+                const uint32_t k0 = ((uint32_t)hv[q].x << 16) | (uint32_t)uv[q].x;
+                const uint32_t k1 = ((uint32_t)hv[q].y << 16) | (uint32_t)uv[q].y;
+                const uint32_t k2 = ((uint32_t)hv[q].z << 16) | (uint32_t)uv[q].z;
+                const uint32_t k3 = ((uint32_t)hv[q].w << 16) | (uint32_t)uv[q].w;
+                if (k0 > bk) { bk = k0; bd = D; }
+                if (k1 > bk) { bk = k1; bd = D + 1; }
+                if (k2 > bk) { bk = k2; bd = D + 2; }
+                if (k3 > bk) { bk = k3; bd = D + 3; }
+            }
+        }
+        if (bk >= 65536u)  // positive score
+            best = ((unsigned long long)bk << ib) | (idmask - (unsigned long long)bd);
+    } else {
+        const unsigned ub = (unsigned)I.u_bits;
+        for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
+            int4 hv[UN], uv[UN];
+#pragma unroll
+            for (int q = 0; q < UN; q++) {
+                const int v = v0 + q * blockDim.x;
+                hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
+                uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
+            }
+#pragma unroll
+            for (int q = 0; q < UN; q++) {
+                const int D = 4 * (v0 + q * blockDim.x);
+                const int32_t sc[4] = {hv[q].x, hv[q].y, hv[q].z, hv[q].w};
+                const int32_t uu[4] = {uv[q].x, uv[q].y, uv[q].z, uv[q].w};
+#pragma unroll
+                for (int c = 0; c < 4; c++) {
+                    if (sc[c] <= 0) continue;
+                    const unsigned long long key = ((unsigned long long)(uint32_t)sc[c] << (ub + ib)) |
+                                                   ((unsigned long long)(uint32_t)uu[c] << ib) |
+                                                   (idmask - (unsigned long long)(D + c));
+                    best = key > best ? key : best;
+                }
+            }
         }
     }
     best = block_max_u64(L, best);
-    if (best == 0ull) return -1;
-    return (int32_t)(idmask - (best & idmask));
+    return best ? (int32_t)(idmask - (best & idmask)) : -1;
 }
 
 // Alg. 5 l.10: plannedTasks_k <- unallocated tasks of Dopt's segment with one
 // missing input (= Dopt), ascending id (ordered block compaction).  Block-wide.
 __device__ void plan(const Inst &I, const View &V, Lead &L, int k, int32_t Dopt) {
-    const int64_t b = __ldg(&I.dptr[Dopt]), e = __ldg(&I.dptr[Dopt + 1]);
+    int64_t b, e;
+    seg_of(I, V, Dopt, b, e);
     const uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int4 *pl = V.plan + (size_t)k * I.plan_cap;
-    int64_t *pt = V.plan_tau ? V.plan_tau + (size_t)k * I.plan_cap : nullptr;
+    int64_t *pt = V.plan_cum ? V.plan_cum + (size_t)k * I.plan_cap : nullptr;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
     int base_out = 0;
@@ -762,6 +934,7 @@ __device__ void plan(const Inst &I, const View &V, Lead &L, int k, int32_t Dopt)
         base_out += tot;
         __syncthreads();
     }
+    if (pt) block_incl_scan(L, pt, 0, base_out, 0);  // tau -> prefix sums
     if (threadIdx.x == 0) {
         L.plan_head[k] = 0;
         L.plan_end[k] = base_out;
@@ -774,7 +947,8 @@ __device__ void plan(const Inst &I, const View &V, Lead &L, int k, int32_t Dopt)
 
 // 3inputs: the lowest-id unallocated task of D2's segment with two missing inputs.
 __device__ int32_t first_cnt2(const Inst &I, const View &V, Lead &L, int k, int32_t D2) {
-    const int64_t b = __ldg(&I.dptr[D2]), e = __ldg(&I.dptr[D2 + 1]);
+    int64_t b, e;
+    seg_of(I, V, D2, b, e);
     const uint32_t *sk = V.s + (size_t)k * I.m_pad;
     for (int64_t base = b; base < e; base += blockDim.x) {
         const int64_t i = base + threadIdx.x;
@@ -830,8 +1004,8 @@ __device__ void verify_scores(const Inst &I, const View &V, Lead &L, int k) {
     }
     __syncthreads();
     for (int D = threadIdx.x; D < I.n; D += blockDim.x)
-        bad += (__ldcg(&vh[D]) != V.h[(size_t)k * I.n + D]) +
-               (__ldcg(&vh2[D]) != V.h2[(size_t)k * I.n + D]) + (__ldcg(&vu[D]) != V.u[D]);
+        bad += (__ldcg(&vh[D]) != V.h[(size_t)k * I.nstr + D]) +
+               (__ldcg(&vh2[D]) != V.h2[(size_t)k * I.nstr + D]) + (__ldcg(&vu[D]) != V.u[D]);
     bad = block_sum(L, bad);
     if (threadIdx.x == 0) L.n_verr += bad;
     __syncthreads();
@@ -912,24 +1086,27 @@ __global__ void __launch_bounds__(512, 1)
         V.resb = I.so_resb >= 0 ? (uint32_t *)(dsm + I.so_resb) : I.resb;
         V.res_list = I.so_res_list >= 0 ? (int32_t *)(dsm + I.so_res_list) : I.res_list;
         V.plan = I.so_plan >= 0 ? (int4 *)(dsm + I.so_plan) : I.plan;
-        V.plan_tau = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
+        V.plan_cum = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
+        V.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
 
         // ---- CTA-local copies of the initial state (global homes were
         //      initialised by dts_init_kernel)
         const int n = I.n, K = I.K;
+        if (I.so_dptr >= 0)
+            for (int D = tid; D <= n; D += blockDim.x) V.dptr32[D] = (int32_t)__ldg(&I.dptr[D]);
         if (I.so_s >= 0) {
             const uint4 *src = reinterpret_cast<const uint4 *>(I.s);
             uint4 *dst = reinterpret_cast<uint4 *>(V.s);
             for (int i = tid; i < (K * I.m_pad) / 4; i += blockDim.x) dst[i] = __ldcg(&src[i]);
         }
         if (I.so_u >= 0)
-            for (int D = tid; D < n; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
+            for (int D = tid; D < I.nstr; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
         if (I.so_h >= 0)
-            for (int i = tid; i < K * n; i += blockDim.x) V.h[i] = __ldcg(&I.h[i]);
+            for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h[i] = __ldcg(&I.h[i]);
         if (I.so_h2 >= 0)
-            for (int i = tid; i < K * n; i += blockDim.x) V.h2[i] = __ldcg(&I.h2[i]);
+            for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h2[i] = __ldcg(&I.h2[i]);
         if (I.so_np >= 0)
-            for (int i = tid; i < K * n; i += blockDim.x) V.np[i] = 0;
+            for (int i = tid; i < K * I.nstr; i += blockDim.x) V.np[i] = 0;
         if (I.so_resb >= 0)
             for (int i = tid; i < K * I.nw; i += blockDim.x) V.resb[i] = 0u;
         if (tid == 0) {
@@ -957,16 +1134,16 @@ __global__ void __launch_bounds__(512, 1)
         // ---- the decision loop
         while (true) {
             PROF_T0(p_pop);
-            if (tid == 0) {
-                // Pops need no other thread: serve them here until a request
-                // finds plannedTasks_k empty (Alg. 5 l.3) or the run ends.
-                int cmd = CMD_DONE;
-                if (!L.error) {
-                    const int r = I.K <= 4 ? pop_run<4>(I, V, L)
-                                           : (I.K <= 8 ? pop_run<8>(I, V, L) : pop_run_smem(I, V, L));
-                    if (r >= 0) cmd = CMD_SCAN;
-                }
-                L.cmd = cmd;
+            int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
+            for (int j = 0; j < K; j++) pending += L.plan_live[j];
+            if (I.max_served < 0 && pending > 16) {
+                pop_batch(I, V, L);
+            } else {  // few pops (or a prefix run that stops at an exact count): thread 0
+                __syncthreads();
+                if (tid == 0)
+                    L.cmd = ((I.max_served < 0 || L.n_served < I.max_served) && pop_run_seq(I, V, L) >= 0)
+                                ? CMD_SCAN
+                                : CMD_DONE;
             }
             PROF_ADD(L, P_POP, p_pop);
             __syncthreads();
@@ -978,7 +1155,7 @@ __global__ void __launch_bounds__(512, 1)
             // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
             int32_t T = -1;
             PROF_T0(p_am);
-            const int32_t Dopt = score_argmax(I, V, L, V.h + (size_t)k * n);
+            const int32_t Dopt = score_argmax(I, V, L, V.h + (size_t)k * I.nstr);
             PROF_ADD(L, P_ARGMAX, p_am);
             PROF_T0(p_pl);
             if (tid == 0) {
@@ -997,7 +1174,7 @@ __global__ void __launch_bounds__(512, 1)
                 PROF_ADD(L, P_PLAN, p_pl);
             } else {
                 if (I.flags & DTS_F_FALLBACK2) {
-                    const int32_t D2 = score_argmax(I, V, L, V.h2 + (size_t)k * n);
+                    const int32_t D2 = score_argmax(I, V, L, V.h2 + (size_t)k * I.nstr);
                     if (D2 >= 0) {
                         T = first_cnt2(I, V, L, k, D2);
                         if (tid == 0) L.n_fb2++;
@@ -1088,6 +1265,14 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
             }
             for (int k = 0; k < I.K; k++) I.s[(size_t)k * I.m_pad + T] = w;
         }
+        for (int64_t D = I.n + tid; D < I.nstr; D += str) {  // row padding: never scores
+            I.u[D] = 0;
+            for (int k = 0; k < I.K; k++) {
+                I.h[(size_t)k * I.nstr + D] = 0;
+                I.h2[(size_t)k * I.nstr + D] = 0;
+                I.np[(size_t)k * I.nstr + D] = 0;
+            }
+        }
         for (int64_t D = tid; D < I.n; D += str) {
             const int64_t b = I.dptr[D], e = I.dptr[D + 1];
             int32_t c1 = 0, c2 = 0;
@@ -1101,9 +1286,9 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
             unsigned __int128 num = (unsigned __int128)I.size[D] * 1000000000ull + (bw - 1);
             delta[D] = (int64_t)(num / bw);
             for (int k = 0; k < I.K; k++) {
-                I.h[(size_t)k * I.n + D] = c1;
-                I.h2[(size_t)k * I.n + D] = c2;
-                I.np[(size_t)k * I.n + D] = 0;
+                I.h[(size_t)k * I.nstr + D] = c1;
+                I.h2[(size_t)k * I.nstr + D] = c2;
+                I.np[(size_t)k * I.nstr + D] = 0;
             }
         }
         for (int64_t i = tid; i < (int64_t)I.K * I.nw; i += str) I.resb[i] = 0u;

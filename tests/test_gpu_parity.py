@@ -236,3 +236,18 @@ def test_many_simulated_gpus(K):
     inst2 = gen.matmul2d(40, M=10, K=K)
     g, o = _both(inst2, smem=-1)
     assert_parity(g, o)
+
+
+def test_hub_datum_64bit_argmax_keys():
+    """A datum used by >= 2^15 tasks disables the packed 32-bit argmax keys
+    (I.key32): the 64-bit (score, u, ~D) path must give the same schedule."""
+    m = 40000
+    rng = np.random.default_rng(3)
+    other = rng.integers(1, 300, size=m)
+    tp = np.arange(0, 2 * m + 1, 2, dtype=np.int64)
+    td = np.empty(2 * m, np.int32)
+    td[0::2] = 0
+    td[1::2] = other
+    inst = gen.Instance("hub", tp, td, np.ones(300, np.uint64), None, 5, 12, 3)
+    g, o = _both(inst, bus=10 ** 9)
+    assert_parity(g, o)

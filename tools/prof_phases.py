@@ -9,16 +9,18 @@ import paper_conf_ipps_gonthiermt22_b200 as dts  # noqa: E402
 
 NAMES = ["pop", "argmax", "plan", "serve_loads", "luf", "evict", "seg_load", "other"]
 cases = [gen.matmul2d(100, M=35, K=4), gen.matmul3d(40, M=142, K=4)]
+blocks = (0, 64, 256)
 if len(sys.argv) > 1 and sys.argv[1] == "big":
-    cases += [gen.config_instances("C4b")[0]]
+    cases = [gen.config_instances("C4a")[0], gen.config_instances("C4b")[0]]
+    blocks = (0,)
 for inst in cases:
-    for block in (0,):
-        for smem in (0, -1):
+    for block in blocks:
+        for smem in (0,):
             dts.schedule(inst, block_threads=block, smem_budget=smem)
             g = dts.schedule(inst, block_threads=block, smem_budget=smem)
             tot = sum(g.prof_cycles[:4]) + g.prof_cycles[7]
             print(f"{inst.name} block={block} smem={smem}: loop {g.loop_ms:.2f} ms, "
-                  f"{g.n_served} dec, {g.n_scans} scans, {g.n_loads} loads, "
+                  f"{g.n_served} dec, {g.n_scans} scans ({g.n_fallback2} fb2, {g.n_fallback_first} fbf), {g.n_loads} loads, "
                   f"{1e6 * g.loop_ms / max(g.n_served, 1):.0f} ns/dec, total_ms {g.total_ms:.2f}")
             print("   cycles/scan: " + ", ".join(
                 f"{n}={c / max(g.n_scans, 1):.0f}" for n, c in zip(NAMES, g.prof_cycles)))
