@@ -157,8 +157,9 @@ typedef struct {
     uint64_t scan_alg_bytes;       /* ... of which in the per-scan pass                       */
     float loop_ms;                 /* device time of the decision-loop kernel (CUDA events)  */
     float total_ms;                /* device time of the whole run (CSR build..assembly)     */
-    int64_t prof_cycles[8];        /* diagnostics: SM cycles of the loop per phase (pop, argmax,
-                                      plan, serve-with-loads, LUF, evict, load-update, other) */
+    int64_t prof_cycles[16];        /* diagnostics: SM cycles of the loop per phase (pop, argmax,
+                                      plan, serve-with-loads, LUF, evict, load-update, other,
+                                      pop-batch warp-0 phase, pop-batch rank phase, #batches, #pops) */
 } dts_result_view;
 
 /* Synchronise on the run's stream, copy the results to host (once) and fill *out. */

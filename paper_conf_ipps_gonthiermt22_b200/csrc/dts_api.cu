@@ -514,11 +514,13 @@ int budget_of(const dts_run_opts &o) {
 // Reuse is ordered on the stream: the H2D copy of a later sweep is enqueued
 // after the previous sweep's kernels on the same stream.
 struct SweepBuf {
-    dts::Inst *d_insts = nullptr;
-    dts::Inst *h_insts = nullptr;  // pinned staging
+    static constexpr int RING = 4;
+    dts::Inst *d_insts = nullptr;        // read by the kernels; reuse is stream-ordered
+    dts::Inst *h_insts[RING] = {};       // pinned staging ring: the host never waits on
+    cudaEvent_t copied[RING] = {};       // the GPU unless it is RING sweeps behind
+    int slot = 0;
     int *d_work = nullptr;
     size_t cap = 0;
-    cudaEvent_t copied = nullptr;   // the last H2D copy out of h_insts
 };
 SweepBuf g_sweep[64];
 
@@ -592,24 +594,26 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
         smem = std::max(smem, insts[i]->h_inst.smem_bytes);
     }
     SweepBuf &B = g_sweep[o.device];
-    if (!B.copied) CK(cudaEventCreateWithFlags(&B.copied, cudaEventDisableTiming), "cudaEventCreate");
-    CK(cudaEventSynchronize(B.copied), "sweep event");
+    if (!B.copied[0])
+        for (auto &e : B.copied) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
     if (B.cap < (size_t)n) {
-        if (B.d_insts) {
-            CK(cudaDeviceSynchronize(), "sync");
-            cudaFree(B.d_insts);
-            cudaFreeHost(B.h_insts);
-        }
+        CK(cudaDeviceSynchronize(), "sync");
+        if (B.d_insts) cudaFree(B.d_insts);
+        for (auto &h : B.h_insts)
+            if (h) cudaFreeHost(h);
         size_t cap = std::max<size_t>((size_t)n, 64);
         CK(cudaMalloc(&B.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
-        CK(cudaMallocHost(&B.h_insts, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
+        for (auto &h : B.h_insts) CK(cudaMallocHost(&h, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
         B.d_work = reinterpret_cast<int *>(B.d_insts + cap);
         B.cap = cap;
     }
-    for (int32_t i = 0; i < n; i++) B.h_insts[i] = insts[i]->h_inst;
-    CK(cudaMemcpyAsync(B.d_insts, B.h_insts, sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
+    const int sl = B.slot;
+    B.slot = (B.slot + 1) % SweepBuf::RING;
+    CK(cudaEventSynchronize(B.copied[sl]), "sweep event");
+    for (int32_t i = 0; i < n; i++) B.h_insts[sl][i] = insts[i]->h_inst;
+    CK(cudaMemcpyAsync(B.d_insts, B.h_insts[sl], sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
        "H2D sweep");
-    CK(cudaEventRecord(B.copied, st), "event");
+    CK(cudaEventRecord(B.copied[sl], st), "event");
     CK(cudaMemsetAsync(B.d_work, 0, sizeof(int), st), "memset");
     CK(dts::launch_init(B.d_insts, n, o.bus_bytes_per_s, work, st), "init");
     int nsm = 0;
@@ -684,7 +688,7 @@ dts_status dts_result(dts_instance *I, dts_result_view *v) {
     v->n_verify_err = I->out.n_verify_err;
     v->alg_bytes = I->out.alg_bytes;
     v->scan_alg_bytes = I->out.scan_alg_bytes;
-    for (int i = 0; i < 8; i++) v->prof_cycles[i] = I->out.prof[i];
+    for (int i = 0; i < 16; i++) v->prof_cycles[i] = I->out.prof[i];
     v->loop_ms = I->loop_ms;
     v->total_ms = I->total_ms;
     return DTS_OK;

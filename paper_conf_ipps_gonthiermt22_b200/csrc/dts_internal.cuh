@@ -52,7 +52,7 @@ struct Out {
     uint64_t alg_bytes, scan_alg_bytes;
     int32_t error;
     int32_t pad;
-    int64_t prof[8];  // SM cycles seen by thread 0 per phase (see PROF_* in dts_loop.cu)
+    int64_t prof[16];  // SM cycles seen by thread 0 per phase (see PROF_* in dts_loop.cu)
 };
 
 // Device descriptor of one instance.

@@ -40,10 +40,19 @@ namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
 
+// CTA barrier that also reconverges each warp.  __syncthreads() alone leaves a
+// warp split after a thread-0-only block (independent thread scheduling), and
+// the split halves then run every later instruction twice and meet again at
+// each full-mask shuffle -- a measured 4x slowdown of the warp-0 phases.
+__device__ __forceinline__ void cta_sync() {
+    __syncthreads();
+    __syncwarp();
+}
+
 enum Cmd : int { CMD_SCAN = 1, CMD_DONE = 2 };
 
 // Per-phase cycle accounting by thread 0 (diagnostics, dts_result_view.prof_cycles).
-enum Prof : int { P_POP = 0, P_ARGMAX, P_PLAN, P_LOADS, P_LUF, P_EVICT, P_SEG, P_OTHER };
+enum Prof : int { P_POP = 0, P_ARGMAX, P_PLAN, P_LOADS, P_LUF, P_EVICT, P_SEG, P_OTHER, P_BW0, P_BD, P_NB, P_NP, P_X1, P_X2, P_X3, P_X4 };
 #define PROF_T0(var) const long long var = (threadIdx.x == 0) ? clock64() : 0
 #define PROF_ADD(L, slot, var) \
     do {                       \
@@ -71,9 +80,9 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     unsigned long long red64b[32];
     int32_t red32[32];
     int32_t wcnt[32];
-    long long prof[8];
-    int64_t bstart[MAX_K], bS[MAX_K];  // pop batch: first start / next scan time per GPU
-    int32_t bcnt[MAX_K], boff[MAX_K + 1];
+    long long prof[16];
+    int64_t bstart[32], breq[32], bns;  // pop batch (K <= 32): per-GPU first start / request
+    int32_t bhead[32], bcnt[32], boff[33];
 };
 
 // Per-instance views: shared-memory arrays where placed, else global homes.
@@ -86,6 +95,13 @@ struct View {
     int64_t *plan_cum;  // inclusive prefix sums of the planned tasks' tau (per-task times only)
     int32_t *dptr32;    // shared-memory copy of dptr, or nullptr
 };
+
+// Per-CTA state at namespace scope, so the (non-inlined) phase functions
+// address it with shared-memory instructions: the leader scalars, this CTA's
+// instance descriptor and its array views.
+__shared__ Lead L;
+__shared__ Inst SI;
+__shared__ View SV;
 
 __device__ __forceinline__ int warp_sum(int v) {
 #pragma unroll
@@ -111,40 +127,44 @@ __device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long v)
 
 // Block reductions (every thread calls; the result is returned to every
 // thread): warp shuffle, one barrier-protected exchange, warp shuffle again.
-__device__ unsigned long long block_max_u64(Lead &L, unsigned long long v) {
+__device__ unsigned long long block_max_u64(unsigned long long v) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     v = warp_max_u64(v);
     if (nw == 1) return v;
-    __syncthreads();
+    cta_sync();
     if (lane == 0) L.red64[w] = v;
-    __syncthreads();
+    cta_sync();
     return warp_max_u64(lane < nw ? L.red64[lane] : 0ull);
 }
-__device__ unsigned long long block_min_u64(Lead &L, unsigned long long v) {
+__device__ unsigned long long block_min_u64(unsigned long long v) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     v = warp_min_u64(v);
     if (nw == 1) return v;
-    __syncthreads();
+    cta_sync();
     if (lane == 0) L.red64[w] = v;
-    __syncthreads();
+    cta_sync();
     return warp_min_u64(lane < nw ? L.red64[lane] : ~0ull);
 }
-__device__ int block_sum(Lead &L, int v) {
+__device__ int block_sum(int v) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     v = warp_sum(v);
     if (nw == 1) return v;
-    __syncthreads();
+    cta_sync();
     if (lane == 0) L.red32[w] = v;
-    __syncthreads();
+    cta_sync();
     return warp_sum(lane < nw ? L.red32[lane] : 0);
 }
 
-__device__ __forceinline__ bool resident(const Inst &I, const View &V, int k, int32_t D) {
+__device__ __forceinline__ bool resident(int k, int32_t D) {
+    const Inst &I = SI;
+    const View &V = SV;
     return (V.resb[(size_t)k * I.nw + (D >> 5)] >> (D & 31)) & 1u;
 }
 
 // Data->task segment bounds of D (int32 copy in shared memory when placed).
-__device__ __forceinline__ void seg_of(const Inst &I, const View &V, int32_t D, int64_t &b, int64_t &e) {
+__device__ __forceinline__ void seg_of(int32_t D, int64_t &b, int64_t &e) {
+    const Inst &I = SI;
+    const View &V = SV;
     if (V.dptr32) {
         b = V.dptr32[D];
         e = V.dptr32[D + 1];
@@ -154,14 +174,17 @@ __device__ __forceinline__ void seg_of(const Inst &I, const View &V, int32_t D, 
     }
 }
 // Size and bus time of D: scalars when all sizes are equal (the paper's model).
-__device__ __forceinline__ uint64_t size_of(const Inst &I, int32_t D) {
+__device__ __forceinline__ uint64_t size_of(int32_t D) {
+    const Inst &I = SI;
     return I.size0 ? I.size0 : __ldg(&I.size[D]);
 }
-__device__ __forceinline__ int64_t delta_of(const Inst &I, int32_t D) {
+__device__ __forceinline__ int64_t delta_of(int32_t D) {
+    const Inst &I = SI;
     return I.size0 ? I.delta0 : __ldg(&I.delta[D]);
 }
 
-__device__ __forceinline__ int64_t tau_of(const Inst &I, int32_t T) {
+__device__ __forceinline__ int64_t tau_of(int32_t T) {
+    const Inst &I = SI;
     return I.tau ? __ldg(&I.tau[T]) : I.default_tau;
 }
 
@@ -171,7 +194,8 @@ struct Row {
     int32_t r0, r1, r2, len;
 };
 
-__device__ __forceinline__ Row row_of_task(const Inst &I, int32_t T) {
+__device__ __forceinline__ Row row_of_task(int32_t T) {
+    const Inst &I = SI;
     const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
     Row r;
     r.len = (int32_t)(re - rb);
@@ -181,28 +205,48 @@ __device__ __forceinline__ Row row_of_task(const Inst &I, int32_t T) {
     return r;
 }
 
-// The (first two) inputs of T not resident on GPU k, skipping `skip`.
-__device__ __forceinline__ void missing_pair(const Inst &I, const View &V, int k, int32_t T, Row r,
-                                             int32_t skip, int32_t &a, int32_t &b) {
+// Rows longer than 3: the (first two) inputs of T not resident on GPU k,
+// skipping `skip`, read from the CSR.
+__device__ __noinline__ void missing_pair_long(int k, int32_t T, int32_t skip, int32_t &a, int32_t &b) {
+    const Inst &I = SI;
     a = -1;
     b = -1;
-    if (r.len <= 3) {
-        const int32_t c[3] = {r.r0, r.r1, r.r2};
-#pragma unroll
-        for (int i = 0; i < 3; i++) {
-            const int32_t D = c[i];
-            if (D < 0 || D == skip || resident(I, V, k, D)) continue;
-            if (a < 0) a = D;
-            else b = D;
-        }
-        return;
-    }
     const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
     for (int64_t i = rb; i < re; i++) {
         const int32_t D = __ldg(&I.tdat[i]);
-        if (D == skip || resident(I, V, k, D)) continue;
+        if (D == skip || resident(k, D)) continue;
         if (a < 0) a = D;
         else if (b < 0) b = D;
+    }
+}
+
+// The (first two) inputs of T not resident on GPU k, skipping `skip`.
+__device__ __forceinline__ void missing_pair(int k, int32_t T, Row r, int32_t skip, int32_t &a, int32_t &b) {
+    if (r.len > 3) {
+        missing_pair_long(k, T, skip, a, b);
+        return;
+    }
+    a = -1;
+    b = -1;
+    const int32_t c[3] = {r.r0, r.r1, r.r2};
+#pragma unroll
+    for (int i = 0; i < 3; i++) {
+        const int32_t D = c[i];
+        if (D < 0 || D == skip || resident(k, D)) continue;
+        if (a < 0) a = D;
+        else b = D;
+    }
+}
+
+// u(D) and np (when plan_k >= 0) of T's inputs for pool_move, long rows.
+__device__ __noinline__ void pool_move_long_row(int32_t T, int sign, int plan_k) {
+    const Inst &I = SI;
+    const View &V = SV;
+    const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+    for (int64_t i = rb; i < re; i++) {
+        const int32_t D = __ldg(&I.tdat[i]);
+        atomicAdd(&V.u[D], sign);
+        if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + D], -sign);
     }
 }
 
@@ -210,45 +254,46 @@ __device__ __forceinline__ void missing_pair(const Inst &I, const View &V, int k
 // tasks (R2, R4): the ALLOC bit in all K state copies, the score buckets of
 // every GPU on which T has one or two missing inputs, u(D) for its inputs,
 // and np_k(D) when it enters / leaves plannedTasks_k (plan_k >= 0).  Called by
-// ONE thread per task; the touched words of s are T's own.  The K state words
-// are loaded together (one round trip), then updated.
-__device__ void pool_move(const Inst &I, const View &V, int32_t T, Row r, int sign, int plan_k) {
-    for (int j0 = 0; j0 < I.K; j0 += 8) {
-        uint32_t w[8];
-#pragma unroll
-        for (int jj = 0; jj < 8; jj++)
-            if (j0 + jj < I.K) w[jj] = V.s[(size_t)(j0 + jj) * I.m_pad + T];
-#pragma unroll
-        for (int jj = 0; jj < 8; jj++) {
+// ONE thread per task; the touched words of s are T's own.  The state words
+// are loaded four at a time (one round trip), then updated by a compact loop
+// (the code stays small: the loop kernel is instruction-cache bound).
+__device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
+    const Inst &I = SI;
+    const View &V = SV;
+    const int K = I.K;
+    for (int j0 = 0; j0 < K; j0 += 4) {
+        uint32_t w0 = 0, w1 = 0, w2 = 0, w3 = 0;
+        w0 = V.s[(size_t)j0 * I.m_pad + T];
+        if (j0 + 1 < K) w1 = V.s[(size_t)(j0 + 1) * I.m_pad + T];
+        if (j0 + 2 < K) w2 = V.s[(size_t)(j0 + 2) * I.m_pad + T];
+        if (j0 + 3 < K) w3 = V.s[(size_t)(j0 + 3) * I.m_pad + T];
+        const int je = K - j0 < 4 ? K - j0 : 4;
+#pragma unroll 1
+        for (int jj = 0; jj < je; jj++) {
+            const uint32_t w = jj == 0 ? w0 : (jj == 1 ? w1 : (jj == 2 ? w2 : w3));
             const int j = j0 + jj;
-            if (j >= I.K) break;
-            V.s[(size_t)j * I.m_pad + T] = sign < 0 ? (w[jj] | ALLOC_BIT) : (w[jj] & ~ALLOC_BIT);
-            const uint32_t c = (w[jj] >> 24) & 0x7fu;
+            V.s[(size_t)j * I.m_pad + T] = sign < 0 ? (w | ALLOC_BIT) : (w & ~ALLOC_BIT);
+            const uint32_t c = (w >> 24) & 0x7fu;
             if (c == 1u) {
-                atomicAdd(&V.h[(size_t)j * I.nstr + (w[jj] & XOR_MASK)], sign);
+                atomicAdd(&V.h[(size_t)j * I.nstr + (w & XOR_MASK)], sign);
             } else if (c == 2u) {
                 int32_t a, b;
-                missing_pair(I, V, j, T, r, -1, a, b);
+                missing_pair(j, T, r, -1, a, b);
                 atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
                 atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
             }
         }
     }
-    if (r.len <= 3) {
-        const int32_t c[3] = {r.r0, r.r1, r.r2};
-#pragma unroll
-        for (int i = 0; i < 3; i++) {
-            if (c[i] < 0) continue;
-            atomicAdd(&V.u[c[i]], sign);
-            if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[i]], -sign);
-        }
+    if (r.len > 3) {
+        pool_move_long_row(T, sign, plan_k);
         return;
     }
-    const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
-    for (int64_t i = rb; i < re; i++) {
-        const int32_t D = __ldg(&I.tdat[i]);
-        atomicAdd(&V.u[D], sign);
-        if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + D], -sign);
+    const int32_t c[3] = {r.r0, r.r1, r.r2};
+#pragma unroll
+    for (int i = 0; i < 3; i++) {
+        if (c[i] < 0) continue;
+        atomicAdd(&V.u[c[i]], sign);
+        if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[i]], -sign);
     }
 }
 
@@ -258,9 +303,11 @@ __device__ void pool_move(const Inst &I, const View &V, int32_t T, Row r, int si
 // the score buckets h (cnt 1) and h2 (cnt 2).  The residency bit of D is
 // already updated.  Each task appears once in the segment, so the state words
 // are plain read-modify-writes; the buckets are atomics.
-__device__ void seg_update(const Inst &I, const View &V, int k, int32_t D, bool load) {
+__device__ void seg_update(int k, int32_t D, bool load) {
+    const Inst &I = SI;
+    const View &V = SV;
     int64_t b, e;
-    seg_of(I, V, D, b, e);
+    seg_of(D, b, e);
     uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int32_t *hk = V.h + (size_t)k * I.nstr;
     int32_t *h2k = V.h2 + (size_t)k * I.nstr;
@@ -282,7 +329,7 @@ __device__ void seg_update(const Inst &I, const View &V, int k, int32_t D, bool 
                 atomicAdd(&hk[o], 1);
             } else if (c == 3u) {  // 3 -> 2: one load away from two data
                 int32_t a2 = ed.y, b2 = ed.z;  // |D(T)| = 3: both others miss
-                if (ed.w > 3) missing_pair(I, V, k, T, Row{-1, -1, -1, ed.w}, -1, a2, b2);
+                if (ed.w > 3) missing_pair(k, T, Row{-1, -1, -1, ed.w}, -1, a2, b2);
                 atomicAdd(&h2k[a2], 1);
                 atomicAdd(&h2k[b2], 1);
             }
@@ -295,7 +342,7 @@ __device__ void seg_update(const Inst &I, const View &V, int k, int32_t D, bool 
                 atomicAdd(&h2k[D], 1);
             } else if (c == 2u) {  // 2 -> 3
                 int32_t a2 = ed.y, b2 = ed.z;  // |D(T)| = 3: both others missed
-                if (ed.w > 3) missing_pair(I, V, k, T, Row{-1, -1, -1, ed.w}, D, a2, b2);
+                if (ed.w > 3) missing_pair(k, T, Row{-1, -1, -1, ed.w}, D, a2, b2);
                 atomicSub(&h2k[a2], 1);
                 atomicSub(&h2k[b2], 1);
             }
@@ -303,8 +350,8 @@ __device__ void seg_update(const Inst &I, const View &V, int k, int32_t D, bool 
     }
 }
 
-__device__ __forceinline__ void push_event(const Inst &I, Lead &L, uint8_t op, int k, int32_t D,
-                                           int32_t T, int64_t t, int64_t te) {
+__device__ __forceinline__ void push_event(uint8_t op, int k, int32_t D, int32_t T, int64_t t, int64_t te) {
+    const Inst &I = SI;
     const int64_t i = L.n_events;
     if (i < I.ev_cap) {
         dts_event ev;
@@ -321,8 +368,8 @@ __device__ __forceinline__ void push_event(const Inst &I, Lead &L, uint8_t op, i
 }
 
 // Thread 0: record the service of T on k (time model of PAPER.md:276-342, R7, R9).
-__device__ __forceinline__ void finish_serve(const Inst &I, Lead &L, int k, int32_t T, int64_t ready,
-                                             int64_t tau) {
+__device__ __forceinline__ void finish_serve(int k, int32_t T, int64_t ready, int64_t tau) {
+    const Inst &I = SI;
     const int64_t start = ready > L.gpu_free[k] ? ready : L.gpu_free[k];
     const int64_t end = start + tau;
     L.gpu_free[k] = end;
@@ -338,7 +385,9 @@ __device__ __forceinline__ void finish_serve(const Inst &I, Lead &L, int k, int3
 
 // Thread 0: pop the smallest planned task of k (Alg. 5 l.2 / l.11, R3); it
 // leaves plannedTasks_k (np_k(D) -= 1 for its inputs).  Returns T and its tau.
-__device__ int32_t pop_planned(const Inst &I, const View &V, Lead &L, int k, int64_t *tau) {
+__device__ int32_t pop_planned(int k, int64_t *tau) {
+    const Inst &I = SI;
+    const View &V = SV;
     const int4 *pl = V.plan + (size_t)k * I.plan_cap;
     int h = L.plan_head[k];
     int4 e = pl[h];
@@ -384,7 +433,9 @@ __device__ int32_t pop_planned(const Inst &I, const View &V, Lead &L, int k, int
 // evicts, Alg. 6 l.8), so serving it is time-model arithmetic.
 // np_k is not maintained by pops: LUF on GPU k only runs while k serves the
 // first task of a new plan (or a fallback task), and every scan resets np_k.
-__device__ int pop_run_seq(const Inst &I, const View &V, Lead &L) {
+__device__ __noinline__ int pop_run_seq() {
+    const Inst &I = SI;
+    const View &V = SV;
     const int K = I.K, W = I.W, pcap = I.plan_cap;
     const int64_t maxs = I.max_served, dtau = I.default_tau;
     int32_t *const sg = I.serve_gpu;
@@ -453,7 +504,7 @@ __device__ int pop_run_seq(const Inst &I, const View &V, Lead &L) {
 
 
 // a[lo..hi) := base + inclusive prefix sums of a[lo..hi).  Block-wide.
-__device__ void block_incl_scan(Lead &L, int64_t *a, int lo, int hi, int64_t base) {
+__device__ __noinline__ void block_incl_scan(int64_t *a, int lo, int hi, int64_t base) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     int64_t carry = base;
     for (int c = lo; c < hi; c += blockDim.x) {
@@ -464,9 +515,9 @@ __device__ void block_incl_scan(Lead &L, int64_t *a, int lo, int hi, int64_t bas
             const int64_t t = __shfl_up_sync(FULL, v, o);
             if (lane >= o) v += t;
         }
-        __syncthreads();
+        cta_sync();
         if (lane == 31) L.red64[w] = (unsigned long long)v;
-        __syncthreads();
+        cta_sync();
         int64_t off = 0, tot = 0;
         for (int j = 0; j < nw; j++) {
             const int64_t x = (int64_t)L.red64[j];
@@ -476,13 +527,15 @@ __device__ void block_incl_scan(Lead &L, int64_t *a, int lo, int hi, int64_t bas
         if (i < hi) a[i] = carry + off + v;
         carry += tot;
     }
-    __syncthreads();
+    cta_sync();
 }
 
 // After LUF removed planned tasks of k (T = -1), close the holes: ordered
 // compaction of [head, end) so the live entries are contiguous (pop_batch
 // indexes them directly), and rebuild their tau prefix sums.  Block-wide.
-__device__ void compact_plan(const Inst &I, const View &V, Lead &L, int k) {
+__device__ __noinline__ void compact_plan(int k) {
+    const Inst &I = SI;
+    const View &V = SV;
     int4 *pl = V.plan + (size_t)k * I.plan_cap;
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
@@ -494,7 +547,7 @@ __device__ void compact_plan(const Inst &I, const View &V, Lead &L, int k) {
         const bool keep = e.x >= 0;
         const unsigned msk = __ballot_sync(FULL, keep);
         if (lane == 0) L.wcnt[w] = __popc(msk);
-        __syncthreads();  // every read of this chunk happened (writes go below its start)
+        cta_sync();  // every read of this chunk happened (writes go below its start)
         int off = out, tot = 0;
         for (int j = 0; j < nw; j++) {
             const int x = L.wcnt[j];
@@ -503,151 +556,184 @@ __device__ void compact_plan(const Inst &I, const View &V, Lead &L, int k) {
         }
         if (keep) pl[off + __popc(msk & lt)] = e;
         out += tot;
-        __syncthreads();
+        cta_sync();
     }
     if (V.plan_cum) {
         int64_t *pc = V.plan_cum + (size_t)k * I.plan_cap;
-        for (int i = ph + threadIdx.x; i < out; i += blockDim.x) pc[i] = tau_of(I, pl[i].x);
-        __syncthreads();
-        block_incl_scan(L, pc, ph, out, ph > 0 ? pc[ph - 1] : 0);
+        for (int i = ph + threadIdx.x; i < out; i += blockDim.x) pc[i] = tau_of(pl[i].x);
+        cta_sync();
+        block_incl_scan(pc, ph, out, ph > 0 ? pc[ph - 1] : 0);
     }
     if (threadIdx.x == 0) L.plan_end[k] = out;
-    __syncthreads();
+    cta_sync();
 }
 
-// Sum of tau over the first c live planned tasks of GPU j (from its head).
-__device__ __forceinline__ int64_t plan_span(const Inst &I, const View &V, const Lead &L, int j, int c) {
+// Sum of tau over the c planned tasks of GPU j starting at plan index h.
+__device__ __forceinline__ int64_t plan_span(int j, int h, int c) {
+    const Inst &I = SI;
+    const View &V = SV;
     if (c <= 0) return 0;
     if (!V.plan_cum) return (int64_t)c * I.default_tau;
     const int64_t *pc = V.plan_cum + (size_t)j * I.plan_cap;
-    const int h = L.plan_head[j];
     return pc[h + c - 1] - (h > 0 ? pc[h - 1] : 0);
 }
 
-// Request time of the i-th pop of GPU j in this batch (W = 0: the GPU asks
-// again when its task ends, R7).
-__device__ __forceinline__ int64_t pop_req(const Inst &I, const View &V, const Lead &L, int j, int i) {
-    return i == 0 ? L.req[j] : L.bstart[j] + plan_span(I, V, L, j, i);
+// Pop batch bookkeeping of GPU j (see pop_batch): its first request time
+// (req), the start of its first pop (start0) and its plan head.  The i-th pop
+// is requested at req (i = 0) or start0 + span(i) (W = 0: a GPU asks again
+// when its task ends, R7).
+struct PopGpu {
+    int64_t req, start0;
+    int head;
+};
+
+__device__ __forceinline__ int64_t pop_req(int j, const PopGpu &g, int i) {
+    return i == 0 ? g.req : g.start0 + plan_span(j, g.head, i);
 }
 
 // #{ i < c : (req_{j,i}, j) < (r, k) } -- the pops of GPU j that precede the
-// event (r, k) in the (time, GPU id) order of requests (R8); binary search.
-__device__ __forceinline__ int pops_before(const Inst &I, const View &V, const Lead &L, int j, int c,
-                                           int64_t r, int k) {
-    int lo = 0, hi = c;  // answer in [lo, hi]
+// request (r, k) in the (time, GPU id) order (R8).  Request times increase
+// with i, so a binary search (multiplications only: 64-bit division is a long
+// software sequence on the SM).
+__device__ int pops_before(int j, PopGpu g, int c, int64_t r, int k) {
+    const Inst &I = SI;
+    const View &V = SV;
+    if (c <= 0) return 0;
+    const bool tie_ok = j < k;  // equal times: the lower GPU id asks first
+    if (!(g.req < r || (g.req == r && tie_ok))) return 0;
+    int lo = 1, hi = c;  // first i in [1, c] whose request does not precede (r, k)
+    if (!V.plan_cum) {
+        const int64_t tau = I.default_tau;
+        while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            const int64_t rm = g.start0 + (int64_t)mid * tau;
+            if (rm < r || (rm == r && tie_ok)) lo = mid + 1;
+            else hi = mid;
+        }
+        return lo;
+    }
     while (lo < hi) {
         const int mid = (lo + hi) >> 1;
-        const int64_t rm = pop_req(I, V, L, j, mid);
-        if (rm < r || (rm == r && j < k)) lo = mid + 1;
+        const int64_t rm = g.start0 + plan_span(j, g.head, mid);
+        if (rm < r || (rm == r && tie_ok)) lo = mid + 1;
         else hi = mid;
     }
     return lo;
 }
 
 // Every request that finds plannedTasks_k non-empty (Alg. 5 l.1-2) up to the
-// next one that finds it empty, served at once by the whole CTA.  Between two
-// scans nothing but pops happens, and a pop only moves time: the popped
-// task's inputs are resident (LUF drops planned tasks whose inputs it evicts,
-// Alg. 6 l.8) and np_k is rebuilt at every scan of k (reset_plan), so each
-// GPU's request times are prefix sums of its planned tasks' tau (PAPER.md:
-// 276-342, W = 0).  The next scan is the earliest (request after the last pop,
-// k) (R8); every pop before it is placed in the global service order by
-// merge ranks.  Sets L.cmd (CMD_SCAN with L.k, L.t, or CMD_DONE).
-__device__ void pop_batch(const Inst &I, const View &V, Lead &L) {
+// next one that finds it empty, served at once.  Between two scans nothing
+// but pops happens, and a pop only moves time: the popped task's inputs are
+// resident (LUF drops planned tasks whose inputs it evicts, Alg. 6 l.8) and
+// np_k is rebuilt at every scan of k (reset_plan), so each GPU's request
+// times are prefix sums of its planned tasks' tau (W = 0).
+// Warp 0 (one lane per simulated GPU, K <= 32) finds the next scan -- the
+// earliest (request after the GPU's last pop, GPU id) (R8) -- and each GPU's
+// pop count before it; then every thread places pops in the global service
+// order by merge ranks.  Sets L.cmd (CMD_SCAN with L.k, L.t, or CMD_DONE).
+__device__ void pop_batch() {
+    const Inst &I = SI;
+    const View &V = SV;
     const int K = I.K;
-    for (int j = threadIdx.x; j < K; j += blockDim.x) {
-        const int live = L.plan_end[j] - L.plan_head[j];
-        const int64_t start0 = L.req[j] > L.gpu_free[j] ? L.req[j] : L.gpu_free[j];
-        L.bstart[j] = start0;
-        L.bS[j] = L.idle[j] ? INT64_MAX : (live == 0 ? L.req[j] : start0 + plan_span(I, V, L, j, live));
-    }
-    __syncthreads();
-    if (threadIdx.x < 32) {  // k* = argmin (S_j, j) over non-idle GPUs
+    PROF_T0(p_w0);
+    if (threadIdx.x == 0) {  // scalar phase: K is small, a serial pass beats warp shuffles
         int kb = -1;
         int64_t sb = INT64_MAX;
-        for (int j = threadIdx.x; j < K; j += 32)
-            if (!L.idle[j] && (kb < 0 || L.bS[j] < sb)) {
+        for (int j = 0; j < K; j++) {  // the next scan: earliest (request after the last pop, j)
+            const int64_t req = L.req[j];
+            const int64_t start0 = req > L.gpu_free[j] ? req : L.gpu_free[j];
+            const int head = L.plan_head[j];
+            L.breq[j] = req;
+            L.bstart[j] = start0;
+            L.bhead[j] = head;
+            if (L.idle[j]) continue;
+            const int live = L.plan_end[j] - head;
+            const int64_t S = live == 0 ? req : start0 + plan_span(j, head, live);
+            if (kb < 0 || S < sb) {
                 kb = j;
-                sb = L.bS[j];
-            }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            const int ko = __shfl_xor_sync(FULL, kb, o);
-            const int64_t so = __shfl_xor_sync(FULL, sb, o);
-            if (ko >= 0 && (kb < 0 || so < sb || (so == sb && ko < kb))) {
-                kb = ko;
-                sb = so;
+                sb = S;
             }
         }
-        if (threadIdx.x == 0) {
-            L.k = kb;
-            L.t = sb;
-            L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
-        }
-    }
-    __syncthreads();
-    const int ks = L.k;
-    const int64_t ts = L.t;
-    if (ks < 0) return;
-    for (int j = threadIdx.x; j < K; j += blockDim.x) {
-        const int live = L.plan_end[j] - L.plan_head[j];
-        L.bcnt[j] = L.idle[j] ? 0 : (j == ks ? live : pops_before(I, V, L, j, live, ts, ks));
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int run = 0;
+        L.prof[P_X2] += clock64() - p_w0;
+        int total = 0;
+        int64_t mk = L.makespan;
         for (int j = 0; j < K; j++) {
-            L.boff[j] = run;
-            run += L.bcnt[j];
+            int c = 0;
+            if (!L.idle[j] && kb >= 0) {
+                const int live = L.plan_end[j] - L.bhead[j];
+                PopGpu g;
+                g.req = L.breq[j];
+                g.start0 = L.bstart[j];
+                g.head = L.bhead[j];
+                c = j == kb ? live : pops_before(j, g, live, sb, kb);
+            }
+            L.bcnt[j] = c;
+            L.boff[j] = total;
+            total += c;
+            if (c > 0) {
+                const int64_t last = L.bstart[j] + plan_span(j, L.bhead[j], c);
+                L.req[j] = last;  // W = 0 (R7)
+                L.gpu_free[j] = last;
+                L.plan_head[j] += c;
+                L.plan_live[j] -= c;
+                mk = last > mk ? last : mk;
+            }
         }
-        L.boff[K] = run;
+        L.prof[P_X4] += clock64() - p_w0;
+        L.boff[K] = total;
+        L.bns = L.n_served;
+        L.n_served += total;
+        L.makespan = mk;
+        L.alg_bytes += 24ull * (uint64_t)total;
+        L.k = kb;
+        L.t = sb;
+        L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
     }
-    __syncthreads();
+    cta_sync();
+    PROF_ADD(L, P_BW0, p_w0);
+    PROF_T0(p_bd);
     const int P = L.boff[K];
-    const int64_t ns = L.n_served;
-    int64_t mk = 0;
-    int32_t *const sg = I.serve_gpu;
-    int32_t *const stk = I.serve_task;
+    const int64_t ns = L.bns;
+    if (threadIdx.x == 0) {
+        L.prof[P_NB] += 1;
+        L.prof[P_NP] += P;
+    }
     for (int p = threadIdx.x; p < P; p += blockDim.x) {
         int j = 0;
         while (L.boff[j + 1] <= p) j++;
         const int i = p - L.boff[j];
-        const int64_t r = pop_req(I, V, L, j, i);
-        const int64_t start = i == 0 ? L.bstart[j] : r;
-        const int64_t end = L.bstart[j] + plan_span(I, V, L, j, i + 1);
-        const int T = V.plan[(size_t)j * I.plan_cap + L.plan_head[j] + i].x;
+        PopGpu g;
+        g.req = L.breq[j];
+        g.start0 = L.bstart[j];
+        g.head = L.bhead[j];
+        const int64_t r = pop_req(j, g, i);
+        const int64_t start = i == 0 ? g.start0 : r;
+        const int64_t end = g.start0 + plan_span(j, g.head, i + 1);
+        const int T = V.plan[(size_t)j * I.plan_cap + g.head + i].x;
         int64_t pos = ns + i;
-        for (int j2 = 0; j2 < K; j2++)
-            if (j2 != j && L.bcnt[j2] > 0) pos += pops_before(I, V, L, j2, L.bcnt[j2], r, j);
+        for (int j2 = 0; j2 < K; j2++) {
+            if (j2 == j) continue;
+            PopGpu g2;
+            g2.req = L.breq[j2];
+            g2.start0 = L.bstart[j2];
+            g2.head = L.bhead[j2];
+            pos += pops_before(j2, g2, L.bcnt[j2], r, j);
+        }
         __stcg(&I.tstart[T], start);
         __stcg(&I.tend[T], end);
-        __stcg(&sg[pos], j);
-        __stcg(&stk[pos], T);
-        mk = end > mk ? end : mk;
+        __stcg(&I.serve_gpu[pos], j);
+        __stcg(&I.serve_task[pos], T);
     }
-    mk = (int64_t)block_max_u64(L, (unsigned long long)mk);
-    for (int j = threadIdx.x; j < K; j += blockDim.x) {
-        const int c = L.bcnt[j];
-        if (c > 0) {
-            const int64_t end = L.bstart[j] + plan_span(I, V, L, j, c);
-            L.req[j] = end;  // W = 0 (R7)
-            L.gpu_free[j] = end;
-            L.plan_head[j] += c;
-            L.plan_live[j] -= c;
-        }
-    }
-    if (threadIdx.x == 0) {
-        L.n_served = ns + P;
-        if (mk > L.makespan) L.makespan = mk;
-        L.alg_bytes += 24ull * (uint64_t)P;
-    }
-    __syncthreads();
+    cta_sync();
+    PROF_ADD(L, P_BD, p_bd);
 }
 
 // CTA-wide, at every scan of GPU k: plannedTasks_k is empty (all popped or
 // removed); clear np_k for every datum its last plan touched, so that np_k
 // counts exactly the plan this scan creates (Alg. 6 l.3).
-__device__ void reset_plan(const Inst &I, const View &V, Lead &L, int k) {
+__device__ void reset_plan(int k) {
+    const Inst &I = SI;
+    const View &V = SV;
     const int4 *pl = V.plan + (size_t)k * I.plan_cap;
     int32_t *npk = V.np + (size_t)k * I.nstr;
     const int pe = L.plan_end[k];
@@ -665,13 +751,13 @@ __device__ void reset_plan(const Inst &I, const View &V, Lead &L, int k) {
             }
         }
     }
-    __syncthreads();
+    cta_sync();
     if (threadIdx.x == 0) {
         L.plan_head[k] = 0;
         L.plan_end[k] = 0;
         L.plan_live[k] = 0;
     }
-    __syncthreads();
+    cta_sync();
 }
 
 __device__ __forceinline__ Row row_of_entry(int4 e) {
@@ -679,7 +765,8 @@ __device__ __forceinline__ Row row_of_entry(int4 e) {
     return Row{e.y, e.z, e.w, (e.y >= 0) + (e.z >= 0) + (e.w >= 0)};
 }
 
-__device__ __forceinline__ bool entry_uses(const Inst &I, int4 e, int32_t D) {
+__device__ __forceinline__ bool entry_uses(int4 e, int32_t D) {
+    const Inst &I = SI;
     if (e.y == D || e.z == D) return true;
     if (e.w != ROW_LONG) return e.w == D;
     const int64_t rb = __ldg(&I.tptr[e.x]), re = __ldg(&I.tptr[e.x + 1]);
@@ -693,7 +780,9 @@ __device__ __forceinline__ bool entry_uses(const Inst &I, int4 e, int32_t D) {
 // the one with the fewest uses in plannedTasks_k, lowest id on ties (R1).
 // Block-wide; returns V (or -1: the Belady branch, unreachable, R7) and sets
 // L.vslot to its index in res_list.
-__device__ int32_t luf_victim(const Inst &I, const View &V, Lead &L, int k) {
+__device__ int32_t luf_victim(int k) {
+    const Inst &I = SI;
+    const View &V = SV;
     const int cnt = L.res_cnt[k];
     const int32_t *rl = V.res_list + (size_t)k * I.res_cap;
     const int32_t *npk = V.np + (size_t)k * I.nstr;
@@ -707,34 +796,35 @@ __device__ int32_t luf_victim(const Inst &I, const View &V, Lead &L, int k) {
             ((unsigned long long)(uint32_t)npk[D] << 32) | (unsigned long long)(uint32_t)D;
         best = key < best ? key : best;
     }
-    best = block_min_u64(L, best);
+    best = block_min_u64(best);
     if (best == ~0ull) return -1;
     const int32_t Vd = (int32_t)(best & 0xffffffffull);
     for (int i = threadIdx.x; i < cnt; i += blockDim.x)
         if (rl[i] == Vd) L.vslot = i;
-    __syncthreads();
+    cta_sync();
     return Vd;
 }
 
 // Alg. 6 l.8-9: planned tasks of k that use V return to the shared pool (R4,
 // idle GPUs wake at t, R18); then V leaves GPU k's memory.  Block-wide.
-__device__ void evict(const Inst &I, const View &V, Lead &L, int k, int32_t Vd, int32_t Tserved,
-                      int64_t t) {
+__device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
+    const Inst &I = SI;
+    const View &V = SV;
     int4 *pl = V.plan + (size_t)k * I.plan_cap;
     int nret = 0;
     unsigned long long tmin = ~0ull;
     const int ph = L.plan_head[k], pe = L.plan_end[k];
     for (int i = ph + threadIdx.x; i < pe; i += blockDim.x) {
         const int4 e = pl[i];
-        if (e.x >= 0 && entry_uses(I, e, Vd)) {
+        if (e.x >= 0 && entry_uses(e, Vd)) {
             pl[i].x = -1;
-            pool_move(I, V, e.x, row_of_entry(e), +1, k);
+            pool_move(e.x, row_of_entry(e), +1, k);
             nret++;
             tmin = (unsigned long long)e.x < tmin ? (unsigned long long)e.x : tmin;
         }
     }
-    nret = block_sum(L, nret);
-    tmin = block_min_u64(L, tmin);
+    nret = block_sum(nret);
+    tmin = block_min_u64(tmin);
     if (threadIdx.x == 0) {
         if (nret > 0) {
             L.plan_live[k] -= nret;
@@ -751,47 +841,49 @@ __device__ void evict(const Inst &I, const View &V, Lead &L, int k, int32_t Vd, 
         rl[L.vslot] = rl[last];
         L.res_cnt[k] = last;
         V.resb[(size_t)k * I.nw + (Vd >> 5)] &= ~(1u << (Vd & 31));
-        L.used[k] -= size_of(I, Vd);
+        L.used[k] -= size_of(Vd);
         L.n_evictions++;
-        push_event(I, L, 1, k, Vd, Tserved, t, t);
+        push_event(1, k, Vd, Tserved, t, t);
         int64_t sb, se;
-        seg_of(I, V, Vd, sb, se);
-        L.alg_bytes += 20ull * (uint64_t)(se - sb) + (uint64_t)nret * (8ull * I.K + 32ull);
+        seg_of(Vd, sb, se);
+        L.alg_bytes += 24ull * (uint64_t)(se - sb) + (uint64_t)nret * (8ull * I.K + 40ull) + 32ull;
     }
-    __syncthreads();
-    if (nret > 0) compact_plan(I, V, L, k);
-    seg_update(I, V, k, Vd, false);
-    __syncthreads();
+    cta_sync();
+    if (nret > 0) compact_plan(k);
+    seg_update(k, Vd, false);
+    cta_sync();
 }
 
 // Serve T on GPU k at time t with loads: evict V(k,i), load the missing inputs
 // in ascending id (R10), process; shared FIFO bus (R9).
 // Block-wide.  L.row holds D(T).
-__device__ void serve_loads(const Inst &I, const View &V, Lead &L, int k, int32_t T, int64_t t) {
+__device__ void serve_loads(int k, int32_t T, int64_t t) {
+    const Inst &I = SI;
+    const View &V = SV;
     if (threadIdx.x == 0) L.ready = t;
-    __syncthreads();
+    cta_sync();
     const int len = L.row_len;
     for (int r = 0; r < len; r++) {
         // every thread reads the shared state before thread 0 may change it
         const int32_t D = L.row[r];
-        const bool res = resident(I, V, k, D);
-        __syncthreads();
+        const bool res = resident(k, D);
+        cta_sync();
         if (res) continue;
-        const uint64_t sz = size_of(I, D);
+        const uint64_t sz = size_of(D);
         while (true) {  // R11: LUF until D fits
             const bool full = L.used[k] + sz > I.cap;
-            __syncthreads();
+            cta_sync();
             if (!full) break;
             PROF_T0(p_luf);
-            const int32_t Vd = luf_victim(I, V, L, k);
+            const int32_t Vd = luf_victim(k);
             PROF_ADD(L, P_LUF, p_luf);
             if (Vd < 0) {
                 if (threadIdx.x == 0) L.error = 1;
-                __syncthreads();
+                cta_sync();
                 return;
             }
             PROF_T0(p_ev);
-            evict(I, V, L, k, Vd, T, t);
+            evict(k, Vd, T, t);
             PROF_ADD(L, P_EVICT, p_ev);
         }
         if (threadIdx.x == 0) {
@@ -800,24 +892,24 @@ __device__ void serve_loads(const Inst &I, const View &V, Lead &L, int k, int32_
             V.resb[(size_t)k * I.nw + (D >> 5)] |= 1u << (D & 31);
             L.used[k] += sz;
             const int64_t st = L.bus_free > t ? L.bus_free : t;
-            const int64_t en = st + delta_of(I, D);
+            const int64_t en = st + delta_of(D);
             L.bus_free = en;
             if (en > L.ready) L.ready = en;
             L.n_loads++;
             L.bytes_loaded += sz;
-            push_event(I, L, 0, k, D, T, st, en);
+            push_event(0, k, D, T, st, en);
             int64_t sb, se;
-            seg_of(I, V, D, sb, se);
-            L.alg_bytes += 20ull * (uint64_t)(se - sb);
+            seg_of(D, sb, se);
+            L.alg_bytes += 24ull * (uint64_t)(se - sb) + 32ull;
         }
-        __syncthreads();
+        cta_sync();
         PROF_T0(p_seg);
-        seg_update(I, V, k, D, true);
-        __syncthreads();
+        seg_update(k, D, true);
+        cta_sync();
         PROF_ADD(L, P_SEG, p_seg);
     }
-    if (threadIdx.x == 0) finish_serve(I, L, k, T, L.ready, tau_of(I, T));
-    __syncthreads();
+    if (threadIdx.x == 0) finish_serve(k, T, L.ready, tau_of(T));
+    cta_sync();
 }
 
 // Alg. 5 l.6-9 (and the 3inputs fallback): block argmax
@@ -830,15 +922,35 @@ __device__ void serve_loads(const Inst &I, const View &V, Lead &L, int k, int32_
 // into one 32-bit key score << 16 | u, and since each thread visits D in
 // increasing order a strict '>' keeps the lowest id among equal keys; the
 // 64-bit (key, ~D) is formed once per thread for the block reduction.
-__device__ int32_t score_argmax(const Inst &I, const View &V, Lead &L, const int32_t *score) {
+// The thread's best 64-bit key (score, u, ~D) when scores may reach 2^15.
+__device__ __noinline__ unsigned long long score_best64(const int32_t *score) {
+    const Inst &I = SI;
+    const View &V = SV;
+    const unsigned ib = (unsigned)I.id_bits, ub = (unsigned)I.u_bits;
+    const unsigned long long idmask = (1ull << ib) - 1ull;
+    unsigned long long best = 0ull;
+    for (int D = threadIdx.x; D < I.n; D += blockDim.x) {
+        const int32_t sc = score[D];
+        if (sc <= 0) continue;
+        const unsigned long long key = ((unsigned long long)(uint32_t)sc << (ub + ib)) |
+                                       ((unsigned long long)(uint32_t)V.u[D] << ib) |
+                                       (idmask - (unsigned long long)D);
+        best = key > best ? key : best;
+    }
+    return best;
+}
+
+__device__ int32_t score_argmax(const int32_t *score) {
+    const Inst &I = SI;
+    const View &V = SV;
     const unsigned ib = (unsigned)I.id_bits;
     const unsigned long long idmask = (1ull << ib) - 1ull;
-    const int4 *h4 = reinterpret_cast<const int4 *>(score);
-    const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
-    const int nv = I.nstr >> 2;
-    constexpr int UN = 4;
     unsigned long long best = 0ull;
     if (I.key32) {
+        const int4 *h4 = reinterpret_cast<const int4 *>(score);
+        const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
+        const int nv = I.nstr >> 2;
+        constexpr int UN = 2;
         uint32_t bk = 0u;
         int32_t bd = 0;
         for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
@@ -865,40 +977,19 @@ __device__ int32_t score_argmax(const Inst &I, const View &V, Lead &L, const int
         if (bk >= 65536u)  // positive score
             best = ((unsigned long long)bk << ib) | (idmask - (unsigned long long)bd);
     } else {
-        const unsigned ub = (unsigned)I.u_bits;
-        for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
-            int4 hv[UN], uv[UN];
-#pragma unroll
-            for (int q = 0; q < UN; q++) {
-                const int v = v0 + q * blockDim.x;
-                hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
-                uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
-            }
-#pragma unroll
-            for (int q = 0; q < UN; q++) {
-                const int D = 4 * (v0 + q * blockDim.x);
-                const int32_t sc[4] = {hv[q].x, hv[q].y, hv[q].z, hv[q].w};
-                const int32_t uu[4] = {uv[q].x, uv[q].y, uv[q].z, uv[q].w};
-#pragma unroll
-                for (int c = 0; c < 4; c++) {
-                    if (sc[c] <= 0) continue;
-                    const unsigned long long key = ((unsigned long long)(uint32_t)sc[c] << (ub + ib)) |
-                                                   ((unsigned long long)(uint32_t)uu[c] << ib) |
-                                                   (idmask - (unsigned long long)(D + c));
-                    best = key > best ? key : best;
-                }
-            }
-        }
+        best = score_best64(score);
     }
-    best = block_max_u64(L, best);
+    best = block_max_u64(best);
     return best ? (int32_t)(idmask - (best & idmask)) : -1;
 }
 
 // Alg. 5 l.10: plannedTasks_k <- unallocated tasks of Dopt's segment with one
 // missing input (= Dopt), ascending id (ordered block compaction).  Block-wide.
-__device__ void plan(const Inst &I, const View &V, Lead &L, int k, int32_t Dopt) {
+__device__ void plan(int k, int32_t Dopt) {
+    const Inst &I = SI;
+    const View &V = SV;
     int64_t b, e;
-    seg_of(I, V, Dopt, b, e);
+    seg_of(Dopt, b, e);
     const uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int4 *pl = V.plan + (size_t)k * I.plan_cap;
     int64_t *pt = V.plan_cum ? V.plan_cum + (size_t)k * I.plan_cap : nullptr;
@@ -917,7 +1008,7 @@ __device__ void plan(const Inst &I, const View &V, Lead &L, int k, int32_t Dopt)
         }
         const unsigned msk = __ballot_sync(FULL, sel);
         if (lane == 0) L.wcnt[w] = __popc(msk);
-        __syncthreads();
+        cta_sync();
         int off = base_out, tot = 0;
         for (int j = 0; j < nw; j++) {
             const int c = L.wcnt[j];
@@ -928,27 +1019,29 @@ __device__ void plan(const Inst &I, const View &V, Lead &L, int k, int32_t Dopt)
             const int pos = off + __popc(msk & lt);
             const Row r = ed.w > 3 ? Row{-1, -1, -1, ed.w} : Row{Dopt, ed.y, ed.z, ed.w};
             pl[pos] = make_int4(T, Dopt, ed.y, ed.w > 3 ? ROW_LONG : ed.z);
-            if (pt) pt[pos] = tau_of(I, T);
-            pool_move(I, V, T, r, -1, k);
+            if (pt) pt[pos] = tau_of(T);
+            pool_move(T, r, -1, k);
         }
         base_out += tot;
-        __syncthreads();
+        cta_sync();
     }
-    if (pt) block_incl_scan(L, pt, 0, base_out, 0);  // tau -> prefix sums
+    if (pt) block_incl_scan(pt, 0, base_out, 0);  // tau -> prefix sums
     if (threadIdx.x == 0) {
         L.plan_head[k] = 0;
         L.plan_end[k] = base_out;
         L.plan_live[k] = base_out;
         L.n_avail -= base_out;
-        L.alg_bytes += 8ull * (uint64_t)(e - b) + (uint64_t)base_out * (8ull * I.K + 48ull);
+        L.alg_bytes += 20ull * (uint64_t)(e - b) + (uint64_t)base_out * (8ull * I.K + 40ull);
     }
-    __syncthreads();
+    cta_sync();
 }
 
 // 3inputs: the lowest-id unallocated task of D2's segment with two missing inputs.
-__device__ int32_t first_cnt2(const Inst &I, const View &V, Lead &L, int k, int32_t D2) {
+__device__ __noinline__ int32_t first_cnt2(int k, int32_t D2) {
+    const Inst &I = SI;
+    const View &V = SV;
     int64_t b, e;
-    seg_of(I, V, D2, b, e);
+    seg_of(D2, b, e);
     const uint32_t *sk = V.s + (size_t)k * I.m_pad;
     for (int64_t base = b; base < e; base += blockDim.x) {
         const int64_t i = base + threadIdx.x;
@@ -957,19 +1050,21 @@ __device__ int32_t first_cnt2(const Inst &I, const View &V, Lead &L, int k, int3
             const int32_t T = __ldg(&I.dedge[i]).x;
             if ((sk[T] >> 24) == 2u) c = (unsigned long long)T;
         }
-        c = block_min_u64(L, c);
+        c = block_min_u64(c);
         if (c != ~0ull) return (int32_t)c;
     }
     return -1;
 }
 
 // Alg. 5 l.13 (R5): the lowest-id unallocated task, scanning up from avail_lo.
-__device__ int32_t first_avail(const Inst &I, const View &V, Lead &L) {
+__device__ __noinline__ int32_t first_avail() {
+    const Inst &I = SI;
+    const View &V = SV;
     for (int64_t base = L.avail_lo; base < I.m; base += blockDim.x) {
         const int64_t T = base + threadIdx.x;
         unsigned long long c = ~0ull;
         if (T < I.m && !(V.s[T] & ALLOC_BIT)) c = (unsigned long long)T;
-        c = block_min_u64(L, c);
+        c = block_min_u64(c);
         if (c != ~0ull) return (int32_t)c;
     }
     return -1;
@@ -978,10 +1073,12 @@ __device__ int32_t first_avail(const Inst &I, const View &V, Lead &L) {
 // DTS_F_VERIFY (P9): recompute n_k(D), n2_k(D), u(D) and cnt_k(T) from their
 // definitions -- the full non-incremental pass of Alg. 5 l.4-5 -- and count
 // mismatches against the incremental state.
-__device__ void verify_scores(const Inst &I, const View &V, Lead &L, int k) {
+__device__ __noinline__ void verify_scores(int k) {
+    const Inst &I = SI;
+    const View &V = SV;
     int32_t *vh = I.vhist, *vh2 = I.vhist + I.n, *vu = I.vhist + 2 * I.n;
     for (int D = threadIdx.x; D < 3 * I.n; D += blockDim.x) vh[D] = 0;
-    __syncthreads();
+    cta_sync();
     const uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int bad = 0;
     for (int T = threadIdx.x; T < I.m; T += blockDim.x) {
@@ -991,37 +1088,38 @@ __device__ void verify_scores(const Inst &I, const View &V, Lead &L, int k) {
         uint32_t x = 0;
         for (int64_t i = rb; i < re; i++) {
             const int32_t D = __ldg(&I.tdat[i]);
-            if (!resident(I, V, k, D)) c++, x ^= (uint32_t)D;
+            if (!resident(k, D)) c++, x ^= (uint32_t)D;
         }
         bad += (c != (int)((w >> 24) & 0x7fu)) || (x != (w & XOR_MASK));
         if (w & ALLOC_BIT) continue;
         for (int64_t i = rb; i < re; i++) {
             const int32_t D = __ldg(&I.tdat[i]);
             atomicAdd(&vu[D], 1);
-            if (c == 2 && !resident(I, V, k, D)) atomicAdd(&vh2[D], 1);
+            if (c == 2 && !resident(k, D)) atomicAdd(&vh2[D], 1);
         }
         if (c == 1) atomicAdd(&vh[x], 1);
     }
-    __syncthreads();
+    cta_sync();
     for (int D = threadIdx.x; D < I.n; D += blockDim.x)
         bad += (__ldcg(&vh[D]) != V.h[(size_t)k * I.nstr + D]) +
                (__ldcg(&vh2[D]) != V.h2[(size_t)k * I.nstr + D]) + (__ldcg(&vu[D]) != V.u[D]);
-    bad = block_sum(L, bad);
+    bad = block_sum(bad);
     if (threadIdx.x == 0) L.n_verr += bad;
-    __syncthreads();
+    cta_sync();
 }
 
 // a8: sigma(k, .) for every k -- stable partition of the service sequence by GPU.
-__device__ void assemble(const Inst &I, int64_t ns) {
+__device__ __noinline__ void assemble(int64_t ns) {
+    const Inst &I = SI;
     __shared__ unsigned long long off[MAX_K];
     __shared__ int tot[MAX_K];
     __shared__ int wk[32][MAX_K];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
     for (int k = threadIdx.x; k < MAX_K; k += blockDim.x) off[k] = 0;
-    __syncthreads();
+    cta_sync();
     for (int64_t i = threadIdx.x; i < ns; i += blockDim.x) atomicAdd(&off[I.serve_gpu[i]], 1ull);
-    __syncthreads();
+    cta_sync();
     if (threadIdx.x == 0) {
         unsigned long long run = 0;
         for (int k = 0; k < I.K; k++) {
@@ -1032,15 +1130,15 @@ __device__ void assemble(const Inst &I, int64_t ns) {
         }
         I.gpu_task_ptr[I.K] = (int64_t)run;
     }
-    __syncthreads();
+    cta_sync();
     for (int64_t base = 0; base < ns; base += blockDim.x) {
         for (int j = threadIdx.x; j < nw * MAX_K; j += blockDim.x) wk[j / MAX_K][j % MAX_K] = 0;
-        __syncthreads();
+        cta_sync();
         const int64_t i = base + threadIdx.x;
         const int k = i < ns ? I.serve_gpu[i] : -1;
         const unsigned peers = __match_any_sync(FULL, k);
         if (k >= 0 && lane == __ffs(peers) - 1) wk[w][k] = __popc(peers);
-        __syncthreads();
+        cta_sync();
         for (int kk = threadIdx.x; kk < I.K; kk += blockDim.x) {  // exclusive prefix over warps
             int run = 0;
             for (int ww = 0; ww < nw; ww++) {
@@ -1050,11 +1148,11 @@ __device__ void assemble(const Inst &I, int64_t ns) {
             }
             tot[kk] = run;
         }
-        __syncthreads();
+        cta_sync();
         if (k >= 0) I.gpu_task_ids[off[k] + wk[w][k] + __popc(peers & lt)] = I.serve_task[i];
-        __syncthreads();
+        cta_sync();
         for (int kk = threadIdx.x; kk < I.K; kk += blockDim.x) off[kk] += tot[kk];
-        __syncthreads();
+        cta_sync();
     }
 }
 
@@ -1064,30 +1162,32 @@ __device__ void assemble(const Inst &I, int64_t ns) {
 __global__ void __launch_bounds__(512, 1)
     dts_cta_kernel(const Inst *__restrict__ insts, int n_inst, int *work_counter) {
     extern __shared__ __align__(16) unsigned char dsm[];
-    __shared__ Lead L;
-    __shared__ Inst SI;  // this CTA's instance descriptor, read at smem latency
     __shared__ int sh_inst;
     const int tid = threadIdx.x;
 
     while (true) {
         if (tid == 0) sh_inst = atomicAdd(work_counter, 1);
-        __syncthreads();
+        cta_sync();
         const int ii = sh_inst;
         if (ii >= n_inst) break;
         if (tid == 0) SI = insts[ii];
-        __syncthreads();
+        cta_sync();
         const Inst &I = SI;
-        View V;
-        V.s = I.so_s >= 0 ? (uint32_t *)(dsm + I.so_s) : I.s;
-        V.u = I.so_u >= 0 ? (int32_t *)(dsm + I.so_u) : I.u;
-        V.h = I.so_h >= 0 ? (int32_t *)(dsm + I.so_h) : I.h;
-        V.h2 = I.so_h2 >= 0 ? (int32_t *)(dsm + I.so_h2) : I.h2;
-        V.np = I.so_np >= 0 ? (int32_t *)(dsm + I.so_np) : I.np;
-        V.resb = I.so_resb >= 0 ? (uint32_t *)(dsm + I.so_resb) : I.resb;
-        V.res_list = I.so_res_list >= 0 ? (int32_t *)(dsm + I.so_res_list) : I.res_list;
-        V.plan = I.so_plan >= 0 ? (int4 *)(dsm + I.so_plan) : I.plan;
-        V.plan_cum = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
-        V.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
+        if (tid == 0) {
+            View &W = SV;
+            W.s = I.so_s >= 0 ? (uint32_t *)(dsm + I.so_s) : I.s;
+            W.u = I.so_u >= 0 ? (int32_t *)(dsm + I.so_u) : I.u;
+            W.h = I.so_h >= 0 ? (int32_t *)(dsm + I.so_h) : I.h;
+            W.h2 = I.so_h2 >= 0 ? (int32_t *)(dsm + I.so_h2) : I.h2;
+            W.np = I.so_np >= 0 ? (int32_t *)(dsm + I.so_np) : I.np;
+            W.resb = I.so_resb >= 0 ? (uint32_t *)(dsm + I.so_resb) : I.resb;
+            W.res_list = I.so_res_list >= 0 ? (int32_t *)(dsm + I.so_res_list) : I.res_list;
+            W.plan = I.so_plan >= 0 ? (int4 *)(dsm + I.so_plan) : I.plan;
+            W.plan_cum = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
+            W.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
+        }
+        cta_sync();
+        const View &V = SV;
 
         // ---- CTA-local copies of the initial state (global homes were
         //      initialised by dts_init_kernel)
@@ -1127,35 +1227,35 @@ __global__ void __launch_bounds__(512, 1)
             L.avail_lo = 0;
             L.error = 0;
             L.row_len = 0;
-            for (int i = 0; i < 8; i++) L.prof[i] = 0;
+            for (int i = 0; i < 16; i++) L.prof[i] = 0;
         }
-        __syncthreads();
+        cta_sync();
 
         // ---- the decision loop
         while (true) {
             PROF_T0(p_pop);
             int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
             for (int j = 0; j < K; j++) pending += L.plan_live[j];
-            if (I.max_served < 0 && pending > 16) {
-                pop_batch(I, V, L);
+            if (I.max_served < 0 && K <= 32 && pending > 10) {
+                pop_batch();
             } else {  // few pops (or a prefix run that stops at an exact count): thread 0
-                __syncthreads();
+                cta_sync();
                 if (tid == 0)
-                    L.cmd = ((I.max_served < 0 || L.n_served < I.max_served) && pop_run_seq(I, V, L) >= 0)
+                    L.cmd = ((I.max_served < 0 || L.n_served < I.max_served) && pop_run_seq() >= 0)
                                 ? CMD_SCAN
                                 : CMD_DONE;
             }
             PROF_ADD(L, P_POP, p_pop);
-            __syncthreads();
+            cta_sync();
             if (L.cmd == CMD_DONE) break;
             const int k = L.k;
             const int64_t t = L.t;
-            reset_plan(I, V, L, k);
-            if (I.flags & DTS_F_VERIFY) verify_scores(I, V, L, k);
+            reset_plan(k);
+            if (I.flags & DTS_F_VERIFY) verify_scores(k);
             // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
             int32_t T = -1;
             PROF_T0(p_am);
-            const int32_t Dopt = score_argmax(I, V, L, V.h + (size_t)k * I.nstr);
+            const int32_t Dopt = score_argmax(V.h + (size_t)k * I.nstr);
             PROF_ADD(L, P_ARGMAX, p_am);
             PROF_T0(p_pl);
             if (tid == 0) {
@@ -1163,25 +1263,29 @@ __global__ void __launch_bounds__(512, 1)
                 L.alg_bytes += 8ull * (uint64_t)n;
             }
             if (Dopt >= 0) {
-                plan(I, V, L, k, Dopt);
+                plan(k, Dopt);
                 if (tid == 0) {
                     int64_t tau;
-                    L.T = pop_planned(I, V, L, k, &tau);
+                    L.T = pop_planned(k, &tau);
                     L.n_scans++;
                 }
-                __syncthreads();
+                cta_sync();
                 T = L.T;
                 PROF_ADD(L, P_PLAN, p_pl);
             } else {
                 if (I.flags & DTS_F_FALLBACK2) {
-                    const int32_t D2 = score_argmax(I, V, L, V.h2 + (size_t)k * I.nstr);
+                    const int32_t D2 = score_argmax(V.h2 + (size_t)k * I.nstr);
+                    if (tid == 0) {
+                        L.scan_alg_bytes += 8ull * (uint64_t)n;
+                        L.alg_bytes += 8ull * (uint64_t)n;
+                    }
                     if (D2 >= 0) {
-                        T = first_cnt2(I, V, L, k, D2);
+                        T = first_cnt2(k, D2);
                         if (tid == 0) L.n_fb2++;
                     }
                 }
                 if (T < 0 && L.n_avail > 0) {
-                    T = first_avail(I, V, L);
+                    T = first_avail();
                     if (tid == 0) {
                         L.n_fbf++;
                         L.avail_lo = T;
@@ -1190,7 +1294,7 @@ __global__ void __launch_bounds__(512, 1)
                 if (T >= 0) {
                     if (tid == 0) {
                         L.row_len = -1;
-                        pool_move(I, V, T, row_of_task(I, T), -1, -1);
+                        pool_move(T, row_of_task(T), -1, -1);
                         L.n_avail--;
                         L.n_scans++;
                     }
@@ -1198,28 +1302,28 @@ __global__ void __launch_bounds__(512, 1)
                     L.idle[k] = 1;
                     L.n_idle++;
                 }
-                __syncthreads();
+                cta_sync();
                 PROF_ADD(L, P_OTHER, p_pl);
                 if (T < 0) continue;
             }
             // serve T with its loads (block-wide); D(T) from the CSR unless cached
             const bool need_row = L.row_len < 0;
-            __syncthreads();
+            cta_sync();
             if (need_row && tid < 32) {
                 const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
                 for (int r = tid; r < (int)(re - rb); r += 32) L.row[r] = __ldg(&I.tdat[rb + r]);
                 if (tid == 0) L.row_len = (int)(re - rb);
             }
-            __syncthreads();
+            cta_sync();
             PROF_T0(p_ld);
-            serve_loads(I, V, L, k, T, t);
+            serve_loads(k, T, t);
             PROF_ADD(L, P_LOADS, p_ld);
             if (L.error) break;
         }
-        __syncthreads();
+        cta_sync();
 
         // ---- a8: per-GPU orders, scalars
-        assemble(I, L.n_served);
+        assemble(L.n_served);
         if (tid == 0) {
             Out *o = I.out;
             o->n_events = L.n_events;
@@ -1237,9 +1341,9 @@ __global__ void __launch_bounds__(512, 1)
             o->alg_bytes = L.alg_bytes;
             o->scan_alg_bytes = L.scan_alg_bytes;
             o->error = L.error;
-            for (int i = 0; i < 8; i++) o->prof[i] = L.prof[i];
+            for (int i = 0; i < 16; i++) o->prof[i] = L.prof[i];
         }
-        __syncthreads();
+        cta_sync();
     }
 }
 

@@ -65,7 +65,7 @@ class dts_result_view(C.Structure):
                 ("n_idle_requests", C.c_int64), ("n_verify_err", C.c_int64),
                 ("alg_bytes", C.c_uint64),
                 ("scan_alg_bytes", C.c_uint64), ("loop_ms", C.c_float), ("total_ms", C.c_float),
-                ("prof_cycles", C.c_int64 * 8)]
+                ("prof_cycles", C.c_int64 * 16)]
 
 
 _lib = None

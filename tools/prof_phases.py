@@ -24,4 +24,8 @@ for inst in cases:
                   f"{1e6 * g.loop_ms / max(g.n_served, 1):.0f} ns/dec, total_ms {g.total_ms:.2f}")
             print("   cycles/scan: " + ", ".join(
                 f"{n}={c / max(g.n_scans, 1):.0f}" for n, c in zip(NAMES, g.prof_cycles)))
-            print(f"   pop cycles/pop: {g.prof_cycles[0] / max(g.n_served - g.n_scans, 1):.0f}")
+            print(f"   pop cycles/pop: {g.prof_cycles[0] / max(g.n_served - g.n_scans, 1):.0f}; "
+                  f"batches {g.prof_cycles[10]} ({g.prof_cycles[11]} pops): warp0 "
+                  f"{g.prof_cycles[8] / max(g.prof_cycles[10], 1):.0f} cyc, rank phase "
+                  f"{g.prof_cycles[9] / max(g.prof_cycles[10], 1):.0f} cyc per batch; w0 checkpoints "
+                  + " ".join(f"{g.prof_cycles[i] / max(g.prof_cycles[10], 1):.0f}" for i in range(12, 16)))
