@@ -136,13 +136,12 @@ class Clocks:
 
 def workload_instances(name, rank, world):
     if name == "C5":
+        from paper_conf_ipps_gonthiermt22_b200.shard import instance_cost, shard
         params = gen.sweep_params()
-        # strong scaling: shard the 4,096 instances; LPT-like round robin on a
-        # cost estimate (m * N, heaviest first) so every rank gets a similar mix
-        cost = [(-(N * N) * N * 1.0, i) for i, (N, M, K) in enumerate(params)]
-        order = [i for _, i in sorted(cost)]
-        mine = order[rank::world]
-        return [gen.sweep_instance(*params[i]) for i in mine], "strong"
+        # strong scaling: the 4,096 independent instances are sharded by LPT on
+        # a cost estimate; no data-path collective
+        costs = [instance_cost(N * N, 2 * N) for (N, M, K) in params]
+        return [gen.sweep_instance(*params[i]) for i in shard(costs, rank, world)], "strong"
     return gen.config_instances(name), "weak"
 
 
@@ -332,14 +331,10 @@ def main():
                   + 128 for r in out)
     e2e_avg = sum(e2e_ms) / len(e2e_ms)
 
-    # ---- max over ranks
-    t = torch.tensor([ms, e2e_avg, loop_ms], dtype=torch.float64, device="cuda")
-    tot = torch.tensor([decisions, alg], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(tot, op=dist.ReduceOp.SUM)
-    ms, e2e_avg, loop_ms_max = [float(x) for x in t.tolist()]
-    all_dec = float(tot[0])
+    # ---- max over ranks (device times), sum of the work
+    from paper_conf_ipps_gonthiermt22_b200.shard import reduce_over_ranks
+    ms, e2e_avg, loop_ms_max = reduce_over_ranks([ms, e2e_avg, loop_ms], "max", device="cuda")
+    all_dec, all_alg = reduce_over_ranks([decisions, alg], "sum", device="cuda")
 
     if rank == 0:
         peak, peak_src = _peaks()

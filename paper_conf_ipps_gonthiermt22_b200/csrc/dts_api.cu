@@ -100,10 +100,17 @@ struct dts_instance {
     bool ran = false;
     bool have_host = false;
     dts::Out out{};
-    std::vector<int64_t> r_gpu_ptr;
-    std::vector<int32_t> r_gpu_ids, r_serve_gpu, r_serve_task;
-    std::vector<int64_t> r_tstart, r_tend;
-    std::vector<dts_event> r_events;
+    // pinned host memory (allocated with the device arena): a mirror of the
+    // inputs for the H2D upload and the result buffers for the D2H read-back
+    char *h_pin = nullptr;
+    int64_t *p_task_ptr = nullptr, *p_task_ns = nullptr;
+    int32_t *p_task_data = nullptr;
+    uint64_t *p_size = nullptr;
+    int64_t *r_gpu_ptr = nullptr, *r_tstart = nullptr, *r_tend = nullptr;
+    int32_t *r_gpu_ids = nullptr, *r_serve_gpu = nullptr, *r_serve_task = nullptr;
+    dts_event *r_events = nullptr;
+    dts::Out *r_out = nullptr;
+    int64_t r_n_events = 0;
     float loop_ms = 0.f, total_ms = 0.f;
 
     ~dts_instance() {
@@ -118,6 +125,7 @@ struct dts_instance {
             cudaSetDevice(cur);
         }
         if (h_pinned) cudaFreeHost(h_pinned);
+        if (h_pin) cudaFreeHost(h_pin);
     }
 };
 
@@ -264,17 +272,20 @@ void dts_instance_destroy(dts_instance *inst) { delete inst; }
 namespace {
 
 dts_status check_device(int device) {
+    // cudaGetDeviceProperties costs milliseconds: query each device once
+    static int checked[64] = {0};  // 0 = unknown, 1 = sm_100, -1 = other
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
     if (e != cudaSuccess || ndev == 0) return fail(DTS_E_CUDA, "no CUDA device (libdts has no CPU path)");
-    if (device < 0 || device >= ndev) return fail(DTS_E_INVAL, "device ordinal out of range");
-    cudaDeviceProp p;
-    CK(cudaGetDeviceProperties(&p, device), "cudaGetDeviceProperties");
-    if (p.major != 10) return fail(DTS_E_CUDA, "libdts is built for sm_100a (B200); device is sm_" +
-                                                   std::to_string(p.major) + std::to_string(p.minor));
+    if (device < 0 || device >= ndev || device >= 64) return fail(DTS_E_INVAL, "device ordinal out of range");
+    if (checked[device] == 0) {
+        int major = 0;
+        CK(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device), "attr major");
+        checked[device] = major == 10 ? 1 : -1;
+    }
+    if (checked[device] < 0) return fail(DTS_E_CUDA, "libdts is built for sm_100a (B200); device is not sm_10x");
     return DTS_OK;
 }
-
 
 dts_status ensure_device(dts_instance *I, int device) {
     if (I->device == device && I->ar.base) return DTS_OK;
@@ -322,6 +333,32 @@ dts_status ensure_device(dts_instance *I, int device) {
     for (auto &ev : I->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
     CK(cudaEventCreateWithFlags(&I->ev_desc, cudaEventDisableTiming), "cudaEventCreate");
     if (!I->h_pinned) CK(cudaMallocHost(&I->h_pinned, sizeof(dts::Inst)), "cudaMallocHost");
+    if (!I->h_pin) {
+        size_t hb = 0;
+        auto hadd = [&](size_t bytes) { size_t o = hb; hb += (bytes + 63) & ~size_t(63); return o; };
+        const size_t o_tp = hadd(8 * (m + 1)), o_td = hadd(4 * (E + 1)), o_sz = hadd(8 * (n + 1)),
+                     o_tn = hadd(8 * (m + 1)), o_gp = hadd(8 * (K + 1)), o_gi = hadd(4 * (m + 1)),
+                     o_sg = hadd(4 * (m + 1)), o_st = hadd(4 * (m + 1)), o_ts = hadd(8 * (m + 1)),
+                     o_te = hadd(8 * (m + 1)), o_ev = hadd(sizeof(dts_event) * ev_cap),
+                     o_out = hadd(sizeof(dts::Out));
+        CK(cudaMallocHost(&I->h_pin, hb), "cudaMallocHost");
+        I->p_task_ptr = (int64_t *)(I->h_pin + o_tp);
+        I->p_task_data = (int32_t *)(I->h_pin + o_td);
+        I->p_size = (uint64_t *)(I->h_pin + o_sz);
+        I->p_task_ns = (int64_t *)(I->h_pin + o_tn);
+        I->r_gpu_ptr = (int64_t *)(I->h_pin + o_gp);
+        I->r_gpu_ids = (int32_t *)(I->h_pin + o_gi);
+        I->r_serve_gpu = (int32_t *)(I->h_pin + o_sg);
+        I->r_serve_task = (int32_t *)(I->h_pin + o_st);
+        I->r_tstart = (int64_t *)(I->h_pin + o_ts);
+        I->r_tend = (int64_t *)(I->h_pin + o_te);
+        I->r_events = (dts_event *)(I->h_pin + o_ev);
+        I->r_out = (dts::Out *)(I->h_pin + o_out);
+        std::memcpy(I->p_task_ptr, I->task_ptr.data(), 8 * (m + 1));
+        if (E) std::memcpy(I->p_task_data, I->task_data.data(), 4 * E);
+        if (n) std::memcpy(I->p_size, I->size.data(), 8 * n);
+        if (I->has_tau && m) std::memcpy(I->p_task_ns, I->task_ns.data(), 8 * m);
+    }
 
     Arena &A = I->ar;
     dts::Inst &h = I->h_inst;
@@ -382,17 +419,16 @@ dts_status ensure_device(dts_instance *I, int device) {
 
 dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
     if (I->uploaded && !force) return DTS_OK;
-    CK(cudaMemcpyAsync(I->d_raw_ptr, I->task_ptr.data(), 8 * ((size_t)I->m + 1), cudaMemcpyHostToDevice, st),
+    // from the pinned mirror of the caller's arrays (asynchronous DMA)
+    CK(cudaMemcpyAsync(I->d_raw_ptr, I->p_task_ptr, 8 * ((size_t)I->m + 1), cudaMemcpyHostToDevice, st),
        "H2D task_ptr");
     if (I->E_raw > 0)
-        CK(cudaMemcpyAsync(I->d_raw_dat, I->task_data.data(), 4 * (size_t)I->E_raw, cudaMemcpyHostToDevice, st),
+        CK(cudaMemcpyAsync(I->d_raw_dat, I->p_task_data, 4 * (size_t)I->E_raw, cudaMemcpyHostToDevice, st),
            "H2D task_data");
     if (I->n > 0)
-        CK(cudaMemcpyAsync(I->d_size, I->size.data(), 8 * (size_t)I->n, cudaMemcpyHostToDevice, st),
-           "H2D data_size");
+        CK(cudaMemcpyAsync(I->d_size, I->p_size, 8 * (size_t)I->n, cudaMemcpyHostToDevice, st), "H2D data_size");
     if (I->has_tau && I->m > 0)
-        CK(cudaMemcpyAsync(I->d_tau, I->task_ns.data(), 8 * (size_t)I->m, cudaMemcpyHostToDevice, st),
-           "H2D task_ns");
+        CK(cudaMemcpyAsync(I->d_tau, I->p_task_ns, 8 * (size_t)I->m, cudaMemcpyHostToDevice, st), "H2D task_ns");
     I->uploaded = true;
     return DTS_OK;
 }
@@ -636,29 +672,28 @@ dts_status dts_result(dts_instance *I, dts_result_view *v) {
     if (!I->have_host) {
         CK(cudaSetDevice(I->device), "cudaSetDevice");
         CK(cudaEventSynchronize(I->ev[3]), "run");
-        CK(cudaMemcpy(&I->out, I->h_inst.out, sizeof I->out, cudaMemcpyDeviceToHost), "D2H out");
+        CK(cudaMemcpyAsync(I->r_out, I->h_inst.out, sizeof I->out, cudaMemcpyDeviceToHost, I->stream), "D2H out");
+        CK(cudaStreamSynchronize(I->stream), "D2H sync");
+        I->out = *I->r_out;
         if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim (Belady branch)");
         const dts::Inst &h = I->h_inst;
         size_t ns = (size_t)I->out.n_served, ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);
         size_t m = (size_t)I->m;
-        I->r_gpu_ptr.resize((size_t)I->K + 1);
-        I->r_gpu_ids.resize(ns);
-        I->r_serve_gpu.resize(ns);
-        I->r_serve_task.resize(ns);
-        I->r_tstart.resize(m);
-        I->r_tend.resize(m);
-        I->r_events.resize(ne);
-        CK(cudaMemcpy(I->r_gpu_ptr.data(), h.gpu_task_ptr, 8 * ((size_t)I->K + 1), cudaMemcpyDeviceToHost), "D2H");
+        cudaStream_t st = I->stream;  // the run's stream: the copies follow the run
+        CK(cudaMemcpyAsync(I->r_gpu_ptr, h.gpu_task_ptr, 8 * ((size_t)I->K + 1), cudaMemcpyDeviceToHost, st), "D2H");
         if (ns) {
-            CK(cudaMemcpy(I->r_gpu_ids.data(), h.gpu_task_ids, 4 * ns, cudaMemcpyDeviceToHost), "D2H");
-            CK(cudaMemcpy(I->r_serve_gpu.data(), h.serve_gpu, 4 * ns, cudaMemcpyDeviceToHost), "D2H");
-            CK(cudaMemcpy(I->r_serve_task.data(), h.serve_task, 4 * ns, cudaMemcpyDeviceToHost), "D2H");
+            CK(cudaMemcpyAsync(I->r_gpu_ids, h.gpu_task_ids, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
+            CK(cudaMemcpyAsync(I->r_serve_gpu, h.serve_gpu, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
+            CK(cudaMemcpyAsync(I->r_serve_task, h.serve_task, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
         }
         if (m) {
-            CK(cudaMemcpy(I->r_tstart.data(), h.tstart, 8 * m, cudaMemcpyDeviceToHost), "D2H");
-            CK(cudaMemcpy(I->r_tend.data(), h.tend, 8 * m, cudaMemcpyDeviceToHost), "D2H");
+            CK(cudaMemcpyAsync(I->r_tstart, h.tstart, 8 * m, cudaMemcpyDeviceToHost, st), "D2H");
+            CK(cudaMemcpyAsync(I->r_tend, h.tend, 8 * m, cudaMemcpyDeviceToHost, st), "D2H");
         }
-        if (ne) CK(cudaMemcpy(I->r_events.data(), h.events, sizeof(dts_event) * ne, cudaMemcpyDeviceToHost), "D2H");
+        if (ne)
+            CK(cudaMemcpyAsync(I->r_events, h.events, sizeof(dts_event) * ne, cudaMemcpyDeviceToHost, st), "D2H");
+        CK(cudaStreamSynchronize(st), "D2H sync");
+        I->r_n_events = (int64_t)ne;
         CK(cudaEventElapsedTime(&I->loop_ms, I->ev[1], I->ev[2]), "elapsed");
         CK(cudaEventElapsedTime(&I->total_ms, I->ev[0], I->ev[3]), "elapsed");
         I->have_host = true;
@@ -666,14 +701,14 @@ dts_status dts_result(dts_instance *I, dts_result_view *v) {
     std::memset(v, 0, sizeof *v);
     v->K = I->K;
     v->n_tasks = I->m;
-    v->gpu_task_ptr = I->r_gpu_ptr.data();
-    v->gpu_task_ids = I->r_gpu_ids.data();
-    v->serve_gpu = I->r_serve_gpu.data();
-    v->serve_task = I->r_serve_task.data();
-    v->task_start_ns = I->r_tstart.data();
-    v->task_end_ns = I->r_tend.data();
-    v->n_events = (int64_t)I->r_events.size();
-    v->events = I->r_events.data();
+    v->gpu_task_ptr = I->r_gpu_ptr;
+    v->gpu_task_ids = I->r_gpu_ids;
+    v->serve_gpu = I->r_serve_gpu;
+    v->serve_task = I->r_serve_task;
+    v->task_start_ns = I->r_tstart;
+    v->task_end_ns = I->r_tend;
+    v->n_events = I->r_n_events;
+    v->events = I->r_events;
     v->bytes_loaded = I->out.bytes_loaded;
     v->n_loads = I->out.n_loads;
     v->n_evictions = I->out.n_evictions;

@@ -1409,10 +1409,27 @@ cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t wo
     return cudaGetLastError();
 }
 
+// cudaFuncSetAttribute is a driver call worth avoiding per launch: raise the
+// kernel's dynamic shared-memory limit only when a launch needs more.
+static cudaError_t ensure_smem_attr(int smem_bytes) {
+    static int cur[64];
+    static bool init = false;
+    if (!init) {
+        for (int &c : cur) c = -1;
+        init = true;
+    }
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (smem_bytes <= cur[dev]) return cudaSuccess;
+    cudaError_t e = cudaFuncSetAttribute(dts_cta_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+    if (e == cudaSuccess) cur[dev] = smem_bytes;
+    return e;
+}
+
 cudaError_t launch_loop(const Inst *d_insts, int n_inst, int block, int grid, int *work_counter,
                         int smem_bytes, cudaStream_t st) {
-    cudaError_t e = cudaFuncSetAttribute(dts_cta_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         smem_bytes);
+    cudaError_t e = ensure_smem_attr(smem_bytes);
     if (e != cudaSuccess) return e;
     dts_cta_kernel<<<grid, block, smem_bytes, st>>>(d_insts, n_inst, work_counter);
     count_launch();
@@ -1421,7 +1438,7 @@ cudaError_t launch_loop(const Inst *d_insts, int n_inst, int block, int grid, in
 
 int loop_max_blocks_per_sm(int block, int smem_bytes) {
     int nb = 0;
-    cudaFuncSetAttribute(dts_cta_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+    if (ensure_smem_attr(smem_bytes) != cudaSuccess) return 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, dts_cta_kernel, block, smem_bytes) != cudaSuccess)
         return 0;
     return nb;

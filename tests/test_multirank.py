@@ -1,0 +1,79 @@
+"""Multi-process (world size 2, gloo, CPU) tests of the multi-GPU host logic:
+LPT sharding of independent instances and the max/sum-over-ranks timing
+reductions bench.py uses.  No GPU needed."""
+import os
+import socket
+
+import pytest
+import torch.multiprocessing as mp
+
+import gen
+from paper_conf_ipps_gonthiermt22_b200.shard import instance_cost, lpt_assign, shard
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, costs, q):
+    import torch.distributed as dist
+    from paper_conf_ipps_gonthiermt22_b200.shard import reduce_over_ranks, shard as shard_fn
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    mine = shard_fn(costs, rank, world)
+    got = [None] * world
+    dist.all_gather_object(got, mine)
+    load = sum(costs[i] for i in mine)
+    mx, = reduce_over_ranks([load], "max")
+    tot, = reduce_over_ranks([load], "sum")
+    dist.barrier()
+    dist.destroy_process_group()
+    q.put((rank, got, load, mx, tot))
+
+
+def _sweep_costs():
+    costs = []
+    for (N, M, K) in gen.sweep_params():
+        costs.append(instance_cost(N * N, 2 * N))
+    return costs
+
+
+def test_lpt_single_process_properties():
+    costs = _sweep_costs()
+    assert len(costs) == 4096
+    for world in (1, 2, 4, 8):
+        parts = lpt_assign(costs, world)
+        flat = sorted(i for p in parts for i in p)
+        assert flat == list(range(len(costs))), "every instance exactly once"
+        loads = [sum(costs[i] for i in p) for p in parts]
+        # LPT bound: max - min <= the largest single cost
+        assert max(loads) - min(loads) <= max(costs) + 1e-6
+        assert max(loads) <= sum(costs) / world + max(costs)
+    assert lpt_assign(costs, 8) == lpt_assign(list(costs), 8), "deterministic"
+
+
+def test_shard_two_ranks_gloo():
+    costs = _sweep_costs()
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, costs, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    (_, got0, load0, mx0, tot0), (_, got1, load1, mx1, tot1) = res
+    assert got0 == got1
+    a, b = got0
+    assert not set(a) & set(b), "shards are disjoint"
+    assert sorted(a + b) == list(range(len(costs))), "shards cover the sweep"
+    assert a == shard(costs, 0, 2) and b == shard(costs, 1, 2)
+    assert mx0 == mx1 == max(load0, load1)
+    assert tot0 == pytest.approx(load0 + load1)
