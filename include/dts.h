@@ -65,7 +65,11 @@ enum {
      * scores n_k(D), n2_k(D), u(D) and every task's missing count from their
      * definitions (a full pass over all tasks) and count disagreements with
      * the incremental state in dts_result_view.n_verify_err.  Slow. */
-    DTS_F_VERIFY = 1u << 1
+    DTS_F_VERIFY = 1u << 1,
+    /* Diagnostic: build the CSR and initial state with the separate grid-wide
+     * kernels even for small instances (default: the loop CTA of an instance
+     * with <= 8 inputs per task and a small n builds them itself). */
+    DTS_F_NOFUSE = 1u << 2
 };
 
 typedef struct {

@@ -7,6 +7,7 @@ fallback: without the library or a B200 the calls raise ``DtsError``.
 from .dts import (  # noqa: F401
     DTS_F_FALLBACK2,
     DTS_F_VERIFY,
+    DTS_F_NOFUSE,
     DTS_POLICY_DARTS_LUF,
     EVENT_DTYPE,
     EXPORTED,

@@ -72,6 +72,8 @@ struct dts_instance {
     std::vector<int64_t> task_ns;
     bool has_tau = false;
     int32_t max_deg_ub = 0;
+    int32_t max_row_len = 0;
+    bool uniform_size = false;
     uint64_t max_row_bytes = 0;
     uint64_t min_size = 1;
     int32_t res_cap = 1;
@@ -248,10 +250,13 @@ dts_status dts_instance_create(int32_t n_tasks, int32_t n_data, const int64_t *t
             }
         }
         I->max_row_bytes = std::max(I->max_row_bytes, bytes);
+        I->max_row_len = std::max(I->max_row_len, q);
     }
     int32_t md = 1;
     for (int32_t D = 0; D < n_data; D++) md = std::max(md, occ[D]);
     I->max_deg_ub = md;
+    I->uniform_size = n_data > 0 && std::all_of(I->size.begin(), I->size.end(),
+                                                [&](uint64_t x) { return x == I->size[0]; });
     I->min_size = min_size;
     uint64_t rc = mem_capacity_bytes / min_size;
     I->res_cap = (int32_t)std::max<uint64_t>(1, std::min<uint64_t>(rc, (uint64_t)std::max(n_data, 1)));
@@ -435,7 +440,8 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
 
 dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_opts *o) {
     if (policy != DTS_POLICY_DARTS_LUF) return fail(DTS_E_UNSUPPORTED, "policy");
-    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY)) return fail(DTS_E_UNSUPPORTED, "unknown flags");
+    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE))
+        return fail(DTS_E_UNSUPPORTED, "unknown flags");
     if (o->lookahead_W != 0) return fail(DTS_E_UNSUPPORTED, "lookahead_W != 0 (NEXT)");
     if (o->bus_bytes_per_s == 0) return fail(DTS_E_INVAL, "bus_bytes_per_s == 0");
     if (o->block_threads != 0 && (o->block_threads < 32 || o->block_threads > 512 || o->block_threads % 32))
@@ -504,7 +510,10 @@ int env_int(const char *name, int dflt) {
 
 // Enqueue everything of one instance up to (not including) the decision loop:
 // upload if needed, CSR build (a1), state init (a2), descriptor H2D.
-dts_status stage(dts_instance *I, const dts_run_opts &o, int budget, cudaStream_t st,
+// Shared scratch of the fused in-CTA CSR build (dts_loop.cu fused_build).
+int fused_scratch_bytes(const dts_instance *I, int block) { return (2 * (block / 32) + 1) * 4 * (I->n + 1); }
+
+dts_status stage(dts_instance *I, const dts_run_opts &o, int budget, int block, cudaStream_t st,
                  bool copy_desc = true) {
     dts_status s = ensure_device(I, o.device);
     if (s != DTS_OK) return s;
@@ -520,17 +529,25 @@ dts_status stage(dts_instance *I, const dts_run_opts &o, int budget, cudaStream_
     h.max_served = o.max_served;
     h.size0 = 0;
     h.delta0 = 0;
-    if (I->n > 0 && std::all_of(I->size.begin(), I->size.end(), [&](uint64_t x) { return x == I->size[0]; })) {
+    h.bw = o.bus_bytes_per_s;
+    h.raw_ptr = I->d_raw_ptr;
+    h.raw_dat = I->d_raw_dat;
+    if (I->uniform_size) {
         h.size0 = I->size[0];
         const unsigned __int128 num = (unsigned __int128)h.size0 * 1000000000u + (o.bus_bytes_per_s - 1);
         h.delta0 = (int64_t)(num / o.bus_bytes_per_s);  // ceil, reading R9 (same as dts_init_kernel)
     }
     place_smem(h, I->has_tau, budget);
+    // small instances: the loop CTA builds its own CSR and state (one launch)
+    const int fs = fused_scratch_bytes(I, block);
+    h.fused = !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
+    if (h.fused) h.smem_bytes = std::max(h.smem_bytes, fs);
     CK(cudaEventRecord(I->ev[0], st), "event");
-    CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
-                      (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, (int4 *)h.dedge,
-                      I->d_csr_scratch, st),
-       "build_csr");
+    if (!h.fused)
+        CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
+                          (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, (int4 *)h.dedge,
+                          I->d_csr_scratch, st),
+           "build_csr");
     if (!copy_desc) return DTS_OK;
     // descriptor H2D from pinned memory (a pageable copy would serialise the host)
     CK(cudaEventSynchronize(I->ev_desc), "desc event");
@@ -583,11 +600,11 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     if (s != DTS_OK) return s;
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
     const int budget = budget_of(o);
-    s = stage(I, o, budget, st);
-    if (s != DTS_OK) return s;
     const int block = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", auto_block(I));
+    s = stage(I, o, budget, block, st);
+    if (s != DTS_OK) return s;
     const int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n + 4);
-    CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
+    if (!I->h_inst.fused) CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
     CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
     CK(cudaEventRecord(I->ev[1], st), "event");
     CK(dts::launch_loop(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");
@@ -622,12 +639,20 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     if (o.block_threads) block = o.block_threads;
     else block = env_int("DTS_BLOCK", block);
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
-    const int budget = budget_of(o);
+    // Each instance is a latency-bound chain: with many more instances than
+    // SMs, run several CTAs per SM (their chains interleave) by default --
+    // a quarter of the shared memory each; few instances get all of it.
+    int nsm = 0;
+    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
+    int budget = budget_of(o);
+    if (o.smem_budget == 0 && n >= 2 * nsm) budget = std::min(budget, (max_dyn_smem(o.device) + 1024) / 4 - 4096);
     int smem = 0;
+    bool any_unfused = false;
     for (int32_t i = 0; i < n; i++) {
-        s = stage(insts[i], o, budget, st, false);
+        s = stage(insts[i], o, budget, block, st, false);
         if (s != DTS_OK) return s;
         smem = std::max(smem, insts[i]->h_inst.smem_bytes);
+        any_unfused |= !insts[i]->h_inst.fused;
     }
     SweepBuf &B = g_sweep[o.device];
     if (!B.copied[0])
@@ -646,14 +671,18 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     const int sl = B.slot;
     B.slot = (B.slot + 1) % SweepBuf::RING;
     CK(cudaEventSynchronize(B.copied[sl]), "sweep event");
-    for (int32_t i = 0; i < n; i++) B.h_insts[sl][i] = insts[i]->h_inst;
+    // longest first (cost ~ m * mean degree), so the device counter hands the
+    // long chains out early and the tail of the batch stays short
+    std::vector<int32_t> ord((size_t)n);
+    for (int32_t i = 0; i < n; i++) ord[(size_t)i] = i;
+    auto cost = [&](int32_t i) { return (double)insts[i]->m * (double)insts[i]->E_raw / std::max(1, insts[i]->n); };
+    std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return cost(a) > cost(b); });
+    for (int32_t i = 0; i < n; i++) B.h_insts[sl][i] = insts[ord[(size_t)i]]->h_inst;
     CK(cudaMemcpyAsync(B.d_insts, B.h_insts[sl], sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
        "H2D sweep");
     CK(cudaEventRecord(B.copied[sl], st), "event");
     CK(cudaMemsetAsync(B.d_work, 0, sizeof(int), st), "memset");
-    CK(dts::launch_init(B.d_insts, n, o.bus_bytes_per_s, work, st), "init");
-    int nsm = 0;
-    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
+    if (any_unfused) CK(dts::launch_init(B.d_insts, n, o.bus_bytes_per_s, work, st), "init");
     const int per = std::max(1, dts::loop_max_blocks_per_sm(block, smem));
     const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
     for (int32_t i = 0; i < n; i++) CK(cudaEventRecord(insts[i]->ev[1], st), "event");

@@ -75,6 +75,11 @@ struct Inst {
     const int32_t *tdat;
     const int64_t *dptr;
     const int32_t *ddat;
+    const int64_t *raw_ptr;  // caller's CSR as uploaded (fused builds read it)
+    const int32_t *raw_dat;
+    int32_t fused;           // 1: the loop CTA builds the CSR and initial state itself
+    int32_t pad2;
+    uint64_t bw;             // bus bytes/s (fused init computes delta)
     const int4 *dedge;     // [E] edge records of the data->task CSR: {T, o1, o2, |D(T)|},
                            // o1/o2 = T's other inputs (-1 if none; first two if |D(T)| > 3)
     const uint64_t *size;

@@ -1156,6 +1156,206 @@ __device__ __noinline__ void assemble(int64_t ns) {
     }
 }
 
+
+// ---------------------------------------------------------------------------
+// Fused a1 + a2 init for small instances (Inst::fused): the CTA that runs the
+// instance first builds its CSR and initial state itself, so a batched sweep
+// is ONE kernel launch instead of ~20 launches per instance.  Same outputs as
+// dts_csr.cu + dts_init_kernel (rows sorted and de-duplicated, D(T) a set,
+// PAPER.md:244-245; each data segment in ascending task id).  Needs rows of
+// <= FUSE_ROW inputs and (2 * warps + 1) * n ints of shared scratch (host-checked).
+constexpr int FUSE_ROW = 8;
+
+// Block-wide exclusive scan of one int per thread; returns the prefix, *total.
+__device__ __forceinline__ int block_excl_scan_int(int v, int *total) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    int x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(FULL, x, o);
+        if (lane >= o) x += t;
+    }
+    cta_sync();
+    if (lane == 31) L.red32[w] = x;
+    cta_sync();
+    int off = 0, tot = 0;
+    for (int j = 0; j < nw; j++) {
+        const int y = L.red32[j];
+        if (j < w) off += y;
+        tot += y;
+    }
+    *total = tot;
+    return off + x - v;
+}
+
+__device__ __noinline__ void fused_build(unsigned char *dsm) {
+    const Inst &I = SI;
+    const int m = I.m, n = I.n, nw = blockDim.x >> 5;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    int64_t *tptr = const_cast<int64_t *>(I.tptr);
+    int32_t *tdat = const_cast<int32_t *>(I.tdat);
+    int64_t *dptr = const_cast<int64_t *>(I.dptr);
+    int32_t *ddat = const_cast<int32_t *>(I.ddat);
+    int4 *dedge = const_cast<int4 *>(I.dedge);
+    int *cnt = reinterpret_cast<int *>(dsm);  // [nw][n] per-warp counts, then bases
+    unsigned *msk = reinterpret_cast<unsigned *>(cnt + nw * n);  // [nw][n] lane masks
+    int *deg = reinterpret_cast<int *>(msk + nw * n);            // [n]
+    for (int i = threadIdx.x; i < nw * n; i += blockDim.x) {
+        cnt[i] = 0;
+        msk[i] = 0u;
+    }
+    for (int i = threadIdx.x; i < n; i += blockDim.x) deg[i] = 0;
+    cta_sync();
+    // 1. rows: sort + de-duplicate (thread per task), tptr by block scans, tdat, deg
+    int64_t carry = 0;
+    for (int c = 0; c < m; c += blockDim.x) {
+        const int T = c + threadIdx.x;
+        int row[FUSE_ROW];
+        int len = 0;
+        if (T < m) {
+            const int64_t rb = I.raw_ptr[T], re = I.raw_ptr[T + 1];
+            for (int64_t i = rb; i < re; i++) {
+                const int v = I.raw_dat[i];
+                int j = len;  // insertion, skipping duplicates
+                bool dup = false;
+                for (int q = 0; q < len; q++) dup |= row[q] == v;
+                if (dup) continue;
+                while (j > 0 && row[j - 1] > v) {
+                    row[j] = row[j - 1];
+                    j--;
+                }
+                row[j] = v;
+                len++;
+            }
+        }
+        int tot;
+        const int off = block_excl_scan_int(len, &tot);
+        if (T < m) {
+            const int64_t o = carry + off;
+            tptr[T] = o;
+            for (int q = 0; q < len; q++) {
+                tdat[o + q] = row[q];
+                atomicAdd(&deg[row[q]], 1);
+            }
+        }
+        carry += tot;
+    }
+    if (threadIdx.x == 0) tptr[m] = carry;
+    cta_sync();
+    // 2. dptr = exclusive scan of deg; per-warp counts over contiguous task ranges
+    int64_t dcarry = 0;
+    for (int c = 0; c < n; c += blockDim.x) {
+        const int D = c + threadIdx.x;
+        const int v = D < n ? deg[D] : 0;
+        int tot;
+        const int off = block_excl_scan_int(v, &tot);
+        if (D < n) dptr[D] = dcarry + off;
+        dcarry += tot;
+    }
+    if (threadIdx.x == 0) dptr[n] = dcarry;
+    const int per = (m + nw - 1) / nw, t0 = w * per, t1 = min(m, t0 + per);
+    for (int T = t0 + lane; T < t1; T += 32) {
+        const int64_t rb = tptr[T], re = tptr[T + 1];
+        for (int64_t i = rb; i < re; i++) atomicAdd(&cnt[w * n + tdat[i]], 1);
+    }
+    cta_sync();
+    for (int D = threadIdx.x; D < n; D += blockDim.x) {  // per-datum bases over warps
+        int64_t run = dptr[D];
+        for (int j = 0; j < nw; j++) {
+            const int x = cnt[j * n + D];
+            cnt[j * n + D] = (int)run;
+            run += x;
+        }
+    }
+    cta_sync();
+    // 3. stable scatter: each warp walks its range 32 tasks at a time; a task's
+    //    rank among the group's tasks with the same datum = lower lanes in the mask
+    const unsigned lt = (1u << lane) - 1u;
+    for (int g = t0; g < t1; g += 32) {
+        const int T = g + lane;
+        int64_t rb = 0, re = 0;
+        if (T < t1) {
+            rb = tptr[T];
+            re = tptr[T + 1];
+        }
+        for (int64_t i = rb; i < re; i++) atomicOr(&msk[w * n + tdat[i]], 1u << lane);
+        __syncwarp();
+        for (int64_t i = rb; i < re; i++) {
+            const int D = tdat[i];
+            const unsigned mk = msk[w * n + D];
+            const int pos = cnt[w * n + D] + __popc(mk & lt);
+            ddat[pos] = T;
+            int4 e;
+            e.x = T;
+            e.y = -1;
+            e.z = -1;
+            e.w = (int)(re - rb);
+            for (int64_t q = rb; q < re; q++) {
+                const int o = tdat[q];
+                if (o == D) continue;
+                if (e.y < 0) e.y = o;
+                else if (e.z < 0) e.z = o;
+            }
+            dedge[pos] = e;
+        }
+        __syncwarp();
+        for (int64_t i = rb; i < re; i++) {
+            const int D = tdat[i];
+            const unsigned mk = msk[w * n + D];
+            if (lane == __ffs(mk) - 1) cnt[w * n + D] += __popc(mk);
+        }
+        __syncwarp();
+        for (int64_t i = rb; i < re; i++) msk[w * n + tdat[i]] = 0u;
+        __syncwarp();
+    }
+    cta_sync();
+}
+
+// a2 initial state for a fused instance, straight into the placed arrays.
+__device__ __noinline__ void fused_init() {
+    const Inst &I = SI;
+    const View &V = SV;
+    const int m = I.m, n = I.n, K = I.K;
+    for (int T = threadIdx.x; T < I.m_pad; T += blockDim.x) {
+        uint32_t w = ALLOC_BIT;
+        if (T < m) {
+            const int64_t b = I.tptr[T], e = I.tptr[T + 1];
+            uint32_t x = 0;
+            for (int64_t i = b; i < e; i++) x ^= (uint32_t)I.tdat[i];
+            w = ((uint32_t)(e - b) << 24) | x;
+            I.tstart[T] = -1;
+            I.tend[T] = -1;
+        }
+        for (int k = 0; k < K; k++) V.s[(size_t)k * I.m_pad + T] = w;
+    }
+    for (int D = threadIdx.x; D < I.nstr; D += blockDim.x) {
+        int32_t c1 = 0, c2 = 0, dg = 0;
+        if (D < n) {
+            const int64_t b = I.dptr[D], e = I.dptr[D + 1];
+            dg = (int32_t)(e - b);
+            for (int64_t i = b; i < e; i++) {
+                const int len = I.dedge[i].w;
+                c1 += len == 1;
+                c2 += len == 2;
+            }
+            if (!I.size0) {
+                const unsigned __int128 num = (unsigned __int128)I.size[D] * 1000000000ull + (I.bw - 1);
+                const_cast<int64_t *>(I.delta)[D] = (int64_t)(num / I.bw);
+            }
+            if (V.dptr32) V.dptr32[D] = (int32_t)b;
+        }
+        V.u[D] = dg;
+        for (int k = 0; k < K; k++) {
+            V.h[(size_t)k * I.nstr + D] = c1;
+            V.h2[(size_t)k * I.nstr + D] = c2;
+            V.np[(size_t)k * I.nstr + D] = 0;
+        }
+    }
+    if (V.dptr32 && threadIdx.x == 0) V.dptr32[n] = (int32_t)I.dptr[n];
+    for (int i = threadIdx.x; i < K * I.nw; i += blockDim.x) V.resb[i] = 0u;
+    cta_sync();
+}
+
 }  // namespace
 
 // One CTA per instance; instances pulled from *work_counter.
@@ -1189,9 +1389,13 @@ __global__ void __launch_bounds__(512, 1)
         cta_sync();
         const View &V = SV;
 
+        const int n = I.n, K = I.K;
+        if (I.fused) {  // a1 + a2 inside this CTA (small instances)
+            fused_build(dsm);
+            fused_init();
+        } else {
         // ---- CTA-local copies of the initial state (global homes were
         //      initialised by dts_init_kernel)
-        const int n = I.n, K = I.K;
         if (I.so_dptr >= 0)
             for (int D = tid; D <= n; D += blockDim.x) V.dptr32[D] = (int32_t)__ldg(&I.dptr[D]);
         if (I.so_s >= 0) {
@@ -1209,6 +1413,7 @@ __global__ void __launch_bounds__(512, 1)
             for (int i = tid; i < K * I.nstr; i += blockDim.x) V.np[i] = 0;
         if (I.so_resb >= 0)
             for (int i = tid; i < K * I.nw; i += blockDim.x) V.resb[i] = 0u;
+        }
         if (tid == 0) {
             for (int k = 0; k < MAX_K; k++) {
                 L.req[k] = 0;
@@ -1354,6 +1559,7 @@ __global__ void __launch_bounds__(512, 1)
 __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint64_t bw) {
     for (int ii = 0; ii < n_inst; ii++) {
         const Inst I = insts[ii];
+        if (I.fused) continue;  // built and initialised inside its loop CTA
         int64_t *delta = const_cast<int64_t *>(I.delta);
         const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
         const int64_t str = (int64_t)gridDim.x * blockDim.x;

@@ -251,3 +251,16 @@ def test_hub_datum_64bit_argmax_keys():
     inst = gen.Instance("hub", tp, td, np.ones(300, np.uint64), None, 5, 12, 3)
     g, o = _both(inst, bus=10 ** 9)
     assert_parity(g, o)
+
+
+@pytest.mark.parametrize("idx", range(12))
+def test_fused_and_separate_csr_build(idx):
+    """Small instances build their CSR and initial state inside the loop CTA
+    (one launch); DTS_F_NOFUSE forces the separate grid-wide kernels.  Both
+    must give the oracle's schedule, with and without shared-memory state."""
+    inst = _shapes()[idx]
+    o = oracle.run(inst)
+    for flags in (dts.DTS_F_FALLBACK2, dts.DTS_F_FALLBACK2 | dts.DTS_F_NOFUSE):
+        for smem in (0, -1):
+            g = dts.schedule(inst, flags=flags, smem_budget=smem)
+            assert_parity(g, o)
