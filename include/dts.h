@@ -69,7 +69,11 @@ enum {
     /* Diagnostic: build the CSR and initial state with the separate grid-wide
      * kernels even for small instances (default: the loop CTA of an instance
      * with <= 8 inputs per task and a small n builds them itself). */
-    DTS_F_NOFUSE = 1u << 2
+    DTS_F_NOFUSE = 1u << 2,
+    /* OPTI variant (§V-F): instead of the datum that frees
+     * the most tasks, take the first one (ascending id) that frees at least
+     * one.  Combines with DTS_F_FALLBACK2 ("DARTS+LUF+OPTI-3inputs"). */
+    DTS_F_OPTI = 1u << 3
 };
 
 typedef struct {

@@ -26,6 +26,7 @@ _SRC = os.path.join(_HERE, "dts_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 F_FALLBACK2 = 1
+F_OPTI = 8
 DEFAULT_BUS_BPS = 12_000_000_000
 
 EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data", "<i4"),

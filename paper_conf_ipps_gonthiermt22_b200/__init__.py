@@ -8,6 +8,7 @@ from .dts import (  # noqa: F401
     DTS_F_FALLBACK2,
     DTS_F_VERIFY,
     DTS_F_NOFUSE,
+    DTS_F_OPTI,
     DTS_POLICY_DARTS_LUF,
     EVENT_DTYPE,
     EXPORTED,

@@ -440,7 +440,7 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
 
 dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_opts *o) {
     if (policy != DTS_POLICY_DARTS_LUF) return fail(DTS_E_UNSUPPORTED, "policy");
-    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE))
+    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI))
         return fail(DTS_E_UNSUPPORTED, "unknown flags");
     if (o->lookahead_W != 0) return fail(DTS_E_UNSUPPORTED, "lookahead_W != 0 (NEXT)");
     if (o->bus_bytes_per_s == 0) return fail(DTS_E_INVAL, "bus_bytes_per_s == 0");

@@ -983,6 +983,27 @@ __device__ int32_t score_argmax(const int32_t *score) {
     return best ? (int32_t)(idmask - (best & idmask)) : -1;
 }
 
+// OPTI (§V-F): "we stop the search as soon as we find a
+// data allowing to compute at least one task" -- dataNotInMem_k searched in
+// ascending id (reading R28), i.e. the lowest D with n_k(D) >= 1.
+__device__ __noinline__ int32_t score_first(const int32_t *score) {
+    const Inst &I = SI;
+    const int4 *h4 = reinterpret_cast<const int4 *>(score);
+    const int nv = I.nstr >> 2;
+    unsigned long long best = ~0ull;
+    for (int v = threadIdx.x; v < nv; v += blockDim.x) {  // increasing D per thread
+        const int4 hv = h4[v];
+        const int D = 4 * v;
+        const int f = hv.x > 0 ? 0 : (hv.y > 0 ? 1 : (hv.z > 0 ? 2 : (hv.w > 0 ? 3 : -1)));
+        if (f >= 0) {
+            best = (unsigned long long)(D + f);
+            break;
+        }
+    }
+    best = block_min_u64(best);
+    return best == ~0ull ? -1 : (int32_t)best;
+}
+
 // Alg. 5 l.10: plannedTasks_k <- unallocated tasks of Dopt's segment with one
 // missing input (= Dopt), ascending id (ordered block compaction).  Block-wide.
 __device__ void plan(int k, int32_t Dopt) {
@@ -1460,7 +1481,8 @@ __global__ void __launch_bounds__(512, 1)
             // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
             int32_t T = -1;
             PROF_T0(p_am);
-            const int32_t Dopt = score_argmax(V.h + (size_t)k * I.nstr);
+            const int32_t Dopt = (I.flags & DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
+                                                        : score_argmax(V.h + (size_t)k * I.nstr);
             PROF_ADD(L, P_ARGMAX, p_am);
             PROF_T0(p_pl);
             if (tid == 0) {

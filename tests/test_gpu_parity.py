@@ -264,3 +264,52 @@ def test_fused_and_separate_csr_build(idx):
         for smem in (0, -1):
             g = dts.schedule(inst, flags=flags, smem_budget=smem)
             assert_parity(g, o)
+
+
+# ------------------------------------------------------------ OPTI (§V-F)
+@pytest.mark.parametrize("idx", range(12))
+@pytest.mark.parametrize("fb2", [1, 0])
+def test_opti_shapes(idx, fb2):
+    inst = _shapes()[idx]
+    flags = dts.DTS_F_OPTI | (dts.DTS_F_FALLBACK2 if fb2 else 0)
+    g, o = _both(inst, flags=flags)
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("N", [4, 6])
+def test_opti_2d_column_major(N):
+    inst = _unit(gen.matmul2d(N, M=2 * N, K=1))
+    g = dts.schedule(inst, bus_bps=10 ** 9, flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_OPTI)
+    assert [int(x) for x in g.orders()[0]] == [i * N + j for j in range(N) for i in range(N)]
+
+
+@pytest.mark.parametrize("cfg", ["C4a", "C4b"])
+def test_opti_config4_prefix(cfg):
+    """DARTS+LUF+OPTI-3inputs (the paper's Cholesky setting, Fig. 11) at full size, prefix."""
+    inst = gen.config_instances(cfg)[0]
+    g, o = _both(inst, flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_OPTI, max_served=1500)
+    assert_parity(g, o, complete=False)
+
+
+def test_opti_config2_batch():
+    insts = gen.config_instances("C2")
+    gs = dts.schedule_batch(insts, flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_OPTI)
+    for inst, g in zip(insts, gs):
+        assert_parity(g, oracle.run(inst, flags=oracle.F_FALLBACK2 | oracle.F_OPTI))
+
+
+# ------------------------------------------------------------ workload variants (§8(f)3)
+def _variants():
+    return [gen.matmul2d(50, M=35, K=2, order="random", seed=11),    # PAPER.md:800, Fig. 9
+            gen.matmul2d(100, M=35, K=4, keep_frac=0.02, seed=12),  # sparse 2D, PAPER.md:813-817
+            gen.matmul2d(60, M=35, K=4, keep_frac=0.3, seed=13),
+            gen.matmul3d(20, M=142, K=4, with_c=True)]              # 3D with C_ij (reading R12)
+
+
+@pytest.mark.parametrize("idx", range(4))
+@pytest.mark.parametrize("flags", [1, 1 | 8])
+def test_workload_variants(idx, flags):
+    inst = _variants()[idx]
+    g, o = _both(inst, flags=flags)
+    assert_parity(g, o)
+    validate(inst, g.serve_gpu, g.serve_task, g.events, g.task_start, g.task_end)

@@ -193,3 +193,30 @@ def test_p6_brute_force_k2(seed):
     bel = belady_loads(r.orders(), ds, 3)
     assert opt <= bel <= r.n_loads
     _check(inst, r, bus=10 ** 9)
+
+
+# ---------------------------------------------------------------- OPTI (§V-F)
+@pytest.mark.parametrize("N", [4, 6])
+def test_opti_2d_ample_memory_column_major(N):
+    """Hand-derived: 2D N x N, K=1, M=2N (everything fits).  The first request
+    falls back to T(0,0) (loads A0, B0).  Then A_i frees only T(i,0) and B_j
+    frees T(0,j) and the rows already loaded, so OPTI (first datum with
+    n(D) >= 1 in id order, PAPER.md:2121-2124, reading R28) loads A1..A_{N-1}
+    one by one, then each B_j plans the whole column j: column-major order,
+    2N loads.  Plain DARTS prefers B1 (n=2) after A1 and differs."""
+    inst = _unit(gen.matmul2d(N, M=2 * N, K=1))
+    r = oracle.run(inst, bus_bps=10 ** 9, flags=oracle.F_FALLBACK2 | oracle.F_OPTI)
+    col_major = [i * N + j for j in range(N) for i in range(N)]
+    assert list(map(int, r.orders()[0])) == col_major
+    assert r.n_loads == 2 * N and r.n_evictions == 0
+    plain = oracle.run(inst, bus_bps=10 ** 9)
+    assert list(map(int, plain.orders()[0])) != col_major
+    _check(inst, r, bus=10 ** 9)
+
+
+@pytest.mark.parametrize("idx", range(8))
+def test_opti_invariants(idx):
+    inst = _small_instances()[idx]
+    r = oracle.run(inst, flags=oracle.F_FALLBACK2 | oracle.F_OPTI)
+    chk = _check(inst, r)
+    assert chk["n_loads"] == r.n_loads and chk["makespan"] == r.makespan
