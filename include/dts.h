@@ -54,7 +54,14 @@ typedef enum {
 } dts_status;
 
 typedef enum {
-    DTS_POLICY_DARTS_LUF = 1 /* Alg. 5 + Alg. 6 */
+    DTS_POLICY_DARTS_LUF = 1, /* Alg. 5 + Alg. 6 */
+    /* Comparison policies of the paper's evaluation, both
+     * with StarPU's default LRU eviction: the resident datum (not an input of
+     * the task being served) whose last use on the GPU is the oldest, lowest id
+     * on ties; an LRU eviction leaves plannedTasks untouched, so a planned task
+     * may reload data (the "domino effect"). */
+    DTS_POLICY_DARTS_LRU = 2, /* "DARTS": Alg. 5 selection, LRU eviction */
+    DTS_POLICY_EAGER_LRU = 3  /* "EAGER": one shared FIFO queue in submission order */
 } dts_policy;
 
 enum {

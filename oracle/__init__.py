@@ -27,6 +27,10 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 
 F_FALLBACK2 = 1
 F_OPTI = 8
+F_LRU = 16     # evict by LRU (not LUF): the paper's plain "DARTS" and "EAGER"
+F_EAGER = 32   # EAGER task choice: shared FIFO queue in submission order
+
+POLICY_FLAGS = {"darts_luf": 0, "darts_lru": F_LRU, "eager_lru": F_EAGER | F_LRU}
 DEFAULT_BUS_BPS = 12_000_000_000
 
 EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data", "<i4"),

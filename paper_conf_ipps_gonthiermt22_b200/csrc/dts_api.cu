@@ -323,6 +323,7 @@ dts_status ensure_device(dts_instance *I, int device) {
     add(4 * K * mp + 16); add(4 * (nstr + 4)); add(4 * K * (nstr + 4)); add(4 * K * (nstr + 4));  // s u h h2
     add(4 * K * (nstr + 4)); add(4 * K * nw); add(4 * K * res_cap);                  // np resb res_list
     add(16 * K * plan_cap); add(8 * K * plan_cap); add(4 * (3 * n + 1));              // plan tau vhist
+    add(4 * K * (nstr + 4));                                                          // lru stamps
     add(sizeof(dts::Out));
     add(4 * (m + 1)); add(4 * (m + 1)); add(8 * (m + 1)); add(8 * (m + 1));          // serve, times
     add(sizeof(dts_event) * ev_cap); add(8 * (K + 1)); add(4 * (m + 1));
@@ -388,6 +389,7 @@ dts_status ensure_device(dts_instance *I, int device) {
     h.plan = A.take<int4>(K * plan_cap);
     h.plan_tau = A.take<int64_t>(K * plan_cap);
     h.vhist = A.take<int32_t>(3 * n + 1);
+    h.lru = A.take<int32_t>(K * (nstr + 4));
     h.out = A.take<dts::Out>(1);
     h.serve_gpu = A.take<int32_t>(m + 1);
     h.serve_task = A.take<int32_t>(m + 1);
@@ -439,7 +441,8 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
 }
 
 dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_opts *o) {
-    if (policy != DTS_POLICY_DARTS_LUF) return fail(DTS_E_UNSUPPORTED, "policy");
+    if (policy != DTS_POLICY_DARTS_LUF && policy != DTS_POLICY_DARTS_LRU && policy != DTS_POLICY_EAGER_LRU)
+        return fail(DTS_E_UNSUPPORTED, "policy");
     if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI))
         return fail(DTS_E_UNSUPPORTED, "unknown flags");
     if (o->lookahead_W != 0) return fail(DTS_E_UNSUPPORTED, "lookahead_W != 0 (NEXT)");
@@ -456,7 +459,7 @@ dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_op
 // Shared-memory placement of one instance's state:
 // greedy, most latency-critical array first, each either fully in the CTA's
 // dynamic shared memory or in its global home.  Returns the bytes used.
-int place_smem(dts::Inst &h, bool has_tau, int budget) {
+int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru) {
     const int64_t K = h.K, n = h.n;
     int used = 0;
     auto put = [&](int32_t &so, int64_t bytes) {
@@ -478,6 +481,8 @@ int place_smem(dts::Inst &h, bool has_tau, int budget) {
     put(h.so_h, 4 * K * (int64_t)h.nstr);
     put(h.so_h2, 4 * K * (int64_t)h.nstr);
     put(h.so_np, 4 * K * (int64_t)h.nstr);
+    if (lru) put(h.so_lru, 4 * K * (int64_t)h.nstr);
+    else h.so_lru = -1;
     put(h.so_s, 4 * K * (int64_t)h.m_pad);  // last: the largest, worth it only when it fits
     h.smem_bytes = used;
     return used;
@@ -513,8 +518,8 @@ int env_int(const char *name, int dflt) {
 // Shared scratch of the fused in-CTA CSR build (dts_loop.cu fused_build).
 int fused_scratch_bytes(const dts_instance *I, int block) { return (2 * (block / 32) + 1) * 4 * (I->n + 1); }
 
-dts_status stage(dts_instance *I, const dts_run_opts &o, int budget, int block, cudaStream_t st,
-                 bool copy_desc = true) {
+dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int budget, int block,
+                 cudaStream_t st, bool copy_desc = true) {
     dts_status s = ensure_device(I, o.device);
     if (s != DTS_OK) return s;
     CK(cudaSetDevice(o.device), "cudaSetDevice");
@@ -527,6 +532,7 @@ dts_status stage(dts_instance *I, const dts_run_opts &o, int budget, int block, 
     h.W = (int32_t)o.lookahead_W;
     h.flags = o.flags;
     h.max_served = o.max_served;
+    h.policy = (int32_t)policy;
     h.size0 = 0;
     h.delta0 = 0;
     h.bw = o.bus_bytes_per_s;
@@ -537,7 +543,7 @@ dts_status stage(dts_instance *I, const dts_run_opts &o, int budget, int block, 
         const unsigned __int128 num = (unsigned __int128)h.size0 * 1000000000u + (o.bus_bytes_per_s - 1);
         h.delta0 = (int64_t)(num / o.bus_bytes_per_s);  // ceil, reading R9 (same as dts_init_kernel)
     }
-    place_smem(h, I->has_tau, budget);
+    place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF);
     // small instances: the loop CTA builds its own CSR and state (one launch)
     const int fs = fused_scratch_bytes(I, block);
     h.fused = !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
@@ -601,7 +607,7 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
     const int budget = budget_of(o);
     const int block = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", auto_block(I));
-    s = stage(I, o, budget, block, st);
+    s = stage(I, policy, o, budget, block, st);
     if (s != DTS_OK) return s;
     const int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n + 4);
     if (!I->h_inst.fused) CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
@@ -649,7 +655,7 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     int smem = 0;
     bool any_unfused = false;
     for (int32_t i = 0; i < n; i++) {
-        s = stage(insts[i], o, budget, block, st, false);
+        s = stage(insts[i], policy, o, budget, block, st, false);
         if (s != DTS_OK) return s;
         smem = std::max(smem, insts[i]->h_inst.smem_bytes);
         any_unfused |= !insts[i]->h_inst.fused;

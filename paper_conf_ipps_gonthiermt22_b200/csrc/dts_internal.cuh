@@ -25,6 +25,7 @@
 //   plan[K][plan_cap] int4 -- plannedTasks_k in ascending id: {T, D0, D1, D2}
 //       (T = -1: removed by LUF; D(T) cached when |D(T)| <= 3, D2 = -2 when
 //       the row is longer)                                           [S/G]
+//   lru[K][nstr] int32 -- serve index of D's last use on GPU k (LRU)   [S/G]
 //   plan_tau[K][plan_cap] int64 -- their durations (per-task times only)  [S/G]
 #pragma once
 #include <cstdint>
@@ -96,6 +97,9 @@ struct Inst {
     int4 *plan;
     int64_t *plan_tau;
     int32_t *vhist;  // DTS_F_VERIFY scratch [3 n]
+    int32_t *lru;    // [K][nstr] last-use stamps (LRU policies)
+    int32_t policy;  // dts_policy
+    int32_t so_lru;
     // shared-memory placement: byte offset in the CTA's dynamic smem, -1 = global home
     int32_t so_u, so_h, so_h2, so_np, so_resb, so_res_list, so_plan, so_plan_tau, so_s, so_dptr;
     int32_t smem_bytes;

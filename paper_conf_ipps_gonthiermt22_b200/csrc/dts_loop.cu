@@ -49,7 +49,7 @@ __device__ __forceinline__ void cta_sync() {
     __syncwarp();
 }
 
-enum Cmd : int { CMD_SCAN = 1, CMD_DONE = 2 };
+enum Cmd : int { CMD_SCAN = 1, CMD_DONE = 2, CMD_POP = 3, CMD_EAGER = 4 };
 
 // Per-phase cycle accounting by thread 0 (diagnostics, dts_result_view.prof_cycles).
 enum Prof : int { P_POP = 0, P_ARGMAX, P_PLAN, P_LOADS, P_LUF, P_EVICT, P_SEG, P_OTHER, P_BW0, P_BD, P_NB, P_NP, P_X1, P_X2, P_X3, P_X4 };
@@ -94,6 +94,7 @@ struct View {
     int4 *plan;
     int64_t *plan_cum;  // inclusive prefix sums of the planned tasks' tau (per-task times only)
     int32_t *dptr32;    // shared-memory copy of dptr, or nullptr
+    int32_t *lru;       // [K][nstr] last-use stamps (LRU policies)
 };
 
 // Per-CTA state at namespace scope, so the (non-inlined) phase functions
@@ -785,7 +786,8 @@ __device__ int32_t luf_victim(int k) {
     const View &V = SV;
     const int cnt = L.res_cnt[k];
     const int32_t *rl = V.res_list + (size_t)k * I.res_cap;
-    const int32_t *npk = V.np + (size_t)k * I.nstr;
+    // LUF key np_k(D); LRU policies: the serve index of D's last use on k
+    const int32_t *npk = (I.policy == DTS_POLICY_DARTS_LUF ? V.np : V.lru) + (size_t)k * I.nstr;
     unsigned long long best = ~0ull;
     for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
         const int32_t D = rl[i];
@@ -813,7 +815,8 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
     int4 *pl = V.plan + (size_t)k * I.plan_cap;
     int nret = 0;
     unsigned long long tmin = ~0ull;
-    const int ph = L.plan_head[k], pe = L.plan_end[k];
+    // Alg. 6 l.8 is LUF's; an LRU eviction leaves plannedTasks_k alone
+    const int ph = L.plan_head[k], pe = I.policy == DTS_POLICY_DARTS_LUF ? L.plan_end[k] : ph;
     for (int i = ph + threadIdx.x; i < pe; i += blockDim.x) {
         const int4 e = pl[i];
         if (e.x >= 0 && entry_uses(e, Vd)) {
@@ -908,7 +911,13 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
         cta_sync();
         PROF_ADD(L, P_SEG, p_seg);
     }
-    if (threadIdx.x == 0) finish_serve(k, T, L.ready, tau_of(T));
+    if (threadIdx.x == 0) {
+        if (I.policy != DTS_POLICY_DARTS_LUF) {  // LRU: D(T) used by the n_served-th task
+            int32_t *lk = V.lru + (size_t)k * I.nstr;
+            for (int r = 0; r < L.row_len; r++) lk[L.row[r]] = (int32_t)L.n_served;
+        }
+        finish_serve(k, T, L.ready, tau_of(T));
+    }
     cta_sync();
 }
 
@@ -1406,6 +1415,7 @@ __global__ void __launch_bounds__(512, 1)
             W.plan = I.so_plan >= 0 ? (int4 *)(dsm + I.so_plan) : I.plan;
             W.plan_cum = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
             W.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
+            W.lru = I.so_lru >= 0 ? (int32_t *)(dsm + I.so_lru) : I.lru;
         }
         cta_sync();
         const View &V = SV;
@@ -1460,26 +1470,76 @@ __global__ void __launch_bounds__(512, 1)
         // ---- the decision loop
         while (true) {
             PROF_T0(p_pop);
-            int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
-            for (int j = 0; j < K; j++) pending += L.plan_live[j];
-            if (I.max_served < 0 && K <= 32 && pending > 10) {
-                pop_batch();
-            } else {  // few pops (or a prefix run that stops at an exact count): thread 0
+            if (I.policy == DTS_POLICY_DARTS_LUF) {
+                int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
+                for (int j = 0; j < K; j++) pending += L.plan_live[j];
+                if (I.max_served < 0 && K <= 32 && pending > 10) {
+                    pop_batch();
+                } else {  // few pops (or a prefix run that stops at an exact count): thread 0
+                    cta_sync();
+                    if (tid == 0)
+                        L.cmd = ((I.max_served < 0 || L.n_served < I.max_served) && pop_run_seq() >= 0)
+                                    ? CMD_SCAN
+                                    : CMD_DONE;
+                }
+            } else {
+                // LRU policies: an LRU eviction does not drop planned tasks, so a
+                // pop may need loads -- every request is served block-wide
                 cta_sync();
-                if (tid == 0)
-                    L.cmd = ((I.max_served < 0 || L.n_served < I.max_served) && pop_run_seq() >= 0)
-                                ? CMD_SCAN
-                                : CMD_DONE;
+                if (tid == 0) {
+                    int cmd = CMD_DONE;
+                    if (I.max_served < 0 || L.n_served < I.max_served) {
+                        int kk = -1;  // next request: smallest (req_k, k), non-idle (R8)
+                        int64_t tb = 0;
+                        for (int j = 0; j < K; j++)
+                            if (!L.idle[j] && (kk < 0 || L.req[j] < tb)) {
+                                kk = j;
+                                tb = L.req[j];
+                            }
+                        if (kk >= 0) {
+                            L.k = kk;
+                            L.t = tb;
+                            if (I.policy == DTS_POLICY_DARTS_LRU && L.plan_live[kk] > 0) {
+                                int64_t tau;
+                                L.T = pop_planned(kk, &tau);
+                                cmd = CMD_POP;
+                            } else {
+                                cmd = I.policy == DTS_POLICY_EAGER_LRU ? CMD_EAGER : CMD_SCAN;
+                            }
+                        }
+                    }
+                    L.cmd = cmd;
+                }
             }
             PROF_ADD(L, P_POP, p_pop);
             cta_sync();
             if (L.cmd == CMD_DONE) break;
             const int k = L.k;
             const int64_t t = L.t;
+            int32_t T = -1;
+            if (L.cmd == CMD_POP) {
+                T = L.T;
+            } else if (L.cmd == CMD_EAGER) {
+                // EAGER: the shared FIFO queue in submission
+                // order -- the lowest-id unallocated task
+                T = L.n_avail > 0 ? first_avail() : -1;
+                if (tid == 0) {
+                    if (T >= 0) {
+                        L.avail_lo = T;
+                        L.row_len = -1;
+                        pool_move(T, row_of_task(T), -1, -1);
+                        L.n_avail--;
+                    } else {
+                        L.idle[k] = 1;
+                        L.n_idle++;
+                    }
+                }
+                cta_sync();
+                if (T < 0) continue;
+            } else {
             reset_plan(k);
             if (I.flags & DTS_F_VERIFY) verify_scores(k);
             // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
-            int32_t T = -1;
             PROF_T0(p_am);
             const int32_t Dopt = (I.flags & DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
                                                         : score_argmax(V.h + (size_t)k * I.nstr);
@@ -1533,6 +1593,7 @@ __global__ void __launch_bounds__(512, 1)
                 PROF_ADD(L, P_OTHER, p_pl);
                 if (T < 0) continue;
             }
+            }  // scan
             // serve T with its loads (block-wide); D(T) from the CSR unless cached
             const bool need_row = L.row_len < 0;
             cta_sync();

@@ -28,6 +28,8 @@ DTS_E_CUDA = -4
 DTS_E_STATE = -5
 DTS_E_UNSUPPORTED = -6
 DTS_POLICY_DARTS_LUF = 1
+DTS_POLICY_DARTS_LRU = 2
+DTS_POLICY_EAGER_LRU = 3
 DTS_F_FALLBACK2 = 1
 DTS_F_VERIFY = 2
 DTS_F_NOFUSE = 4
@@ -233,7 +235,8 @@ def dts_version() -> int:
     return int(load_library().dts_version())
 
 
-def schedule(inst, *, W: int = 0, flags: int = DTS_F_FALLBACK2, bus_bps: int = 12_000_000_000,
+def schedule(inst, *, policy: int = DTS_POLICY_DARTS_LUF, W: int = 0, flags: int = DTS_F_FALLBACK2,
+             bus_bps: int = 12_000_000_000,
              device: int = 0, block_threads: int = 0, smem_budget: int = 0,
              max_served: int = -1, stream: int = 0) -> Result:
     """One call: create the instance from host arrays (a ``gen.Instance``-like
@@ -243,7 +246,7 @@ def schedule(inst, *, W: int = 0, flags: int = DTS_F_FALLBACK2, bus_bps: int = 1
     o = dts_run_opts_default(flags=flags, lookahead_W=W, bus_bytes_per_s=bus_bps, device=device,
                              block_threads=block_threads, smem_budget=smem_budget,
                              max_served=max_served, cuda_stream=stream or None)
-    dts_run(h, DTS_POLICY_DARTS_LUF, o)
+    dts_run(h, policy, o)
     return dts_result(h)
 
 
@@ -253,7 +256,7 @@ def create(inst) -> Instance:
                                inst.default_task_ns, inst.mem_capacity, inst.K)
 
 
-def schedule_batch(insts, *, W: int = 0, flags: int = DTS_F_FALLBACK2,
+def schedule_batch(insts, *, policy: int = DTS_POLICY_DARTS_LUF, W: int = 0, flags: int = DTS_F_FALLBACK2,
                    bus_bps: int = 12_000_000_000, device: int = 0, block_threads: int = 0,
                    smem_budget: int = 0, stream: int = 0):
     """Run many independent instances in ONE batched launch (dts_sweep_run,
@@ -262,5 +265,5 @@ def schedule_batch(insts, *, W: int = 0, flags: int = DTS_F_FALLBACK2,
     o = dts_run_opts_default(flags=flags, lookahead_W=W, bus_bytes_per_s=bus_bps, device=device,
                              block_threads=block_threads, smem_budget=smem_budget,
                              max_served=-1, cuda_stream=stream or None)
-    dts_sweep_run(hs, DTS_POLICY_DARTS_LUF, o)
+    dts_sweep_run(hs, policy, o)
     return [dts_result(h) for h in hs]

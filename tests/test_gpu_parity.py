@@ -313,3 +313,55 @@ def test_workload_variants(idx, flags):
     g, o = _both(inst, flags=flags)
     assert_parity(g, o)
     validate(inst, g.serve_gpu, g.serve_task, g.events, g.task_start, g.task_end)
+
+
+# ------------------------------------------------------------ DARTS+LRU, EAGER+LRU (§8(f)2)
+_POL = {"darts_lru": (dts.DTS_POLICY_DARTS_LRU, oracle.F_LRU),
+        "eager_lru": (dts.DTS_POLICY_EAGER_LRU, oracle.F_EAGER | oracle.F_LRU)}
+
+
+def _both_policy(inst, name, bus=oracle.DEFAULT_BUS_BPS, flags=1, smem=0, max_served=-1):
+    pol, of = _POL[name]
+    g = dts.schedule(inst, policy=pol, bus_bps=bus, flags=flags, smem_budget=smem,
+                     max_served=max_served)
+    o = oracle.run(inst, bus_bps=bus, flags=flags | of, max_served=max_served)
+    return g, o
+
+
+@pytest.mark.parametrize("name", ["darts_lru", "eager_lru"])
+@pytest.mark.parametrize("idx", range(12))
+def test_lru_policies_shapes(name, idx):
+    inst = _shapes()[idx]
+    for smem in (0, -1):
+        g, o = _both_policy(inst, name, smem=smem)
+        assert_parity(g, o)
+        validate(inst, g.serve_gpu, g.serve_task, g.events, g.task_start, g.task_end)
+
+
+def test_eager_lru_hand_trace_gpu():
+    inst = _unit(gen.matmul2d(3, M=4, K=1))
+    g = dts.schedule(inst, policy=dts.DTS_POLICY_EAGER_LRU, bus_bps=10 ** 9)
+    assert [int(e["data"]) for e in g.events if e["op"] == 0] == [0, 3, 4, 5, 1, 4, 2, 4]
+    assert [int(e["data"]) for e in g.events if e["op"] == 1] == [4, 0, 4, 1]
+
+
+@pytest.mark.parametrize("name", ["darts_lru", "eager_lru"])
+def test_lru_policies_config2_batch(name):
+    pol, of = _POL[name]
+    insts = gen.config_instances("C2")
+    gs = dts.schedule_batch(insts, policy=pol)
+    for inst, g in zip(insts, gs):
+        assert_parity(g, oracle.run(inst, flags=1 | of))
+
+
+@pytest.mark.parametrize("name", ["darts_lru", "eager_lru"])
+def test_lru_policies_config3(name):
+    g, o = _both_policy(gen.config_instances("C3")[0], name)
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("name", ["darts_lru", "eager_lru"])
+@pytest.mark.parametrize("cfg", ["C4a", "C4b"])
+def test_lru_policies_config4_prefix(name, cfg):
+    g, o = _both_policy(gen.config_instances(cfg)[0], name, max_served=1500)
+    assert_parity(g, o, complete=False)

@@ -220,3 +220,67 @@ def test_opti_invariants(idx):
     r = oracle.run(inst, flags=oracle.F_FALLBACK2 | oracle.F_OPTI)
     chk = _check(inst, r)
     assert chk["n_loads"] == r.n_loads and chk["makespan"] == r.makespan
+
+
+# ---------------------------------------------------- EAGER / LRU (§8(f)2)
+def lru_replay_one(order, dsets, M):
+    """Independent LRU replay of a FIXED per-GPU order with unit sizes: before
+    each task, load its missing inputs in ascending id, evicting the resident
+    datum (not an input of the task) whose last use is the oldest, lowest id on
+    ties; then every input is 'used' by this task.  Returns (loads, evicts)
+    as lists of data ids in event order."""
+    mem, last, loads, evicts = set(), {}, [], []
+    for idx, T in enumerate(order):
+        need = dsets[T]
+        for D in sorted(need - mem):
+            if len(mem) >= M:
+                cand = sorted(mem - need)
+                V = min(cand, key=lambda x: (last[x], x))
+                mem.remove(V)
+                evicts.append(V)
+            mem.add(D)
+            loads.append(D)
+        for D in need:
+            last[D] = idx
+    return loads, evicts
+
+
+def test_eager_lru_2d_hand_trace():
+    """Hand trace (EAGER = shared FIFO in submission order, PAPER.md:819-825;
+    LRU eviction): 2D N=3, K=1, M=4.  Loads A0 B0 B1 B2 A1 B1 A2 B1, evictions
+    B1 A0 B1 A1 (ids: A_i = i, B_j = 3 + j); 8 loads."""
+    inst = _unit(gen.matmul2d(3, M=4, K=1))
+    r = oracle.run(inst, bus_bps=10 ** 9, flags=oracle.POLICY_FLAGS["eager_lru"])
+    assert list(map(int, r.orders()[0])) == list(range(9))
+    assert [int(e["data"]) for e in r.events if e["op"] == 0] == [0, 3, 4, 5, 1, 4, 2, 4]
+    assert [int(e["data"]) for e in r.events if e["op"] == 1] == [4, 0, 4, 1]
+    assert r.n_scans == 0
+    _check(inst, r, bus=10 ** 9)
+
+
+@pytest.mark.parametrize("policy", ["eager_lru", "darts_lru"])
+@pytest.mark.parametrize("idx", range(8))
+def test_lru_matches_independent_replay(policy, idx):
+    """Every GPU's load/evict sequence equals an independent LRU replay of its
+    task order (LRU decisions depend only on the GPU's own order)."""
+    inst = _unit(_small_instances()[idx])
+    M = int(inst.mem_capacity)
+    r = oracle.run(inst, bus_bps=10 ** 9, flags=oracle.F_FALLBACK2 | oracle.POLICY_FLAGS[policy])
+    _check(inst, r, bus=10 ** 9)
+    ds = dsets_of(inst)
+    for k, order in enumerate(r.orders()):
+        loads, evicts = lru_replay_one(list(map(int, order)), ds, M)
+        ev = r.events[r.events["gpu"] == k]
+        assert [int(e["data"]) for e in ev if e["op"] == 0] == loads
+        assert [int(e["data"]) for e in ev if e["op"] == 1] == evicts
+    if policy == "eager_lru" and inst.K == 1:
+        assert list(map(int, r.orders()[0])) == list(range(inst.m))
+
+
+def test_eager_lru_collapse_when_one_matrix_fits():
+    """EAGER+LRU collapses once only one matrix fits:
+    2D N=20 with M = N+1 reloads far more than DARTS+LUF."""
+    inst = gen.matmul2d(20, M=21, K=1)
+    eager = oracle.run(inst, flags=oracle.POLICY_FLAGS["eager_lru"])
+    darts = oracle.run(inst)
+    assert eager.n_loads > 2 * darts.n_loads
