@@ -146,6 +146,9 @@ def workload_instances(name, rank, world):
 
 
 # ------------------------------------------------------------------ oracle
+ORACLE_FLAGS = 1  # set in main(): FALLBACK2 | policy | OPTI
+
+
 def oracle_sample(insts, budget_s, threads):
     """Time the plain CPU oracle (as it stands) over the batch, repeated until
     budget_s elapsed; one instance per thread (ctypes releases the GIL)."""
@@ -158,7 +161,7 @@ def oracle_sample(insts, budget_s, threads):
         while True:
             # biggest instances first so the pool stays busy
             order = sorted(insts, key=lambda i: -i.E)
-            rs = list(ex.map(lambda i: oracle.run(i), order))
+            rs = list(ex.map(lambda i: oracle.run(i, flags=ORACLE_FLAGS), order))
             done_dec += sum(r.n_served for r in rs)
             n_batches += 1
             if time.perf_counter() - t0 >= budget_s:
@@ -174,7 +177,7 @@ def oracle_prefix_sample(inst, budget_s):
     n = 200
     while True:
         t0 = time.perf_counter()
-        r = oracle.run(inst, max_served=n)
+        r = oracle.run(inst, max_served=n, flags=ORACLE_FLAGS)
         dt = time.perf_counter() - t0
         if dt >= budget_s / 4 or n >= inst.m:
             return r.n_served / dt, dt, r.n_served
@@ -211,7 +214,8 @@ def run_reference(args, rank, world):
             "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
             "scaling": scaling, "vs_baseline": None, "dtype": "int64", "data": "synthetic",
-            "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload]}"},
+            "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload]}",
+                       "policy": args.policy + ("+opti" if args.opti else "") + " (3inputs fallback on)"},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": thr, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -226,11 +230,16 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="C2", choices=list(WORKLOADS))
+    ap.add_argument("--policy", default="darts_luf", choices=["darts_luf", "darts_lru", "eager_lru"],
+                    help="DARTS+LUF (the method) or a comparison policy of the paper")
+    ap.add_argument("--opti", action="store_true", help="OPTI variant (PAPER.md:2121-2124)")
     ap.add_argument("--cpu-budget", type=float, default=10.0,
                     help="seconds of oracle time for cpu_baseline (rank 0, N=1)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
 
+    global ORACLE_FLAGS
+    ORACLE_FLAGS = 1 | {"darts_luf": 0, "darts_lru": 16, "eager_lru": 48}[args.policy] | (8 if args.opti else 0)
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
@@ -256,7 +265,10 @@ def main():
     insts, scaling = workload_instances(args.workload, rank, world)
     single = args.workload in ("C3", "C4a", "C4b")  # one large instance: grouped CTAs
     handles = [dts.create(i) for i in insts]
-    opts = dts.dts_run_opts_default(device=dev, cuda_stream=sptr)
+    policy = {"darts_luf": dts.DTS_POLICY_DARTS_LUF, "darts_lru": dts.DTS_POLICY_DARTS_LRU,
+              "eager_lru": dts.DTS_POLICY_EAGER_LRU}[args.policy]
+    opts = dts.dts_run_opts_default(device=dev, cuda_stream=sptr,
+                                    flags=dts.DTS_F_FALLBACK2 | (dts.DTS_F_OPTI if args.opti else 0))
     for h in handles:
         dts.dts_instance_upload(h, dev, sptr)
     torch.cuda.synchronize()
@@ -264,9 +276,9 @@ def main():
     def step():
         if single:
             for h in handles:
-                dts.dts_run(h, dts.DTS_POLICY_DARTS_LUF, opts)
+                dts.dts_run(h, policy, opts)
         else:
-            dts.dts_sweep_run(handles, dts.DTS_POLICY_DARTS_LUF, opts)
+            dts.dts_sweep_run(handles, policy, opts)
 
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.int32, device="cuda")  # > 126 MB L2
 
@@ -359,6 +371,7 @@ def main():
             "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
             "dtype": "int32", "data": "synthetic",
             "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload]}",
+                       "policy": args.policy + ("+opti" if args.opti else "") + " (3inputs fallback on)",
                        "instances_per_rank": len(insts), "decisions_per_step": int(all_dec),
                        "l2": "flushed between timed steps (256 MiB write)",
                        "launch": "one batched loop launch, one CTA per instance" if not single
