@@ -49,6 +49,8 @@ __device__ __forceinline__ void cta_sync() {
     __syncwarp();
 }
 
+constexpr int POP_RANK_MAX = 256;  // pops ranked by counting in one pass
+
 enum Cmd : int { CMD_SCAN = 1, CMD_DONE = 2, CMD_POP = 3, CMD_EAGER = 4 };
 
 // Per-phase cycle accounting by thread 0 (diagnostics, dts_result_view.prof_cycles).
@@ -83,6 +85,8 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     long long prof[16];
     int64_t bstart[32], breq[32], bns;  // pop batch (K <= 32): per-GPU first start / request
     int32_t bhead[32], bcnt[32], boff[33];
+    int64_t rkey[POP_RANK_MAX];  // pop batch: request time of each pop (merge ranks)
+    int32_t rgpu[POP_RANK_MAX];
 };
 
 // Per-instance views: shared-memory arrays where placed, else global homes.
@@ -596,28 +600,31 @@ __device__ __forceinline__ int64_t pop_req(int j, const PopGpu &g, int i) {
 // request (r, k) in the (time, GPU id) order (R8).  Request times increase
 // with i, so a binary search (multiplications only: 64-bit division is a long
 // software sequence on the SM).
-__device__ int pops_before(int j, PopGpu g, int c, int64_t r, int k) {
+__device__ __forceinline__ int pops_before(int j, PopGpu g, int c, int64_t r, int k) {
     const Inst &I = SI;
     const View &V = SV;
     if (c <= 0) return 0;
     const bool tie_ok = j < k;  // equal times: the lower GPU id asks first
     if (!(g.req < r || (g.req == r && tie_ok))) return 0;
-    int lo = 1, hi = c;  // first i in [1, c] whose request does not precede (r, k)
-    if (!V.plan_cum) {
+    if (!V.plan_cum) {  // i >= 1 asks at start0 + i * tau: binary search, multiplications only
         const int64_t tau = I.default_tau;
+        int lo = 1, hi = c;
         while (lo < hi) {
             const int mid = (lo + hi) >> 1;
             const int64_t rm = g.start0 + (int64_t)mid * tau;
-            if (rm < r || (rm == r && tie_ok)) lo = mid + 1;
-            else hi = mid;
+            const bool b = (rm < r) | ((rm == r) & tie_ok);
+            lo = b ? mid + 1 : lo;
+            hi = b ? hi : mid;
         }
         return lo;
     }
+    int lo = 1, hi = c;  // first i in [1, c] whose request does not precede (r, k)
     while (lo < hi) {
         const int mid = (lo + hi) >> 1;
         const int64_t rm = g.start0 + plan_span(j, g.head, mid);
-        if (rm < r || (rm == r && tie_ok)) lo = mid + 1;
-        else hi = mid;
+        const bool b = (rm < r) | ((rm == r) & tie_ok);
+        lo = b ? mid + 1 : lo;
+        hi = b ? hi : mid;
     }
     return lo;
 }
@@ -632,63 +639,136 @@ __device__ int pops_before(int j, PopGpu g, int c, int64_t r, int k) {
 // earliest (request after the GPU's last pop, GPU id) (R8) -- and each GPU's
 // pop count before it; then every thread places pops in the global service
 // order by merge ranks.  Sets L.cmd (CMD_SCAN with L.k, L.t, or CMD_DONE).
+// Scalar phase of pop_batch for K <= KR with the per-GPU values in registers
+// (fully unrolled over KR): the next scan (earliest request after a GPU's last
+// pop, R8), each GPU's pop count before it, the new request times.
+template <int KR>
+__device__ __forceinline__ void pop_batch_scalar() {
+    const Inst &I = SI;
+    const int K = I.K;
+    int64_t rq[KR], st[KR], S[KR];
+    int hd[KR], lv[KR];
+    bool act[KR];
+#pragma unroll
+    for (int j = 0; j < KR; j++) {
+        act[j] = j < K && !L.idle[j];
+        rq[j] = j < K ? L.req[j] : 0;
+        const int64_t gf = j < K ? L.gpu_free[j] : 0;
+        st[j] = rq[j] > gf ? rq[j] : gf;
+        hd[j] = j < K ? L.plan_head[j] : 0;
+        lv[j] = j < K ? L.plan_end[j] - hd[j] : 0;
+    }
+    int kb = -1;
+    int64_t sb = INT64_MAX;
+#pragma unroll
+    for (int j = 0; j < KR; j++) {
+        S[j] = lv[j] == 0 ? rq[j] : st[j] + plan_span(j, hd[j], lv[j]);
+        const bool take = act[j] & ((kb < 0) | (S[j] < sb));
+        kb = take ? j : kb;
+        sb = take ? S[j] : sb;
+    }
+    int total = 0;
+    int64_t mk = L.makespan;
+#pragma unroll
+    for (int j = 0; j < KR; j++) {
+        if (j >= K) break;
+        int c = 0;
+        if (act[j] && kb >= 0) {
+            PopGpu g;
+            g.req = rq[j];
+            g.start0 = st[j];
+            g.head = hd[j];
+            c = j == kb ? lv[j] : pops_before(j, g, lv[j], sb, kb);
+        }
+        L.breq[j] = rq[j];
+        L.bstart[j] = st[j];
+        L.bhead[j] = hd[j];
+        L.bcnt[j] = c;
+        L.boff[j] = total;
+        total += c;
+        if (c > 0) {
+            const int64_t last = st[j] + plan_span(j, hd[j], c);
+            L.req[j] = last;  // W = 0 (R7)
+            L.gpu_free[j] = last;
+            L.plan_head[j] = hd[j] + c;
+            L.plan_live[j] -= c;
+            mk = last > mk ? last : mk;
+        }
+    }
+    L.boff[K] = total;
+    L.bns = L.n_served;
+    L.n_served += total;
+    L.makespan = mk;
+    L.alg_bytes += 24ull * (uint64_t)total;
+    L.k = kb;
+    L.t = sb;
+    L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
+}
+
+// The same for 8 < K <= 32, values left in shared memory.
+__device__ __noinline__ void pop_batch_scalar_smem() {
+    const Inst &I = SI;
+    const int K = I.K;
+    int kb = -1;
+    int64_t sb = INT64_MAX;
+    for (int j = 0; j < K; j++) {
+        const int64_t req = L.req[j];
+        const int64_t start0 = req > L.gpu_free[j] ? req : L.gpu_free[j];
+        const int head = L.plan_head[j];
+        L.breq[j] = req;
+        L.bstart[j] = start0;
+        L.bhead[j] = head;
+        if (L.idle[j]) continue;
+        const int live = L.plan_end[j] - head;
+        const int64_t S = live == 0 ? req : start0 + plan_span(j, head, live);
+        if (kb < 0 || S < sb) {
+            kb = j;
+            sb = S;
+        }
+    }
+    int total = 0;
+    int64_t mk = L.makespan;
+    for (int j = 0; j < K; j++) {
+        int c = 0;
+        if (!L.idle[j] && kb >= 0) {
+            const int live = L.plan_end[j] - L.bhead[j];
+            PopGpu g;
+            g.req = L.breq[j];
+            g.start0 = L.bstart[j];
+            g.head = L.bhead[j];
+            c = j == kb ? live : pops_before(j, g, live, sb, kb);
+        }
+        L.bcnt[j] = c;
+        L.boff[j] = total;
+        total += c;
+        if (c > 0) {
+            const int64_t last = L.bstart[j] + plan_span(j, L.bhead[j], c);
+            L.req[j] = last;  // W = 0 (R7)
+            L.gpu_free[j] = last;
+            L.plan_head[j] += c;
+            L.plan_live[j] -= c;
+            mk = last > mk ? last : mk;
+        }
+    }
+    L.boff[K] = total;
+    L.bns = L.n_served;
+    L.n_served += total;
+    L.makespan = mk;
+    L.alg_bytes += 24ull * (uint64_t)total;
+    L.k = kb;
+    L.t = sb;
+    L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
+}
+
 __device__ void pop_batch() {
     const Inst &I = SI;
     const View &V = SV;
     const int K = I.K;
     PROF_T0(p_w0);
-    if (threadIdx.x == 0) {  // scalar phase: K is small, a serial pass beats warp shuffles
-        int kb = -1;
-        int64_t sb = INT64_MAX;
-        for (int j = 0; j < K; j++) {  // the next scan: earliest (request after the last pop, j)
-            const int64_t req = L.req[j];
-            const int64_t start0 = req > L.gpu_free[j] ? req : L.gpu_free[j];
-            const int head = L.plan_head[j];
-            L.breq[j] = req;
-            L.bstart[j] = start0;
-            L.bhead[j] = head;
-            if (L.idle[j]) continue;
-            const int live = L.plan_end[j] - head;
-            const int64_t S = live == 0 ? req : start0 + plan_span(j, head, live);
-            if (kb < 0 || S < sb) {
-                kb = j;
-                sb = S;
-            }
-        }
-        L.prof[P_X2] += clock64() - p_w0;
-        int total = 0;
-        int64_t mk = L.makespan;
-        for (int j = 0; j < K; j++) {
-            int c = 0;
-            if (!L.idle[j] && kb >= 0) {
-                const int live = L.plan_end[j] - L.bhead[j];
-                PopGpu g;
-                g.req = L.breq[j];
-                g.start0 = L.bstart[j];
-                g.head = L.bhead[j];
-                c = j == kb ? live : pops_before(j, g, live, sb, kb);
-            }
-            L.bcnt[j] = c;
-            L.boff[j] = total;
-            total += c;
-            if (c > 0) {
-                const int64_t last = L.bstart[j] + plan_span(j, L.bhead[j], c);
-                L.req[j] = last;  // W = 0 (R7)
-                L.gpu_free[j] = last;
-                L.plan_head[j] += c;
-                L.plan_live[j] -= c;
-                mk = last > mk ? last : mk;
-            }
-        }
-        L.prof[P_X4] += clock64() - p_w0;
-        L.boff[K] = total;
-        L.bns = L.n_served;
-        L.n_served += total;
-        L.makespan = mk;
-        L.alg_bytes += 24ull * (uint64_t)total;
-        L.k = kb;
-        L.t = sb;
-        L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
+    if (threadIdx.x == 0) {
+        if (K <= 4) pop_batch_scalar<4>();
+        else if (K <= 8) pop_batch_scalar<8>();
+        else pop_batch_scalar_smem();
     }
     cta_sync();
     PROF_ADD(L, P_BW0, p_w0);
@@ -699,6 +779,41 @@ __device__ void pop_batch() {
         L.prof[P_NB] += 1;
         L.prof[P_NP] += P;
     }
+    if (P <= (int)blockDim.x && P <= POP_RANK_MAX) {
+        // merge ranks by counting: each pop's key (request time, GPU) in shared
+        // memory, position = #keys before it (ties inside a GPU keep pop order)
+        int j = 0, i = 0, T = -1;
+        int64_t r = 0, start = 0, end = 0;
+        const int p = threadIdx.x;
+        if (p < P) {
+            while (L.boff[j + 1] <= p) j++;
+            i = p - L.boff[j];
+            PopGpu g;
+            g.req = L.breq[j];
+            g.start0 = L.bstart[j];
+            g.head = L.bhead[j];
+            r = pop_req(j, g, i);
+            start = i == 0 ? g.start0 : r;
+            end = g.start0 + plan_span(j, g.head, i + 1);
+            T = V.plan[(size_t)j * I.plan_cap + g.head + i].x;
+            L.rkey[p] = r;
+            L.rgpu[p] = j;
+        }
+        cta_sync();
+        if (p < P) {
+            int64_t pos = ns;
+            for (int q = 0; q < P; q++) {
+                const int64_t rq = L.rkey[q];
+                const int jq = L.rgpu[q];
+                // bitwise, not short-circuit: one predicated chain, no branches
+                pos += (int)((rq < r) | ((rq == r) & ((jq < j) | ((jq == j) & (q < p)))));
+            }
+            __stcg(&I.tstart[T], start);
+            __stcg(&I.tend[T], end);
+            __stcg(&I.serve_gpu[pos], j);
+            __stcg(&I.serve_task[pos], T);
+        }
+    } else {
     for (int p = threadIdx.x; p < P; p += blockDim.x) {
         int j = 0;
         while (L.boff[j + 1] <= p) j++;
@@ -724,6 +839,7 @@ __device__ void pop_batch() {
         __stcg(&I.tend[T], end);
         __stcg(&I.serve_gpu[pos], j);
         __stcg(&I.serve_task[pos], T);
+    }
     }
     cta_sync();
     PROF_ADD(L, P_BD, p_bd);
@@ -793,10 +909,9 @@ __device__ int32_t luf_victim(int k) {
         const int32_t D = rl[i];
         bool in_buf = false;
         for (int r = 0; r < L.row_len; r++) in_buf |= (L.row[r] == D);
-        if (in_buf) continue;
         const unsigned long long key =
             ((unsigned long long)(uint32_t)npk[D] << 32) | (unsigned long long)(uint32_t)D;
-        best = key < best ? key : best;
+        best = (!in_buf & (key < best)) ? key : best;
     }
     best = block_min_u64(best);
     if (best == ~0ull) return -1;
