@@ -85,8 +85,11 @@ enum {
 
 typedef struct {
     uint32_t flags;           /* DTS_F_* ; default DTS_F_FALLBACK2 */
-    uint32_t lookahead_W;     /* taskBuffer depth beyond the served task;
-                                 0 (default, the formal model of §III) -- others: UNSUPPORTED */
+    uint32_t lookahead_W;     /* taskBuffer depth beyond the served task:
+                                 0 (default, the formal model of §III: a GPU asks for its
+                                 next task when the current one ends) or 1 (StarPU's
+                                 prefetch: it asks when the current one starts, and LUF
+                                 protects both tasks' inputs; reading R7); >1: UNSUPPORTED */
     uint64_t bus_bytes_per_s; /* shared host->GPU bus bandwidth; default 12e9 (reading R9) */
     int32_t device;           /* CUDA device ordinal; default 0 */
     int32_t block_threads;    /* threads of the ONE CTA that runs an instance: a multiple of

@@ -445,7 +445,7 @@ dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_op
         return fail(DTS_E_UNSUPPORTED, "policy");
     if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI))
         return fail(DTS_E_UNSUPPORTED, "unknown flags");
-    if (o->lookahead_W != 0) return fail(DTS_E_UNSUPPORTED, "lookahead_W != 0 (NEXT)");
+    if (o->lookahead_W > 1) return fail(DTS_E_UNSUPPORTED, "lookahead_W > 1");
     if (o->bus_bytes_per_s == 0) return fail(DTS_E_INVAL, "bus_bytes_per_s == 0");
     if (o->block_threads != 0 && (o->block_threads < 32 || o->block_threads > 512 || o->block_threads % 32))
         return fail(DTS_E_INVAL, "block_threads must be 0 or a multiple of 32 in [32, 512]");

@@ -68,6 +68,10 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     int32_t plan_head[MAX_K], plan_end[MAX_K], plan_live[MAX_K];
     int32_t res_cnt[MAX_K];
     int32_t idle[MAX_K];
+    int32_t last_task[MAX_K];  // W = 1: the task that may still run when k asks again
+    int64_t last_end[MAX_K];
+    int32_t row2[MAX_ROW + 1];  // its inputs (taskBuffer_k = {running, served}, R7)
+    int32_t row2_len;
     int64_t bus_free;
     int64_t n_events, n_served, n_loads, n_evictions, n_scans, n_fb2, n_fbf, n_belady, n_idle,
         n_verr;
@@ -385,6 +389,8 @@ __device__ __forceinline__ void finish_serve(int k, int32_t T, int64_t ready, in
     I.serve_task[L.n_served] = T;
     L.n_served++;
     L.req[k] = (I.W == 0) ? end : start;  // R7
+    L.last_task[k] = T;
+    L.last_end[k] = end;
     L.alg_bytes += 24;
 }
 
@@ -493,6 +499,8 @@ __device__ __noinline__ int pop_run_seq() {
             ns++;
             pops++;
             req = (W == 0) ? end : start;  // R7
+            L.last_task[k] = T;
+            L.last_end[k] = end;
             if (live == 0 || (maxs >= 0 && ns >= maxs)) break;
             if (k2 >= 0 && (req > t2 || (req == t2 && k2 < k))) break;
         }
@@ -907,8 +915,9 @@ __device__ int32_t luf_victim(int k) {
     unsigned long long best = ~0ull;
     for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
         const int32_t D = rl[i];
-        bool in_buf = false;
+        bool in_buf = false;  // nb(D) > 0: an input of a taskBuffer_k task
         for (int r = 0; r < L.row_len; r++) in_buf |= (L.row[r] == D);
+        for (int r = 0; r < L.row2_len; r++) in_buf |= (L.row2[r] == D);
         const unsigned long long key =
             ((unsigned long long)(uint32_t)npk[D] << 32) | (unsigned long long)(uint32_t)D;
         best = (!in_buf & (key < best)) ? key : best;
@@ -978,7 +987,18 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
 __device__ void serve_loads(int k, int32_t T, int64_t t) {
     const Inst &I = SI;
     const View &V = SV;
-    if (threadIdx.x == 0) L.ready = t;
+    if (threadIdx.x == 0) {
+        L.ready = t;
+        L.row2_len = 0;
+    }
+    cta_sync();
+    // W = 1: taskBuffer_k also holds the task still running on k (R7)
+    if (I.W >= 1 && L.last_task[k] >= 0 && L.last_end[k] > t && threadIdx.x < 32) {
+        const int32_t Tr = L.last_task[k];
+        const int64_t rb = __ldg(&I.tptr[Tr]), re = __ldg(&I.tptr[Tr + 1]);
+        for (int r = threadIdx.x; r < (int)(re - rb); r += 32) L.row2[r] = __ldg(&I.tdat[rb + r]);
+        if (threadIdx.x == 0) L.row2_len = (int)(re - rb);
+    }
     cta_sync();
     const int len = L.row_len;
     for (int r = 0; r < len; r++) {
@@ -1568,6 +1588,8 @@ __global__ void __launch_bounds__(512, 1)
                 L.plan_head[k] = L.plan_end[k] = L.plan_live[k] = 0;
                 L.res_cnt[k] = 0;
                 L.idle[k] = 0;
+                L.last_task[k] = -1;
+                L.last_end[k] = 0;
             }
             L.bus_free = 0;
             L.n_events = L.n_served = L.n_loads = L.n_evictions = L.n_scans = L.n_fb2 = L.n_fbf =
@@ -1588,7 +1610,7 @@ __global__ void __launch_bounds__(512, 1)
             if (I.policy == DTS_POLICY_DARTS_LUF) {
                 int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
                 for (int j = 0; j < K; j++) pending += L.plan_live[j];
-                if (I.max_served < 0 && K <= 32 && pending > 10) {
+                if (I.max_served < 0 && I.W == 0 && K <= 32 && pending > 10) {
                     pop_batch();
                 } else {  // few pops (or a prefix run that stops at an exact count): thread 0
                     cta_sync();

@@ -365,3 +365,35 @@ def test_lru_policies_config3(name):
 def test_lru_policies_config4_prefix(name, cfg):
     g, o = _both_policy(gen.config_instances(cfg)[0], name, max_served=1500)
     assert_parity(g, o, complete=False)
+
+
+# ------------------------------------------------------------ W = 1 prefetch window (§8(f)4)
+def _w1(inst):
+    """Room for two tasks' inputs (the capacity check for W = 1)."""
+    return inst.with_(mem_capacity=int(inst.mem_capacity) + 3 * int(inst.data_size.max()))
+
+
+@pytest.mark.parametrize("idx", range(12))
+@pytest.mark.parametrize("name", ["darts_luf", "darts_lru", "eager_lru"])
+def test_w1_shapes(idx, name):
+    inst = _w1(_shapes()[idx])
+    pol = {"darts_luf": (dts.DTS_POLICY_DARTS_LUF, 0), **_POL}[name]
+    g = dts.schedule(inst, policy=pol[0], W=1)
+    o = oracle.run(inst, W=1, flags=1 | pol[1])
+    assert_parity(g, o)
+    validate(inst, g.serve_gpu, g.serve_task, g.events, g.task_start, g.task_end, W=1)
+
+
+def test_w1_config2_and_3():
+    for inst in gen.config_instances("C2")[::3] + gen.config_instances("C3"):
+        g = dts.schedule(inst, W=1)
+        o = oracle.run(inst, W=1)
+        assert_parity(g, o)
+
+
+@pytest.mark.parametrize("cfg", ["C4a", "C4b"])
+def test_w1_config4_prefix(cfg):
+    inst = gen.config_instances(cfg)[0]
+    g = dts.schedule(inst, W=1, max_served=1500)
+    o = oracle.run(inst, W=1, max_served=1500)
+    assert_parity(g, o, complete=False)
