@@ -236,6 +236,13 @@ def main():
     ap.add_argument("--cpu-budget", type=float, default=10.0,
                     help="seconds of oracle time for cpu_baseline (rank 0, N=1)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--mode", default="replica", choices=["replica", "shard"],
+                    help="N>1 with a single-instance workload (C3/C4): 'replica' = every rank "
+                         "schedules its own copy (weak); 'shard' = ONE instance task-sharded over "
+                         "the ranks, exchanging through NVLink peer memory (strong, SURVEY §8(e))")
+    ap.add_argument("--shards", type=int, default=1,
+                    help="single-instance workloads at N=1: task shards as co-resident CTAs of "
+                         "one B200 (dts_shard_group_run)")
     args = ap.parse_args()
 
     global ORACLE_FLAGS
@@ -263,18 +270,33 @@ def main():
     sptr = stream.cuda_stream
 
     insts, scaling = workload_instances(args.workload, rank, world)
-    single = args.workload in ("C3", "C4a", "C4b")  # one large instance: grouped CTAs
-    handles = [dts.create(i) for i in insts]
+    single = args.workload in ("C3", "C4a", "C4b")  # one large instance
+    xsh = single and world > 1 and args.mode == "shard"  # one instance over the ranks
+    gsh = single and not xsh and args.shards > 1          # one instance over CTAs of this GPU
+    if gsh:
+        handles = [dts.create(insts[0]) for _ in range(args.shards)]
+    else:
+        handles = [dts.create(i) for i in insts]
+    if xsh:
+        scaling = "strong"
     policy = {"darts_luf": dts.DTS_POLICY_DARTS_LUF, "darts_lru": dts.DTS_POLICY_DARTS_LRU,
               "eager_lru": dts.DTS_POLICY_EAGER_LRU}[args.policy]
     opts = dts.dts_run_opts_default(device=dev, cuda_stream=sptr,
                                     flags=dts.DTS_F_FALLBACK2 | (dts.DTS_F_OPTI if args.opti else 0))
+    if xsh:  # map the peers' shard state (CUDA IPC over NVLink); handles are host blobs
+        dts.dts_shard_set(handles[0], world, rank)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, dts.dts_shard_export(handles[0], dev))
+        dts.dts_shard_connect(handles[0], blobs)
+        dist.barrier()
     for h in handles:
         dts.dts_instance_upload(h, dev, sptr)
     torch.cuda.synchronize()
 
     def step():
-        if single:
+        if gsh:
+            dts.dts_shard_group_run(handles, policy, opts)
+        elif single:
             for h in handles:
                 dts.dts_run(h, policy, opts)
         else:
@@ -293,7 +315,9 @@ def main():
     barrier()
     res0 = [dts.dts_result(h) for h in handles]
     decisions = sum(r.n_served for r in res0)
-    assert decisions == sum(i.m for i in insts), "not every task scheduled"
+    if gsh or xsh:  # every shard holds the (same) whole schedule: count it once
+        decisions = res0[0].n_served if (gsh or rank == 0) else 0
+    assert decisions == sum(i.m for i in insts) or (xsh and rank > 0), "not every task scheduled"
 
     # ---- device-resident timed region
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
@@ -324,7 +348,7 @@ def main():
     # ---- e2e: host arrays -> device, run, results -> host, every step
     e2e_ms = []
     h2d = sum(8 * (i.m + 1) + 4 * i.E + 8 * i.n + (8 * i.m if i.task_ns is not None else 0)
-              for i in insts)
+              for i in insts) * (args.shards if gsh else 1)
     d2h = 0
     barrier()
     for i in range(max(2, args.steps // 2)):
@@ -375,7 +399,10 @@ def main():
                        "instances_per_rank": len(insts), "decisions_per_step": int(all_dec),
                        "l2": "flushed between timed steps (256 MiB write)",
                        "launch": "one batched loop launch, one CTA per instance" if not single
-                       else "one cooperative launch per instance (CTA group)"},
+                       else (f"one cooperative launch: the instance task-sharded over {args.shards} CTAs"
+                             if gsh else f"one loop launch per rank: the instance task-sharded over "
+                             f"{world} B200s, peer-memory exchanges" if xsh
+                             else "one loop launch (one CTA) per instance")},
             "e2e": {"value": all_dec / (e2e_avg / 1e3), "unit": UNIT,
                     "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h)},
             "gpu_launches": int(launches),

@@ -193,6 +193,47 @@ dts_status dts_result(dts_instance *inst, dts_result_view *out);
 dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy,
                          const dts_run_opts *opts);
 
+/* ---- Task-sharded single instance (second mode) ----------
+ * One instance whose tasks are split into G consecutive id ranges with about
+ * E/G edges each; shard g keeps the packed state, the data->task edges and
+ * PARTIAL scores n_k(D), n2_k(D), u(D) of its own tasks, and every decision of
+ * Alg. 5 / Alg. 6 is replicated on all shards from the
+ * exchanged values: per scan, a reduce-scatter of the partial scores by datum
+ * slice plus the max of the G slice keys (the "allreduce + argmax" of the
+ * north_star, done inside the kernel through the shards' memory); per plan,
+ * one exchange of each shard's part of plannedTasks_k (Alg. 5 l.10); per
+ * fallback pick (Alg. 5 l.13, 3inputs), one min-exchange.  The schedule is
+ * the same as dts_run's on the whole instance, bit for bit; every shard's
+ * dts_result returns all of it.
+ *
+ * Multi-GPU (one process per B200): every rank creates the SAME instance,
+ *   dts_shard_set(inst, G, rank); dts_shard_export(inst, device, my_handle);
+ *   all-gather the handles (any transport, rank order);
+ *   dts_shard_connect(inst, all_handles);  then each run: dts_run(inst, ...)
+ *   on every rank concurrently (each launches one CTA that exchanges with its
+ *   peers over NVLink through CUDA IPC mappings; a peer missing for 5 s ends
+ *   the run with DTS_E_STATE from dts_result instead of a hang).
+ * One device: dts_shard_group_run runs G shards as G co-resident CTAs. */
+#define DTS_SHARD_HANDLE_BYTES 128
+
+/* Make `inst` shard g of G (G = 1: the whole instance).  Host only. */
+dts_status dts_shard_set(dts_instance *inst, int32_t G, int32_t g);
+/* The task range [*t_lo, *t_hi) the instance owns. */
+dts_status dts_shard_range(const dts_instance *inst, int32_t *t_lo, int32_t *t_hi);
+/* Allocate the shard's device state on `device` and write its IPC handle
+ * (DTS_SHARD_HANDLE_BYTES bytes) to `handle`. */
+dts_status dts_shard_export(dts_instance *inst, int32_t device, void *handle);
+/* Map the peers' state: `handles` = G handles in shard order (this shard's
+ * own included, ignored).  Resets this shard's exchange numbers: every rank
+ * must finish dts_shard_connect (a barrier) before any rank runs, and the
+ * ranks then call dts_run the same number of times.  Needs every peer alive
+ * (exported) at this call. */
+dts_status dts_shard_connect(dts_instance *inst, const void *handles);
+/* One device: shards[i] becomes shard i of G (same instance in every entry)
+ * and all G run in ONE cooperative launch on opts->device. */
+dts_status dts_shard_group_run(dts_instance *const *shards, int32_t G, dts_policy policy,
+                               const dts_run_opts *opts);
+
 void dts_instance_destroy(dts_instance *inst);
 const char *dts_status_str(dts_status s);
 const char *dts_last_error(void);

@@ -30,4 +30,11 @@ from .dts import (  # noqa: F401
     schedule_batch,
     load_library,
     schedule,
+    schedule_sharded,
+    dts_shard_set,
+    dts_shard_range,
+    dts_shard_export,
+    dts_shard_connect,
+    dts_shard_group_run,
+    DTS_SHARD_HANDLE_BYTES,
 )

@@ -115,11 +115,22 @@ struct dts_instance {
     int64_t r_n_events = 0;
     float loop_ms = 0.f, total_ms = 0.f;
 
+    // task shard (§8(e)): shard g of G owns tasks [t_lo, t_hi)
+    int32_t G = 1, g = 0, t_lo = 0, t_hi = 0;
+    uint64_t runs = 0;                       // runs so far: exchange numbers of run r start at r << 32
+    unsigned long long *d_epoch = nullptr;   // this shard's published exchange number
+    unsigned char *d_box = nullptr;          // its two payload slots
+    int64_t box_bytes = 0;
+    dts::ShardPeer *d_peers = nullptr;       // [MAX_G] peer table read by the kernel
+    bool connected = false;
+    std::vector<void *> ipc_open;            // peers' arenas mapped through CUDA IPC
+
     ~dts_instance() {
         if (device >= 0) {
             int cur = 0;
             cudaGetDevice(&cur);
             cudaSetDevice(device);
+            for (void *p : ipc_open) cudaIpcCloseMemHandle(p);
             if (ar.base) cudaFree(ar.base);
             for (auto &e : ev)
                 if (e) cudaEventDestroy(e);
@@ -295,6 +306,8 @@ dts_status check_device(int device) {
 dts_status ensure_device(dts_instance *I, int device) {
     if (I->device == device && I->ar.base) return DTS_OK;
     if (I->device >= 0 && I->ar.base) {
+        if (I->connected && I->G > 1)
+            return fail(DTS_E_STATE, "a connected task shard cannot move to another device");
         cudaSetDevice(I->device);
         cudaFree(I->ar.base);
         for (auto &e : I->ev)
@@ -329,6 +342,8 @@ dts_status ensure_device(dts_instance *I, int device) {
     add(sizeof(dts_event) * ev_cap); add(8 * (K + 1)); add(4 * (m + 1));
     add(sizeof(dts::Inst)); add(64);
     add(dts::csr_scratch_bytes(I->m, I->n, I->E_raw));
+    const int64_t box_bytes = (int64_t)sizeof(dts::ShardSlot) + 16 * (int64_t)plan_cap;
+    add(256); add(2 * (size_t)box_bytes); add(sizeof(dts::ShardPeer) * dts::MAX_G);  // shard exchange
     char *base = nullptr;
     cudaError_t e = cudaMalloc(&base, need);
     if (e != cudaSuccess) return fail(DTS_E_NOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
@@ -401,7 +416,14 @@ dts_status ensure_device(dts_instance *I, int device) {
     I->d_inst = A.take<dts::Inst>(1);
     I->d_work = A.take<int>(16);
     I->d_csr_scratch = A.take<char>(dts::csr_scratch_bytes(I->m, I->n, I->E_raw));
+    I->d_epoch = A.take<unsigned long long>(32);
+    I->box_bytes = box_bytes;
+    I->d_box = A.take<unsigned char>(2 * (size_t)box_bytes);
+    I->d_peers = A.take<dts::ShardPeer>(dts::MAX_G);
     if (A.used > A.size) return fail(DTS_E_NOMEM, "arena overflow (internal)");
+    CK(cudaMemset(I->d_epoch, 0, 256), "memset epoch");  // exchange numbers start at 0, once
+    I->connected = false;
+    I->runs = 0;
 
     h.m = I->m;
     h.n = I->n;
@@ -459,12 +481,13 @@ dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_op
 // Shared-memory placement of one instance's state:
 // greedy, most latency-critical array first, each either fully in the CTA's
 // dynamic shared memory or in its global home.  Returns the bytes used.
-int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru) {
+int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard) {
     const int64_t K = h.K, n = h.n;
     int used = 0;
     auto put = [&](int32_t &so, int64_t bytes) {
         bytes = (bytes + 15) & ~int64_t(15);
-        if (budget > 0 && used + bytes <= budget) {
+        const bool peer_read = shard && (&so == &h.so_u || &so == &h.so_h || &so == &h.so_h2);
+        if (budget > 0 && !peer_read && used + bytes <= budget) {
             so = used;
             used += (int)bytes;
         } else {
@@ -543,16 +566,23 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
         const unsigned __int128 num = (unsigned __int128)h.size0 * 1000000000u + (o.bus_bytes_per_s - 1);
         h.delta0 = (int64_t)(num / o.bus_bytes_per_s);  // ceil, reading R9 (same as dts_init_kernel)
     }
-    place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF);
+    place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF, I->G > 1);
+    h.G = I->G;
+    h.g = I->g;
+    h.t_lo = I->G > 1 ? I->t_lo : 0;
+    h.t_hi = I->G > 1 ? I->t_hi : I->m;
+    h.peers = I->G > 1 ? I->d_peers : nullptr;
+    h.ep_base = (unsigned long long)(++I->runs) << 32;
+    h.box_bytes = I->box_bytes;
     // small instances: the loop CTA builds its own CSR and state (one launch)
     const int fs = fused_scratch_bytes(I, block);
-    h.fused = !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
+    h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
     if (h.fused) h.smem_bytes = std::max(h.smem_bytes, fs);
     CK(cudaEventRecord(I->ev[0], st), "event");
     if (!h.fused)
         CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
                           (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, (int4 *)h.dedge,
-                          I->d_csr_scratch, st),
+                          I->d_csr_scratch, st, h.t_lo, h.t_hi),
            "build_csr");
     if (!copy_desc) return DTS_OK;
     // descriptor H2D from pinned memory (a pageable copy would serialise the host)
@@ -604,6 +634,9 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     if (s != DTS_OK) return s;
     s = check_device(o.device);
     if (s != DTS_OK) return s;
+    if (I->G > 1 && !I->connected)
+        return fail(DTS_E_STATE, "task shard not connected (dts_shard_connect) -- or use dts_shard_group_run");
+    if (I->G > 1 && I->device != o.device) return fail(DTS_E_INVAL, "task shard: opts.device != exported device");
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
     const int budget = budget_of(o);
     const int block = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", auto_block(I));
@@ -701,6 +734,224 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     return DTS_OK;
 }
 
+
+}  // extern "C"
+
+// ---------------------------------------------------------------- task shards
+namespace {
+
+// Consecutive task ranges with about E/G edges each (§8(e)); the last shard
+// ends at m.
+void shard_bounds(const dts_instance *I, int32_t G, int32_t g, int32_t *lo, int32_t *hi) {
+    auto start = [&](int32_t q) -> int32_t {
+        if (q <= 0) return 0;
+        if (q >= G) return I->m;
+        const int64_t E = I->E_raw;
+        if (E == 0) return (int32_t)((int64_t)I->m * q / G);
+        const int64_t target = (E * q + G - 1) / G;
+        return (int32_t)(std::lower_bound(I->task_ptr.begin(), I->task_ptr.begin() + I->m, target) -
+                         I->task_ptr.begin());
+    };
+    *lo = start(g);
+    *hi = g == G - 1 ? I->m : std::max(*lo, start(g + 1));
+}
+
+constexpr uint32_t SHARD_MAGIC = 0x48535444u;  // "DTSH"
+struct ShardHandle {
+    cudaIpcMemHandle_t mem;      // the shard's device arena
+    int64_t off_epoch, off_box, off_h, off_h2, off_u;
+    int32_t G, g;
+    int64_t box_bytes;
+    uint32_t magic, pad;
+};
+static_assert(sizeof(ShardHandle) <= DTS_SHARD_HANDLE_BYTES, "handle size");
+
+dts::ShardPeer own_peer(const dts_instance *I) {
+    dts::ShardPeer p;
+    p.epoch = I->d_epoch;
+    p.box = I->d_box;
+    p.h = I->h_inst.h;
+    p.h2 = I->h_inst.h2;
+    p.u = I->h_inst.u;
+    return p;
+}
+
+dts_status write_peers(dts_instance *I, const std::vector<dts::ShardPeer> &tab) {
+    CK(cudaSetDevice(I->device), "cudaSetDevice");
+    CK(cudaMemcpy(I->d_peers, tab.data(), sizeof(dts::ShardPeer) * tab.size(), cudaMemcpyHostToDevice),
+       "H2D peers");
+    I->connected = true;
+    return DTS_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+dts_status dts_shard_set(dts_instance *I, int32_t G, int32_t g) {
+    if (!I) return fail(DTS_E_INVAL, "instance is NULL");
+    if (G < 1 || G > dts::MAX_G) return fail(DTS_E_UNSUPPORTED, "G must be in [1, 64]");
+    if (g < 0 || g >= G) return fail(DTS_E_INVAL, "g must be in [0, G)");
+    for (void *p : I->ipc_open) cudaIpcCloseMemHandle(p);
+    I->ipc_open.clear();
+    I->G = G;
+    I->g = g;
+    shard_bounds(I, G, g, &I->t_lo, &I->t_hi);
+    I->connected = false;
+    return DTS_OK;
+}
+
+dts_status dts_shard_range(const dts_instance *I, int32_t *t_lo, int32_t *t_hi) {
+    if (!I || !t_lo || !t_hi) return fail(DTS_E_INVAL, "NULL argument");
+    *t_lo = I->G > 1 ? I->t_lo : 0;
+    *t_hi = I->G > 1 ? I->t_hi : I->m;
+    return DTS_OK;
+}
+
+dts_status dts_shard_export(dts_instance *I, int32_t device, void *handle) {
+    if (!I || !handle) return fail(DTS_E_INVAL, "NULL argument");
+    if (I->G < 2) return fail(DTS_E_STATE, "not a task shard (dts_shard_set with G >= 2 first)");
+    dts_status s = ensure_device(I, device);
+    if (s != DTS_OK) return s;
+    ShardHandle hd;
+    std::memset(&hd, 0, sizeof hd);
+    CK(cudaIpcGetMemHandle(&hd.mem, I->ar.base), "cudaIpcGetMemHandle");
+    const char *b = I->ar.base;
+    hd.off_epoch = (const char *)I->d_epoch - b;
+    hd.off_box = (const char *)I->d_box - b;
+    hd.off_h = (const char *)I->h_inst.h - b;
+    hd.off_h2 = (const char *)I->h_inst.h2 - b;
+    hd.off_u = (const char *)I->h_inst.u - b;
+    hd.G = I->G;
+    hd.g = I->g;
+    hd.box_bytes = I->box_bytes;
+    hd.magic = SHARD_MAGIC;
+    std::memset(handle, 0, DTS_SHARD_HANDLE_BYTES);
+    std::memcpy(handle, &hd, sizeof hd);
+    return DTS_OK;
+}
+
+dts_status dts_shard_connect(dts_instance *I, const void *handles) {
+    if (!I || !handles) return fail(DTS_E_INVAL, "NULL argument");
+    if (I->G < 2 || !I->ar.base) return fail(DTS_E_STATE, "dts_shard_export first");
+    CK(cudaSetDevice(I->device), "cudaSetDevice");
+    // a new connection starts every shard's exchange numbers at 0 (the caller
+    // makes all ranks connect before any of them runs: include/dts.h)
+    CK(cudaDeviceSynchronize(), "sync");
+    CK(cudaMemset(I->d_epoch, 0, 256), "memset epoch");
+    CK(cudaDeviceSynchronize(), "sync");
+    I->runs = 0;
+    for (void *p : I->ipc_open) cudaIpcCloseMemHandle(p);
+    I->ipc_open.clear();
+    std::vector<dts::ShardPeer> tab((size_t)I->G);
+    for (int32_t p = 0; p < I->G; p++) {
+        ShardHandle hd;
+        std::memcpy(&hd, (const char *)handles + (size_t)p * DTS_SHARD_HANDLE_BYTES, sizeof hd);
+        if (hd.magic != SHARD_MAGIC || hd.G != I->G || hd.g != p || hd.box_bytes != I->box_bytes)
+            return fail(DTS_E_INVAL, "shard handle " + std::to_string(p) + " does not match this instance");
+        if (p == I->g) {
+            tab[(size_t)p] = own_peer(I);
+            continue;
+        }
+        void *base = nullptr;
+        CK(cudaIpcOpenMemHandle(&base, hd.mem, cudaIpcMemLazyEnablePeerAccess), "cudaIpcOpenMemHandle");
+        I->ipc_open.push_back(base);
+        char *c = (char *)base;
+        tab[(size_t)p].epoch = (unsigned long long *)(c + hd.off_epoch);
+        tab[(size_t)p].box = (unsigned char *)(c + hd.off_box);
+        tab[(size_t)p].h = (const int32_t *)(c + hd.off_h);
+        tab[(size_t)p].h2 = (const int32_t *)(c + hd.off_h2);
+        tab[(size_t)p].u = (const int32_t *)(c + hd.off_u);
+    }
+    return write_peers(I, tab);
+}
+
+dts_status dts_shard_group_run(dts_instance *const *shards, int32_t G, dts_policy policy,
+                               const dts_run_opts *opts) {
+    if (G < 1 || G > dts::MAX_G || !shards) return fail(DTS_E_INVAL, "G must be in [1, 64]");
+    dts_run_opts o;
+    if (opts) o = *opts;
+    else dts_run_opts_default(&o);
+    dts_status s = check_device(o.device);
+    if (s != DTS_OK) return s;
+    std::vector<dts_instance *> seen(shards, shards + G);
+    std::sort(seen.begin(), seen.end());
+    if (std::adjacent_find(seen.begin(), seen.end()) != seen.end()) return fail(DTS_E_INVAL, "shard listed twice");
+    int block = 32;
+    int64_t work = 1;
+    for (int32_t i = 0; i < G; i++) {
+        dts_instance *I = shards[i];
+        if (!I) return fail(DTS_E_INVAL, "shard is NULL");
+        if (I->m != shards[0]->m || I->n != shards[0]->n || I->K != shards[0]->K || I->E_raw != shards[0]->E_raw)
+            return fail(DTS_E_INVAL, "shards must hold the same instance");
+        s = check_opts(I, policy, &o);
+        if (s != DTS_OK) return s;
+        if (I->G != G || I->g != i || (G > 1 && !I->connected) || I->device != o.device) {
+            s = dts_shard_set(I, G, i);
+            if (s != DTS_OK) return s;
+            s = ensure_device(I, o.device);
+            if (s != DTS_OK) return s;
+        }
+        block = std::max(block, auto_block(I));
+        work = std::max<int64_t>(work, std::max<int64_t>(I->m_pad, (int64_t)I->n * I->K));
+    }
+    if (G > 1 && !shards[0]->connected) {  // same device: the peers' own pointers
+        std::vector<dts::ShardPeer> tab((size_t)G);
+        for (int32_t p = 0; p < G; p++) tab[(size_t)p] = own_peer(shards[p]);
+        for (int32_t i = 0; i < G; i++) {
+            s = write_peers(shards[i], tab);
+            if (s != DTS_OK) return s;
+        }
+    }
+    if (o.block_threads) block = o.block_threads;
+    else block = env_int("DTS_BLOCK", block);
+    cudaStream_t st = (cudaStream_t)o.cuda_stream;
+    const int budget = budget_of(o);
+    // one exchange-number range for the whole group: above every shard's last
+    uint64_t runs = 0;
+    for (int32_t i = 0; i < G; i++) runs = std::max(runs, shards[i]->runs);
+    int smem = 0;
+    for (int32_t i = 0; i < G; i++) {
+        shards[i]->runs = runs;
+        s = stage(shards[i], policy, o, budget, block, st, false);
+        if (s != DTS_OK) return s;
+        smem = std::max(smem, shards[i]->h_inst.smem_bytes);
+    }
+    SweepBuf &B = g_sweep[o.device];
+    if (!B.copied[0])
+        for (auto &e : B.copied) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
+    if (B.cap < (size_t)G) {
+        CK(cudaDeviceSynchronize(), "sync");
+        if (B.d_insts) cudaFree(B.d_insts);
+        for (auto &h : B.h_insts)
+            if (h) cudaFreeHost(h);
+        size_t cap = std::max<size_t>((size_t)G, 64);
+        CK(cudaMalloc(&B.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
+        for (auto &h : B.h_insts) CK(cudaMallocHost(&h, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
+        B.d_work = reinterpret_cast<int *>(B.d_insts + cap);
+        B.cap = cap;
+    }
+    const int sl = B.slot;
+    B.slot = (B.slot + 1) % SweepBuf::RING;
+    CK(cudaEventSynchronize(B.copied[sl]), "sweep event");
+    for (int32_t i = 0; i < G; i++) B.h_insts[sl][i] = shards[i]->h_inst;
+    CK(cudaMemcpyAsync(B.d_insts, B.h_insts[sl], sizeof(dts::Inst) * (size_t)G, cudaMemcpyHostToDevice, st),
+       "H2D shards");
+    CK(cudaEventRecord(B.copied[sl], st), "event");
+    CK(cudaMemsetAsync(B.d_work, 0, sizeof(int), st), "memset");
+    CK(dts::launch_init(B.d_insts, G, o.bus_bytes_per_s, work, st), "init");
+    for (int32_t i = 0; i < G; i++) CK(cudaEventRecord(shards[i]->ev[1], st), "event");
+    // the G shards exchange inside the kernel: they must be co-resident
+    CK(dts::launch_loop_coop(B.d_insts, G, block, B.d_work, smem, st), "loop (cooperative)");
+    for (int32_t i = 0; i < G; i++) {
+        CK(cudaEventRecord(shards[i]->ev[2], st), "event");
+        CK(cudaEventRecord(shards[i]->ev[3], st), "event");
+        shards[i]->ran = true;
+    }
+    return DTS_OK;
+}
+
+
 dts_status dts_result(dts_instance *I, dts_result_view *v) {
     if (!I || !v) return fail(DTS_E_INVAL, "NULL argument");
     if (!I->ran) return fail(DTS_E_STATE, "dts_result before dts_run");
@@ -710,6 +961,7 @@ dts_status dts_result(dts_instance *I, dts_result_view *v) {
         CK(cudaMemcpyAsync(I->r_out, I->h_inst.out, sizeof I->out, cudaMemcpyDeviceToHost, I->stream), "D2H out");
         CK(cudaStreamSynchronize(I->stream), "D2H sync");
         I->out = *I->r_out;
+        if (I->out.error == 2) return fail(DTS_E_STATE, "task shards: a peer did not reach an exchange in time");
         if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim (Belady branch)");
         const dts::Inst &h = I->h_inst;
         size_t ns = (size_t)I->out.n_served, ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);

@@ -131,19 +131,23 @@ __global__ void k_rows(const int64_t *__restrict__ raw_ptr, const int32_t *__res
 }
 
 // 3. compact rows into tdat, write the (datum, task) edges, count degrees.
+//    Only the tasks of [t_lo, t_hi) enter the data->task side (a task shard,
+//    §8(e); the whole range otherwise); the other edges get key n and sort
+//    past dptr[n].  The task->data side always holds every row.
 __global__ void k_compact(const int64_t *__restrict__ raw_ptr, const int32_t *__restrict__ tmp,
-                          const int64_t *__restrict__ tptr, int32_t m, int32_t *__restrict__ tdat,
-                          int32_t *__restrict__ ekey, int32_t *__restrict__ eval,
-                          unsigned long long *__restrict__ deg) {
+                          const int64_t *__restrict__ tptr, int32_t m, int32_t n, int32_t t_lo,
+                          int32_t t_hi, int32_t *__restrict__ tdat, int32_t *__restrict__ ekey,
+                          int32_t *__restrict__ eval, unsigned long long *__restrict__ deg) {
     int32_t T = blockIdx.x * blockDim.x + threadIdx.x;
     if (T >= m) return;
+    const bool own = T >= t_lo && T < t_hi;
     int64_t b = raw_ptr[T], o = tptr[T], q = tptr[T + 1] - o;
     for (int64_t i = 0; i < q; i++) {
         int32_t D = tmp[b + i];
         tdat[o + i] = D;
-        ekey[o + i] = D;
+        ekey[o + i] = own ? D : n;
         eval[o + i] = T;
-        atomicAdd(&deg[D], 1ull);
+        if (own) atomicAdd(&deg[D], 1ull);
     }
 }
 
@@ -281,7 +285,7 @@ static inline char *carve(char *&p, size_t bytes) {
 
 cudaError_t build_csr(const int64_t *raw_ptr, const int32_t *raw_dat, int32_t m, int32_t n,
                       int64_t E_raw, int64_t *tptr, int32_t *tdat, int64_t *dptr, int32_t *ddat,
-                      int4 *dedge, void *scratch, cudaStream_t st) {
+                      int4 *dedge, void *scratch, cudaStream_t st, int32_t t_lo, int32_t t_hi) {
     char *p = (char *)scratch;
     int32_t *tmp = (int32_t *)carve(p, sizeof(int32_t) * (size_t)(E_raw + 4));
     int64_t *nlen = (int64_t *)carve(p, sizeof(int64_t) * (size_t)(m + 4));
@@ -306,7 +310,7 @@ cudaError_t build_csr(const int64_t *raw_ptr, const int32_t *raw_dat, int32_t m,
     }
     scan_excl<int64_t>(nlen, m, tptr, sscr, st);
     if (m > 0) {
-        k_compact<<<(m + 255) / 256, 256, 0, st>>>(raw_ptr, tmp, tptr, m, tdat, k0, v0, deg);
+        k_compact<<<(m + 255) / 256, 256, 0, st>>>(raw_ptr, tmp, tptr, m, n, t_lo, t_hi, tdat, k0, v0, deg);
         count_launch();
     }
     scan_excl<unsigned long long>(deg, n, dptr, sscr, st);

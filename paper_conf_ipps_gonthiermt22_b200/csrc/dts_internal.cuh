@@ -56,6 +56,27 @@ struct Out {
     int64_t prof[16];  // SM cycles seen by thread 0 per phase (see PROF_* in dts_loop.cu)
 };
 
+// Task-sharded single instance (second mode): shard g of G
+// owns the tasks [t_lo, t_hi) -- their packed state s, their data->task edges
+// and PARTIAL score arrays h, h2, u -- while every decision (residency, plans,
+// np, the time model, the trace) is replicated on all shards.  Shards meet at
+// exchange points through each other's memory (same device: other CTAs; other
+// B200s: CUDA IPC mappings over NVLink).  One entry per shard, pointers valid
+// in the address space of the shard that reads the table.
+constexpr int MAX_G = 64;
+struct ShardPeer {
+    unsigned long long *epoch;  // the shard's last published exchange number
+    unsigned char *box;         // its two payload slots (by exchange parity)
+    const int32_t *h, *h2, *u;  // its partial score arrays (global homes)
+};
+// Payload slot: keys / candidate ids, then the shard's part of a new plan.
+struct ShardSlot {
+    unsigned long long key[2];
+    int32_t cnt;
+    int32_t pad[3];
+    // int4 ents[plan_cap] follow
+};
+
 // Device descriptor of one instance.
 struct Inst {
     int32_t m, n, K, W;
@@ -115,6 +136,12 @@ struct Inst {
     // result assembly
     int64_t *gpu_task_ptr;  // [K+1]
     int32_t *gpu_task_ids;  // [m]
+    // task sharding (G = 1: the whole instance on one CTA)
+    int32_t G, g;             // shards, this shard
+    int32_t t_lo, t_hi;       // owned task range
+    const ShardPeer *peers;   // [G] (device), nullptr when G = 1
+    unsigned long long ep_base;  // exchange numbers of this run: ep_base + 1, 2, ...
+    int64_t box_bytes;        // bytes of one payload slot
 };
 
 }  // namespace dts

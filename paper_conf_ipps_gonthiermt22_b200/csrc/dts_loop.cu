@@ -91,6 +91,9 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     int32_t bhead[32], bcnt[32], boff[33];
     int64_t rkey[POP_RANK_MAX];  // pop batch: request time of each pop (merge ranks)
     int32_t rgpu[POP_RANK_MAX];
+    int64_t xe;      // task shards: exchanges done in this run
+    int32_t xerr;    // task shards: a peer did not arrive in time (the run is abandoned)
+    int32_t xoff[MAX_G + 1];  // plan exchange: each shard's offset in the merged plan
 };
 
 // Per-instance views: shared-memory arrays where placed, else global homes.
@@ -247,14 +250,14 @@ __device__ __forceinline__ void missing_pair(int k, int32_t T, Row r, int32_t sk
     }
 }
 
-// u(D) and np (when plan_k >= 0) of T's inputs for pool_move, long rows.
-__device__ __noinline__ void pool_move_long_row(int32_t T, int sign, int plan_k) {
+// u(D) (own tasks) and np (when plan_k >= 0) of T's inputs for pool_move, long rows.
+__device__ __noinline__ void pool_move_long_row(int32_t T, int sign, int plan_k, bool own) {
     const Inst &I = SI;
     const View &V = SV;
     const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
     for (int64_t i = rb; i < re; i++) {
         const int32_t D = __ldg(&I.tdat[i]);
-        atomicAdd(&V.u[D], sign);
+        if (own) atomicAdd(&V.u[D], sign);
         if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + D], -sign);
     }
 }
@@ -266,11 +269,15 @@ __device__ __noinline__ void pool_move_long_row(int32_t T, int sign, int plan_k)
 // ONE thread per task; the touched words of s are T's own.  The state words
 // are loaded four at a time (one round trip), then updated by a compact loop
 // (the code stays small: the loop kernel is instruction-cache bound).
+// Task shards (§8(e)): s, h, h2 and u are the owner's (partial) arrays, np is
+// replicated -- a shard applies np for every task of a plan, the rest only
+// for its own tasks.
 __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
     const Inst &I = SI;
     const View &V = SV;
     const int K = I.K;
-    for (int j0 = 0; j0 < K; j0 += 4) {
+    const bool own = T >= I.t_lo && T < I.t_hi;
+    for (int j0 = 0; own && j0 < K; j0 += 4) {
         uint32_t w0 = 0, w1 = 0, w2 = 0, w3 = 0;
         w0 = V.s[(size_t)j0 * I.m_pad + T];
         if (j0 + 1 < K) w1 = V.s[(size_t)(j0 + 1) * I.m_pad + T];
@@ -294,14 +301,14 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
         }
     }
     if (r.len > 3) {
-        pool_move_long_row(T, sign, plan_k);
+        pool_move_long_row(T, sign, plan_k, own);
         return;
     }
     const int32_t c[3] = {r.r0, r.r1, r.r2};
 #pragma unroll
     for (int i = 0; i < 3; i++) {
         if (c[i] < 0) continue;
-        atomicAdd(&V.u[c[i]], sign);
+        if (own) atomicAdd(&V.u[c[i]], sign);
         if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[i]], -sign);
     }
 }
@@ -1221,18 +1228,280 @@ __device__ __noinline__ int32_t first_cnt2(int k, int32_t D2) {
     return -1;
 }
 
-// Alg. 5 l.13 (R5): the lowest-id unallocated task, scanning up from avail_lo.
+// Alg. 5 l.13 (R5): the lowest-id unallocated task, scanning up from avail_lo
+// (over the owned range [t_lo, t_hi) = all tasks unless sharded).
 __device__ __noinline__ int32_t first_avail() {
     const Inst &I = SI;
     const View &V = SV;
-    for (int64_t base = L.avail_lo; base < I.m; base += blockDim.x) {
+    for (int64_t base = L.avail_lo > I.t_lo ? L.avail_lo : I.t_lo; base < I.t_hi; base += blockDim.x) {
         const int64_t T = base + threadIdx.x;
         unsigned long long c = ~0ull;
-        if (T < I.m && !(V.s[T] & ALLOC_BIT)) c = (unsigned long long)T;
+        if (T < I.t_hi && !(V.s[T] & ALLOC_BIT)) c = (unsigned long long)T;
         c = block_min_u64(c);
         if (c != ~0ull) return (int32_t)c;
     }
     return -1;
+}
+
+// ---------------------------------------------------------------------------
+// Task shards (the north_star's second multi-GPU mode): one
+// instance, its tasks split into G consecutive id ranges.  Shard g keeps the
+// packed state and the data->task edges of its own tasks and PARTIAL score
+// arrays (h, h2, u count only its tasks); everything the decisions depend on
+// afterwards (residency, plannedTasks, np, the bus and time model, the trace)
+// is replicated: every shard takes the same decision from the same exchanged
+// values.  Exchanges go through the shards' memory -- other CTAs of the same
+// launch, or other B200s through CUDA IPC mappings over NVLink -- inside the
+// kernel: no host round trip per decision.  Per scan: exchange 1 (partials
+// final), a reduce-scatter of (h, u[, h2]) by datum slice with the slice's best
+// key, exchange 2, max of G keys; per plan: one exchange of the shards' parts.
+
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long global_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+constexpr unsigned long long XCH_TIMEOUT_NS = 5000000000ull;
+
+// Payload slot of exchange number x (1-based within the run) of shard p.
+__device__ __forceinline__ ShardSlot *xch_slot(int p, int64_t x) {
+    const Inst &I = SI;
+    unsigned char *box = (unsigned char *)__ldg((const unsigned long long *)&I.peers[p].box);
+    return reinterpret_cast<ShardSlot *>(box + (x & 1) * I.box_bytes);
+}
+
+// Block-wide: publish this shard's slot of the next exchange (every thread's
+// writes to it precede the barrier) and wait until every shard published the
+// same exchange.  Thread 0 releases at system scope (peers may be other GPUs);
+// warp 0 acquires the peers' exchange numbers.  Two slots by parity suffice: a
+// shard reuses a slot only after every peer published the exchange in between,
+// which they do only after reading this one.  A peer missing for
+// XCH_TIMEOUT_NS sets L.xerr -- the run ends with an error instead of a hang.
+__device__ __noinline__ void xch_sync() {
+    const Inst &I = SI;
+    const unsigned long long e = I.ep_base + (unsigned long long)L.xe + 1ull;
+    cta_sync();
+    if (threadIdx.x == 0) {
+        __threadfence_system();
+        st_release_sys((unsigned long long *)__ldg((const unsigned long long *)&I.peers[I.g].epoch), e);
+    }
+    if (threadIdx.x < 32) {
+        const unsigned long long t0 = global_ns();
+        for (int p = threadIdx.x; p < I.G; p += 32) {
+            const unsigned long long *f =
+                (const unsigned long long *)__ldg((const unsigned long long *)&I.peers[p].epoch);
+            while (ld_acquire_sys(f) < e) {
+                if (global_ns() - t0 > XCH_TIMEOUT_NS) {
+                    L.xerr = 1;
+                    break;
+                }
+            }
+        }
+        __syncwarp();
+        if (threadIdx.x == 0) L.xe = L.xe + 1;
+    }
+    cta_sync();
+}
+
+// Block-wide: minimum over shards of one block-uniform candidate (~0 = none).
+__device__ __noinline__ unsigned long long xch_min(unsigned long long v) {
+    const Inst &I = SI;
+    if (threadIdx.x == 0) xch_slot(I.g, L.xe + 1)->key[0] = v;
+    xch_sync();
+    if (L.xerr) return ~0ull;
+    unsigned long long r = ~0ull;
+    for (int p = 0; p < I.G; p++) {
+        const unsigned long long x = __ldcg(&xch_slot(p, L.xe)->key[0]);
+        r = x < r ? x : r;
+    }
+    return r == ~0ull || r < (unsigned long long)I.m ? r : ~0ull;  // (a task id or none)
+}
+
+__device__ __forceinline__ unsigned long long score_key(int32_t sc, int32_t u, int32_t D, unsigned ub, unsigned ib,
+                                                        unsigned long long idmask) {
+    return sc > 0 ? ((unsigned long long)(uint32_t)sc << (ub + ib)) | ((unsigned long long)(uint32_t)u << ib) |
+                        (idmask - (unsigned long long)D)
+                  : 0ull;
+}
+
+// Alg. 5 l.4-9 (+ the 3inputs score when fb2, OPTI's first positive datum
+// when opti) over the shards: n_k(D) = sum of the shards' h_k(D), u(D) = sum
+// of their u(D).  Shard g reduces the datum slice g of every shard's partials
+// and publishes the slice's best keys; the max over shards is the argmax of
+// the whole instance with the same (score, u, -D) order as one shard.
+// Returns D* (or -1); *d2 = the 3inputs D2 (or -1).
+__device__ __noinline__ int32_t shard_scan(int k, bool fb2, bool opti, int32_t *d2) {
+    const Inst &I = SI;
+    const unsigned ib = (unsigned)I.id_bits, ub = (unsigned)I.u_bits;
+    const unsigned long long idmask = (1ull << ib) - 1ull;
+    xch_sync();  // every shard's partial scores are final
+    const int nv = I.nstr >> 2;
+    const int per = (nv + I.G - 1) / I.G;
+    const int v0 = I.g * per, v1 = nv < v0 + per ? nv : v0 + per;
+    unsigned long long b1 = 0ull, b2 = 0ull;
+    if (!L.xerr) {
+        for (int v = v0 + threadIdx.x; v < v1; v += blockDim.x) {
+            int4 hs = make_int4(0, 0, 0, 0), us = hs, h2s = hs;
+            for (int p = 0; p < I.G; p++) {
+                const ShardPeer *P = &I.peers[p];
+                const int4 *ph = (const int4 *)((const int32_t *)__ldg((const unsigned long long *)&P->h) +
+                                                (size_t)k * I.nstr);
+                const int4 *pu = (const int4 *)__ldg((const unsigned long long *)&P->u);
+                const int4 a = __ldcg(ph + v), c = __ldcg(pu + v);
+                hs.x += a.x; hs.y += a.y; hs.z += a.z; hs.w += a.w;
+                us.x += c.x; us.y += c.y; us.z += c.z; us.w += c.w;
+                if (fb2) {
+                    const int4 *ph2 = (const int4 *)((const int32_t *)__ldg((const unsigned long long *)&P->h2) +
+                                                     (size_t)k * I.nstr);
+                    const int4 d = __ldcg(ph2 + v);
+                    h2s.x += d.x; h2s.y += d.y; h2s.z += d.z; h2s.w += d.w;
+                }
+            }
+            const int D = 4 * v;
+            const int32_t hh[4] = {hs.x, hs.y, hs.z, hs.w}, uu[4] = {us.x, us.y, us.z, us.w},
+                          h2h[4] = {h2s.x, h2s.y, h2s.z, h2s.w};
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const unsigned long long k1 =
+                    opti ? (hh[q] > 0 ? idmask - (unsigned long long)(D + q) + 1ull : 0ull)
+                         : score_key(hh[q], uu[q], D + q, ub, ib, idmask);
+                const unsigned long long k2 = score_key(h2h[q], uu[q], D + q, ub, ib, idmask);
+                b1 = k1 > b1 ? k1 : b1;
+                b2 = k2 > b2 ? k2 : b2;
+            }
+        }
+    }
+    b1 = block_max_u64(b1);
+    b2 = block_max_u64(b2);
+    if (threadIdx.x == 0) {
+        ShardSlot *my = xch_slot(I.g, L.xe + 1);
+        my->key[0] = b1;
+        my->key[1] = b2;
+    }
+    xch_sync();
+    *d2 = -1;
+    if (L.xerr) return -1;
+    unsigned long long m1 = 0ull, m2 = 0ull;
+    for (int p = 0; p < I.G; p++) {
+        const ShardSlot *sl = xch_slot(p, L.xe);
+        const unsigned long long x1 = __ldcg(&sl->key[0]), x2 = __ldcg(&sl->key[1]);
+        m1 = x1 > m1 ? x1 : m1;
+        m2 = x2 > m2 ? x2 : m2;
+    }
+    if (m2) *d2 = (int32_t)(idmask - (m2 & idmask));
+    const int32_t D = !m1 ? -1 : opti ? (int32_t)(idmask - (m1 - 1ull)) : (int32_t)(idmask - (m1 & idmask));
+    if (D >= I.n || *d2 >= I.n) {  // not a peer of this run: abandon
+        cta_sync();
+        if (threadIdx.x == 0) L.xerr = 1;
+        cta_sync();
+        *d2 = -1;
+        return -1;
+    }
+    return D;
+}
+
+// Alg. 5 l.10 over the shards: each shard compacts the unallocated tasks of
+// ITS part of Dopt's segment with one missing input (ascending id) into its
+// slot; after the exchange every shard concatenates the G parts in shard order
+// (= ascending id: shards own consecutive ranges) into its replicated
+// plannedTasks_k and moves them out of the pool (pool_move: np for all, the
+// partial state for its own).  Block-wide.
+__device__ __noinline__ void plan_shard(int k, int32_t Dopt) {
+    const Inst &I = SI;
+    const View &V = SV;
+    int64_t b, e;
+    seg_of(Dopt, b, e);
+    const uint32_t *sk = V.s + (size_t)k * I.m_pad;
+    ShardSlot *my = xch_slot(I.g, L.xe + 1);
+    int4 *ents = reinterpret_cast<int4 *>(my + 1);
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    int base_out = 0;
+    for (int64_t base = b; base < e; base += blockDim.x) {
+        const int64_t i = base + threadIdx.x;
+        bool sel = false;
+        int4 ed = make_int4(-1, -1, -1, 0);
+        if (i < e) {
+            ed = __ldg(&I.dedge[i]);
+            sel = (sk[ed.x] >> 24) == 1u;
+        }
+        const unsigned msk = __ballot_sync(FULL, sel);
+        if (lane == 0) L.wcnt[w] = __popc(msk);
+        cta_sync();
+        int off = base_out, tot = 0;
+        for (int j = 0; j < nw; j++) {
+            const int c = L.wcnt[j];
+            if (j < w) off += c;
+            tot += c;
+        }
+        if (sel) ents[off + __popc(msk & lt)] = make_int4(ed.x, Dopt, ed.y, ed.w > 3 ? ROW_LONG : ed.z);
+        base_out += tot;
+        cta_sync();
+    }
+    if (threadIdx.x == 0) my->cnt = base_out;
+    xch_sync();
+    if (threadIdx.x == 0) {
+        int run = 0;
+        for (int p = 0; p < I.G; p++) {
+            L.xoff[p] = run;
+            const int c = L.xerr ? 0 : __ldcg(&xch_slot(p, L.xe)->cnt);
+            run += c;
+            if (c < 0 || run > I.plan_cap) {  // not a peer of this run: abandon, do not index
+                L.xerr = 1;
+                run -= c;
+            }
+        }
+        L.xoff[I.G] = L.xerr ? 0 : run;
+    }
+    cta_sync();
+    const int total = L.xoff[I.G];
+    int4 *pl = V.plan + (size_t)k * I.plan_cap;
+    int64_t *pt = V.plan_cum ? V.plan_cum + (size_t)k * I.plan_cap : nullptr;
+    for (int i = threadIdx.x; i < total; i += blockDim.x) {
+        int p = 0;
+        while (L.xoff[p + 1] <= i) p++;
+        const int4 en = __ldcg(reinterpret_cast<const int4 *>(xch_slot(p, L.xe) + 1) + (i - L.xoff[p]));
+        pl[i] = en;
+        if (pt) pt[i] = tau_of(en.x);
+        pool_move(en.x, row_of_entry(en), -1, k);
+    }
+    cta_sync();
+    if (pt) block_incl_scan(pt, 0, total, 0);
+    if (threadIdx.x == 0) {
+        L.plan_head[k] = 0;
+        L.plan_end[k] = total;
+        L.plan_live[k] = total;
+        L.n_avail -= total;
+        L.alg_bytes += 20ull * (uint64_t)(e - b) + (uint64_t)total * (8ull * I.K + 40ull);
+    }
+    cta_sync();
+}
+
+// Alg. 5 l.13 / the 3inputs pick over the shards: each shard's lowest
+// candidate, then the minimum.
+__device__ __noinline__ int32_t any_first_avail() {
+    int32_t T = first_avail();
+    if (SI.G > 1) {
+        const unsigned long long r = xch_min(T < 0 ? ~0ull : (unsigned long long)T);
+        T = r == ~0ull ? -1 : (int32_t)r;
+    }
+    return T;
+}
+__device__ __noinline__ int32_t any_first_cnt2(int k, int32_t D2) {
+    int32_t T = first_cnt2(k, D2);
+    if (SI.G > 1) {
+        const unsigned long long r = xch_min(T < 0 ? ~0ull : (unsigned long long)T);
+        T = r == ~0ull ? -1 : (int32_t)r;
+    }
+    return T;
 }
 
 // DTS_F_VERIFY (P9): recompute n_k(D), n2_k(D), u(D) and cnt_k(T) from their
@@ -1246,7 +1515,7 @@ __device__ __noinline__ void verify_scores(int k) {
     cta_sync();
     const uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int bad = 0;
-    for (int T = threadIdx.x; T < I.m; T += blockDim.x) {
+    for (int T = I.t_lo + threadIdx.x; T < I.t_hi; T += blockDim.x) {  // owned tasks
         const uint32_t w = sk[T];
         const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
         int c = 0;
@@ -1600,6 +1869,8 @@ __global__ void __launch_bounds__(512, 1)
             L.avail_lo = 0;
             L.error = 0;
             L.row_len = 0;
+            L.xe = 0;
+            L.xerr = 0;
             for (int i = 0; i < 16; i++) L.prof[i] = 0;
         }
         cta_sync();
@@ -1650,7 +1921,7 @@ __global__ void __launch_bounds__(512, 1)
             }
             PROF_ADD(L, P_POP, p_pop);
             cta_sync();
-            if (L.cmd == CMD_DONE) break;
+            if (L.cmd == CMD_DONE || L.xerr) break;
             const int k = L.k;
             const int64_t t = L.t;
             int32_t T = -1;
@@ -1659,7 +1930,7 @@ __global__ void __launch_bounds__(512, 1)
             } else if (L.cmd == CMD_EAGER) {
                 // EAGER: the shared FIFO queue in submission
                 // order -- the lowest-id unallocated task
-                T = L.n_avail > 0 ? first_avail() : -1;
+                T = L.n_avail > 0 ? any_first_avail() : -1;
                 if (tid == 0) {
                     if (T >= 0) {
                         L.avail_lo = T;
@@ -1678,8 +1949,11 @@ __global__ void __launch_bounds__(512, 1)
             if (I.flags & DTS_F_VERIFY) verify_scores(k);
             // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
             PROF_T0(p_am);
-            const int32_t Dopt = (I.flags & DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
-                                                        : score_argmax(V.h + (size_t)k * I.nstr);
+            int32_t D2s = -1;  // task shards: the 3inputs argmax comes with the main one
+            const int32_t Dopt = I.G > 1 ? shard_scan(k, (I.flags & DTS_F_FALLBACK2) != 0,
+                                                      (I.flags & DTS_F_OPTI) != 0, &D2s)
+                                 : (I.flags & DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
+                                                          : score_argmax(V.h + (size_t)k * I.nstr);
             PROF_ADD(L, P_ARGMAX, p_am);
             PROF_T0(p_pl);
             if (tid == 0) {
@@ -1687,7 +1961,8 @@ __global__ void __launch_bounds__(512, 1)
                 L.alg_bytes += 8ull * (uint64_t)n;
             }
             if (Dopt >= 0) {
-                plan(k, Dopt);
+                if (I.G > 1) plan_shard(k, Dopt);
+                else plan(k, Dopt);
                 if (tid == 0) {
                     int64_t tau;
                     L.T = pop_planned(k, &tau);
@@ -1698,18 +1973,18 @@ __global__ void __launch_bounds__(512, 1)
                 PROF_ADD(L, P_PLAN, p_pl);
             } else {
                 if (I.flags & DTS_F_FALLBACK2) {
-                    const int32_t D2 = score_argmax(V.h2 + (size_t)k * I.nstr);
+                    const int32_t D2 = I.G > 1 ? D2s : score_argmax(V.h2 + (size_t)k * I.nstr);
                     if (tid == 0) {
                         L.scan_alg_bytes += 8ull * (uint64_t)n;
                         L.alg_bytes += 8ull * (uint64_t)n;
                     }
                     if (D2 >= 0) {
-                        T = first_cnt2(k, D2);
+                        T = any_first_cnt2(k, D2);
                         if (tid == 0) L.n_fb2++;
                     }
                 }
                 if (T < 0 && L.n_avail > 0) {
-                    T = first_avail();
+                    T = any_first_avail();
                     if (tid == 0) {
                         L.n_fbf++;
                         L.avail_lo = T;
@@ -1743,9 +2018,14 @@ __global__ void __launch_bounds__(512, 1)
             PROF_T0(p_ld);
             serve_loads(k, T, t);
             PROF_ADD(L, P_LOADS, p_ld);
-            if (L.error) break;
+            if (L.error || L.xerr) break;
         }
         cta_sync();
+        if (I.G > 1) {  // no shard leaves while a peer may still read its slots
+            xch_sync();
+            if (tid == 0 && L.xerr && !L.error) L.error = 2;
+            cta_sync();
+        }
 
         // ---- a8: per-GPU orders, scalars
         assemble(L.n_served);
@@ -1790,6 +2070,7 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
                 uint32_t x = 0;
                 for (int64_t i = b; i < e; i++) x ^= (uint32_t)I.tdat[i];
                 w = ((uint32_t)(e - b) << 24) | x;
+                if (T < I.t_lo || T >= I.t_hi) w |= ALLOC_BIT;  // another shard's task
                 I.tstart[T] = -1;
                 I.tend[T] = -1;
             }
@@ -1860,6 +2141,17 @@ cudaError_t launch_loop(const Inst *d_insts, int n_inst, int block, int grid, in
     dts_cta_kernel<<<grid, block, smem_bytes, st>>>(d_insts, n_inst, work_counter);
     count_launch();
     return cudaGetLastError();
+}
+
+cudaError_t launch_loop_coop(const Inst *d_insts, int n_inst, int block, int *work_counter, int smem_bytes,
+                             cudaStream_t st) {
+    cudaError_t e = ensure_smem_attr(smem_bytes);
+    if (e != cudaSuccess) return e;
+    void *args[] = {(void *)&d_insts, (void *)&n_inst, (void *)&work_counter};
+    e = cudaLaunchCooperativeKernel((const void *)dts_cta_kernel, dim3(n_inst), dim3(block), args,
+                                    (size_t)smem_bytes, st);
+    count_launch();
+    return e;
 }
 
 int loop_max_blocks_per_sm(int block, int smem_bytes) {

@@ -11,6 +11,10 @@ cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t wo
 // One CTA per instance (grid CTAs pull instances from *work_counter).
 cudaError_t launch_loop(const Inst *d_insts, int n_inst, int block, int grid, int *work_counter,
                         int smem_bytes, cudaStream_t st);
+// Task shards (§8(e)) of one instance on one device: n_inst CTAs that
+// exchange inside the kernel, so a cooperative launch (all co-resident).
+cudaError_t launch_loop_coop(const Inst *d_insts, int n_inst, int block, int *work_counter, int smem_bytes,
+                             cudaStream_t st);
 int loop_max_blocks_per_sm(int block, int smem_bytes);
 int loop_static_smem();
 }  // namespace dts

@@ -40,7 +40,10 @@ EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data",
 
 EXPORTED = ["dts_run_opts_default", "dts_instance_create", "dts_instance_upload", "dts_run",
             "dts_result", "dts_sweep_run", "dts_instance_destroy", "dts_status_str",
-            "dts_last_error", "dts_version", "dts_kernel_launches"]
+            "dts_last_error", "dts_version", "dts_kernel_launches",
+            "dts_shard_set", "dts_shard_range", "dts_shard_export", "dts_shard_connect",
+            "dts_shard_group_run"]
+DTS_SHARD_HANDLE_BYTES = 128
 
 
 class DtsError(RuntimeError):
@@ -108,6 +111,17 @@ def load_library(path: str = LIB_PATH):
     lib.dts_kernel_launches.restype = C.c_uint64
     lib.dts_version.argtypes = []
     lib.dts_version.restype = C.c_uint32
+    lib.dts_shard_set.argtypes = [P, C.c_int32, C.c_int32]
+    lib.dts_shard_set.restype = C.c_int
+    lib.dts_shard_range.argtypes = [P, C.POINTER(C.c_int32), C.POINTER(C.c_int32)]
+    lib.dts_shard_range.restype = C.c_int
+    lib.dts_shard_export.argtypes = [P, C.c_int32, P]
+    lib.dts_shard_export.restype = C.c_int
+    lib.dts_shard_connect.argtypes = [P, P]
+    lib.dts_shard_connect.restype = C.c_int
+    lib.dts_shard_group_run.argtypes = [C.POINTER(C.c_void_p), C.c_int32, C.c_int,
+                                        C.POINTER(dts_run_opts)]
+    lib.dts_shard_group_run.restype = C.c_int
     _lib = lib
     return lib
 
@@ -170,6 +184,39 @@ def dts_sweep_run(insts, policy: int = DTS_POLICY_DARTS_LUF, opts: Optional[dts_
     arr = (C.c_void_p * len(insts))(*[i.handle for i in insts])
     _check(load_library().dts_sweep_run(arr, len(insts), int(policy),
                                         None if opts is None else C.byref(opts)))
+
+
+# ---- task-sharded single instance (include/dts.h, SURVEY.md §8(e) second mode)
+
+def dts_shard_set(inst: Instance, G: int, g: int):
+    _check(load_library().dts_shard_set(inst.handle, int(G), int(g)))
+
+
+def dts_shard_range(inst: Instance):
+    lo, hi = C.c_int32(), C.c_int32()
+    _check(load_library().dts_shard_range(inst.handle, C.byref(lo), C.byref(hi)))
+    return int(lo.value), int(hi.value)
+
+
+def dts_shard_export(inst: Instance, device: int = 0) -> bytes:
+    buf = (C.c_char * DTS_SHARD_HANDLE_BYTES)()
+    _check(load_library().dts_shard_export(inst.handle, int(device), buf))
+    return bytes(buf)
+
+
+def dts_shard_connect(inst: Instance, handles) -> None:
+    """handles: the G exported handles in shard order."""
+    blob = b"".join(bytes(h) for h in handles)
+    if len(blob) % DTS_SHARD_HANDLE_BYTES:
+        raise DtsError(DTS_E_INVAL, "shard handles must be DTS_SHARD_HANDLE_BYTES each")
+    buf = C.create_string_buffer(blob, len(blob))
+    _check(load_library().dts_shard_connect(inst.handle, buf))
+
+
+def dts_shard_group_run(shards, policy: int = DTS_POLICY_DARTS_LUF, opts: Optional[dts_run_opts] = None):
+    arr = (C.c_void_p * len(shards))(*[i.handle for i in shards])
+    _check(load_library().dts_shard_group_run(arr, len(shards), int(policy),
+                                              None if opts is None else C.byref(opts)))
 
 
 @dataclass
@@ -266,4 +313,18 @@ def schedule_batch(insts, *, policy: int = DTS_POLICY_DARTS_LUF, W: int = 0, fla
                              block_threads=block_threads, smem_budget=smem_budget,
                              max_served=-1, cuda_stream=stream or None)
     dts_sweep_run(hs, policy, o)
+    return [dts_result(h) for h in hs]
+
+
+def schedule_sharded(inst, G: int, *, policy: int = DTS_POLICY_DARTS_LUF, W: int = 0,
+                     flags: int = DTS_F_FALLBACK2, bus_bps: int = 12_000_000_000, device: int = 0,
+                     block_threads: int = 0, smem_budget: int = 0, max_served: int = -1,
+                     stream: int = 0):
+    """One instance, its tasks sharded over G co-resident CTAs of one device
+    (dts_shard_group_run); returns every shard's result (all equal)."""
+    hs = [create(inst) for _ in range(G)]
+    o = dts_run_opts_default(flags=flags, lookahead_W=W, bus_bytes_per_s=bus_bps, device=device,
+                             block_threads=block_threads, smem_budget=smem_budget,
+                             max_served=max_served, cuda_stream=stream or None)
+    dts_shard_group_run(hs, policy, o)
     return [dts_result(h) for h in hs]
