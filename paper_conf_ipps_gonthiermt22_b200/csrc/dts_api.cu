@@ -123,6 +123,7 @@ struct dts_instance {
     int64_t box_bytes = 0;
     dts::ShardPeer *d_peers = nullptr;       // [MAX_G] peer table read by the kernel
     bool connected = false;
+    bool xsys = false;                       // peers mapped through CUDA IPC (other processes / GPUs)
     std::vector<void *> ipc_open;            // peers' arenas mapped through CUDA IPC
 
     ~dts_instance() {
@@ -574,6 +575,7 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     h.peers = I->G > 1 ? I->d_peers : nullptr;
     h.ep_base = (unsigned long long)(++I->runs) << 32;
     h.box_bytes = I->box_bytes;
+    h.xsys = I->xsys ? 1 : 0;
     // small instances: the loop CTA builds its own CSR and state (one launch)
     const int fs = fused_scratch_bytes(I, block);
     h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
@@ -863,6 +865,7 @@ dts_status dts_shard_connect(dts_instance *I, const void *handles) {
         tab[(size_t)p].h2 = (const int32_t *)(c + hd.off_h2);
         tab[(size_t)p].u = (const int32_t *)(c + hd.off_u);
     }
+    I->xsys = true;
     return write_peers(I, tab);
 }
 
@@ -901,6 +904,7 @@ dts_status dts_shard_group_run(dts_instance *const *shards, int32_t G, dts_polic
         for (int32_t i = 0; i < G; i++) {
             s = write_peers(shards[i], tab);
             if (s != DTS_OK) return s;
+            shards[i]->xsys = false;
         }
     }
     if (o.block_threads) block = o.block_threads;

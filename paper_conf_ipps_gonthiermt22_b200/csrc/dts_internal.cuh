@@ -142,6 +142,8 @@ struct Inst {
     const ShardPeer *peers;   // [G] (device), nullptr when G = 1
     unsigned long long ep_base;  // exchange numbers of this run: ep_base + 1, 2, ...
     int64_t box_bytes;        // bytes of one payload slot
+    int32_t xsys;             // 1: peers on other devices (system-scope release/acquire)
+    int32_t pad3;
 };
 
 }  // namespace dts

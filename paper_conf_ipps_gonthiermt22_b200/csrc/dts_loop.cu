@@ -114,6 +114,7 @@ struct View {
 __shared__ Lead L;
 __shared__ Inst SI;
 __shared__ View SV;
+__shared__ ShardPeer SP[MAX_G];  // task shards: the peer table (copied at instance start)
 
 __device__ __forceinline__ int warp_sum(int v) {
 #pragma unroll
@@ -1271,34 +1272,44 @@ __device__ __forceinline__ unsigned long long global_ns() {
 }
 constexpr unsigned long long XCH_TIMEOUT_NS = 5000000000ull;
 
+__device__ __forceinline__ unsigned long long ld_acquire_gpu(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_gpu(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
 // Payload slot of exchange number x (1-based within the run) of shard p.
 __device__ __forceinline__ ShardSlot *xch_slot(int p, int64_t x) {
     const Inst &I = SI;
-    unsigned char *box = (unsigned char *)__ldg((const unsigned long long *)&I.peers[p].box);
-    return reinterpret_cast<ShardSlot *>(box + (x & 1) * I.box_bytes);
+    return reinterpret_cast<ShardSlot *>(SP[p].box + (x & 1) * I.box_bytes);
 }
 
 // Block-wide: publish this shard's slot of the next exchange (every thread's
 // writes to it precede the barrier) and wait until every shard published the
-// same exchange.  Thread 0 releases at system scope (peers may be other GPUs);
-// warp 0 acquires the peers' exchange numbers.  Two slots by parity suffice: a
+// same exchange.  Thread 0 releases (system scope when the peers are other
+// GPUs, I.xsys; GPU scope for CTAs of one device) -- the barrier orders the
+// other threads' writes before it -- and warp 0 acquires the peers' exchange
+// numbers.  Two slots by parity suffice: a
 // shard reuses a slot only after every peer published the exchange in between,
 // which they do only after reading this one.  A peer missing for
 // XCH_TIMEOUT_NS sets L.xerr -- the run ends with an error instead of a hang.
 __device__ __noinline__ void xch_sync() {
     const Inst &I = SI;
     const unsigned long long e = I.ep_base + (unsigned long long)L.xe + 1ull;
+    PROF_T0(p_x);
     cta_sync();
     if (threadIdx.x == 0) {
-        __threadfence_system();
-        st_release_sys((unsigned long long *)__ldg((const unsigned long long *)&I.peers[I.g].epoch), e);
+        if (I.xsys) st_release_sys(SP[I.g].epoch, e);
+        else st_release_gpu(SP[I.g].epoch, e);
     }
     if (threadIdx.x < 32) {
         const unsigned long long t0 = global_ns();
         for (int p = threadIdx.x; p < I.G; p += 32) {
-            const unsigned long long *f =
-                (const unsigned long long *)__ldg((const unsigned long long *)&I.peers[p].epoch);
-            while (ld_acquire_sys(f) < e) {
+            const unsigned long long *f = SP[p].epoch;
+            while ((I.xsys ? ld_acquire_sys(f) : ld_acquire_gpu(f)) < e) {
                 if (global_ns() - t0 > XCH_TIMEOUT_NS) {
                     L.xerr = 1;
                     break;
@@ -1306,9 +1317,13 @@ __device__ __noinline__ void xch_sync() {
             }
         }
         __syncwarp();
-        if (threadIdx.x == 0) L.xe = L.xe + 1;
+        if (threadIdx.x == 0) {
+            L.xe = L.xe + 1;
+            L.prof[P_X2] += 1;
+        }
     }
     cta_sync();
+    PROF_ADD(L, P_X1, p_x);
 }
 
 // Block-wide: minimum over shards of one block-uniform candidate (~0 = none).
@@ -1351,16 +1366,14 @@ __device__ __noinline__ int32_t shard_scan(int k, bool fb2, bool opti, int32_t *
         for (int v = v0 + threadIdx.x; v < v1; v += blockDim.x) {
             int4 hs = make_int4(0, 0, 0, 0), us = hs, h2s = hs;
             for (int p = 0; p < I.G; p++) {
-                const ShardPeer *P = &I.peers[p];
-                const int4 *ph = (const int4 *)((const int32_t *)__ldg((const unsigned long long *)&P->h) +
-                                                (size_t)k * I.nstr);
-                const int4 *pu = (const int4 *)__ldg((const unsigned long long *)&P->u);
+                const ShardPeer *P = &SP[p];
+                const int4 *ph = (const int4 *)(P->h + (size_t)k * I.nstr);
+                const int4 *pu = (const int4 *)P->u;
                 const int4 a = __ldcg(ph + v), c = __ldcg(pu + v);
                 hs.x += a.x; hs.y += a.y; hs.z += a.z; hs.w += a.w;
                 us.x += c.x; us.y += c.y; us.z += c.z; us.w += c.w;
                 if (fb2) {
-                    const int4 *ph2 = (const int4 *)((const int32_t *)__ldg((const unsigned long long *)&P->h2) +
-                                                     (size_t)k * I.nstr);
+                    const int4 *ph2 = (const int4 *)(P->h2 + (size_t)k * I.nstr);
                     const int4 d = __ldcg(ph2 + v);
                     h2s.x += d.x; h2s.y += d.y; h2s.z += d.z; h2s.w += d.w;
                 }
@@ -1823,6 +1836,8 @@ __global__ void __launch_bounds__(512, 1)
         }
         cta_sync();
         const View &V = SV;
+        if (I.G > 1)
+            for (int p = tid; p < I.G; p += blockDim.x) SP[p] = I.peers[p];
 
         const int n = I.n, K = I.K;
         if (I.fused) {  // a1 + a2 inside this CTA (small instances)
