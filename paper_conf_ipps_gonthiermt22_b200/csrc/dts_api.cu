@@ -438,6 +438,7 @@ dts_status ensure_device(dts_instance *I, int device) {
     h.id_bits = bits_for(I->n > 0 ? (uint64_t)(I->n - 1) : 0);
     h.u_bits = bits_for((uint64_t)I->max_deg_ub);
     h.key32 = I->max_deg_ub < 32768 ? 1 : 0;  // n(D), n2(D), u(D) <= deg(D)
+    h.max_row = I->max_row_len;
     h.E = I->E_raw;
     h.size = I->d_size;
     h.delta = I->d_delta;

@@ -88,7 +88,7 @@ struct Inst {
     int32_t res_cap;     // >= max resident data per GPU
     int32_t id_bits, u_bits;
     int32_t key32;       // scores and u(D) < 2^15: 32-bit argmax keys (score << 16 | u)
-    int32_t pad0;
+    int32_t max_row;     // max |D(T)|
     int32_t nw;          // 32-bit words per residency bitmap row
     int32_t nstr;        // row stride of h, h2, np (and length of u): n rounded up to 4
     int64_t E;

@@ -91,6 +91,9 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     int32_t bhead[32], bcnt[32], boff[33];
     int64_t rkey[POP_RANK_MAX];  // pop batch: request time of each pop (merge ranks)
     int32_t rgpu[POP_RANK_MAX];
+    int4 fent;       // a fallback / EAGER pick as a plan entry (pool_move_many)
+    int32_t miss[MAX_ROW + 1];  // serve_loads: D(T) \ R_k in ascending id (R10)
+    int32_t nmiss;
     int64_t xe;      // task shards: exchanges done in this run
     int32_t xerr;    // task shards: a peer did not arrive in time (the run is abandoned)
     int32_t xoff[MAX_G + 1];  // plan exchange: each shard's offset in the merged plan
@@ -116,26 +119,22 @@ __shared__ Inst SI;
 __shared__ View SV;
 __shared__ ShardPeer SP[MAX_G];  // task shards: the peer table (copied at instance start)
 
-__device__ __forceinline__ int warp_sum(int v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
-    return v;
-}
+// Warp reductions with redux.sync (one instruction per 32-bit reduction): a
+// 64-bit max / min is the high words' extremum, then the low words' among the
+// lanes that hold it -- 56 cycles on the B200 against 200 for five 64-bit
+// shuffle rounds (tools/micro/redux_micro.cu).  Every lane must take part.
+__device__ __forceinline__ int warp_sum(int v) { return (int)__reduce_add_sync(FULL, (unsigned)v); }
 __device__ __forceinline__ unsigned long long warp_max_u64(unsigned long long v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        unsigned long long t = __shfl_xor_sync(FULL, v, o);
-        v = t > v ? t : v;
-    }
-    return v;
+    const unsigned hi = (unsigned)(v >> 32), lo = (unsigned)v;
+    const unsigned mh = __reduce_max_sync(FULL, hi);
+    const unsigned ml = __reduce_max_sync(FULL, hi == mh ? lo : 0u);
+    return ((unsigned long long)mh << 32) | ml;
 }
 __device__ __forceinline__ unsigned long long warp_min_u64(unsigned long long v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        unsigned long long t = __shfl_xor_sync(FULL, v, o);
-        v = t < v ? t : v;
-    }
-    return v;
+    const unsigned hi = (unsigned)(v >> 32), lo = (unsigned)v;
+    const unsigned mh = __reduce_min_sync(FULL, hi);
+    const unsigned ml = __reduce_min_sync(FULL, hi == mh ? lo : 0xffffffffu);
+    return ((unsigned long long)mh << 32) | ml;
 }
 
 // Block reductions (every thread calls; the result is returned to every
@@ -157,6 +156,21 @@ __device__ unsigned long long block_min_u64(unsigned long long v) {
     if (lane == 0) L.red64[w] = v;
     cta_sync();
     return warp_min_u64(lane < nw ? L.red64[lane] : ~0ull);
+}
+// Sum of one int and min of one unsigned per thread, in one exchange.
+__device__ void block_sum_min(int &sum, unsigned &mn) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    sum = warp_sum(sum);
+    mn = __reduce_min_sync(FULL, mn);
+    if (nw == 1) return;
+    cta_sync();
+    if (lane == 0) {
+        L.red32[w] = sum;
+        L.wcnt[w] = (int)mn;
+    }
+    cta_sync();
+    sum = warp_sum(lane < nw ? L.red32[lane] : 0);
+    mn = __reduce_min_sync(FULL, lane < nw ? (unsigned)L.wcnt[lane] : 0xffffffffu);
 }
 __device__ int block_sum(int v) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
@@ -207,16 +221,6 @@ struct Row {
     int32_t r0, r1, r2, len;
 };
 
-__device__ __forceinline__ Row row_of_task(int32_t T) {
-    const Inst &I = SI;
-    const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
-    Row r;
-    r.len = (int32_t)(re - rb);
-    r.r0 = r.len > 0 ? __ldg(&I.tdat[rb]) : -1;
-    r.r1 = r.len > 1 ? __ldg(&I.tdat[rb + 1]) : -1;
-    r.r2 = r.len > 2 ? __ldg(&I.tdat[rb + 2]) : -1;
-    return r;
-}
 
 // Rows longer than 3: the (first two) inputs of T not resident on GPU k,
 // skipping `skip`, read from the CSR.
@@ -312,6 +316,73 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
         if (own) atomicAdd(&V.u[c[i]], sign);
         if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[i]], -sign);
     }
+}
+
+// Block-wide pool_move of P tasks given as plan entries {T, D0, D1, D2}
+// (-1 = absent input, D2 = ROW_LONG: read the row from the CSR).  The
+// (task, simulated GPU) state items and the per-task input counts (u, np) are
+// spread over the CTA: one short dependent chain per item instead of K
+// divergent ones per task on one thread.  Entries must be visible to every
+// thread (written before a barrier); the caller synchronises afterwards.
+__device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, int plan_k) {
+    const Inst &I = SI;
+    const View &V = SV;
+    const int K = I.K;
+    const int n_state = P * K;
+    for (int idx = threadIdx.x; idx < n_state + P; idx += blockDim.x) {
+        if (idx < n_state) {
+            const int p = idx / K, j = idx - p * K;
+            const int4 e = ents[p];
+            const int32_t T = e.x;
+            if (T < I.t_lo || T >= I.t_hi) continue;  // another shard's task
+            uint32_t *sp = &V.s[(size_t)j * I.m_pad + T];
+            const uint32_t w = *sp;
+            *sp = sign < 0 ? (w | ALLOC_BIT) : (w & ~ALLOC_BIT);
+            const uint32_t c = (w >> 24) & 0x7fu;
+            if (c == 1u) {
+                atomicAdd(&V.h[(size_t)j * I.nstr + (w & XOR_MASK)], sign);
+            } else if (c == 2u) {
+                int32_t a, b;
+                const bool lng = e.w == ROW_LONG;
+                const int len = lng ? 4 : (e.y >= 0) + (e.z >= 0) + (e.w >= 0);
+                if (len == 2) {  // both inputs miss: no residency lookups
+                    a = e.y;
+                    b = e.z >= 0 ? e.z : e.w;
+                } else {
+                    missing_pair(j, T, Row{e.y, e.z, lng ? -1 : e.w, len}, -1, a, b);
+                }
+                atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+                atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
+            }
+        } else {
+            const int4 e = ents[idx - n_state];
+            const int32_t T = e.x;
+            const bool own = T >= I.t_lo && T < I.t_hi;
+            if (e.w == ROW_LONG) {
+                pool_move_long_row(T, sign, plan_k, own);
+                continue;
+            }
+            const int32_t c[3] = {e.y, e.z, e.w};
+#pragma unroll
+            for (int q = 0; q < 3; q++) {
+                if (c[q] < 0) continue;
+                if (own) atomicAdd(&V.u[c[q]], sign);
+                if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[q]], -sign);
+            }
+        }
+    }
+}
+
+// D(T) of task T as a plan entry {T, D0, D1, D2 | ROW_LONG} (thread-local).
+__device__ __forceinline__ int4 entry_of_task(int32_t T) {
+    const Inst &I = SI;
+    const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+    const int len = (int)(re - rb);
+    int4 e = make_int4(T, -1, -1, -1);
+    if (len > 0) e.y = __ldg(&I.tdat[rb]);
+    if (len > 1) e.z = __ldg(&I.tdat[rb + 1]);
+    if (len > 2) e.w = len > 3 ? ROW_LONG : __ldg(&I.tdat[rb + 2]);
+    return e;
 }
 
 // a2: datum D becomes resident (load) / leaves (evict) on GPU k.  Walk D's
@@ -651,129 +722,67 @@ __device__ __forceinline__ int pops_before(int j, PopGpu g, int c, int64_t r, in
 // resident (LUF drops planned tasks whose inputs it evicts, Alg. 6 l.8) and
 // np_k is rebuilt at every scan of k (reset_plan), so each GPU's request
 // times are prefix sums of its planned tasks' tau (W = 0).
-// Warp 0 (one lane per simulated GPU, K <= 32) finds the next scan -- the
-// earliest (request after the GPU's last pop, GPU id) (R8) -- and each GPU's
-// pop count before it; then every thread places pops in the global service
-// order by merge ranks.  Sets L.cmd (CMD_SCAN with L.k, L.t, or CMD_DONE).
-// Scalar phase of pop_batch for K <= KR with the per-GPU values in registers
-// (fully unrolled over KR): the next scan (earliest request after a GPU's last
-// pop, R8), each GPU's pop count before it, the new request times.
-template <int KR>
-__device__ __forceinline__ void pop_batch_scalar() {
+// Scalar phase on warp 0, lane j = simulated GPU j (K <= 32): the next scan
+// -- the earliest (request after the GPU's last pop, GPU id) (R8), a warp min
+// plus the lowest lane holding it -- each GPU's pop count before it (binary
+// searches in parallel), their offsets (lane prefix sum), the new request
+// times.  Sets L.cmd (CMD_SCAN with L.k, L.t, or CMD_DONE).
+__device__ __noinline__ void pop_batch_warp() {
     const Inst &I = SI;
-    const int K = I.K;
-    int64_t rq[KR], st[KR], S[KR];
-    int hd[KR], lv[KR];
-    bool act[KR];
-#pragma unroll
-    for (int j = 0; j < KR; j++) {
-        act[j] = j < K && !L.idle[j];
-        rq[j] = j < K ? L.req[j] : 0;
-        const int64_t gf = j < K ? L.gpu_free[j] : 0;
-        st[j] = rq[j] > gf ? rq[j] : gf;
-        hd[j] = j < K ? L.plan_head[j] : 0;
-        lv[j] = j < K ? L.plan_end[j] - hd[j] : 0;
+    const int K = I.K, j = threadIdx.x;
+    const bool in = j < K;
+    const bool act = in && !L.idle[j];
+    const int64_t rq = in ? L.req[j] : 0;
+    const int64_t gf = in ? L.gpu_free[j] : 0;
+    const int64_t st = rq > gf ? rq : gf;
+    const int hd = in ? L.plan_head[j] : 0;
+    const int lv = in ? L.plan_end[j] - hd : 0;
+    const int64_t S = lv == 0 ? rq : st + plan_span(j, hd, lv);
+    const unsigned long long key = act ? (unsigned long long)S : ~0ull;  // times >= 0
+    const unsigned long long mk = warp_min_u64(key);
+    const unsigned am = __ballot_sync(FULL, act && key == mk);
+    const int kb = am ? __ffs(am) - 1 : -1;
+    const int64_t sb = (int64_t)mk;
+    int c = 0;
+    if (act && kb >= 0) {
+        PopGpu g;
+        g.req = rq;
+        g.start0 = st;
+        g.head = hd;
+        c = j == kb ? lv : pops_before(j, g, lv, sb, kb);
     }
-    int kb = -1;
-    int64_t sb = INT64_MAX;
-#pragma unroll
-    for (int j = 0; j < KR; j++) {
-        S[j] = lv[j] == 0 ? rq[j] : st[j] + plan_span(j, hd[j], lv[j]);
-        const bool take = act[j] & ((kb < 0) | (S[j] < sb));
-        kb = take ? j : kb;
-        sb = take ? S[j] : sb;
+    int x = c;  // inclusive prefix over lanes 0..K-1
+    for (int o = 1; o < K; o <<= 1) {
+        const int t = __shfl_up_sync(FULL, x, o);
+        if (j >= o) x += t;
     }
-    int total = 0;
-    int64_t mk = L.makespan;
-#pragma unroll
-    for (int j = 0; j < KR; j++) {
-        if (j >= K) break;
-        int c = 0;
-        if (act[j] && kb >= 0) {
-            PopGpu g;
-            g.req = rq[j];
-            g.start0 = st[j];
-            g.head = hd[j];
-            c = j == kb ? lv[j] : pops_before(j, g, lv[j], sb, kb);
-        }
-        L.breq[j] = rq[j];
-        L.bstart[j] = st[j];
-        L.bhead[j] = hd[j];
+    const int total = __shfl_sync(FULL, x, K - 1);
+    int64_t last = 0;
+    if (in) {
+        L.breq[j] = rq;
+        L.bstart[j] = st;
+        L.bhead[j] = hd;
         L.bcnt[j] = c;
-        L.boff[j] = total;
-        total += c;
+        L.boff[j] = x - c;
         if (c > 0) {
-            const int64_t last = st[j] + plan_span(j, hd[j], c);
+            last = st + plan_span(j, hd, c);
             L.req[j] = last;  // W = 0 (R7)
             L.gpu_free[j] = last;
-            L.plan_head[j] = hd[j] + c;
+            L.plan_head[j] = hd + c;
             L.plan_live[j] -= c;
-            mk = last > mk ? last : mk;
         }
     }
-    L.boff[K] = total;
-    L.bns = L.n_served;
-    L.n_served += total;
-    L.makespan = mk;
-    L.alg_bytes += 24ull * (uint64_t)total;
-    L.k = kb;
-    L.t = sb;
-    L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
-}
-
-// The same for 8 < K <= 32, values left in shared memory.
-__device__ __noinline__ void pop_batch_scalar_smem() {
-    const Inst &I = SI;
-    const int K = I.K;
-    int kb = -1;
-    int64_t sb = INT64_MAX;
-    for (int j = 0; j < K; j++) {
-        const int64_t req = L.req[j];
-        const int64_t start0 = req > L.gpu_free[j] ? req : L.gpu_free[j];
-        const int head = L.plan_head[j];
-        L.breq[j] = req;
-        L.bstart[j] = start0;
-        L.bhead[j] = head;
-        if (L.idle[j]) continue;
-        const int live = L.plan_end[j] - head;
-        const int64_t S = live == 0 ? req : start0 + plan_span(j, head, live);
-        if (kb < 0 || S < sb) {
-            kb = j;
-            sb = S;
-        }
+    const int64_t mkx = (int64_t)warp_max_u64((unsigned long long)last);
+    if (j == 0) {
+        L.boff[K] = total;
+        L.bns = L.n_served;
+        L.n_served += total;
+        if (mkx > L.makespan) L.makespan = mkx;
+        L.alg_bytes += 24ull * (uint64_t)total;
+        L.k = kb;
+        L.t = sb;
+        L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
     }
-    int total = 0;
-    int64_t mk = L.makespan;
-    for (int j = 0; j < K; j++) {
-        int c = 0;
-        if (!L.idle[j] && kb >= 0) {
-            const int live = L.plan_end[j] - L.bhead[j];
-            PopGpu g;
-            g.req = L.breq[j];
-            g.start0 = L.bstart[j];
-            g.head = L.bhead[j];
-            c = j == kb ? live : pops_before(j, g, live, sb, kb);
-        }
-        L.bcnt[j] = c;
-        L.boff[j] = total;
-        total += c;
-        if (c > 0) {
-            const int64_t last = L.bstart[j] + plan_span(j, L.bhead[j], c);
-            L.req[j] = last;  // W = 0 (R7)
-            L.gpu_free[j] = last;
-            L.plan_head[j] += c;
-            L.plan_live[j] -= c;
-            mk = last > mk ? last : mk;
-        }
-    }
-    L.boff[K] = total;
-    L.bns = L.n_served;
-    L.n_served += total;
-    L.makespan = mk;
-    L.alg_bytes += 24ull * (uint64_t)total;
-    L.k = kb;
-    L.t = sb;
-    L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
 }
 
 __device__ void pop_batch() {
@@ -781,11 +790,7 @@ __device__ void pop_batch() {
     const View &V = SV;
     const int K = I.K;
     PROF_T0(p_w0);
-    if (threadIdx.x == 0) {
-        if (K <= 4) pop_batch_scalar<4>();
-        else if (K <= 8) pop_batch_scalar<8>();
-        else pop_batch_scalar_smem();
-    }
+    if (threadIdx.x < 32) pop_batch_warp();
     cta_sync();
     PROF_ADD(L, P_BW0, p_w0);
     PROF_T0(p_bd);
@@ -921,6 +926,7 @@ __device__ int32_t luf_victim(int k) {
     // LUF key np_k(D); LRU policies: the serve index of D's last use on k
     const int32_t *npk = (I.policy == DTS_POLICY_DARTS_LUF ? V.np : V.lru) + (size_t)k * I.nstr;
     unsigned long long best = ~0ull;
+    int bslot = -1;
     for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
         const int32_t D = rl[i];
         bool in_buf = false;  // nb(D) > 0: an input of a taskBuffer_k task
@@ -928,15 +934,16 @@ __device__ int32_t luf_victim(int k) {
         for (int r = 0; r < L.row2_len; r++) in_buf |= (L.row2[r] == D);
         const unsigned long long key =
             ((unsigned long long)(uint32_t)npk[D] << 32) | (unsigned long long)(uint32_t)D;
-        best = (!in_buf & (key < best)) ? key : best;
+        const bool take = !in_buf & (key < best);
+        best = take ? key : best;
+        bslot = take ? i : bslot;
     }
+    const unsigned long long mine = best;
     best = block_min_u64(best);
     if (best == ~0ull) return -1;
-    const int32_t Vd = (int32_t)(best & 0xffffffffull);
-    for (int i = threadIdx.x; i < cnt; i += blockDim.x)
-        if (rl[i] == Vd) L.vslot = i;
+    if (mine == best) L.vslot = bslot;  // the one thread holding V (ids are unique)
     cta_sync();
-    return Vd;
+    return (int32_t)(best & 0xffffffffull);
 }
 
 // Alg. 6 l.8-9: planned tasks of k that use V return to the shared pool (R4,
@@ -946,7 +953,7 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
     const View &V = SV;
     int4 *pl = V.plan + (size_t)k * I.plan_cap;
     int nret = 0;
-    unsigned long long tmin = ~0ull;
+    unsigned tmin = 0xffffffffu;
     // Alg. 6 l.8 is LUF's; an LRU eviction leaves plannedTasks_k alone
     const int ph = L.plan_head[k], pe = I.policy == DTS_POLICY_DARTS_LUF ? L.plan_end[k] : ph;
     for (int i = ph + threadIdx.x; i < pe; i += blockDim.x) {
@@ -955,11 +962,10 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
             pl[i].x = -1;
             pool_move(e.x, row_of_entry(e), +1, k);
             nret++;
-            tmin = (unsigned long long)e.x < tmin ? (unsigned long long)e.x : tmin;
+            tmin = (unsigned)e.x < tmin ? (unsigned)e.x : tmin;
         }
     }
-    nret = block_sum(nret);
-    tmin = block_min_u64(tmin);
+    block_sum_min(nret, tmin);
     if (threadIdx.x == 0) {
         if (nret > 0) {
             L.plan_live[k] -= nret;
@@ -995,11 +1001,17 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
 __device__ void serve_loads(int k, int32_t T, int64_t t) {
     const Inst &I = SI;
     const View &V = SV;
+    // Thread 0: the missing inputs, ascending (R10).  Residency of D(T) only
+    // changes by these loads while T is served (LUF never evicts an input of
+    // a taskBuffer task), so the list is fixed up front: one barrier.
     if (threadIdx.x == 0) {
         L.ready = t;
         L.row2_len = 0;
+        int nm = 0;
+        for (int r = 0; r < L.row_len; r++)
+            if (!resident(k, L.row[r])) L.miss[nm++] = L.row[r];
+        L.nmiss = nm;
     }
-    cta_sync();
     // W = 1: taskBuffer_k also holds the task still running on k (R7)
     if (I.W >= 1 && L.last_task[k] >= 0 && L.last_end[k] > t && threadIdx.x < 32) {
         const int32_t Tr = L.last_task[k];
@@ -1008,13 +1020,9 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
         if (threadIdx.x == 0) L.row2_len = (int)(re - rb);
     }
     cta_sync();
-    const int len = L.row_len;
-    for (int r = 0; r < len; r++) {
-        // every thread reads the shared state before thread 0 may change it
-        const int32_t D = L.row[r];
-        const bool res = resident(k, D);
-        cta_sync();
-        if (res) continue;
+    const int nmiss = L.nmiss;
+    for (int r = 0; r < nmiss; r++) {
+        const int32_t D = L.miss[r];
         const uint64_t sz = size_of(D);
         while (true) {  // R11: LUF until D fits
             const bool full = L.used[k] + sz > I.cap;
@@ -1048,7 +1056,9 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
             seg_of(D, sb, se);
             L.alg_bytes += 24ull * (uint64_t)(se - sb) + 32ull;
         }
-        cta_sync();
+        // seg_update reads nothing thread 0 just wrote unless a row is longer
+        // than its edge record (missing_pair reads the residency bitmap)
+        if (I.max_row > 3) cta_sync();
         PROF_T0(p_seg);
         seg_update(k, D, true);
         cta_sync();
@@ -1169,6 +1179,7 @@ __device__ void plan(int k, int32_t Dopt) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
     int base_out = 0;
+    PROF_T0(p_q3);
     for (int64_t base = b; base < e; base += blockDim.x) {
         const int64_t i = base + threadIdx.x;
         int32_t T = -1;
@@ -1190,14 +1201,18 @@ __device__ void plan(int k, int32_t Dopt) {
         }
         if (sel) {
             const int pos = off + __popc(msk & lt);
-            const Row r = ed.w > 3 ? Row{-1, -1, -1, ed.w} : Row{Dopt, ed.y, ed.z, ed.w};
             pl[pos] = make_int4(T, Dopt, ed.y, ed.w > 3 ? ROW_LONG : ed.z);
             if (pt) pt[pos] = tau_of(T);
-            pool_move(T, r, -1, k);
         }
         base_out += tot;
         cta_sync();
     }
+    PROF_T0(p_pm);
+    pool_move_many(pl, base_out, -1, k);
+    cta_sync();
+    PROF_ADD(L, P_X1, p_pm);
+    PROF_ADD(L, P_X3, p_q3);
+    PROF_T0(p_q4);
     if (pt) block_incl_scan(pt, 0, base_out, 0);  // tau -> prefix sums
     if (threadIdx.x == 0) {
         L.plan_head[k] = 0;
@@ -1207,6 +1222,7 @@ __device__ void plan(int k, int32_t Dopt) {
         L.alg_bytes += 20ull * (uint64_t)(e - b) + (uint64_t)base_out * (8ull * I.K + 40ull);
     }
     cta_sync();
+    PROF_ADD(L, P_X4, p_q4);
 }
 
 // 3inputs: the lowest-id unallocated task of D2's segment with two missing inputs.
@@ -1484,8 +1500,9 @@ __device__ __noinline__ void plan_shard(int k, int32_t Dopt) {
         const int4 en = __ldcg(reinterpret_cast<const int4 *>(xch_slot(p, L.xe) + 1) + (i - L.xoff[p]));
         pl[i] = en;
         if (pt) pt[i] = tau_of(en.x);
-        pool_move(en.x, row_of_entry(en), -1, k);
     }
+    cta_sync();
+    pool_move_many(pl, total, -1, k);
     cta_sync();
     if (pt) block_incl_scan(pt, 0, total, 0);
     if (threadIdx.x == 0) {
@@ -1950,7 +1967,7 @@ __global__ void __launch_bounds__(512, 1)
                     if (T >= 0) {
                         L.avail_lo = T;
                         L.row_len = -1;
-                        pool_move(T, row_of_task(T), -1, -1);
+                        L.fent = entry_of_task(T);
                         L.n_avail--;
                     } else {
                         L.idle[k] = 1;
@@ -1959,6 +1976,8 @@ __global__ void __launch_bounds__(512, 1)
                 }
                 cta_sync();
                 if (T < 0) continue;
+                pool_move_many(&L.fent, 1, -1, -1);
+                cta_sync();
             } else {
             reset_plan(k);
             if (I.flags & DTS_F_VERIFY) verify_scores(k);
@@ -2008,10 +2027,12 @@ __global__ void __launch_bounds__(512, 1)
                 if (T >= 0) {
                     if (tid == 0) {
                         L.row_len = -1;
-                        pool_move(T, row_of_task(T), -1, -1);
+                        L.fent = entry_of_task(T);
                         L.n_avail--;
                         L.n_scans++;
                     }
+                    cta_sync();
+                    pool_move_many(&L.fent, 1, -1, -1);
                 } else if (tid == 0) {
                     L.idle[k] = 1;
                     L.n_idle++;

@@ -1,0 +1,6 @@
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:dts_cta_kernel -s 1 -c 1 -o gpurun_out/c2n100 python tools/one_instance.py C2 19 > gpurun_out/ncu_src.log 2>&1
+echo "ncu rc=$?"; tail -3 gpurun_out/ncu_src.log
+ncu -i gpurun_out/c2n100.ncu-rep --page source --csv --print-source sass > gpurun_out/c2n100_sass.csv 2>&1
+ncu -i gpurun_out/c2n100.ncu-rep --page source --csv > gpurun_out/c2n100_src.csv 2>&1
+ls -la gpurun_out/
