@@ -722,67 +722,129 @@ __device__ __forceinline__ int pops_before(int j, PopGpu g, int c, int64_t r, in
 // resident (LUF drops planned tasks whose inputs it evicts, Alg. 6 l.8) and
 // np_k is rebuilt at every scan of k (reset_plan), so each GPU's request
 // times are prefix sums of its planned tasks' tau (W = 0).
-// Scalar phase on warp 0, lane j = simulated GPU j (K <= 32): the next scan
-// -- the earliest (request after the GPU's last pop, GPU id) (R8), a warp min
-// plus the lowest lane holding it -- each GPU's pop count before it (binary
-// searches in parallel), their offsets (lane prefix sum), the new request
-// times.  Sets L.cmd (CMD_SCAN with L.k, L.t, or CMD_DONE).
-__device__ __noinline__ void pop_batch_warp() {
+// Warp 0 (one lane per simulated GPU, K <= 32) finds the next scan -- the
+// earliest (request after the GPU's last pop, GPU id) (R8) -- and each GPU's
+// pop count before it; then every thread places pops in the global service
+// order by merge ranks.  Sets L.cmd (CMD_SCAN with L.k, L.t, or CMD_DONE).
+// Scalar phase of pop_batch for K <= KR with the per-GPU values in registers
+// (fully unrolled over KR): the next scan (earliest request after a GPU's last
+// pop, R8), each GPU's pop count before it, the new request times.
+template <int KR>
+__device__ __forceinline__ void pop_batch_scalar() {
     const Inst &I = SI;
-    const int K = I.K, j = threadIdx.x;
-    const bool in = j < K;
-    const bool act = in && !L.idle[j];
-    const int64_t rq = in ? L.req[j] : 0;
-    const int64_t gf = in ? L.gpu_free[j] : 0;
-    const int64_t st = rq > gf ? rq : gf;
-    const int hd = in ? L.plan_head[j] : 0;
-    const int lv = in ? L.plan_end[j] - hd : 0;
-    const int64_t S = lv == 0 ? rq : st + plan_span(j, hd, lv);
-    const unsigned long long key = act ? (unsigned long long)S : ~0ull;  // times >= 0
-    const unsigned long long mk = warp_min_u64(key);
-    const unsigned am = __ballot_sync(FULL, act && key == mk);
-    const int kb = am ? __ffs(am) - 1 : -1;
-    const int64_t sb = (int64_t)mk;
-    int c = 0;
-    if (act && kb >= 0) {
-        PopGpu g;
-        g.req = rq;
-        g.start0 = st;
-        g.head = hd;
-        c = j == kb ? lv : pops_before(j, g, lv, sb, kb);
+    const int K = I.K;
+    int64_t rq[KR], st[KR], S[KR];
+    int hd[KR], lv[KR];
+    bool act[KR];
+#pragma unroll
+    for (int j = 0; j < KR; j++) {
+        act[j] = j < K && !L.idle[j];
+        rq[j] = j < K ? L.req[j] : 0;
+        const int64_t gf = j < K ? L.gpu_free[j] : 0;
+        st[j] = rq[j] > gf ? rq[j] : gf;
+        hd[j] = j < K ? L.plan_head[j] : 0;
+        lv[j] = j < K ? L.plan_end[j] - hd[j] : 0;
     }
-    int x = c;  // inclusive prefix over lanes 0..K-1
-    for (int o = 1; o < K; o <<= 1) {
-        const int t = __shfl_up_sync(FULL, x, o);
-        if (j >= o) x += t;
+    int kb = -1;
+    int64_t sb = INT64_MAX;
+#pragma unroll
+    for (int j = 0; j < KR; j++) {
+        S[j] = lv[j] == 0 ? rq[j] : st[j] + plan_span(j, hd[j], lv[j]);
+        const bool take = act[j] & ((kb < 0) | (S[j] < sb));
+        kb = take ? j : kb;
+        sb = take ? S[j] : sb;
     }
-    const int total = __shfl_sync(FULL, x, K - 1);
-    int64_t last = 0;
-    if (in) {
-        L.breq[j] = rq;
-        L.bstart[j] = st;
-        L.bhead[j] = hd;
+    int total = 0;
+    int64_t mk = L.makespan;
+#pragma unroll
+    for (int j = 0; j < KR; j++) {
+        if (j >= K) break;
+        int c = 0;
+        if (act[j] && kb >= 0) {
+            PopGpu g;
+            g.req = rq[j];
+            g.start0 = st[j];
+            g.head = hd[j];
+            c = j == kb ? lv[j] : pops_before(j, g, lv[j], sb, kb);
+        }
+        L.breq[j] = rq[j];
+        L.bstart[j] = st[j];
+        L.bhead[j] = hd[j];
         L.bcnt[j] = c;
-        L.boff[j] = x - c;
+        L.boff[j] = total;
+        total += c;
         if (c > 0) {
-            last = st + plan_span(j, hd, c);
+            const int64_t last = st[j] + plan_span(j, hd[j], c);
             L.req[j] = last;  // W = 0 (R7)
             L.gpu_free[j] = last;
-            L.plan_head[j] = hd + c;
+            L.plan_head[j] = hd[j] + c;
             L.plan_live[j] -= c;
+            mk = last > mk ? last : mk;
         }
     }
-    const int64_t mkx = (int64_t)warp_max_u64((unsigned long long)last);
-    if (j == 0) {
-        L.boff[K] = total;
-        L.bns = L.n_served;
-        L.n_served += total;
-        if (mkx > L.makespan) L.makespan = mkx;
-        L.alg_bytes += 24ull * (uint64_t)total;
-        L.k = kb;
-        L.t = sb;
-        L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
+    L.boff[K] = total;
+    L.bns = L.n_served;
+    L.n_served += total;
+    L.makespan = mk;
+    L.alg_bytes += 24ull * (uint64_t)total;
+    L.k = kb;
+    L.t = sb;
+    L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
+}
+
+// The same for 8 < K <= 32, values left in shared memory.
+__device__ __noinline__ void pop_batch_scalar_smem() {
+    const Inst &I = SI;
+    const int K = I.K;
+    int kb = -1;
+    int64_t sb = INT64_MAX;
+    for (int j = 0; j < K; j++) {
+        const int64_t req = L.req[j];
+        const int64_t start0 = req > L.gpu_free[j] ? req : L.gpu_free[j];
+        const int head = L.plan_head[j];
+        L.breq[j] = req;
+        L.bstart[j] = start0;
+        L.bhead[j] = head;
+        if (L.idle[j]) continue;
+        const int live = L.plan_end[j] - head;
+        const int64_t S = live == 0 ? req : start0 + plan_span(j, head, live);
+        if (kb < 0 || S < sb) {
+            kb = j;
+            sb = S;
+        }
     }
+    int total = 0;
+    int64_t mk = L.makespan;
+    for (int j = 0; j < K; j++) {
+        int c = 0;
+        if (!L.idle[j] && kb >= 0) {
+            const int live = L.plan_end[j] - L.bhead[j];
+            PopGpu g;
+            g.req = L.breq[j];
+            g.start0 = L.bstart[j];
+            g.head = L.bhead[j];
+            c = j == kb ? live : pops_before(j, g, live, sb, kb);
+        }
+        L.bcnt[j] = c;
+        L.boff[j] = total;
+        total += c;
+        if (c > 0) {
+            const int64_t last = L.bstart[j] + plan_span(j, L.bhead[j], c);
+            L.req[j] = last;  // W = 0 (R7)
+            L.gpu_free[j] = last;
+            L.plan_head[j] += c;
+            L.plan_live[j] -= c;
+            mk = last > mk ? last : mk;
+        }
+    }
+    L.boff[K] = total;
+    L.bns = L.n_served;
+    L.n_served += total;
+    L.makespan = mk;
+    L.alg_bytes += 24ull * (uint64_t)total;
+    L.k = kb;
+    L.t = sb;
+    L.cmd = kb < 0 ? CMD_DONE : CMD_SCAN;
 }
 
 __device__ void pop_batch() {
@@ -790,7 +852,11 @@ __device__ void pop_batch() {
     const View &V = SV;
     const int K = I.K;
     PROF_T0(p_w0);
-    if (threadIdx.x < 32) pop_batch_warp();
+    if (threadIdx.x == 0) {
+        if (K <= 4) pop_batch_scalar<4>();
+        else if (K <= 8) pop_batch_scalar<8>();
+        else pop_batch_scalar_smem();
+    }
     cta_sync();
     PROF_ADD(L, P_BW0, p_w0);
     PROF_T0(p_bd);

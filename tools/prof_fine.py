@@ -2,7 +2,7 @@ import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import gen
 import paper_conf_ipps_gonthiermt22_b200 as dts
-NAMES = ["pop", "argmax", "plan", "serve_loads", "luf", "evict", "seg_load", "other", "bw0", "bd", "nb", "np", "x1", "x2", "plan_loop", "plan_tail"]
+NAMES = ["pop", "argmax", "plan", "serve_loads", "luf", "evict", "seg_load", "other", "bw0", "bd", "nb", "np", "x1", "x2", "x3", "x4"]
 for inst in [gen.config_instances("C2")[19], gen.config_instances("C2")[18], gen.config_instances("C3")[0]]:
     dts.schedule(inst)
     g = dts.schedule(inst)
