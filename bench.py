@@ -408,7 +408,7 @@ def main():
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": _traffic(args.workload),
-                         "kernel": "dts_loop_kernel", "peak_source": peak_src,
+                         "kernel": "dts_cta_kernel", "peak_source": peak_src,
                          "alg_bytes_per_launch": int(alg), "launch_ms": loop_ms},
             "hbm_gbs": achieved,
             "bytes_loaded": int(bytes_loaded), "n_loads": int(n_loads), "n_scans": int(n_scans),
