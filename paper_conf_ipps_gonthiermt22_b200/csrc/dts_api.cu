@@ -577,6 +577,7 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     h.ep_base = (unsigned long long)(++I->runs) << 32;
     h.box_bytes = I->box_bytes;
     h.xsys = I->xsys ? 1 : 0;
+    h.pop_batch_min = env_int("DTS_POP_BATCH_MIN", 10);
     // small instances: the loop CTA builds its own CSR and state (one launch)
     const int fs = fused_scratch_bytes(I, block);
     h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;

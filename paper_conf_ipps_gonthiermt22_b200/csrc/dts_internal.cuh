@@ -143,7 +143,7 @@ struct Inst {
     unsigned long long ep_base;  // exchange numbers of this run: ep_base + 1, 2, ...
     int64_t box_bytes;        // bytes of one payload slot
     int32_t xsys;             // 1: peers on other devices (system-scope release/acquire)
-    int32_t pad3;
+    int32_t pop_batch_min;    // serve pops in one batch when more than this many are planned
 };
 
 }  // namespace dts

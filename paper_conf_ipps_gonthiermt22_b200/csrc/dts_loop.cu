@@ -1979,7 +1979,7 @@ __global__ void __launch_bounds__(512, 1)
             if (I.policy == DTS_POLICY_DARTS_LUF) {
                 int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
                 for (int j = 0; j < K; j++) pending += L.plan_live[j];
-                if (I.max_served < 0 && I.W == 0 && K <= 32 && pending > 10) {
+                if (I.max_served < 0 && I.W == 0 && K <= 32 && pending > I.pop_batch_min) {
                     pop_batch();
                 } else {  // few pops (or a prefix run that stops at an exact count): thread 0
                     cta_sync();
