@@ -53,13 +53,30 @@ constexpr int POP_RANK_MAX = 256;  // pops ranked by counting in one pass
 
 enum Cmd : int { CMD_SCAN = 1, CMD_DONE = 2, CMD_POP = 3, CMD_EAGER = 4 };
 
-// Per-phase cycle accounting by thread 0 (diagnostics, dts_result_view.prof_cycles).
+// Per-phase cycle accounting by thread 0 (diagnostics, dts_result_view.prof_cycles),
+// compiled only into the profiling build (lib/libdts_prof.so, -DDTS_PROF): the
+// probes are thread-0 branches plus shared read-modify-writes on the critical
+// path, so the production library leaves them out (prof_cycles reads 0).
 enum Prof : int { P_POP = 0, P_ARGMAX, P_PLAN, P_LOADS, P_LUF, P_EVICT, P_SEG, P_OTHER, P_BW0, P_BD, P_NB, P_NP, P_X1, P_X2, P_X3, P_X4 };
+#ifdef DTS_PROF
 #define PROF_T0(var) const long long var = (threadIdx.x == 0) ? clock64() : 0
 #define PROF_ADD(L, slot, var) \
     do {                       \
         if (threadIdx.x == 0) (L).prof[slot] += clock64() - (var); \
     } while (0)
+#define PROF_CNT(L, slot, v) \
+    do {                     \
+        if (threadIdx.x == 0) (L).prof[slot] += (v); \
+    } while (0)
+#else
+#define PROF_T0(var)
+#define PROF_ADD(L, slot, var) \
+    do {                       \
+    } while (0)
+#define PROF_CNT(L, slot, v) \
+    do {                     \
+    } while (0)
+#endif
 
 struct Lead {  // leader scalars + broadcast slots (static shared memory)
     int64_t req[MAX_K];
@@ -523,7 +540,7 @@ __device__ int32_t pop_planned(int k, int64_t *tau) {
 // evicts, Alg. 6 l.8), so serving it is time-model arithmetic.
 // np_k is not maintained by pops: LUF on GPU k only runs while k serves the
 // first task of a new plan (or a fallback task), and every scan resets np_k.
-__device__ __noinline__ int pop_run_seq() {
+__device__ __forceinline__ int pop_run_seq() {
     const Inst &I = SI;
     const View &V = SV;
     const int K = I.K, W = I.W, pcap = I.plan_cap;
@@ -535,19 +552,28 @@ __device__ __noinline__ int pop_run_seq() {
     int64_t ns = L.n_served, mk = L.makespan, pops = 0;
     int ret = -1;
     while (maxs < 0 || ns < maxs) {
+        // the next request and the one after it: the two smallest (req_j, j)
+        // over the non-idle GPUs (R8); eight GPUs' words loaded before any
+        // compare, the compares branch-free (an idle GPU's key is INT64_MAX)
         int k = -1, k2 = -1;
-        int64_t t1 = 0, t2 = 0;
-        for (int j = 0; j < K; j++) {
-            if (L.idle[j]) continue;
-            const int64_t r = L.req[j];
-            if (k < 0 || r < t1) {
-                k2 = k;
-                t2 = t1;
-                k = j;
-                t1 = r;
-            } else if (k2 < 0 || r < t2) {
-                k2 = j;
-                t2 = r;
+        int64_t t1 = INT64_MAX, t2 = INT64_MAX;
+        for (int j0 = 0; j0 < K; j0 += 8) {
+            int64_t r[8];
+#pragma unroll
+            for (int q = 0; q < 8; q++) {
+                const int j = j0 + q;
+                r[q] = (j < K && !L.idle[j]) ? L.req[j] : INT64_MAX;
+            }
+#pragma unroll
+            for (int q = 0; q < 8; q++) {
+                const int j = j0 + q;
+                const bool ok = r[q] != INT64_MAX;
+                const bool b1 = ok & (r[q] < t1);
+                const bool b2 = ok & !b1 & (r[q] < t2);
+                k2 = b1 ? k : (b2 ? j : k2);
+                t2 = b1 ? t1 : (b2 ? r[q] : t2);
+                k = b1 ? j : k;
+                t1 = b1 ? r[q] : t1;
             }
         }
         if (k < 0) break;
@@ -862,10 +888,8 @@ __device__ void pop_batch() {
     PROF_T0(p_bd);
     const int P = L.boff[K];
     const int64_t ns = L.bns;
-    if (threadIdx.x == 0) {
-        L.prof[P_NB] += 1;
-        L.prof[P_NP] += P;
-    }
+    PROF_CNT(L, P_NB, 1);
+    PROF_CNT(L, P_NP, P);
     if (P <= (int)blockDim.x && P <= POP_RANK_MAX) {
         // merge ranks by counting: each pop's key (request time, GPU) in shared
         // memory, position = #keys before it (ties inside a GPU keep pop order)
@@ -1399,12 +1423,10 @@ __device__ __noinline__ void xch_sync() {
             }
         }
         __syncwarp();
-        if (threadIdx.x == 0) {
-            L.xe = L.xe + 1;
-            L.prof[P_X2] += 1;
-        }
+        if (threadIdx.x == 0) L.xe = L.xe + 1;
     }
     cta_sync();
+    PROF_CNT(L, P_X2, 1);
     PROF_ADD(L, P_X1, p_x);
 }
 

@@ -18,7 +18,10 @@ from typing import Optional
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "lib", "libdts.so")
+# DTS_PROFILE=1 loads the profiling build (per-phase cycle probes in
+# dts_result_view.prof_cycles); otherwise prof_cycles reads 0.
+LIB_PATH = os.path.join(_PKG, "lib", "libdts_prof.so" if os.environ.get("DTS_PROFILE") == "1"
+                        else "libdts.so")
 
 DTS_OK = 0
 DTS_E_INVAL = -1

@@ -1,6 +1,7 @@
 """Print the per-phase cycle split of the decision loop (dts_result_view.prof_cycles)
 for a few instances, plus loop time per decision.  Needs a B200."""
 import os
+os.environ.setdefault("DTS_PROFILE", "1")
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))

@@ -1,6 +1,7 @@
 """Exchange cost of the task-sharded single instance (dts_shard_group_run):
 loop time, exchanges, and thread-0 cycles inside xch_sync per exchange.  Needs a B200."""
 import os
+os.environ.setdefault("DTS_PROFILE", "1")
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
