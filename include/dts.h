@@ -80,7 +80,12 @@ enum {
     /* OPTI variant (§V-F): instead of the datum that frees
      * the most tasks, take the first one (ascending id) that frees at least
      * one.  Combines with DTS_F_FALLBACK2 ("DARTS+LUF+OPTI-3inputs"). */
-    DTS_F_OPTI = 1u << 3
+    DTS_F_OPTI = 1u << 3,
+    /* Diagnostic: keep the packed per-(simulated GPU, task) state word
+     * (cnt:7 | xor:24, 4 K m bytes) even when every task has <= 3 inputs
+     * (default then: no per-GPU task state, the missing inputs are read off
+     * the task's row and the residency bitmaps). */
+    DTS_F_PACKED = 1u << 4
 };
 
 typedef struct {

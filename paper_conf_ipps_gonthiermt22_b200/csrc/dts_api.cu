@@ -338,6 +338,7 @@ dts_status ensure_device(dts_instance *I, int device) {
     add(4 * K * (nstr + 4)); add(4 * K * nw); add(4 * K * res_cap);                  // np resb res_list
     add(16 * K * plan_cap); add(8 * K * plan_cap); add(4 * (3 * n + 1));              // plan tau vhist
     add(4 * K * (nstr + 4));                                                          // lru stamps
+    add(4 * (mp / 32 + 2));                                                           // alloc bitmap
     add(sizeof(dts::Out));
     add(4 * (m + 1)); add(4 * (m + 1)); add(8 * (m + 1)); add(8 * (m + 1));          // serve, times
     add(sizeof(dts_event) * ev_cap); add(8 * (K + 1)); add(4 * (m + 1));
@@ -406,6 +407,7 @@ dts_status ensure_device(dts_instance *I, int device) {
     h.plan_tau = A.take<int64_t>(K * plan_cap);
     h.vhist = A.take<int32_t>(3 * n + 1);
     h.lru = A.take<int32_t>(K * (nstr + 4));
+    h.al = A.take<uint32_t>(mp / 32 + 2);
     h.out = A.take<dts::Out>(1);
     h.serve_gpu = A.take<int32_t>(m + 1);
     h.serve_task = A.take<int32_t>(m + 1);
@@ -467,7 +469,7 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
 dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_opts *o) {
     if (policy != DTS_POLICY_DARTS_LUF && policy != DTS_POLICY_DARTS_LRU && policy != DTS_POLICY_EAGER_LRU)
         return fail(DTS_E_UNSUPPORTED, "policy");
-    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI))
+    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI | DTS_F_PACKED))
         return fail(DTS_E_UNSUPPORTED, "unknown flags");
     if (o->lookahead_W > 1) return fail(DTS_E_UNSUPPORTED, "lookahead_W > 1");
     if (o->bus_bytes_per_s == 0) return fail(DTS_E_INVAL, "bus_bytes_per_s == 0");
@@ -483,7 +485,7 @@ dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_op
 // Shared-memory placement of one instance's state:
 // greedy, most latency-critical array first, each either fully in the CTA's
 // dynamic shared memory or in its global home.  Returns the bytes used.
-int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard) {
+int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard, bool sl) {
     const int64_t K = h.K, n = h.n;
     int used = 0;
     auto put = [&](int32_t &so, int64_t bytes) {
@@ -497,6 +499,8 @@ int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard) {
         }
     };
     put(h.so_resb, 4 * K * h.nw);
+    if (sl) put(h.so_al, 4 * (int64_t)(h.m_pad / 32 + 1));  // read by every segment walk
+    else h.so_al = -1;
     put(h.so_dptr, 4 * (n + 1));
     put(h.so_plan, 16 * K * h.plan_cap);
     if (has_tau) put(h.so_plan_tau, 8 * K * h.plan_cap);
@@ -508,7 +512,8 @@ int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard) {
     put(h.so_np, 4 * K * (int64_t)h.nstr);
     if (lru) put(h.so_lru, 4 * K * (int64_t)h.nstr);
     else h.so_lru = -1;
-    put(h.so_s, 4 * K * (int64_t)h.m_pad);  // last: the largest, worth it only when it fits
+    if (!sl) put(h.so_s, 4 * K * (int64_t)h.m_pad);  // last: the largest, worth it only when it fits
+    else h.so_s = -1;
     h.smem_bytes = used;
     return used;
 }
@@ -568,7 +573,9 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
         const unsigned __int128 num = (unsigned __int128)h.size0 * 1000000000u + (o.bus_bytes_per_s - 1);
         h.delta0 = (int64_t)(num / o.bus_bytes_per_s);  // ceil, reading R9 (same as dts_init_kernel)
     }
-    place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF, I->G > 1);
+    // row-derived state (no per-(GPU, task) words) when every edge record holds its row
+    h.sl = I->G == 1 && I->max_row_len <= 3 && !(o.flags & DTS_F_PACKED) ? 1 : 0;
+    place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF, I->G > 1, h.sl != 0);
     h.G = I->G;
     h.g = I->g;
     h.t_lo = I->G > 1 ? I->t_lo : 0;
@@ -688,7 +695,9 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     int nsm = 0;
     CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
     int budget = budget_of(o);
-    if (o.smem_budget == 0 && n >= 2 * nsm) budget = std::min(budget, (max_dyn_smem(o.device) + 1024) / 4 - 4096);
+    const int smem_div = std::max(1, env_int("DTS_SWEEP_SMEM_DIV", 4));
+    if (o.smem_budget == 0 && n >= 2 * nsm)
+        budget = std::min(budget, (max_dyn_smem(o.device) + 1024) / smem_div - 4096);
     int smem = 0;
     bool any_unfused = false;
     for (int32_t i = 0; i < n; i++) {

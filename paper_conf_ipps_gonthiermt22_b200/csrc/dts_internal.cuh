@@ -14,6 +14,12 @@
 //       bits 24..30 : cnt_k(T) = |D(T) \ R_k|   (<= 127)
 //       bits  0..23 : x_k(T)   = XOR of the ids in D(T) \ R_k   (n < 2^24)
 //     so a task with cnt 1 NAMES its one missing datum: x_k(T).
+//   al[m_pad/32 + 1] uint32 -- allocation bitmap (bit set: T left the shared
+//       pool, R2; pad bits set).  The "row-derived" state mode (Inst::sl,
+//       every row <= 3 inputs, one shard): s is not kept at all -- cnt_k(T) and
+//       the missing ids are read off T's row (edge record / plan entry) and the
+//       residency bitmap, so the per-(GPU, task) state shrinks from 4 K m bytes
+//       to m / 8 and fits in shared memory for every config        [S/G]
 //   h[K][nstr] int32 -- n_k(D)  = #unallocated T with cnt_k(T)=1, x_k(T)=D: the
 //       DARTS score of Alg. 5 l.4-5, kept incrementally [S/G]
 //   h2[K][nstr] int32 -- n2_k(D) = #unallocated T with cnt_k(T)=2, D missing:
@@ -144,6 +150,10 @@ struct Inst {
     int64_t box_bytes;        // bytes of one payload slot
     int32_t xsys;             // 1: peers on other devices (system-scope release/acquire)
     int32_t pop_batch_min;    // serve pops in one batch when more than this many are planned
+    // row-derived state mode (sl = 1): no s; allocation bitmap al instead
+    int32_t sl;
+    int32_t so_al;            // shared-memory offset of al, -1 = global home
+    uint32_t *al;             // [m_pad / 32 + 1] global home
 };
 
 }  // namespace dts

@@ -126,6 +126,7 @@ struct View {
     int64_t *plan_cum;  // inclusive prefix sums of the planned tasks' tau (per-task times only)
     int32_t *dptr32;    // shared-memory copy of dptr, or nullptr
     int32_t *lru;       // [K][nstr] last-use stamps (LRU policies)
+    uint32_t *al;       // row-derived mode: allocation bitmap (bit set = left the pool)
 };
 
 // Per-CTA state at namespace scope, so the (non-inlined) phase functions
@@ -203,6 +204,21 @@ __device__ __forceinline__ bool resident(int k, int32_t D) {
     const Inst &I = SI;
     const View &V = SV;
     return (V.resb[(size_t)k * I.nw + (D >> 5)] >> (D & 31)) & 1u;
+}
+
+// Row-derived mode (Inst::sl): T has left the shared pool (R2).
+__device__ __forceinline__ bool allocated(int32_t T) { return (SV.al[T >> 5] >> (T & 31)) & 1u; }
+__device__ __forceinline__ void set_alloc(int32_t T, int sign) {
+    if (sign < 0) atomicOr(&SV.al[T >> 5], 1u << (T & 31));
+    else atomicAnd(&SV.al[T >> 5], ~(1u << (T & 31)));
+}
+// Row-derived mode: the inputs of a <= 3-input row {a, b, c} (-1 = absent)
+// not resident on GPU k -- their count cnt_k(T) and the first two of them.
+__device__ __forceinline__ int missing_of(int k, int32_t a, int32_t b, int32_t c, int32_t &m0, int32_t &m1) {
+    const bool ma = a >= 0 && !resident(k, a), mb = b >= 0 && !resident(k, b), mc = c >= 0 && !resident(k, c);
+    m0 = ma ? a : (mb ? b : c);
+    m1 = ma ? (mb ? b : c) : c;
+    return (int)ma + (int)mb + (int)mc;
 }
 
 // Data->task segment bounds of D (int32 copy in shared memory when placed).
@@ -299,7 +315,21 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
     const View &V = SV;
     const int K = I.K;
     const bool own = T >= I.t_lo && T < I.t_hi;
-    for (int j0 = 0; own && j0 < K; j0 += 4) {
+    if (I.sl) {  // row-derived state: the allocation bit, then each GPU's buckets
+        set_alloc(T, sign);
+#pragma unroll 1
+        for (int j = 0; j < K; j++) {
+            int32_t a, b;
+            const int c = missing_of(j, r.r0, r.r1, r.r2, a, b);
+            if (c == 1) {
+                atomicAdd(&V.h[(size_t)j * I.nstr + a], sign);
+            } else if (c == 2) {
+                atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+                atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
+            }
+        }
+    }
+    for (int j0 = 0; own && !I.sl && j0 < K; j0 += 4) {
         uint32_t w0 = 0, w1 = 0, w2 = 0, w3 = 0;
         w0 = V.s[(size_t)j0 * I.m_pad + T];
         if (j0 + 1 < K) w1 = V.s[(size_t)(j0 + 1) * I.m_pad + T];
@@ -351,6 +381,17 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
             const int p = idx / K, j = idx - p * K;
             const int4 e = ents[p];
             const int32_t T = e.x;
+            if (I.sl) {  // row-derived state: T's missing inputs on GPU j from its row
+                int32_t a, b;
+                const int c = missing_of(j, e.y, e.z, e.w, a, b);
+                if (c == 1) {
+                    atomicAdd(&V.h[(size_t)j * I.nstr + a], sign);
+                } else if (c == 2) {
+                    atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+                    atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
+                }
+                continue;
+            }
             if (T < I.t_lo || T >= I.t_hi) continue;  // another shard's task
             uint32_t *sp = &V.s[(size_t)j * I.m_pad + T];
             const uint32_t w = *sp;
@@ -375,6 +416,7 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
             const int4 e = ents[idx - n_state];
             const int32_t T = e.x;
             const bool own = T >= I.t_lo && T < I.t_hi;
+            if (I.sl) set_alloc(T, sign);
             if (e.w == ROW_LONG) {
                 pool_move_long_row(T, sign, plan_k, own);
                 continue;
@@ -416,6 +458,39 @@ __device__ void seg_update(int k, int32_t D, bool load) {
     uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int32_t *hk = V.h + (size_t)k * I.nstr;
     int32_t *h2k = V.h2 + (size_t)k * I.nstr;
+    if (I.sl) {  // row-derived state: cnt_k(T) before the change from T's other inputs
+        for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
+            const int4 ed = __ldg(&I.dedge[i]);
+            if (allocated(ed.x)) continue;
+            const bool my = ed.y >= 0 && !resident(k, ed.y), mz = ed.z >= 0 && !resident(k, ed.z);
+            const int c = (int)my + (int)mz + (load ? 1 : 0);  // missing inputs before
+            const int32_t o = my ? ed.y : ed.z;                 // the other missing one (c == 2 / 1)
+            if (load) {
+                if (c == 1) {  // 1 -> 0
+                    atomicSub(&hk[D], 1);
+                } else if (c == 2) {  // 2 -> 1: now freed by o
+                    atomicSub(&h2k[D], 1);
+                    atomicSub(&h2k[o], 1);
+                    atomicAdd(&hk[o], 1);
+                } else if (c == 3) {  // 3 -> 2
+                    atomicAdd(&h2k[ed.y], 1);
+                    atomicAdd(&h2k[ed.z], 1);
+                }
+            } else {
+                if (c == 0) {  // 0 -> 1
+                    atomicAdd(&hk[D], 1);
+                } else if (c == 1) {  // 1 -> 2: missing {o, D}
+                    atomicSub(&hk[o], 1);
+                    atomicAdd(&h2k[o], 1);
+                    atomicAdd(&h2k[D], 1);
+                } else if (c == 2) {  // 2 -> 3
+                    atomicSub(&h2k[ed.y], 1);
+                    atomicSub(&h2k[ed.z], 1);
+                }
+            }
+        }
+        return;
+    }
     for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
         const int4 ed = __ldg(&I.dedge[i]);
         const int32_t T = ed.x;
@@ -1278,7 +1353,8 @@ __device__ void plan(int k, int32_t Dopt) {
         if (i < e) {
             ed = __ldg(&I.dedge[i]);
             T = ed.x;
-            sel = (sk[T] >> 24) == 1u;
+            sel = I.sl ? !allocated(T) && (ed.y < 0 || resident(k, ed.y)) && (ed.z < 0 || resident(k, ed.z))
+                       : (sk[T] >> 24) == 1u;
         }
         const unsigned msk = __ballot_sync(FULL, sel);
         if (lane == 0) L.wcnt[w] = __popc(msk);
@@ -1326,8 +1402,14 @@ __device__ __noinline__ int32_t first_cnt2(int k, int32_t D2) {
         const int64_t i = base + threadIdx.x;
         unsigned long long c = ~0ull;
         if (i < e) {
-            const int32_t T = __ldg(&I.dedge[i]).x;
-            if ((sk[T] >> 24) == 2u) c = (unsigned long long)T;
+            if (I.sl) {  // D2 misses (n2(D2) > 0): exactly one other input misses
+                const int4 ed = __ldg(&I.dedge[i]);
+                const int mo = (int)(ed.y >= 0 && !resident(k, ed.y)) + (int)(ed.z >= 0 && !resident(k, ed.z));
+                if (!allocated(ed.x) && mo == 1) c = (unsigned long long)ed.x;
+            } else {
+                const int32_t T = __ldg(&I.dedge[i]).x;
+                if ((sk[T] >> 24) == 2u) c = (unsigned long long)T;
+            }
         }
         c = block_min_u64(c);
         if (c != ~0ull) return (int32_t)c;
@@ -1340,6 +1422,22 @@ __device__ __noinline__ int32_t first_cnt2(int k, int32_t D2) {
 __device__ __noinline__ int32_t first_avail() {
     const Inst &I = SI;
     const View &V = SV;
+    if (I.sl) {  // the allocation bitmap, a word per thread (bits past m are set)
+        const int lo = L.avail_lo;
+        const int nwd = (I.m + 31) >> 5;
+        for (int w0 = lo >> 5; w0 < nwd; w0 += blockDim.x) {
+            const int wd = w0 + threadIdx.x;
+            unsigned long long c = ~0ull;
+            if (wd < nwd) {
+                uint32_t free_bits = ~V.al[wd];
+                if (wd == (lo >> 5)) free_bits &= ~((1u << (lo & 31)) - 1u);
+                if (free_bits) c = (unsigned long long)(32 * wd + __ffs(free_bits) - 1);
+            }
+            c = block_min_u64(c);
+            if (c != ~0ull) return (int32_t)c;
+        }
+        return -1;
+    }
     for (int64_t base = L.avail_lo > I.t_lo ? L.avail_lo : I.t_lo; base < I.t_hi; base += blockDim.x) {
         const int64_t T = base + threadIdx.x;
         unsigned long long c = ~0ull;
@@ -1634,7 +1732,7 @@ __device__ __noinline__ void verify_scores(int k) {
     const uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int bad = 0;
     for (int T = I.t_lo + threadIdx.x; T < I.t_hi; T += blockDim.x) {  // owned tasks
-        const uint32_t w = sk[T];
+        const uint32_t w = I.sl ? 0u : sk[T];
         const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
         int c = 0;
         uint32_t x = 0;
@@ -1642,8 +1740,12 @@ __device__ __noinline__ void verify_scores(int k) {
             const int32_t D = __ldg(&I.tdat[i]);
             if (!resident(k, D)) c++, x ^= (uint32_t)D;
         }
-        bad += (c != (int)((w >> 24) & 0x7fu)) || (x != (w & XOR_MASK));
-        if (w & ALLOC_BIT) continue;
+        if (I.sl) {
+            if (allocated(T)) continue;
+        } else {
+            bad += (c != (int)((w >> 24) & 0x7fu)) || (x != (w & XOR_MASK));
+            if (w & ALLOC_BIT) continue;
+        }
         for (int64_t i = rb; i < re; i++) {
             const int32_t D = __ldg(&I.tdat[i]);
             atomicAdd(&vu[D], 1);
@@ -1878,8 +1980,14 @@ __device__ __noinline__ void fused_init() {
             I.tstart[T] = -1;
             I.tend[T] = -1;
         }
-        for (int k = 0; k < K; k++) V.s[(size_t)k * I.m_pad + T] = w;
+        if (!I.sl)
+            for (int k = 0; k < K; k++) V.s[(size_t)k * I.m_pad + T] = w;
     }
+    if (I.sl)  // nothing allocated; bits past m set
+        for (int wd = threadIdx.x; wd <= I.m_pad / 32; wd += blockDim.x) {
+            const int t0 = 32 * wd;
+            V.al[wd] = t0 >= m ? ~0u : (m - t0 >= 32 ? 0u : ~((1u << (m - t0)) - 1u));
+        }
     for (int D = threadIdx.x; D < I.nstr; D += blockDim.x) {
         int32_t c1 = 0, c2 = 0, dg = 0;
         if (D < n) {
@@ -1938,6 +2046,7 @@ __global__ void __launch_bounds__(512, 1)
             W.plan_cum = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
             W.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
             W.lru = I.so_lru >= 0 ? (int32_t *)(dsm + I.so_lru) : I.lru;
+            W.al = I.so_al >= 0 ? (uint32_t *)(dsm + I.so_al) : I.al;
         }
         cta_sync();
         const View &V = SV;
@@ -1958,6 +2067,8 @@ __global__ void __launch_bounds__(512, 1)
             uint4 *dst = reinterpret_cast<uint4 *>(V.s);
             for (int i = tid; i < (K * I.m_pad) / 4; i += blockDim.x) dst[i] = __ldcg(&src[i]);
         }
+        if (I.sl && I.so_al >= 0)
+            for (int i = tid; i <= I.m_pad / 32; i += blockDim.x) V.al[i] = __ldcg(&I.al[i]);
         if (I.so_u >= 0)
             for (int D = tid; D < I.nstr; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
         if (I.so_h >= 0)
@@ -2198,8 +2309,14 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
                 I.tstart[T] = -1;
                 I.tend[T] = -1;
             }
-            for (int k = 0; k < I.K; k++) I.s[(size_t)k * I.m_pad + T] = w;
+            if (!I.sl)
+                for (int k = 0; k < I.K; k++) I.s[(size_t)k * I.m_pad + T] = w;
         }
+        if (I.sl)  // allocation bitmap: nothing allocated, bits past m set
+            for (int64_t wd = tid; wd <= I.m_pad / 32; wd += str) {
+                const int64_t t0 = 32 * wd;
+                I.al[wd] = t0 >= I.m ? ~0u : (I.m - t0 >= 32 ? 0u : ~((1u << (I.m - t0)) - 1u));
+            }
         for (int64_t D = I.n + tid; D < I.nstr; D += str) {  // row padding: never scores
             I.u[D] = 0;
             for (int k = 0; k < I.K; k++) {

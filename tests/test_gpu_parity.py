@@ -168,6 +168,53 @@ def test_long_rows():
         assert_parity(g, oracle.run(inst, bus_bps=10 ** 9))
 
 
+# ------------------------------------------------------------ state modes
+# Rows of <= 3 inputs run in the row-derived state mode by default (no
+# per-(GPU, task) words: missing inputs read off the row and the residency
+# bitmaps); DTS_F_PACKED keeps the packed cnt:7|xor:24 words.  Both must give
+# the oracle's schedule.
+PACKED = dts.DTS_F_FALLBACK2 | dts.DTS_F_PACKED
+
+
+@pytest.mark.parametrize("idx", range(12))
+@pytest.mark.parametrize("smem", [0, -1])
+def test_packed_state_mode_shapes(idx, smem):
+    inst = _shapes()[idx]
+    g = dts.schedule(inst, flags=PACKED | dts.DTS_F_VERIFY, smem_budget=smem)
+    assert g.n_verify_err == 0
+    assert_parity(g, oracle.run(inst))
+
+
+@pytest.mark.parametrize("name", ["darts_luf", "darts_lru", "eager_lru"])
+@pytest.mark.parametrize("W", [0, 1])
+def test_packed_state_mode_policies(name, W):
+    pol, of = {"darts_luf": (dts.DTS_POLICY_DARTS_LUF, 0),
+               "darts_lru": (dts.DTS_POLICY_DARTS_LRU, oracle.F_LRU),
+               "eager_lru": (dts.DTS_POLICY_EAGER_LRU, oracle.F_EAGER | oracle.F_LRU)}[name]
+    for inst in (_shapes()[5], _shapes()[9]):
+        o = oracle.run(inst, W=W, flags=oracle.F_FALLBACK2 | of)
+        assert_parity(dts.schedule(inst, policy=pol, W=W, flags=PACKED), o)
+        assert_parity(dts.schedule(inst, policy=pol, W=W), o)  # row-derived
+
+
+def test_packed_state_mode_config3_and_4_prefix():
+    inst = gen.config_instances("C3")[0]
+    assert_parity(dts.schedule(inst, flags=PACKED), oracle.run(inst))
+    for cfg in ("C4a", "C4b"):
+        inst = gen.config_instances(cfg)[0]
+        g = dts.schedule(inst, flags=PACKED, max_served=800)
+        assert_parity(g, oracle.run(inst, max_served=800), complete=False)
+
+
+def test_row_derived_verify_partial_placement():
+    """P9 in the row-derived mode with the allocation bitmap in HBM / partly placed."""
+    for inst in (_shapes()[8], _shapes()[10]):
+        for smem in (-1, 2000, 0):
+            g = dts.schedule(inst, flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_VERIFY, smem_budget=smem)
+            assert g.n_verify_err == 0
+            assert_parity(g, oracle.run(inst))
+
+
 # ------------------------------------------------------------ larger configs
 def test_config3():
     inst = gen.config_instances("C3")[0]
