@@ -398,7 +398,9 @@ def main():
                        "policy": args.policy + ("+opti" if args.opti else "") + " (3inputs fallback on)",
                        "instances_per_rank": len(insts), "decisions_per_step": int(all_dec),
                        "l2": "flushed between timed steps (256 MiB write)",
-                       "launch": "one batched loop launch, one CTA per instance" if not single
+                       "launch": ("one batched loop launch, one CTA per instance" if len(insts) < 296 else
+                                  "two concurrent batched loop launches (256-thread CTAs for the long-segment "
+                                  "instances, <= 128 for the rest), one CTA per instance") if not single
                        else (f"one cooperative launch: the instance task-sharded over {args.shards} CTAs"
                              if gsh else f"one loop launch per rank: the instance task-sharded over "
                              f"{world} B200s, peer-memory exchanges" if xsh

@@ -514,6 +514,8 @@ int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard, boo
     else h.so_lru = -1;
     if (!sl) put(h.so_s, 4 * K * (int64_t)h.m_pad);  // last: the largest, worth it only when it fits
     else h.so_s = -1;
+    if (sl && h.ce_bytes > 0) put(h.so_ce, (int64_t)h.ce_bytes * h.E);  // edge records, when all else fits
+    else h.so_ce = -1;
     h.smem_bytes = used;
     return used;
 }
@@ -575,6 +577,15 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     }
     // row-derived state (no per-(GPU, task) words) when every edge record holds its row
     h.sl = I->G == 1 && I->max_row_len <= 3 && !(o.flags & DTS_F_PACKED) ? 1 : 0;
+    {  // compact edge records: T, then the (<= 2) other inputs, value n = absent
+        const int tb = bits_for(I->m > 0 ? (uint64_t)(I->m - 1) : 0), db = bits_for((uint64_t)I->n);
+        const int one = I->max_row_len <= 2 ? 1 : 0;
+        const int need = tb + (one ? 1 : 2) * db;
+        h.ce_tb = tb;
+        h.ce_db = db;
+        h.ce_one = one;
+        h.ce_bytes = !h.sl ? 0 : (need <= 32 ? 4 : (need <= 64 ? 8 : 0));
+    }
     place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF, I->G > 1, h.sl != 0);
     h.G = I->G;
     h.g = I->g;
@@ -585,6 +596,7 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     h.box_bytes = I->box_bytes;
     h.xsys = I->xsys ? 1 : 0;
     h.pop_batch_min = env_int("DTS_POP_BATCH_MIN", 10);
+    h.poison = env_int("DTS_POISON", 0);
     // small instances: the loop CTA builds its own CSR and state (one launch)
     const int fs = fused_scratch_bytes(I, block);
     h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
@@ -619,8 +631,10 @@ struct SweepBuf {
     dts::Inst *h_insts[RING] = {};       // pinned staging ring: the host never waits on
     cudaEvent_t copied[RING] = {};       // the GPU unless it is RING sweeps behind
     int slot = 0;
-    int *d_work = nullptr;
+    int *d_work = nullptr;               // [0]: group A's instance counter, [1]: group B's
     size_t cap = 0;
+    cudaStream_t side = nullptr;         // group B of a split batch (forked from / joined into the caller's stream)
+    cudaEvent_t fork = nullptr, join = nullptr;
 };
 SweepBuf g_sweep[64];
 
@@ -673,7 +687,6 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     else dts_run_opts_default(&o);
     dts_status s = check_device(o.device);
     if (s != DTS_OK) return s;
-    int block = 32;
     int64_t work = 1;
     std::vector<dts_instance *> seen(insts, insts + n);
     std::sort(seen.begin(), seen.end());
@@ -683,32 +696,59 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
         if (!insts[i]) return fail(DTS_E_INVAL, "instance is NULL");
         s = check_opts(insts[i], policy, &o);
         if (s != DTS_OK) return s;
-        block = std::max(block, auto_block(insts[i]));
         work = std::max<int64_t>(work, std::max<int64_t>(insts[i]->m_pad, (int64_t)insts[i]->n * insts[i]->K));
     }
-    if (o.block_threads) block = o.block_threads;
-    else block = env_int("DTS_BLOCK", block);
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
     // Each instance is a latency-bound chain: with many more instances than
     // SMs, run several CTAs per SM (their chains interleave) by default --
-    // a quarter of the shared memory each; few instances get all of it.
+    // a share of the shared memory each; few instances get all of it.
     int nsm = 0;
     CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
+    const bool many = n >= 2 * nsm;
     int budget = budget_of(o);
-    const int smem_div = std::max(1, env_int("DTS_SWEEP_SMEM_DIV", 4));
-    if (o.smem_budget == 0 && n >= 2 * nsm)
-        budget = std::min(budget, (max_dyn_smem(o.device) + 1024) / smem_div - 4096);
-    int smem = 0;
+    const int smem_div = std::max(1, env_int("DTS_SWEEP_SMEM_DIV", 6));
+    if (o.smem_budget == 0 && many) budget = std::min(budget, (max_dyn_smem(o.device) + 1024) / smem_div - 4096);
+    // longest first (cost ~ m * mean degree), so the device counter hands the
+    // long chains out early and the tail of the batch stays short
+    std::vector<int32_t> ord((size_t)n);
+    for (int32_t i = 0; i < n; i++) ord[(size_t)i] = i;
+    auto cost = [&](int32_t i) { return (double)insts[i]->m * (double)insts[i]->E_raw / std::max(1, insts[i]->n); };
+    std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return cost(a) > cost(b); });
+    // CTA size per group: a batch of many instances runs as two concurrent
+    // launches -- the instances whose segments want wide CTAs (auto_block >=
+    // 256) with those, the rest with small CTAs so more chains share an SM.
+    // Few instances, or a forced size: one launch.
+    const int forced = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", 0);
+    const int small_max = env_int("DTS_SWEEP_SMALL_BLOCK", 128);
+    int nb = n, block_a = 32, block_b = 32;  // group A = ord[0, nb), group B = ord[nb, n)
+    if (!forced && many && small_max > 0) {
+        nb = 0;
+        for (int32_t i = 0; i < n; i++)
+            if (auto_block(insts[ord[(size_t)i]]) > small_max) nb = i + 1;  // the long ones come first
+        // group B: every instance after the last wide one (cost order ~ width order)
+    }
+    for (int32_t i = 0; i < n; i++) {
+        const int ab = auto_block(insts[ord[(size_t)i]]);
+        if (i < nb) block_a = std::max(block_a, ab);
+        else block_b = std::max(block_b, std::min(ab, small_max));
+    }
+    if (forced) block_a = block_b = forced;
+    int smem_a = 0, smem_b = 0;
     bool any_unfused = false;
     for (int32_t i = 0; i < n; i++) {
-        s = stage(insts[i], policy, o, budget, block, st, false);
+        dts_instance *I = insts[ord[(size_t)i]];
+        s = stage(I, policy, o, budget, i < nb ? block_a : block_b, st, false);
         if (s != DTS_OK) return s;
-        smem = std::max(smem, insts[i]->h_inst.smem_bytes);
-        any_unfused |= !insts[i]->h_inst.fused;
+        (i < nb ? smem_a : smem_b) = std::max(i < nb ? smem_a : smem_b, I->h_inst.smem_bytes);
+        any_unfused |= !I->h_inst.fused;
     }
     SweepBuf &B = g_sweep[o.device];
-    if (!B.copied[0])
+    if (!B.copied[0]) {
         for (auto &e : B.copied) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
+        CK(cudaEventCreateWithFlags(&B.fork, cudaEventDisableTiming), "cudaEventCreate");
+        CK(cudaEventCreateWithFlags(&B.join, cudaEventDisableTiming), "cudaEventCreate");
+        CK(cudaStreamCreateWithFlags(&B.side, cudaStreamNonBlocking), "cudaStreamCreate");
+    }
     if (B.cap < (size_t)n) {
         CK(cudaDeviceSynchronize(), "sync");
         if (B.d_insts) cudaFree(B.d_insts);
@@ -723,22 +763,29 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     const int sl = B.slot;
     B.slot = (B.slot + 1) % SweepBuf::RING;
     CK(cudaEventSynchronize(B.copied[sl]), "sweep event");
-    // longest first (cost ~ m * mean degree), so the device counter hands the
-    // long chains out early and the tail of the batch stays short
-    std::vector<int32_t> ord((size_t)n);
-    for (int32_t i = 0; i < n; i++) ord[(size_t)i] = i;
-    auto cost = [&](int32_t i) { return (double)insts[i]->m * (double)insts[i]->E_raw / std::max(1, insts[i]->n); };
-    std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return cost(a) > cost(b); });
     for (int32_t i = 0; i < n; i++) B.h_insts[sl][i] = insts[ord[(size_t)i]]->h_inst;
     CK(cudaMemcpyAsync(B.d_insts, B.h_insts[sl], sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
        "H2D sweep");
     CK(cudaEventRecord(B.copied[sl], st), "event");
-    CK(cudaMemsetAsync(B.d_work, 0, sizeof(int), st), "memset");
+    CK(cudaMemsetAsync(B.d_work, 0, 2 * sizeof(int), st), "memset");
     if (any_unfused) CK(dts::launch_init(B.d_insts, n, o.bus_bytes_per_s, work, st), "init");
-    const int per = std::max(1, dts::loop_max_blocks_per_sm(block, smem));
-    const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
     for (int32_t i = 0; i < n; i++) CK(cudaEventRecord(insts[i]->ev[1], st), "event");
-    CK(dts::launch_loop(B.d_insts, n, block, grid, B.d_work, smem, st), "loop");
+    const bool two = nb > 0 && nb < n;
+    if (two) {  // group B on the side stream, forked from and joined back into st
+        CK(cudaEventRecord(B.fork, st), "event");
+        CK(cudaStreamWaitEvent(B.side, B.fork, 0), "wait");
+        const int per_b = std::max(1, dts::loop_max_blocks_per_sm(block_b, smem_b));
+        const int grid_b = (int)std::min<int64_t>((int64_t)(n - nb), (int64_t)per_b * nsm);
+        CK(dts::launch_loop(B.d_insts + nb, n - nb, block_b, grid_b, B.d_work + 1, smem_b, B.side), "loop B");
+        CK(cudaEventRecord(B.join, B.side), "event");
+    }
+    const int na = two ? nb : n;
+    const int blk = two ? block_a : std::max(block_a, block_b);
+    const int sm = two ? smem_a : std::max(smem_a, smem_b);
+    const int per = std::max(1, dts::loop_max_blocks_per_sm(blk, sm));
+    const int grid = (int)std::min<int64_t>((int64_t)na, (int64_t)per * nsm);
+    CK(dts::launch_loop(B.d_insts, na, blk, grid, B.d_work, sm, st), "loop");
+    if (two) CK(cudaStreamWaitEvent(st, B.join, 0), "wait");
     for (int32_t i = 0; i < n; i++) {
         CK(cudaEventRecord(insts[i]->ev[2], st), "event");
         CK(cudaEventRecord(insts[i]->ev[3], st), "event");

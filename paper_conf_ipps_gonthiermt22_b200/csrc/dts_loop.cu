@@ -44,6 +44,10 @@ constexpr unsigned FULL = 0xffffffffu;
 // warp split after a thread-0-only block (independent thread scheduling), and
 // the split halves then run every later instruction twice and meet again at
 // each full-mask shuffle -- a measured 4x slowdown of the warp-0 phases.
+// Every value a thread reads to choose a path must be final before the
+// barrier that precedes the read and stay unchanged until the next barrier
+// (see pop_batch: a violation shows up as divergent barriers in
+// compute-sanitizer synccheck).
 __device__ __forceinline__ void cta_sync() {
     __syncthreads();
     __syncwarp();
@@ -127,6 +131,8 @@ struct View {
     int32_t *dptr32;    // shared-memory copy of dptr, or nullptr
     int32_t *lru;       // [K][nstr] last-use stamps (LRU policies)
     uint32_t *al;       // row-derived mode: allocation bitmap (bit set = left the pool)
+    uint32_t *ce4;      // row-derived mode: 4-byte compact edge records (shared), or
+    unsigned long long *ce8;  // 8-byte ones, or neither (edge records from dedge)
 };
 
 // Per-CTA state at namespace scope, so the (non-inlined) phase functions
@@ -219,6 +225,24 @@ __device__ __forceinline__ int missing_of(int k, int32_t a, int32_t b, int32_t c
     m0 = ma ? a : (mb ? b : c);
     m1 = ma ? (mb ? b : c) : c;
     return (int)ma + (int)mb + (int)mc;
+}
+
+// Edge record i of the data->task CSR as {T, o1, o2, -} (row-derived mode:
+// rows <= 3, the 4th field unused): decoded from the compact shared-memory
+// copy when placed, else the 16-byte record from global memory.
+__device__ __forceinline__ int4 edge_at(int64_t i) {
+    const Inst &I = SI;
+    const View &V = SV;
+    if (V.ce4 || V.ce8) {
+        const unsigned long long v = V.ce4 ? (unsigned long long)V.ce4[i] : V.ce8[i];
+        const unsigned tb = (unsigned)I.ce_tb, db = (unsigned)I.ce_db;
+        const unsigned long long dm = (1ull << db) - 1ull;
+        const int32_t T = (int32_t)(v & ((1ull << tb) - 1ull));
+        const int32_t y = (int32_t)((v >> tb) & dm);
+        const int32_t z = I.ce_one ? I.n : (int32_t)((v >> (tb + db)) & dm);
+        return make_int4(T, y == I.n ? -1 : y, z == I.n ? -1 : z, 0);
+    }
+    return __ldg(&I.dedge[i]);
 }
 
 // Data->task segment bounds of D (int32 copy in shared memory when placed).
@@ -460,7 +484,7 @@ __device__ void seg_update(int k, int32_t D, bool load) {
     int32_t *h2k = V.h2 + (size_t)k * I.nstr;
     if (I.sl) {  // row-derived state: cnt_k(T) before the change from T's other inputs
         for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
-            const int4 ed = __ldg(&I.dedge[i]);
+            const int4 ed = edge_at(i);
             if (allocated(ed.x)) continue;
             const bool my = ed.y >= 0 && !resident(k, ed.y), mz = ed.z >= 0 && !resident(k, ed.z);
             const int c = (int)my + (int)mz + (load ? 1 : 0);  // missing inputs before
@@ -878,8 +902,7 @@ __device__ __forceinline__ void pop_batch_scalar() {
             const int64_t last = st[j] + plan_span(j, hd[j], c);
             L.req[j] = last;  // W = 0 (R7)
             L.gpu_free[j] = last;
-            L.plan_head[j] = hd[j] + c;
-            L.plan_live[j] -= c;
+            L.plan_head[j] = hd[j] + c;  // plan_live: after the barrier (pop_batch)
             mk = last > mk ? last : mk;
         }
     }
@@ -933,8 +956,7 @@ __device__ __noinline__ void pop_batch_scalar_smem() {
             const int64_t last = L.bstart[j] + plan_span(j, L.bhead[j], c);
             L.req[j] = last;  // W = 0 (R7)
             L.gpu_free[j] = last;
-            L.plan_head[j] += c;
-            L.plan_live[j] -= c;
+            L.plan_head[j] += c;  // plan_live: after the barrier (pop_batch)
             mk = last > mk ? last : mk;
         }
     }
@@ -959,6 +981,12 @@ __device__ void pop_batch() {
         else pop_batch_scalar_smem();
     }
     cta_sync();
+    // plan_live is what every thread summed at the top of the loop iteration to
+    // choose this path: thread 0 may change it only once all have passed the
+    // barrier above (changing it in the scalar phase let a late warp take the
+    // other path -- divergent barriers, found by compute-sanitizer synccheck)
+    if (threadIdx.x == 0)
+        for (int j = 0; j < K; j++) L.plan_live[j] -= L.bcnt[j];
     PROF_ADD(L, P_BW0, p_w0);
     PROF_T0(p_bd);
     const int P = L.boff[K];
@@ -1351,7 +1379,7 @@ __device__ void plan(int k, int32_t Dopt) {
         bool sel = false;
         int4 ed = make_int4(-1, -1, -1, 0);
         if (i < e) {
-            ed = __ldg(&I.dedge[i]);
+            ed = I.sl ? edge_at(i) : __ldg(&I.dedge[i]);
             T = ed.x;
             sel = I.sl ? !allocated(T) && (ed.y < 0 || resident(k, ed.y)) && (ed.z < 0 || resident(k, ed.z))
                        : (sk[T] >> 24) == 1u;
@@ -1403,7 +1431,7 @@ __device__ __noinline__ int32_t first_cnt2(int k, int32_t D2) {
         unsigned long long c = ~0ull;
         if (i < e) {
             if (I.sl) {  // D2 misses (n2(D2) > 0): exactly one other input misses
-                const int4 ed = __ldg(&I.dedge[i]);
+                const int4 ed = edge_at(i);
                 const int mo = (int)(ed.y >= 0 && !resident(k, ed.y)) + (int)(ed.z >= 0 && !resident(k, ed.z));
                 if (!allocated(ed.x) && mo == 1) c = (unsigned long long)ed.x;
             } else {
@@ -1767,7 +1795,7 @@ __device__ __noinline__ void assemble(int64_t ns) {
     const Inst &I = SI;
     __shared__ unsigned long long off[MAX_K];
     __shared__ int tot[MAX_K];
-    __shared__ int wk[32][MAX_K];
+    __shared__ int wk[16][MAX_K];  // [warp][GPU]: blocks of <= 512 threads
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
     for (int k = threadIdx.x; k < MAX_K; k += blockDim.x) off[k] = 0;
@@ -2033,6 +2061,14 @@ __global__ void __launch_bounds__(512, 1)
         if (tid == 0) SI = insts[ii];
         cta_sync();
         const Inst &I = SI;
+        if (I.poison) {  // debug: nothing may depend on the previous instance's shared memory
+            for (int i = tid; i < I.smem_bytes / 4; i += blockDim.x) reinterpret_cast<uint32_t *>(dsm)[i] = 0xA5A5A5A5u;
+            if (tid == 0) {
+                uint32_t *l = reinterpret_cast<uint32_t *>(&L);
+                for (size_t i = 0; i < sizeof(Lead) / 4; i++) l[i] = 0x5A5A5A5Au;
+            }
+            cta_sync();
+        }
         if (tid == 0) {
             View &W = SV;
             W.s = I.so_s >= 0 ? (uint32_t *)(dsm + I.so_s) : I.s;
@@ -2047,6 +2083,8 @@ __global__ void __launch_bounds__(512, 1)
             W.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
             W.lru = I.so_lru >= 0 ? (int32_t *)(dsm + I.so_lru) : I.lru;
             W.al = I.so_al >= 0 ? (uint32_t *)(dsm + I.so_al) : I.al;
+            W.ce4 = I.so_ce >= 0 && I.ce_bytes == 4 ? (uint32_t *)(dsm + I.so_ce) : nullptr;
+            W.ce8 = I.so_ce >= 0 && I.ce_bytes == 8 ? (unsigned long long *)(dsm + I.so_ce) : nullptr;
         }
         cta_sync();
         const View &V = SV;
@@ -2079,6 +2117,19 @@ __global__ void __launch_bounds__(512, 1)
             for (int i = tid; i < K * I.nstr; i += blockDim.x) V.np[i] = 0;
         if (I.so_resb >= 0)
             for (int i = tid; i < K * I.nw; i += blockDim.x) V.resb[i] = 0u;
+        }
+        if (I.so_ce >= 0) {  // compact edge records (the CSR was built by this CTA or the grid)
+            cta_sync();
+            const int64_t E = I.dptr[n];
+            const unsigned tb = (unsigned)I.ce_tb, db = (unsigned)I.ce_db;
+            for (int64_t i = tid; i < E; i += blockDim.x) {
+                const int4 ed = __ldcg(&I.dedge[i]);
+                const unsigned long long y = ed.y < 0 ? (unsigned long long)n : (unsigned long long)ed.y;
+                const unsigned long long z = ed.z < 0 ? (unsigned long long)n : (unsigned long long)ed.z;
+                const unsigned long long v = (unsigned long long)ed.x | (y << tb) | (I.ce_one ? 0ull : z << (tb + db));
+                if (I.ce_bytes == 4) V.ce4[i] = (uint32_t)v;
+                else V.ce8[i] = v;
+            }
         }
         if (tid == 0) {
             for (int k = 0; k < MAX_K; k++) {

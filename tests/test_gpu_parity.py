@@ -215,6 +215,26 @@ def test_row_derived_verify_partial_placement():
             assert_parity(g, oracle.run(inst))
 
 
+def test_compact_edge_records():
+    """Row-derived mode with the edge records packed into shared memory: 4-byte
+    records for 2-input rows (o2 not stored) and for 3-input rows, 8-byte
+    records when T and two ids need more than 32 bits; each against the
+    oracle with P9 on, placed and unplaced."""
+    cases = [gen.matmul2d(40, M=10, K=3),                       # 12 + 7 bits: 4 B, one other
+             gen.random_shared(5000, 256, 3, M=20, K=4, seed=21),  # 13 + 2 * 9: 4 B
+             gen.random_shared(6000, 1024, 3, M=24, K=2, seed=22),  # 13 + 2 * 11: 8 B
+             gen.cholesky(12, M=20, K=3)]                        # rows of 1..3 inputs
+    for inst in cases:
+        o = oracle.run(inst)
+        for smem in (0, -1):
+            g = dts.schedule(inst, flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_VERIFY, smem_budget=smem)
+            assert g.n_verify_err == 0
+            assert_parity(g, o)
+    gs = dts.schedule_batch(cases)
+    for inst, g in zip(cases, gs):
+        assert_parity(g, oracle.run(inst))
+
+
 # ------------------------------------------------------------ larger configs
 def test_config3():
     inst = gen.config_instances("C3")[0]
@@ -272,6 +292,21 @@ def test_sweep_sample_config5():
     gs = dts.schedule_batch(insts)
     for inst, g in zip(insts, gs):
         assert_parity(g, oracle.run(inst))
+
+
+def test_sweep_split_launch():
+    """A batch of >= 2 x 148 instances runs as two concurrent launches (wide
+    CTAs for the instances with long segments, <= 128-thread CTAs for the rest),
+    each on its own device counter; every instance must match the oracle."""
+    params = [(N, M, K) for N in (5, 10, 15) for M in (4, 6, 8, 12) for K in (1, 2, 3, 4)]
+    insts = [gen.sweep_instance(*p) for p in params] * 7                 # 336 narrow
+    insts += [gen.sweep_instance(70, 8, 2), gen.sweep_instance(140, 12, 3)]  # 128 (B), 256 (A)
+    gs = dts.schedule_batch(insts)
+    cache = {}
+    for inst, g in zip(insts, gs):
+        if inst.name not in cache:
+            cache[inst.name] = oracle.run(inst)
+        assert_parity(g, cache[inst.name])
 
 
 @pytest.mark.parametrize("K", [5, 9, 16, 64])
