@@ -482,6 +482,11 @@ dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_op
     return DTS_OK;
 }
 
+int env_int(const char *name, int dflt) {
+    const char *v = std::getenv(name);
+    return v ? std::atoi(v) : dflt;
+}
+
 // Shared-memory placement of one instance's state:
 // greedy, most latency-critical array first, each either fully in the CTA's
 // dynamic shared memory or in its global home.  Returns the bytes used.
@@ -499,14 +504,18 @@ int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard, boo
         }
     };
     put(h.so_resb, 4 * K * h.nw);
-    if (sl) put(h.so_al, 4 * (int64_t)(h.m_pad / 32 + 1));  // read by every segment walk
-    else h.so_al = -1;
+    // the allocation bitmap is read by every segment walk; DTS_AL_LATE=1 (experiment)
+    // places it after u instead, for instances where both do not fit (C4)
+    const bool al_late = env_int("DTS_AL_LATE", 0) != 0;
+    h.so_al = -1;
+    if (sl && !al_late) put(h.so_al, 4 * (int64_t)(h.m_pad / 32 + 1));
     put(h.so_dptr, 4 * (n + 1));
     put(h.so_plan, 16 * K * h.plan_cap);
     if (has_tau) put(h.so_plan_tau, 8 * K * h.plan_cap);
     else h.so_plan_tau = -1;
     put(h.so_res_list, 4 * K * h.res_cap);
     put(h.so_u, 4 * (int64_t)h.nstr);
+    if (sl && al_late) put(h.so_al, 4 * (int64_t)(h.m_pad / 32 + 1));
     put(h.so_h, 4 * K * (int64_t)h.nstr);
     put(h.so_h2, 4 * K * (int64_t)h.nstr);
     put(h.so_np, 4 * K * (int64_t)h.nstr);
@@ -540,10 +549,6 @@ int auto_block(const dts_instance *I) {
     return b;
 }
 
-int env_int(const char *name, int dflt) {
-    const char *v = std::getenv(name);
-    return v ? std::atoi(v) : dflt;
-}
 
 // Enqueue everything of one instance up to (not including) the decision loop:
 // upload if needed, CSR build (a1), state init (a2), descriptor H2D.

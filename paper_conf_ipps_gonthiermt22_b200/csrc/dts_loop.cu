@@ -468,6 +468,21 @@ __device__ __forceinline__ int4 entry_of_task(int32_t T) {
     return e;
 }
 
+// Thread 0: D(T) for serve_loads straight from a fallback / EAGER pick's
+// entry (rows are sorted, so the entry lists them ascending, R10) -- no second
+// CSR read; a longer row is read by the serve path (row_len = -1).
+__device__ __forceinline__ void row_from_entry(int4 e) {
+    if (e.w == ROW_LONG) {
+        L.row_len = -1;
+        return;
+    }
+    int len = 0;
+    if (e.y >= 0) L.row[len++] = e.y;
+    if (e.z >= 0) L.row[len++] = e.z;
+    if (e.w >= 0) L.row[len++] = e.w;
+    L.row_len = len;
+}
+
 // a2: datum D becomes resident (load) / leaves (evict) on GPU k.  Walk D's
 // data->task segment (edge records: the task and its other inputs in one 16 B
 // load): cnt_k(T) -/+= 1, x_k(T) ^= D, and move every unallocated task between
@@ -1295,42 +1310,54 @@ __device__ __noinline__ unsigned long long score_best64(const int32_t *score) {
     return best;
 }
 
+// The thread's best (score << 16 | u, then lowest D) over its slice, UN
+// 16-byte vectors of h and u in flight per thread: 2 when the rows are in
+// shared memory, 8 when they are global (C4: 16,471 data from L2, one round
+// trip per 8 vectors instead of per 2).
+template <int UN>
+__device__ __noinline__ unsigned long long score_best32(const int32_t *score) {
+    const Inst &I = SI;
+    const View &V = SV;
+    const unsigned ib = (unsigned)I.id_bits;
+    const unsigned long long idmask = (1ull << ib) - 1ull;
+    const int4 *h4 = reinterpret_cast<const int4 *>(score);
+    const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
+    const int nv = I.nstr >> 2;
+    uint32_t bk = 0u;
+    int32_t bd = 0;
+    for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
+        int4 hv[UN], uv[UN];
+#pragma unroll
+        for (int q = 0; q < UN; q++) {
+            const int v = v0 + q * blockDim.x;
+            hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
+            uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
+        }
+#pragma unroll
+        for (int q = 0; q < UN; q++) {
+            const int D = 4 * (v0 + q * blockDim.x);
+            const uint32_t k0 = ((uint32_t)hv[q].x << 16) | (uint32_t)uv[q].x;
+            const uint32_t k1 = ((uint32_t)hv[q].y << 16) | (uint32_t)uv[q].y;
+            const uint32_t k2 = ((uint32_t)hv[q].z << 16) | (uint32_t)uv[q].z;
+            const uint32_t k3 = ((uint32_t)hv[q].w << 16) | (uint32_t)uv[q].w;
+            if (k0 > bk) { bk = k0; bd = D; }
+            if (k1 > bk) { bk = k1; bd = D + 1; }
+            if (k2 > bk) { bk = k2; bd = D + 2; }
+            if (k3 > bk) { bk = k3; bd = D + 3; }
+        }
+    }
+    return bk >= 65536u ? ((unsigned long long)bk << ib) | (idmask - (unsigned long long)bd) : 0ull;  // positive score
+}
+
 __device__ int32_t score_argmax(const int32_t *score) {
     const Inst &I = SI;
     const View &V = SV;
     const unsigned ib = (unsigned)I.id_bits;
     const unsigned long long idmask = (1ull << ib) - 1ull;
-    unsigned long long best = 0ull;
+    unsigned long long best;
     if (I.key32) {
-        const int4 *h4 = reinterpret_cast<const int4 *>(score);
-        const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
-        const int nv = I.nstr >> 2;
-        constexpr int UN = 2;
-        uint32_t bk = 0u;
-        int32_t bd = 0;
-        for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
-            int4 hv[UN], uv[UN];
-#pragma unroll
-            for (int q = 0; q < UN; q++) {
-                const int v = v0 + q * blockDim.x;
-                hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
-                uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
-            }
-#pragma unroll
-            for (int q = 0; q < UN; q++) {
-                const int D = 4 * (v0 + q * blockDim.x);
-                const uint32_t k0 = ((uint32_t)hv[q].x << 16) | (uint32_t)uv[q].x;
-                const uint32_t k1 = ((uint32_t)hv[q].y << 16) | (uint32_t)uv[q].y;
-                const uint32_t k2 = ((uint32_t)hv[q].z << 16) | (uint32_t)uv[q].z;
-                const uint32_t k3 = ((uint32_t)hv[q].w << 16) | (uint32_t)uv[q].w;
-                if (k0 > bk) { bk = k0; bd = D; }
-                if (k1 > bk) { bk = k1; bd = D + 1; }
-                if (k2 > bk) { bk = k2; bd = D + 2; }
-                if (k3 > bk) { bk = k3; bd = D + 3; }
-            }
-        }
-        if (bk >= 65536u)  // positive score
-            best = ((unsigned long long)bk << ib) | (idmask - (unsigned long long)bd);
+        // shared rows: __isShared is one instruction; global rows want more loads in flight
+        best = __isShared(score) && __isShared(V.u) ? score_best32<2>(score) : score_best32<8>(score);
     } else {
         best = score_best64(score);
     }
@@ -2216,8 +2243,8 @@ __global__ void __launch_bounds__(512, 1)
                 if (tid == 0) {
                     if (T >= 0) {
                         L.avail_lo = T;
-                        L.row_len = -1;
                         L.fent = entry_of_task(T);
+                        row_from_entry(L.fent);
                         L.n_avail--;
                     } else {
                         L.idle[k] = 1;
@@ -2276,8 +2303,8 @@ __global__ void __launch_bounds__(512, 1)
                 }
                 if (T >= 0) {
                     if (tid == 0) {
-                        L.row_len = -1;
                         L.fent = entry_of_task(T);
+                        row_from_entry(L.fent);
                         L.n_avail--;
                         L.n_scans++;
                     }

@@ -309,6 +309,28 @@ def test_sweep_split_launch():
         assert_parity(g, cache[inst.name])
 
 
+@pytest.mark.parametrize("block", [0, 128])
+def test_sweep_config5_repeated(block):
+    """The full 4,096-instance sweep (bench launch configuration, and forced
+    128-thread CTAs) three times: every repetition schedules every task and
+    gives the same schedules (guards the block-level pop-batch race), and a
+    sample matches the oracle."""
+    insts = gen.config_instances("C5")
+    hs = [dts.create(i) for i in insts]
+    o = dts.dts_run_opts_default(flags=dts.DTS_F_FALLBACK2, block_threads=block)
+    ref = None
+    for _ in range(3):
+        dts.dts_sweep_run(hs, dts.DTS_POLICY_DARTS_LUF, o)
+        res = [dts.dts_result(h) for h in hs]
+        assert all(g.n_served == i.m for g, i in zip(res, insts))
+        sig = [(g.n_loads, g.n_evictions, g.makespan, g.n_scans) for g in res]
+        ref = ref or sig
+        assert sig == ref
+    for i in range(0, len(insts), 409):
+        if insts[i].m <= 12000:
+            assert_parity(res[i], oracle.run(insts[i]))
+
+
 @pytest.mark.parametrize("K", [5, 9, 16, 64])
 def test_many_simulated_gpus(K):
     """K beyond the register-resident pop path (K <= 8) and up to MAX_K = 64."""

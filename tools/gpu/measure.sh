@@ -12,5 +12,5 @@ timeout 600 python bench.py --workload C3 --shards 4 --steps 5 --no-cpu-baseline
 timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > $O/${TAG}_bench_reference_C2.json 2> $O/${TAG}_ref.err; echo "ref rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/${TAG}_launches_C2.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_bench.log 2>&1; echo "launches rc=$?"
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:dts_cta_kernel -s 3 -c 1 -o $O/${TAG}_full_C2 python bench.py --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C2.log 2>&1; echo "full C2 rc=$?"
-timeout 900 ncu --set full --clock-control none -k regex:dts_cta_kernel -s 3 -c 1 -o $O/${TAG}_full_C5 python bench.py --workload C5 --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C5.log 2>&1; echo "full C5 rc=$?"
+timeout 900 ncu --set full --clock-control none -k regex:dts_cta_kernel -s 6 -c 2 -o $O/${TAG}_full_C5 python bench.py --workload C5 --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C5.log 2>&1; echo "full C5 rc=$?"
 ls $O | grep $TAG
