@@ -359,6 +359,7 @@ def main():
         for h in handles:
             dts.dts_instance_upload(h, dev, sptr)
         step()
+        dts.dts_fetch_results(handles)  # all instances' results to host, two waits
         out = [dts.dts_result(h) for h in handles]
         t1.record(stream)
         t1.synchronize()

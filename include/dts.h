@@ -188,6 +188,14 @@ typedef struct {
 /* Synchronise on the run's stream, copy the results to host (once) and fill *out. */
 dts_status dts_result(dts_instance *inst, dts_result_view *out);
 
+/* Copy the results of insts[0..n) to host in two batched phases -- every
+ * instance's scalars, one wait per distinct stream, then every instance's
+ * arrays, one more wait per stream -- instead of two waits per instance.
+ * dts_result on these instances then returns without device work.  The
+ * instances must have run (DTS_E_STATE otherwise); the first failing
+ * instance's status is returned. */
+dts_status dts_fetch_results(dts_instance *const *insts, int32_t n);
+
 /* Sweep (BASELINE config 5) / batch: run every instance of insts[0..n) on
  * ONE device (opts->device) in a single batched launch of the decision loop,
  * one CTA per instance, CTAs pulling instances from a device counter (no

@@ -504,18 +504,16 @@ int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard, boo
         }
     };
     put(h.so_resb, 4 * K * h.nw);
-    // the allocation bitmap is read by every segment walk; DTS_AL_LATE=1 (experiment)
-    // places it after u instead, for instances where both do not fit (C4)
-    const bool al_late = env_int("DTS_AL_LATE", 0) != 0;
+    // the allocation bitmap is read by every segment walk (placing it after u
+    // instead made C4 1 % slower, profiles/r01i_c4_placement.txt)
     h.so_al = -1;
-    if (sl && !al_late) put(h.so_al, 4 * (int64_t)(h.m_pad / 32 + 1));
+    if (sl) put(h.so_al, 4 * (int64_t)(h.m_pad / 32 + 1));
     put(h.so_dptr, 4 * (n + 1));
     put(h.so_plan, 16 * K * h.plan_cap);
     if (has_tau) put(h.so_plan_tau, 8 * K * h.plan_cap);
     else h.so_plan_tau = -1;
     put(h.so_res_list, 4 * K * h.res_cap);
     put(h.so_u, 4 * (int64_t)h.nstr);
-    if (sl && al_late) put(h.so_al, 4 * (int64_t)(h.m_pad / 32 + 1));
     put(h.so_h, 4 * K * (int64_t)h.nstr);
     put(h.so_h2, 4 * K * (int64_t)h.nstr);
     put(h.so_np, 4 * K * (int64_t)h.nstr);
@@ -523,8 +521,6 @@ int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard, boo
     else h.so_lru = -1;
     if (!sl) put(h.so_s, 4 * K * (int64_t)h.m_pad);  // last: the largest, worth it only when it fits
     else h.so_s = -1;
-    if (sl && h.ce_bytes > 0) put(h.so_ce, (int64_t)h.ce_bytes * h.E);  // edge records, when all else fits
-    else h.so_ce = -1;
     h.smem_bytes = used;
     return used;
 }
@@ -582,15 +578,6 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     }
     // row-derived state (no per-(GPU, task) words) when every edge record holds its row
     h.sl = I->G == 1 && I->max_row_len <= 3 && !(o.flags & DTS_F_PACKED) ? 1 : 0;
-    {  // compact edge records: T, then the (<= 2) other inputs, value n = absent
-        const int tb = bits_for(I->m > 0 ? (uint64_t)(I->m - 1) : 0), db = bits_for((uint64_t)I->n);
-        const int one = I->max_row_len <= 2 ? 1 : 0;
-        const int need = tb + (one ? 1 : 2) * db;
-        h.ce_tb = tb;
-        h.ce_db = db;
-        h.ce_one = one;
-        h.ce_bytes = !h.sl ? 0 : (need <= 32 ? 4 : (need <= 64 ? 8 : 0));
-    }
     place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF, I->G > 1, h.sl != 0);
     h.G = I->G;
     h.g = I->g;
@@ -1019,38 +1006,81 @@ dts_status dts_shard_group_run(dts_instance *const *shards, int32_t G, dts_polic
 }
 
 
+// Result copies in two phases so that many instances share the waits
+// (dts_fetch_results): the scalars first (they size the rest), then the arrays.
+static dts_status fetch_out(dts_instance *I) {
+    CK(cudaSetDevice(I->device), "cudaSetDevice");
+    CK(cudaMemcpyAsync(I->r_out, I->h_inst.out, sizeof I->out, cudaMemcpyDeviceToHost, I->stream), "D2H out");
+    return DTS_OK;
+}
+static dts_status fetch_arrays(dts_instance *I) {
+    I->out = *I->r_out;
+    if (I->out.error == 2) return fail(DTS_E_STATE, "task shards: a peer did not reach an exchange in time");
+    if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim (Belady branch)");
+    const dts::Inst &h = I->h_inst;
+    size_t ns = (size_t)I->out.n_served, ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);
+    size_t m = (size_t)I->m;
+    cudaStream_t st = I->stream;  // the run's stream: the copies follow the run
+    CK(cudaSetDevice(I->device), "cudaSetDevice");
+    CK(cudaMemcpyAsync(I->r_gpu_ptr, h.gpu_task_ptr, 8 * ((size_t)I->K + 1), cudaMemcpyDeviceToHost, st), "D2H");
+    if (ns) {
+        CK(cudaMemcpyAsync(I->r_gpu_ids, h.gpu_task_ids, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
+        CK(cudaMemcpyAsync(I->r_serve_gpu, h.serve_gpu, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
+        CK(cudaMemcpyAsync(I->r_serve_task, h.serve_task, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
+    }
+    if (m) {
+        CK(cudaMemcpyAsync(I->r_tstart, h.tstart, 8 * m, cudaMemcpyDeviceToHost, st), "D2H");
+        CK(cudaMemcpyAsync(I->r_tend, h.tend, 8 * m, cudaMemcpyDeviceToHost, st), "D2H");
+    }
+    if (ne)
+        CK(cudaMemcpyAsync(I->r_events, h.events, sizeof(dts_event) * ne, cudaMemcpyDeviceToHost, st), "D2H");
+    I->r_n_events = (int64_t)ne;
+    return DTS_OK;
+}
+static dts_status fetch_done(dts_instance *I) {
+    CK(cudaEventElapsedTime(&I->loop_ms, I->ev[1], I->ev[2]), "elapsed");
+    CK(cudaEventElapsedTime(&I->total_ms, I->ev[0], I->ev[3]), "elapsed");
+    I->have_host = true;
+    return DTS_OK;
+}
+// Wait for every distinct (device, stream) of the list once.
+static dts_status sync_streams(dts_instance *const *insts, int32_t n) {
+    std::vector<std::pair<int, cudaStream_t>> seen;
+    for (int32_t i = 0; i < n; i++) {
+        const std::pair<int, cudaStream_t> key(insts[i]->device, insts[i]->stream);
+        if (insts[i]->have_host || std::find(seen.begin(), seen.end(), key) != seen.end()) continue;
+        seen.push_back(key);
+        CK(cudaSetDevice(key.first), "cudaSetDevice");
+        CK(cudaStreamSynchronize(key.second), "D2H sync");
+    }
+    return DTS_OK;
+}
+
+dts_status dts_fetch_results(dts_instance *const *insts, int32_t n) {
+    if (n < 0 || (n > 0 && !insts)) return fail(DTS_E_INVAL, "insts");
+    for (int32_t i = 0; i < n; i++) {
+        if (!insts[i]) return fail(DTS_E_INVAL, "instance is NULL");
+        if (!insts[i]->ran) return fail(DTS_E_STATE, "dts_fetch_results before dts_run");
+    }
+    dts_status s;
+    for (int32_t i = 0; i < n; i++)
+        if (!insts[i]->have_host && (s = fetch_out(insts[i])) != DTS_OK) return s;
+    if ((s = sync_streams(insts, n)) != DTS_OK) return s;
+    for (int32_t i = 0; i < n; i++)
+        if (!insts[i]->have_host && (s = fetch_arrays(insts[i])) != DTS_OK) return s;
+    if ((s = sync_streams(insts, n)) != DTS_OK) return s;
+    for (int32_t i = 0; i < n; i++)
+        if (!insts[i]->have_host && (s = fetch_done(insts[i])) != DTS_OK) return s;
+    return DTS_OK;
+}
+
 dts_status dts_result(dts_instance *I, dts_result_view *v) {
     if (!I || !v) return fail(DTS_E_INVAL, "NULL argument");
     if (!I->ran) return fail(DTS_E_STATE, "dts_result before dts_run");
     if (!I->have_host) {
-        CK(cudaSetDevice(I->device), "cudaSetDevice");
-        CK(cudaEventSynchronize(I->ev[3]), "run");
-        CK(cudaMemcpyAsync(I->r_out, I->h_inst.out, sizeof I->out, cudaMemcpyDeviceToHost, I->stream), "D2H out");
-        CK(cudaStreamSynchronize(I->stream), "D2H sync");
-        I->out = *I->r_out;
-        if (I->out.error == 2) return fail(DTS_E_STATE, "task shards: a peer did not reach an exchange in time");
-        if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim (Belady branch)");
-        const dts::Inst &h = I->h_inst;
-        size_t ns = (size_t)I->out.n_served, ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);
-        size_t m = (size_t)I->m;
-        cudaStream_t st = I->stream;  // the run's stream: the copies follow the run
-        CK(cudaMemcpyAsync(I->r_gpu_ptr, h.gpu_task_ptr, 8 * ((size_t)I->K + 1), cudaMemcpyDeviceToHost, st), "D2H");
-        if (ns) {
-            CK(cudaMemcpyAsync(I->r_gpu_ids, h.gpu_task_ids, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
-            CK(cudaMemcpyAsync(I->r_serve_gpu, h.serve_gpu, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
-            CK(cudaMemcpyAsync(I->r_serve_task, h.serve_task, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
-        }
-        if (m) {
-            CK(cudaMemcpyAsync(I->r_tstart, h.tstart, 8 * m, cudaMemcpyDeviceToHost, st), "D2H");
-            CK(cudaMemcpyAsync(I->r_tend, h.tend, 8 * m, cudaMemcpyDeviceToHost, st), "D2H");
-        }
-        if (ne)
-            CK(cudaMemcpyAsync(I->r_events, h.events, sizeof(dts_event) * ne, cudaMemcpyDeviceToHost, st), "D2H");
-        CK(cudaStreamSynchronize(st), "D2H sync");
-        I->r_n_events = (int64_t)ne;
-        CK(cudaEventElapsedTime(&I->loop_ms, I->ev[1], I->ev[2]), "elapsed");
-        CK(cudaEventElapsedTime(&I->total_ms, I->ev[0], I->ev[3]), "elapsed");
-        I->have_host = true;
+        dts_instance *one[1] = {I};
+        dts_status s = dts_fetch_results(one, 1);
+        if (s != DTS_OK) return s;
     }
     std::memset(v, 0, sizeof *v);
     v->K = I->K;

@@ -154,13 +154,6 @@ struct Inst {
     int32_t sl;
     int32_t so_al;            // shared-memory offset of al, -1 = global home
     uint32_t *al;             // [m_pad / 32 + 1] global home
-    // row-derived mode: compact edge records in shared memory (so_ce >= 0):
-    // {T, o1, o2} bit-packed into ce_bytes = 4 or 8 bytes (T in ce_tb bits,
-    // each other input in ce_db bits, value n = absent; ce_one: rows <= 2,
-    // o2 not stored) -- the data->task segments read by every scan, load and
-    // eviction come from shared memory instead of L2
-    int32_t ce_bytes, ce_tb, ce_db, ce_one;
-    int32_t so_ce;
     int32_t poison;  // debug (env DTS_POISON=1): fill the CTA's dynamic shared memory at instance start
 };
 

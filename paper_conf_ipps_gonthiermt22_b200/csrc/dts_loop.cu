@@ -131,8 +131,6 @@ struct View {
     int32_t *dptr32;    // shared-memory copy of dptr, or nullptr
     int32_t *lru;       // [K][nstr] last-use stamps (LRU policies)
     uint32_t *al;       // row-derived mode: allocation bitmap (bit set = left the pool)
-    uint32_t *ce4;      // row-derived mode: 4-byte compact edge records (shared), or
-    unsigned long long *ce8;  // 8-byte ones, or neither (edge records from dedge)
 };
 
 // Per-CTA state at namespace scope, so the (non-inlined) phase functions
@@ -225,24 +223,6 @@ __device__ __forceinline__ int missing_of(int k, int32_t a, int32_t b, int32_t c
     m0 = ma ? a : (mb ? b : c);
     m1 = ma ? (mb ? b : c) : c;
     return (int)ma + (int)mb + (int)mc;
-}
-
-// Edge record i of the data->task CSR as {T, o1, o2, -} (row-derived mode:
-// rows <= 3, the 4th field unused): decoded from the compact shared-memory
-// copy when placed, else the 16-byte record from global memory.
-__device__ __forceinline__ int4 edge_at(int64_t i) {
-    const Inst &I = SI;
-    const View &V = SV;
-    if (V.ce4 || V.ce8) {
-        const unsigned long long v = V.ce4 ? (unsigned long long)V.ce4[i] : V.ce8[i];
-        const unsigned tb = (unsigned)I.ce_tb, db = (unsigned)I.ce_db;
-        const unsigned long long dm = (1ull << db) - 1ull;
-        const int32_t T = (int32_t)(v & ((1ull << tb) - 1ull));
-        const int32_t y = (int32_t)((v >> tb) & dm);
-        const int32_t z = I.ce_one ? I.n : (int32_t)((v >> (tb + db)) & dm);
-        return make_int4(T, y == I.n ? -1 : y, z == I.n ? -1 : z, 0);
-    }
-    return __ldg(&I.dedge[i]);
 }
 
 // Data->task segment bounds of D (int32 copy in shared memory when placed).
@@ -499,7 +479,7 @@ __device__ void seg_update(int k, int32_t D, bool load) {
     int32_t *h2k = V.h2 + (size_t)k * I.nstr;
     if (I.sl) {  // row-derived state: cnt_k(T) before the change from T's other inputs
         for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
-            const int4 ed = edge_at(i);
+            const int4 ed = __ldg(&I.dedge[i]);
             if (allocated(ed.x)) continue;
             const bool my = ed.y >= 0 && !resident(k, ed.y), mz = ed.z >= 0 && !resident(k, ed.z);
             const int c = (int)my + (int)mz + (load ? 1 : 0);  // missing inputs before
@@ -1000,8 +980,10 @@ __device__ void pop_batch() {
     // choose this path: thread 0 may change it only once all have passed the
     // barrier above (changing it in the scalar phase let a late warp take the
     // other path -- divergent barriers, found by compute-sanitizer synccheck)
-    if (threadIdx.x == 0)
-        for (int j = 0; j < K; j++) L.plan_live[j] -= L.bcnt[j];
+    {  // one GPU per thread, from the top of the CTA (idle in the rank phase below)
+        const int j = (int)blockDim.x - 1 - (int)threadIdx.x;
+        for (int jj = j; jj >= 0 && jj < K; jj += blockDim.x) L.plan_live[jj] -= L.bcnt[jj];
+    }
     PROF_ADD(L, P_BW0, p_w0);
     PROF_T0(p_bd);
     const int P = L.boff[K];
@@ -1310,54 +1292,42 @@ __device__ __noinline__ unsigned long long score_best64(const int32_t *score) {
     return best;
 }
 
-// The thread's best (score << 16 | u, then lowest D) over its slice, UN
-// 16-byte vectors of h and u in flight per thread: 2 when the rows are in
-// shared memory, 8 when they are global (C4: 16,471 data from L2, one round
-// trip per 8 vectors instead of per 2).
-template <int UN>
-__device__ __noinline__ unsigned long long score_best32(const int32_t *score) {
-    const Inst &I = SI;
-    const View &V = SV;
-    const unsigned ib = (unsigned)I.id_bits;
-    const unsigned long long idmask = (1ull << ib) - 1ull;
-    const int4 *h4 = reinterpret_cast<const int4 *>(score);
-    const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
-    const int nv = I.nstr >> 2;
-    uint32_t bk = 0u;
-    int32_t bd = 0;
-    for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
-        int4 hv[UN], uv[UN];
-#pragma unroll
-        for (int q = 0; q < UN; q++) {
-            const int v = v0 + q * blockDim.x;
-            hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
-            uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
-        }
-#pragma unroll
-        for (int q = 0; q < UN; q++) {
-            const int D = 4 * (v0 + q * blockDim.x);
-            const uint32_t k0 = ((uint32_t)hv[q].x << 16) | (uint32_t)uv[q].x;
-            const uint32_t k1 = ((uint32_t)hv[q].y << 16) | (uint32_t)uv[q].y;
-            const uint32_t k2 = ((uint32_t)hv[q].z << 16) | (uint32_t)uv[q].z;
-            const uint32_t k3 = ((uint32_t)hv[q].w << 16) | (uint32_t)uv[q].w;
-            if (k0 > bk) { bk = k0; bd = D; }
-            if (k1 > bk) { bk = k1; bd = D + 1; }
-            if (k2 > bk) { bk = k2; bd = D + 2; }
-            if (k3 > bk) { bk = k3; bd = D + 3; }
-        }
-    }
-    return bk >= 65536u ? ((unsigned long long)bk << ib) | (idmask - (unsigned long long)bd) : 0ull;  // positive score
-}
-
 __device__ int32_t score_argmax(const int32_t *score) {
     const Inst &I = SI;
     const View &V = SV;
     const unsigned ib = (unsigned)I.id_bits;
     const unsigned long long idmask = (1ull << ib) - 1ull;
-    unsigned long long best;
+    unsigned long long best = 0ull;
     if (I.key32) {
-        // shared rows: __isShared is one instruction; global rows want more loads in flight
-        best = __isShared(score) && __isShared(V.u) ? score_best32<2>(score) : score_best32<8>(score);
+        const int4 *h4 = reinterpret_cast<const int4 *>(score);
+        const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
+        const int nv = I.nstr >> 2;
+        constexpr int UN = 2;
+        uint32_t bk = 0u;
+        int32_t bd = 0;
+        for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
+            int4 hv[UN], uv[UN];
+#pragma unroll
+            for (int q = 0; q < UN; q++) {
+                const int v = v0 + q * blockDim.x;
+                hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
+                uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
+            }
+#pragma unroll
+            for (int q = 0; q < UN; q++) {
+                const int D = 4 * (v0 + q * blockDim.x);
+                const uint32_t k0 = ((uint32_t)hv[q].x << 16) | (uint32_t)uv[q].x;
+                const uint32_t k1 = ((uint32_t)hv[q].y << 16) | (uint32_t)uv[q].y;
+                const uint32_t k2 = ((uint32_t)hv[q].z << 16) | (uint32_t)uv[q].z;
+                const uint32_t k3 = ((uint32_t)hv[q].w << 16) | (uint32_t)uv[q].w;
+                if (k0 > bk) { bk = k0; bd = D; }
+                if (k1 > bk) { bk = k1; bd = D + 1; }
+                if (k2 > bk) { bk = k2; bd = D + 2; }
+                if (k3 > bk) { bk = k3; bd = D + 3; }
+            }
+        }
+        if (bk >= 65536u)  // positive score
+            best = ((unsigned long long)bk << ib) | (idmask - (unsigned long long)bd);
     } else {
         best = score_best64(score);
     }
@@ -1406,7 +1376,7 @@ __device__ void plan(int k, int32_t Dopt) {
         bool sel = false;
         int4 ed = make_int4(-1, -1, -1, 0);
         if (i < e) {
-            ed = I.sl ? edge_at(i) : __ldg(&I.dedge[i]);
+            ed = __ldg(&I.dedge[i]);
             T = ed.x;
             sel = I.sl ? !allocated(T) && (ed.y < 0 || resident(k, ed.y)) && (ed.z < 0 || resident(k, ed.z))
                        : (sk[T] >> 24) == 1u;
@@ -1458,7 +1428,7 @@ __device__ __noinline__ int32_t first_cnt2(int k, int32_t D2) {
         unsigned long long c = ~0ull;
         if (i < e) {
             if (I.sl) {  // D2 misses (n2(D2) > 0): exactly one other input misses
-                const int4 ed = edge_at(i);
+                const int4 ed = __ldg(&I.dedge[i]);
                 const int mo = (int)(ed.y >= 0 && !resident(k, ed.y)) + (int)(ed.z >= 0 && !resident(k, ed.z));
                 if (!allocated(ed.x) && mo == 1) c = (unsigned long long)ed.x;
             } else {
@@ -2110,8 +2080,6 @@ __global__ void __launch_bounds__(512, 1)
             W.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
             W.lru = I.so_lru >= 0 ? (int32_t *)(dsm + I.so_lru) : I.lru;
             W.al = I.so_al >= 0 ? (uint32_t *)(dsm + I.so_al) : I.al;
-            W.ce4 = I.so_ce >= 0 && I.ce_bytes == 4 ? (uint32_t *)(dsm + I.so_ce) : nullptr;
-            W.ce8 = I.so_ce >= 0 && I.ce_bytes == 8 ? (unsigned long long *)(dsm + I.so_ce) : nullptr;
         }
         cta_sync();
         const View &V = SV;
@@ -2144,19 +2112,6 @@ __global__ void __launch_bounds__(512, 1)
             for (int i = tid; i < K * I.nstr; i += blockDim.x) V.np[i] = 0;
         if (I.so_resb >= 0)
             for (int i = tid; i < K * I.nw; i += blockDim.x) V.resb[i] = 0u;
-        }
-        if (I.so_ce >= 0) {  // compact edge records (the CSR was built by this CTA or the grid)
-            cta_sync();
-            const int64_t E = I.dptr[n];
-            const unsigned tb = (unsigned)I.ce_tb, db = (unsigned)I.ce_db;
-            for (int64_t i = tid; i < E; i += blockDim.x) {
-                const int4 ed = __ldcg(&I.dedge[i]);
-                const unsigned long long y = ed.y < 0 ? (unsigned long long)n : (unsigned long long)ed.y;
-                const unsigned long long z = ed.z < 0 ? (unsigned long long)n : (unsigned long long)ed.z;
-                const unsigned long long v = (unsigned long long)ed.x | (y << tb) | (I.ce_one ? 0ull : z << (tb + db));
-                if (I.ce_bytes == 4) V.ce4[i] = (uint32_t)v;
-                else V.ce8[i] = v;
-            }
         }
         if (tid == 0) {
             for (int k = 0; k < MAX_K; k++) {

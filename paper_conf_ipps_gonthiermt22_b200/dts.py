@@ -43,7 +43,7 @@ EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data",
                         ("task", "<i4"), ("op", "u1"), ("pad", "u1", (3,))])
 
 EXPORTED = ["dts_run_opts_default", "dts_instance_create", "dts_instance_upload", "dts_run",
-            "dts_result", "dts_sweep_run", "dts_instance_destroy", "dts_status_str",
+            "dts_result", "dts_fetch_results", "dts_sweep_run", "dts_instance_destroy", "dts_status_str",
             "dts_last_error", "dts_version", "dts_kernel_launches",
             "dts_shard_set", "dts_shard_range", "dts_shard_export", "dts_shard_connect",
             "dts_shard_group_run"]
@@ -105,6 +105,9 @@ def load_library(path: str = LIB_PATH):
     lib.dts_sweep_run.argtypes = [C.POINTER(C.c_void_p), C.c_int32, C.c_int,
                                   C.POINTER(dts_run_opts)]
     lib.dts_sweep_run.restype = C.c_int
+    if hasattr(lib, "dts_fetch_results"):  # (older builds, tools/lib_ab.py, lack it)
+        lib.dts_fetch_results.argtypes = [C.POINTER(C.c_void_p), C.c_int32]
+        lib.dts_fetch_results.restype = C.c_int
     lib.dts_instance_destroy.argtypes = [P]
     lib.dts_instance_destroy.restype = None
     lib.dts_status_str.argtypes = [C.c_int]
@@ -278,6 +281,13 @@ def dts_result(inst: Instance) -> Result:
                   float(v.loop_ms), float(v.total_ms), tuple(int(x) for x in v.prof_cycles))
 
 
+def dts_fetch_results(insts) -> None:
+    """Batched device->host copy of many instances' results (two waits in
+    total); dts_result afterwards reads host memory only."""
+    arr = (C.c_void_p * len(insts))(*[i.handle for i in insts])
+    _check(load_library().dts_fetch_results(arr, len(insts)))
+
+
 def dts_kernel_launches() -> int:
     return int(load_library().dts_kernel_launches())
 
@@ -317,6 +327,7 @@ def schedule_batch(insts, *, policy: int = DTS_POLICY_DARTS_LUF, W: int = 0, fla
                              block_threads=block_threads, smem_budget=smem_budget,
                              max_served=-1, cuda_stream=stream or None)
     dts_sweep_run(hs, policy, o)
+    dts_fetch_results(hs)
     return [dts_result(h) for h in hs]
 
 

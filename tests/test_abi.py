@@ -98,3 +98,12 @@ def test_no_gpu_fails_loudly():
     with pytest.raises(dts.DtsError) as e:
         dts.schedule(i)
     assert e.value.status == B.DTS_E_CUDA
+
+
+def test_fetch_results_before_run_is_state_error():
+    i = gen.fig1()
+    hs = [dts.dts_instance_create(i.task_ptr, i.task_data, i.data_size, None, 1, 2, 2) for _ in range(2)]
+    with pytest.raises(dts.DtsError) as e:
+        dts.dts_fetch_results(hs)
+    assert e.value.status == B.DTS_E_STATE
+    dts.dts_fetch_results([])  # nothing to do

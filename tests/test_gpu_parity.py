@@ -215,14 +215,13 @@ def test_row_derived_verify_partial_placement():
             assert_parity(g, oracle.run(inst))
 
 
-def test_compact_edge_records():
-    """Row-derived mode with the edge records packed into shared memory: 4-byte
-    records for 2-input rows (o2 not stored) and for 3-input rows, 8-byte
-    records when T and two ids need more than 32 bits; each against the
-    oracle with P9 on, placed and unplaced."""
-    cases = [gen.matmul2d(40, M=10, K=3),                       # 12 + 7 bits: 4 B, one other
-             gen.random_shared(5000, 256, 3, M=20, K=4, seed=21),  # 13 + 2 * 9: 4 B
-             gen.random_shared(6000, 1024, 3, M=24, K=2, seed=22),  # 13 + 2 * 11: 8 B
+def test_row_derived_mode_row_widths():
+    """Row-derived mode on rows of 1, 2 and 3 inputs and on ids wider than 32
+    bits in total (T and two other inputs), each against the oracle with P9
+    on, state placed and unplaced, alone and batched."""
+    cases = [gen.matmul2d(40, M=10, K=3),                       # rows of 2
+             gen.random_shared(5000, 256, 3, M=20, K=4, seed=21),  # rows of 3
+             gen.random_shared(6000, 1024, 3, M=24, K=2, seed=22),  # 13 + 2 * 11 id bits
              gen.cholesky(12, M=20, K=3)]                        # rows of 1..3 inputs
     for inst in cases:
         o = oracle.run(inst)
@@ -501,3 +500,17 @@ def test_w1_config4_prefix(cfg):
     g = dts.schedule(inst, W=1, max_served=1500)
     o = oracle.run(inst, W=1, max_served=1500)
     assert_parity(g, o, complete=False)
+
+
+def test_fetch_results_matches_per_instance_result():
+    """dts_fetch_results (batched copies, two waits) returns what dts_result
+    alone would, for a sweep and for separately run instances."""
+    insts = gen.config_instances("C2")[:6]
+    a = dts.schedule_batch(insts)  # fetch + result
+    hs = [dts.create(i) for i in insts]
+    for h in hs:
+        dts.dts_run(h, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default())
+    b = [dts.dts_result(h) for h in hs]  # one at a time
+    for x, y, inst in zip(a, b, insts):
+        assert np.array_equal(x.serve_task, y.serve_task) and np.array_equal(x.events, y.events)
+        assert_parity(x, oracle.run(inst))
