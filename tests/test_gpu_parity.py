@@ -514,3 +514,4 @@ def test_fetch_results_matches_per_instance_result():
     for x, y, inst in zip(a, b, insts):
         assert np.array_equal(x.serve_task, y.serve_task) and np.array_equal(x.events, y.events)
         assert_parity(x, oracle.run(inst))
+
