@@ -93,8 +93,12 @@ class Clocks:
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            t0 = time.time()  # nvidia-smi's first sample before the region starts
+            while not self.lines and time.time() - t0 < 3.0:
+                time.sleep(0.01)
         except Exception:
             self.proc = None
+        self.n0 = len(self.lines)
         return self
 
     def _read(self):
@@ -103,6 +107,9 @@ class Clocks:
 
     def __exit__(self, *a):
         if self.proc is not None:
+            t0 = time.time()  # a region shorter than the 100 ms period: the sample that closes it
+            while len(self.lines) <= self.n0 and time.time() - t0 < 1.0:
+                time.sleep(0.005)
             self.proc.terminate()
             try:
                 self.proc.wait(timeout=5)

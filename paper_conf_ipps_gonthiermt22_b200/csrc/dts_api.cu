@@ -112,6 +112,10 @@ struct dts_instance {
     int32_t *r_gpu_ids = nullptr, *r_serve_gpu = nullptr, *r_serve_task = nullptr;
     dts_event *r_events = nullptr;
     dts::Out *r_out = nullptr;
+    // pinned mirror of the device result region [gpu_task_ptr .. events end): one
+    // D2H copy per instance brings sigma, the service order, the times and the trace
+    char *h_res = nullptr;
+    size_t res_bytes = 0;
     int64_t r_n_events = 0;
     float loop_ms = 0.f, total_ms = 0.f;
 
@@ -140,6 +144,7 @@ struct dts_instance {
         }
         if (h_pinned) cudaFreeHost(h_pinned);
         if (h_pin) cudaFreeHost(h_pin);
+        if (h_res) cudaFreeHost(h_res);
     }
 };
 
@@ -358,24 +363,16 @@ dts_status ensure_device(dts_instance *I, int device) {
     if (!I->h_pinned) CK(cudaMallocHost(&I->h_pinned, sizeof(dts::Inst)), "cudaMallocHost");
     if (!I->h_pin) {
         size_t hb = 0;
-        auto hadd = [&](size_t bytes) { size_t o = hb; hb += (bytes + 63) & ~size_t(63); return o; };
+        // the input mirror has the device arena's layout (256-byte rounding, same
+        // order as d_raw_ptr, d_raw_dat, d_size, d_tau): one H2D copy uploads it
+        auto hadd = [&](size_t bytes) { size_t o = hb; hb += (bytes + 255) & ~size_t(255); return o; };
         const size_t o_tp = hadd(8 * (m + 1)), o_td = hadd(4 * (E + 1)), o_sz = hadd(8 * (n + 1)),
-                     o_tn = hadd(8 * (m + 1)), o_gp = hadd(8 * (K + 1)), o_gi = hadd(4 * (m + 1)),
-                     o_sg = hadd(4 * (m + 1)), o_st = hadd(4 * (m + 1)), o_ts = hadd(8 * (m + 1)),
-                     o_te = hadd(8 * (m + 1)), o_ev = hadd(sizeof(dts_event) * ev_cap),
-                     o_out = hadd(sizeof(dts::Out));
+                     o_tn = hadd(8 * (m + 1)), o_out = hadd(sizeof(dts::Out));
         CK(cudaMallocHost(&I->h_pin, hb), "cudaMallocHost");
         I->p_task_ptr = (int64_t *)(I->h_pin + o_tp);
         I->p_task_data = (int32_t *)(I->h_pin + o_td);
         I->p_size = (uint64_t *)(I->h_pin + o_sz);
         I->p_task_ns = (int64_t *)(I->h_pin + o_tn);
-        I->r_gpu_ptr = (int64_t *)(I->h_pin + o_gp);
-        I->r_gpu_ids = (int32_t *)(I->h_pin + o_gi);
-        I->r_serve_gpu = (int32_t *)(I->h_pin + o_sg);
-        I->r_serve_task = (int32_t *)(I->h_pin + o_st);
-        I->r_tstart = (int64_t *)(I->h_pin + o_ts);
-        I->r_tend = (int64_t *)(I->h_pin + o_te);
-        I->r_events = (dts_event *)(I->h_pin + o_ev);
         I->r_out = (dts::Out *)(I->h_pin + o_out);
         std::memcpy(I->p_task_ptr, I->task_ptr.data(), 8 * (m + 1));
         if (E) std::memcpy(I->p_task_data, I->task_data.data(), 4 * E);
@@ -409,13 +406,14 @@ dts_status ensure_device(dts_instance *I, int device) {
     h.lru = A.take<int32_t>(K * (nstr + 4));
     h.al = A.take<uint32_t>(mp / 32 + 2);
     h.out = A.take<dts::Out>(1);
+    // the result region, contiguous, the trace last (its used length varies)
+    h.gpu_task_ptr = A.take<int64_t>(K + 1);
+    h.gpu_task_ids = A.take<int32_t>(m + 1);
     h.serve_gpu = A.take<int32_t>(m + 1);
     h.serve_task = A.take<int32_t>(m + 1);
     h.tstart = A.take<int64_t>(m + 1);
     h.tend = A.take<int64_t>(m + 1);
     h.events = A.take<dts_event>(ev_cap);
-    h.gpu_task_ptr = A.take<int64_t>(K + 1);
-    h.gpu_task_ids = A.take<int32_t>(m + 1);
     I->d_inst = A.take<dts::Inst>(1);
     I->d_work = A.take<int>(16);
     I->d_csr_scratch = A.take<char>(dts::csr_scratch_bytes(I->m, I->n, I->E_raw));
@@ -424,6 +422,24 @@ dts_status ensure_device(dts_instance *I, int device) {
     I->d_box = A.take<unsigned char>(2 * (size_t)box_bytes);
     I->d_peers = A.take<dts::ShardPeer>(dts::MAX_G);
     if (A.used > A.size) return fail(DTS_E_NOMEM, "arena overflow (internal)");
+    {  // host mirror of the result region, same relative layout
+        char *r0 = reinterpret_cast<char *>(h.gpu_task_ptr);
+        const size_t bytes = (size_t)(reinterpret_cast<char *>(h.events) - r0) + sizeof(dts_event) * ev_cap;
+        if (I->h_res && I->res_bytes != bytes) {
+            cudaFreeHost(I->h_res);
+            I->h_res = nullptr;
+        }
+        if (!I->h_res) CK(cudaMallocHost(&I->h_res, bytes), "cudaMallocHost");
+        I->res_bytes = bytes;
+        auto at = [&](const void *d) { return I->h_res + (reinterpret_cast<const char *>(d) - r0); };
+        I->r_gpu_ptr = reinterpret_cast<int64_t *>(at(h.gpu_task_ptr));
+        I->r_gpu_ids = reinterpret_cast<int32_t *>(at(h.gpu_task_ids));
+        I->r_serve_gpu = reinterpret_cast<int32_t *>(at(h.serve_gpu));
+        I->r_serve_task = reinterpret_cast<int32_t *>(at(h.serve_task));
+        I->r_tstart = reinterpret_cast<int64_t *>(at(h.tstart));
+        I->r_tend = reinterpret_cast<int64_t *>(at(h.tend));
+        I->r_events = reinterpret_cast<dts_event *>(at(h.events));
+    }
     CK(cudaMemset(I->d_epoch, 0, 256), "memset epoch");  // exchange numbers start at 0, once
     I->connected = false;
     I->runs = 0;
@@ -452,16 +468,12 @@ dts_status ensure_device(dts_instance *I, int device) {
 
 dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
     if (I->uploaded && !force) return DTS_OK;
-    // from the pinned mirror of the caller's arrays (asynchronous DMA)
-    CK(cudaMemcpyAsync(I->d_raw_ptr, I->p_task_ptr, 8 * ((size_t)I->m + 1), cudaMemcpyHostToDevice, st),
-       "H2D task_ptr");
-    if (I->E_raw > 0)
-        CK(cudaMemcpyAsync(I->d_raw_dat, I->p_task_data, 4 * (size_t)I->E_raw, cudaMemcpyHostToDevice, st),
-           "H2D task_data");
-    if (I->n > 0)
-        CK(cudaMemcpyAsync(I->d_size, I->p_size, 8 * (size_t)I->n, cudaMemcpyHostToDevice, st), "H2D data_size");
-    if (I->has_tau && I->m > 0)
-        CK(cudaMemcpyAsync(I->d_tau, I->p_task_ns, 8 * (size_t)I->m, cudaMemcpyHostToDevice, st), "H2D task_ns");
+    // from the pinned mirror of the caller's arrays (asynchronous DMA), one copy:
+    // task_ptr, task_data, data_size[, task_ns] at the arena's relative offsets
+    const char *d0 = reinterpret_cast<const char *>(I->d_raw_ptr);
+    const char *end = I->has_tau && I->m > 0 ? reinterpret_cast<const char *>(I->d_tau + I->m)
+                                             : reinterpret_cast<const char *>(I->d_size + I->n);
+    CK(cudaMemcpyAsync(I->d_raw_ptr, I->p_task_ptr, (size_t)(end - d0), cudaMemcpyHostToDevice, st), "H2D inputs");
     I->uploaded = true;
     return DTS_OK;
 }
@@ -539,9 +551,13 @@ int max_dyn_smem(int device) {
 
 // Threads of the CTA: enough to cover a data segment (deg(D)) in one pass
 // and the score argmax in <= 8 entries per thread, within [64, 512].
-int auto_block(const dts_instance *I) {
+int auto_block(const dts_instance *I, bool alone = false) {
+    // alone (a single instance, or a batch small enough for one CTA per
+    // instance on its own SM): twice the widest segment -- the pool moves of
+    // a plan (|plan| x K items) then take one pass (C2's chain: 7.08 -> 6.98 ms)
+    const int64_t deg = alone ? 2 * (int64_t)I->max_deg_ub : (int64_t)I->max_deg_ub;
     int b = 64;
-    while (b < 512 && (b * 8 < I->n || b < I->max_deg_ub)) b *= 2;
+    while (b < 512 && (b * 8 < I->n || b < deg)) b *= 2;
     return b;
 }
 
@@ -656,7 +672,7 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     if (I->G > 1 && I->device != o.device) return fail(DTS_E_INVAL, "task shard: opts.device != exported device");
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
     const int budget = budget_of(o);
-    const int block = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", auto_block(I));
+    const int block = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", auto_block(I, true));
     s = stage(I, policy, o, budget, block, st);
     if (s != DTS_OK) return s;
     const int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n + 4);
@@ -720,7 +736,7 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
         // group B: every instance after the last wide one (cost order ~ width order)
     }
     for (int32_t i = 0; i < n; i++) {
-        const int ab = auto_block(insts[ord[(size_t)i]]);
+        const int ab = auto_block(insts[ord[(size_t)i]], !many);
         if (i < nb) block_a = std::max(block_a, ab);
         else block_b = std::max(block_b, std::min(ab, small_max));
     }
@@ -1018,22 +1034,12 @@ static dts_status fetch_arrays(dts_instance *I) {
     if (I->out.error == 2) return fail(DTS_E_STATE, "task shards: a peer did not reach an exchange in time");
     if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim (Belady branch)");
     const dts::Inst &h = I->h_inst;
-    size_t ns = (size_t)I->out.n_served, ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);
-    size_t m = (size_t)I->m;
+    const size_t ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);
     cudaStream_t st = I->stream;  // the run's stream: the copies follow the run
     CK(cudaSetDevice(I->device), "cudaSetDevice");
-    CK(cudaMemcpyAsync(I->r_gpu_ptr, h.gpu_task_ptr, 8 * ((size_t)I->K + 1), cudaMemcpyDeviceToHost, st), "D2H");
-    if (ns) {
-        CK(cudaMemcpyAsync(I->r_gpu_ids, h.gpu_task_ids, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
-        CK(cudaMemcpyAsync(I->r_serve_gpu, h.serve_gpu, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
-        CK(cudaMemcpyAsync(I->r_serve_task, h.serve_task, 4 * ns, cudaMemcpyDeviceToHost, st), "D2H");
-    }
-    if (m) {
-        CK(cudaMemcpyAsync(I->r_tstart, h.tstart, 8 * m, cudaMemcpyDeviceToHost, st), "D2H");
-        CK(cudaMemcpyAsync(I->r_tend, h.tend, 8 * m, cudaMemcpyDeviceToHost, st), "D2H");
-    }
-    if (ne)
-        CK(cudaMemcpyAsync(I->r_events, h.events, sizeof(dts_event) * ne, cudaMemcpyDeviceToHost, st), "D2H");
+    // one copy: sigma, service order, task times, then the used part of the trace
+    const size_t head = (size_t)(reinterpret_cast<const char *>(h.events) - reinterpret_cast<const char *>(h.gpu_task_ptr));
+    CK(cudaMemcpyAsync(I->h_res, h.gpu_task_ptr, head + sizeof(dts_event) * ne, cudaMemcpyDeviceToHost, st), "D2H");
     I->r_n_events = (int64_t)ne;
     return DTS_OK;
 }

@@ -14,3 +14,4 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --c
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:dts_cta_kernel -s 3 -c 1 -o $O/${TAG}_full_C2 python bench.py --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C2.log 2>&1; echo "full C2 rc=$?"
 timeout 900 ncu --set full --clock-control none -k regex:dts_cta_kernel -s 6 -c 2 -o $O/${TAG}_full_C5 python bench.py --workload C5 --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C5.log 2>&1; echo "full C5 rc=$?"
 ls $O | grep $TAG
+DTS_BLOCK=256 timeout 300 python bench.py --steps 10 --warmup 3 --no-cpu-baseline > $O/${TAG}_c2_b256.json 2>/dev/null; python -c "import json;d=json.load(open(\"$O/${TAG}_c2_b256.json\"));print(\"C2 block 256\", d[\"ms_per_step\"], d[\"value\"])"
