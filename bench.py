@@ -367,7 +367,7 @@ def main():
             dts.dts_instance_upload(h, dev, sptr)
         step()
         dts.dts_fetch_results(handles)  # all instances' results to host, two waits
-        out = [dts.dts_result(h) for h in handles]
+        out = [dts.dts_result(h, copy=False) for h in handles]  # views of the pinned result buffers
         t1.record(stream)
         t1.synchronize()
         e2e_ms.append(t0.elapsed_time(t1))

@@ -13,6 +13,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <memory>
 #include <vector>
 
 #include "dts.h"
@@ -61,6 +62,22 @@ struct Arena {
 
 }  // namespace
 
+// The events of one batched launch, shared by all its instances: recording
+// two events per instance after a long launch fills the device work queue and
+// blocks the host until the launch ends (4,096 instances: the whole sweep).
+struct SweepEvents {
+    int device = 0;
+    cudaEvent_t begin = nullptr, loop_begin = nullptr, loop_end = nullptr;
+    ~SweepEvents() {
+        int cur = 0;
+        cudaGetDevice(&cur);
+        cudaSetDevice(device);
+        for (cudaEvent_t e : {begin, loop_begin, loop_end})
+            if (e) cudaEventDestroy(e);
+        cudaSetDevice(cur);
+    }
+};
+
 struct dts_instance {
     int32_t m = 0, n = 0, K = 1;
     int64_t E_raw = 0;
@@ -97,6 +114,7 @@ struct dts_instance {
     dts::Inst *d_inst = nullptr;
     cudaStream_t stream = nullptr;
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    std::shared_ptr<SweepEvents> sev;  // set by a batched launch: its events replace ev[]
 
     // run state / results
     bool ran = false;
@@ -568,7 +586,7 @@ int auto_block(const dts_instance *I, bool alone = false) {
 int fused_scratch_bytes(const dts_instance *I, int block) { return (2 * (block / 32) + 1) * 4 * (I->n + 1); }
 
 dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int budget, int block,
-                 cudaStream_t st, bool copy_desc = true) {
+                 cudaStream_t st, bool copy_desc = true, bool own_events = true) {
     dts_status s = ensure_device(I, o.device);
     if (s != DTS_OK) return s;
     CK(cudaSetDevice(o.device), "cudaSetDevice");
@@ -609,7 +627,10 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     const int fs = fused_scratch_bytes(I, block);
     h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
     if (h.fused) h.smem_bytes = std::max(h.smem_bytes, fs);
-    CK(cudaEventRecord(I->ev[0], st), "event");
+    if (own_events) {
+        I->sev.reset();
+        CK(cudaEventRecord(I->ev[0], st), "event");
+    }
     if (!h.fused)
         CK(dts::build_csr(I->d_raw_ptr, I->d_raw_dat, I->m, I->n, I->E_raw, (int64_t *)h.tptr,
                           (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, (int4 *)h.dedge,
@@ -743,9 +764,16 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     if (forced) block_a = block_b = forced;
     int smem_a = 0, smem_b = 0;
     bool any_unfused = false;
+    auto sev = std::make_shared<SweepEvents>();
+    sev->device = o.device;
+    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    CK(cudaEventCreate(&sev->begin), "cudaEventCreate");
+    CK(cudaEventCreate(&sev->loop_begin), "cudaEventCreate");
+    CK(cudaEventCreate(&sev->loop_end), "cudaEventCreate");
+    CK(cudaEventRecord(sev->begin, st), "event");
     for (int32_t i = 0; i < n; i++) {
         dts_instance *I = insts[ord[(size_t)i]];
-        s = stage(I, policy, o, budget, i < nb ? block_a : block_b, st, false);
+        s = stage(I, policy, o, budget, i < nb ? block_a : block_b, st, false, false);
         if (s != DTS_OK) return s;
         (i < nb ? smem_a : smem_b) = std::max(i < nb ? smem_a : smem_b, I->h_inst.smem_bytes);
         any_unfused |= !I->h_inst.fused;
@@ -777,7 +805,7 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     CK(cudaEventRecord(B.copied[sl], st), "event");
     CK(cudaMemsetAsync(B.d_work, 0, 2 * sizeof(int), st), "memset");
     if (any_unfused) CK(dts::launch_init(B.d_insts, n, o.bus_bytes_per_s, work, st), "init");
-    for (int32_t i = 0; i < n; i++) CK(cudaEventRecord(insts[i]->ev[1], st), "event");
+    CK(cudaEventRecord(sev->loop_begin, st), "event");
     const bool two = nb > 0 && nb < n;
     if (two) {  // group B on the side stream, forked from and joined back into st
         CK(cudaEventRecord(B.fork, st), "event");
@@ -794,9 +822,9 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
     const int grid = (int)std::min<int64_t>((int64_t)na, (int64_t)per * nsm);
     CK(dts::launch_loop(B.d_insts, na, blk, grid, B.d_work, sm, st), "loop");
     if (two) CK(cudaStreamWaitEvent(st, B.join, 0), "wait");
+    CK(cudaEventRecord(sev->loop_end, st), "event");
     for (int32_t i = 0; i < n; i++) {
-        CK(cudaEventRecord(insts[i]->ev[2], st), "event");
-        CK(cudaEventRecord(insts[i]->ev[3], st), "event");
+        insts[i]->sev = sev;
         insts[i]->ran = true;
     }
     return DTS_OK;
@@ -1044,8 +1072,13 @@ static dts_status fetch_arrays(dts_instance *I) {
     return DTS_OK;
 }
 static dts_status fetch_done(dts_instance *I) {
-    CK(cudaEventElapsedTime(&I->loop_ms, I->ev[1], I->ev[2]), "elapsed");
-    CK(cudaEventElapsedTime(&I->total_ms, I->ev[0], I->ev[3]), "elapsed");
+    if (I->sev) {
+        CK(cudaEventElapsedTime(&I->loop_ms, I->sev->loop_begin, I->sev->loop_end), "elapsed");
+        CK(cudaEventElapsedTime(&I->total_ms, I->sev->begin, I->sev->loop_end), "elapsed");
+    } else {
+        CK(cudaEventElapsedTime(&I->loop_ms, I->ev[1], I->ev[2]), "elapsed");
+        CK(cudaEventElapsedTime(&I->total_ms, I->ev[0], I->ev[3]), "elapsed");
+    }
     I->have_host = true;
     return DTS_OK;
 }

@@ -259,21 +259,30 @@ class Result:
         return [self.gpu_task_ids[p[k]:p[k + 1]] for k in range(self.K)]
 
 
-def _arr(ptr, n, dtype):
+def _arr(ptr, n, dtype, copy=True):
     if n == 0 or not ptr:
         return np.zeros(0, dtype)
     buf = (C.c_char * (int(n) * np.dtype(dtype).itemsize)).from_address(ptr)
-    return np.frombuffer(buf, dtype=dtype).copy()
+    a = np.frombuffer(buf, dtype=dtype)
+    if copy:
+        return a.copy()
+    a.flags.writeable = False
+    return a
 
 
-def dts_result(inst: Instance) -> Result:
+def dts_result(inst: Instance, copy: bool = True) -> Result:
+    """The run's results.  copy=False returns read-only numpy views of the
+    library's pinned host buffers instead of copies (no host memcpy): like the
+    C ABI's dts_result_view they stay valid until the instance runs again or is
+    destroyed."""
     v = dts_result_view()
     _check(load_library().dts_result(inst.handle, C.byref(v)))
     ns = int(v.n_served)
-    return Result(int(v.K), _arr(v.gpu_task_ptr, v.K + 1, np.int64), _arr(v.gpu_task_ids, ns, np.int32),
-                  _arr(v.serve_gpu, ns, np.int32), _arr(v.serve_task, ns, np.int32),
-                  _arr(v.task_start_ns, v.n_tasks, np.int64), _arr(v.task_end_ns, v.n_tasks, np.int64),
-                  _arr(v.events, v.n_events, EVENT_DTYPE), int(v.bytes_loaded), int(v.n_loads),
+    A = (lambda p, n, dt: _arr(p, n, dt, copy))
+    return Result(int(v.K), A(v.gpu_task_ptr, v.K + 1, np.int64), A(v.gpu_task_ids, ns, np.int32),
+                  A(v.serve_gpu, ns, np.int32), A(v.serve_task, ns, np.int32),
+                  A(v.task_start_ns, v.n_tasks, np.int64), A(v.task_end_ns, v.n_tasks, np.int64),
+                  A(v.events, v.n_events, EVENT_DTYPE), int(v.bytes_loaded), int(v.n_loads),
                   int(v.n_evictions), int(v.makespan_ns), float(v.makespan_s), ns, int(v.n_scans),
                   int(v.n_fallback2), int(v.n_fallback_first), int(v.n_belady),
                   int(v.n_idle_requests), int(v.n_verify_err), int(v.alg_bytes),

@@ -515,3 +515,18 @@ def test_fetch_results_matches_per_instance_result():
         assert np.array_equal(x.serve_task, y.serve_task) and np.array_equal(x.events, y.events)
         assert_parity(x, oracle.run(inst))
 
+
+
+def test_result_views_without_copy():
+    """dts_result(copy=False): read-only views of the pinned result buffers,
+    equal to the copies, valid until the instance runs again."""
+    insts = gen.config_instances("C2")[:4]
+    hs = [dts.create(i) for i in insts]
+    dts.dts_sweep_run(hs, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default())
+    dts.dts_fetch_results(hs)
+    for h, inst in zip(hs, insts):
+        v = dts.dts_result(h, copy=False)
+        c = dts.dts_result(h)
+        assert not v.serve_task.flags.writeable
+        assert np.array_equal(v.serve_task, c.serve_task) and np.array_equal(v.events, c.events)
+        assert_parity(v, oracle.run(inst))
