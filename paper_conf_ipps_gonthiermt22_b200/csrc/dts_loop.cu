@@ -369,6 +369,33 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
     }
 }
 
+// One (task, GPU) item of pool_move_many in the packed-state mode, out of line
+// (keeps the hot row-derived loop compact).
+__device__ __noinline__ void pool_item_packed(int4 e, int j, int sign) {
+    const Inst &I = SI;
+    const View &V = SV;
+    const int32_t T = e.x;
+    uint32_t *sp = &V.s[(size_t)j * I.m_pad + T];
+    const uint32_t w = *sp;
+    *sp = sign < 0 ? (w | ALLOC_BIT) : (w & ~ALLOC_BIT);
+    const uint32_t c = (w >> 24) & 0x7fu;
+    if (c == 1u) {
+        atomicAdd(&V.h[(size_t)j * I.nstr + (w & XOR_MASK)], sign);
+    } else if (c == 2u) {
+        int32_t a, b;
+        const bool lng = e.w == ROW_LONG;
+        const int len = lng ? 4 : (e.y >= 0) + (e.z >= 0) + (e.w >= 0);
+        if (len == 2) {  // both inputs miss: no residency lookups
+            a = e.y;
+            b = e.z >= 0 ? e.z : e.w;
+        } else {
+            missing_pair(j, T, Row{e.y, e.z, lng ? -1 : e.w, len}, -1, a, b);
+        }
+        atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+        atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
+    }
+}
+
 // Block-wide pool_move of P tasks given as plan entries {T, D0, D1, D2}
 // (-1 = absent input, D2 = ROW_LONG: read the row from the CSR).  The
 // (task, simulated GPU) state items and the per-task input counts (u, np) are
@@ -397,25 +424,7 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
                 continue;
             }
             if (T < I.t_lo || T >= I.t_hi) continue;  // another shard's task
-            uint32_t *sp = &V.s[(size_t)j * I.m_pad + T];
-            const uint32_t w = *sp;
-            *sp = sign < 0 ? (w | ALLOC_BIT) : (w & ~ALLOC_BIT);
-            const uint32_t c = (w >> 24) & 0x7fu;
-            if (c == 1u) {
-                atomicAdd(&V.h[(size_t)j * I.nstr + (w & XOR_MASK)], sign);
-            } else if (c == 2u) {
-                int32_t a, b;
-                const bool lng = e.w == ROW_LONG;
-                const int len = lng ? 4 : (e.y >= 0) + (e.z >= 0) + (e.w >= 0);
-                if (len == 2) {  // both inputs miss: no residency lookups
-                    a = e.y;
-                    b = e.z >= 0 ? e.z : e.w;
-                } else {
-                    missing_pair(j, T, Row{e.y, e.z, lng ? -1 : e.w, len}, -1, a, b);
-                }
-                atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
-                atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
-            }
+            pool_item_packed(e, j, sign);
         } else {
             const int4 e = ents[idx - n_state];
             const int32_t T = e.x;
@@ -463,13 +472,9 @@ __device__ __forceinline__ void row_from_entry(int4 e) {
     L.row_len = len;
 }
 
-// a2: datum D becomes resident (load) / leaves (evict) on GPU k.  Walk D's
-// data->task segment (edge records: the task and its other inputs in one 16 B
-// load): cnt_k(T) -/+= 1, x_k(T) ^= D, and move every unallocated task between
-// the score buckets h (cnt 1) and h2 (cnt 2).  The residency bit of D is
-// already updated.  Each task appears once in the segment, so the state words
-// are plain read-modify-writes; the buckets are atomics.
-__device__ void seg_update(int k, int32_t D, bool load) {
+// Packed-state mode of seg_update, out of line: the hot row-derived path stays
+// compact (the loop kernel is instruction-cache bound).
+__device__ __noinline__ void seg_update_packed(int k, int32_t D, bool load) {
     const Inst &I = SI;
     const View &V = SV;
     int64_t b, e;
@@ -477,39 +482,6 @@ __device__ void seg_update(int k, int32_t D, bool load) {
     uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int32_t *hk = V.h + (size_t)k * I.nstr;
     int32_t *h2k = V.h2 + (size_t)k * I.nstr;
-    if (I.sl) {  // row-derived state: cnt_k(T) before the change from T's other inputs
-        for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
-            const int4 ed = __ldg(&I.dedge[i]);
-            if (allocated(ed.x)) continue;
-            const bool my = ed.y >= 0 && !resident(k, ed.y), mz = ed.z >= 0 && !resident(k, ed.z);
-            const int c = (int)my + (int)mz + (load ? 1 : 0);  // missing inputs before
-            const int32_t o = my ? ed.y : ed.z;                 // the other missing one (c == 2 / 1)
-            if (load) {
-                if (c == 1) {  // 1 -> 0
-                    atomicSub(&hk[D], 1);
-                } else if (c == 2) {  // 2 -> 1: now freed by o
-                    atomicSub(&h2k[D], 1);
-                    atomicSub(&h2k[o], 1);
-                    atomicAdd(&hk[o], 1);
-                } else if (c == 3) {  // 3 -> 2
-                    atomicAdd(&h2k[ed.y], 1);
-                    atomicAdd(&h2k[ed.z], 1);
-                }
-            } else {
-                if (c == 0) {  // 0 -> 1
-                    atomicAdd(&hk[D], 1);
-                } else if (c == 1) {  // 1 -> 2: missing {o, D}
-                    atomicSub(&hk[o], 1);
-                    atomicAdd(&h2k[o], 1);
-                    atomicAdd(&h2k[D], 1);
-                } else if (c == 2) {  // 2 -> 3
-                    atomicSub(&h2k[ed.y], 1);
-                    atomicSub(&h2k[ed.z], 1);
-                }
-            }
-        }
-        return;
-    }
     for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
         const int4 ed = __ldg(&I.dedge[i]);
         const int32_t T = ed.x;
@@ -546,6 +518,59 @@ __device__ void seg_update(int k, int32_t D, bool load) {
                 atomicSub(&h2k[b2], 1);
             }
         }
+    }
+}
+
+
+// a2: datum D becomes resident (load) / leaves (evict) on GPU k.  Walk D's
+// data->task segment (edge records: the task and its other inputs in one 16 B
+// load): cnt_k(T) -/+= 1, x_k(T) ^= D, and move every unallocated task between
+// the score buckets h (cnt 1) and h2 (cnt 2).  The residency bit of D is
+// already updated.  Each task appears once in the segment, so the state words
+// are plain read-modify-writes; the buckets are atomics.
+__device__ void seg_update(int k, int32_t D, bool load) {
+    const Inst &I = SI;
+    const View &V = SV;
+    if (!I.sl) {
+        seg_update_packed(k, D, load);
+        return;
+    }
+    int64_t b, e;
+    seg_of(D, b, e);
+    int32_t *hk = V.h + (size_t)k * I.nstr;
+    int32_t *h2k = V.h2 + (size_t)k * I.nstr;
+    {  // row-derived state: cnt_k(T) before the change from T's other inputs
+        for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
+            const int4 ed = __ldg(&I.dedge[i]);
+            if (allocated(ed.x)) continue;
+            const bool my = ed.y >= 0 && !resident(k, ed.y), mz = ed.z >= 0 && !resident(k, ed.z);
+            const int c = (int)my + (int)mz + (load ? 1 : 0);  // missing inputs before
+            const int32_t o = my ? ed.y : ed.z;                 // the other missing one (c == 2 / 1)
+            if (load) {
+                if (c == 1) {  // 1 -> 0
+                    atomicSub(&hk[D], 1);
+                } else if (c == 2) {  // 2 -> 1: now freed by o
+                    atomicSub(&h2k[D], 1);
+                    atomicSub(&h2k[o], 1);
+                    atomicAdd(&hk[o], 1);
+                } else if (c == 3) {  // 3 -> 2
+                    atomicAdd(&h2k[ed.y], 1);
+                    atomicAdd(&h2k[ed.z], 1);
+                }
+            } else {
+                if (c == 0) {  // 0 -> 1
+                    atomicAdd(&hk[D], 1);
+                } else if (c == 1) {  // 1 -> 2: missing {o, D}
+                    atomicSub(&hk[o], 1);
+                    atomicAdd(&h2k[o], 1);
+                    atomicAdd(&h2k[D], 1);
+                } else if (c == 2) {  // 2 -> 3
+                    atomicSub(&h2k[ed.y], 1);
+                    atomicSub(&h2k[ed.z], 1);
+                }
+            }
+        }
+        return;
     }
 }
 

@@ -12,7 +12,8 @@ import paper_conf_ipps_gonthiermt22_b200 as dts  # noqa: E402
 NAMES = ["pop", "argmax", "plan", "serve_loads", "luf", "evict", "seg_load", "other"]
 SETS = {"c2": lambda: [gen.config_instances("C2")[19], gen.config_instances("C2")[18]],
         "c3": lambda: [gen.config_instances("C3")[0]],
-        "c5long": lambda: [gen.sweep_instance(160, 4, 7), gen.sweep_instance(160, 6, 6)],
+        "c5long": lambda: [gen.sweep_instance(160, 4, 7), gen.sweep_instance(160, 6, 6),
+                           gen.sweep_instance(160, 4, 1)],
         "c4": lambda: [gen.config_instances("C4a")[0], gen.config_instances("C4b")[0]]}
 prof = os.environ.get("DTS_PROFILE") == "1"
 for name in (sys.argv[1:] or ["c2", "c3", "c5long"]):

@@ -12,7 +12,7 @@ NAMES = ["pop", "argmax", "plan", "serve_loads", "luf", "evict", "seg_load", "ot
          "nb", "np", "x1", "x2", "x3", "x4"]
 SETS = {"c2": [gen.config_instances("C2")[19], gen.config_instances("C2")[18]],
         "c3": [gen.config_instances("C3")[0]],
-        "c5long": [gen.sweep_instance(160, 4, 7), gen.sweep_instance(160, 6, 6)]}
+        "c5long": [gen.sweep_instance(160, 4, 7), gen.sweep_instance(160, 4, 1)]}
 for name in (sys.argv[1:] or ["c2", "c3"]):
     for inst in SETS[name]:
         dts.schedule(inst)
