@@ -52,7 +52,7 @@ class _Result(C.Structure):
                 ("n_evictions", C.c_int64), ("n_scans", C.c_int64), ("n_fallback2", C.c_int64),
                 ("n_fallback_first", C.c_int64), ("n_belady", C.c_int64),
                 ("n_idle_requests", C.c_int64), ("bytes_loaded", C.c_uint64),
-                ("makespan", C.c_int64)]
+                ("makespan", C.c_int64), ("n_wakes", C.c_int64)]
 
 
 _lib = None
@@ -61,7 +61,9 @@ _lib = None
 def _load():
     global _lib
     if _lib is None:
-        _lib = C.CDLL(build())
+        # DTS_ORACLE_LIB: a deliberately mutated build of dts_oracle.c
+        # (tools/oracle_mutants.py checks that the pins reject it)
+        _lib = C.CDLL(os.environ.get("DTS_ORACLE_LIB") or build())
         _lib.or_run.restype = C.c_int
         _lib.or_run.argtypes = [C.c_int32, C.c_int32, C.c_void_p, C.c_void_p, C.c_void_p,
                                 C.c_void_p, C.c_int64, C.c_uint64, C.c_int32, C.c_int32,
@@ -88,6 +90,7 @@ class OracleResult:
     bytes_loaded: int
     makespan: int
     K: int
+    n_wakes: int = 0
 
     def orders(self):
         """Per-GPU task order sigma(k, .)."""
@@ -121,4 +124,4 @@ def run(inst, W: int = 0, flags: int = F_FALLBACK2, bus_bps: int = DEFAULT_BUS_B
     return OracleResult(sg[:ns].copy(), st[:ns].copy(), ts[:m].copy(), te[:m].copy(),
                         ev[:r.n_events].copy(), ns, r.n_loads, r.n_evictions, r.n_scans,
                         r.n_fallback2, r.n_fallback_first, r.n_belady, r.n_idle_requests,
-                        r.bytes_loaded, r.makespan, int(inst.K))
+                        r.bytes_loaded, r.makespan, int(inst.K), r.n_wakes)

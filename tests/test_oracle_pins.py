@@ -142,6 +142,7 @@ def test_p5_invariants(idx, W):
     assert chk["n_loads"] == r.n_loads and chk["n_evictions"] == r.n_evictions
     assert chk["bytes_loaded"] == r.bytes_loaded and chk["makespan"] == r.makespan
     assert r.n_belady == 0  # unreachable with the capacity check (reading R7)
+    assert r.n_wakes == 0   # unreachable (reading R18)
     assert sum(len(o) for o in r.orders()) == inst.m
 
 
@@ -284,3 +285,61 @@ def test_eager_lru_collapse_when_one_matrix_fits():
     eager = oracle.run(inst, flags=oracle.POLICY_FLAGS["eager_lru"])
     darts = oracle.run(inst)
     assert eager.n_loads > 2 * darts.n_loads
+
+
+# ------------------------------------------------ F1: the 3inputs fallback (§V-E)
+def f1_instance(g=None):
+    """The hand-traced fallback instance of tests/golden/f1_fallback2_hand.json
+    (unit sizes, delta = tau = 1 tick)."""
+    g = g or _golden("f1_fallback2_hand.json")
+    rows = g["rows"]
+    tp = np.zeros(len(rows) + 1, np.int64)
+    tp[1:] = np.cumsum([len(r) for r in rows])
+    td = np.array([d for r in rows for d in r], np.int32)
+    return gen.Instance("f1_fallback2", tp, td, np.ones(g["data"], np.uint64), None, g["tau"],
+                        g["M"], g["K"])
+
+
+def test_f1_fallback2_hand_trace():
+    """Pins the 3inputs scoring (readings R6, R24): n2
+    credits both missing inputs, the key is (n2, u, -id), the task is the
+    lowest-id one with D2 and one other input missing.  Each plausible
+    mistake changes the first pick (see the golden's derivation)."""
+    g = _golden("f1_fallback2_hand.json")
+    inst = f1_instance(g)
+    r = oracle.run(inst, bus_bps=10 ** 9)
+    assert list(map(int, r.orders()[0])) == g["order"]
+    ev = [["L" if e["op"] == 0 else "E", int(e["data"]), int(e["task"]), int(e["t"]), int(e["t_end"])]
+          for e in r.events]
+    assert ev == g["events"]
+    assert (r.n_loads, r.n_evictions, r.n_scans) == (g["n_loads"], g["n_evictions"], g["n_scans"])
+    assert (r.n_fallback2, r.n_fallback_first) == (g["n_fallback2"], g["n_fallback_first"])
+    assert r.n_idle_requests == g["n_idle_requests"] and r.n_served - r.n_scans == g["pops"]
+    assert r.makespan == g["makespan"]
+    _check(inst, r, bus=10 ** 9)
+
+
+def test_f1_fallback_off_takes_lowest_id_task():
+    """Without the 3inputs variant the first request falls to Alg. 5 l.13
+    (R5): the lowest-id available task, T0, which does not use D2 = D5."""
+    inst = f1_instance()
+    r = oracle.run(inst, bus_bps=10 ** 9, flags=0)
+    assert int(r.serve_task[0]) == 0 and r.n_fallback_first >= 1 and r.n_fallback2 == 0
+    _check(inst, r, bus=10 ** 9)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_r18_idle_wake_never_fires(seed):
+    """Reading R18 (wake idle GPUs when LUF returns planned tasks, Alg. 6
+    l.8) is unreachable: a return happens while serving the first task of a
+    plan made at the same request out of a non-empty pool, an idle GPU saw
+    an empty pool, and the pool refills only by returns.  Checked here on
+    small random instances with K = 2..4 and tight memory (many returns)."""
+    K = 2 + seed % 3
+    inst = _tiny(2000 + seed, m=40 + seed, n=12, K=K, M=3 + seed % 2)
+    for W in (0, 1):
+        if W and inst.mem_capacity < 6:
+            continue
+        for flags in (oracle.F_FALLBACK2, 0, oracle.F_FALLBACK2 | oracle.F_OPTI):
+            r = oracle.run(inst, W=W, bus_bps=10 ** 9, flags=flags)
+            assert r.n_wakes == 0 and r.n_served == inst.m
