@@ -7,20 +7,26 @@
 A *step* is one pass of the whole hot path (device CSR
 build, state init, the device-resident DARTS+LUF decision loop, result
 assembly) over one batch of synthetic instances.  Default workload = BASELINE
-config 2 (configs[1]): the 20 2D tiled-matmul instances N = 10..100 (step 10)
-x K in {2, 4} simulated GPUs, M = 35 data (500 MiB) per simulated GPU, all
-scheduled by ONE batched launch (one CTA per instance).
+config 4, the largest single-GPU configuration: the Cholesky task set (C4a,
+1,004,731 tasks) and the random shared-input task set (C4b, 2^20 tasks x 3
+inputs), K = 8 simulated GPUs, both scheduled by ONE batched launch of the
+decision loop (one CTA each, dts_sweep_run).  C1, C2, C3, C4a, C4b and C5
+are available with --workload.
 
-Multi-GPU (torchrun, one process per B200): each rank schedules its own copy
-of the batch -- independent problems, no data-path collective -- so scaling
-is "weak"; C5 (the 4,096-instance sweep) is sharded across ranks instead
-("strong").  Time = max over ranks of the device time (CUDA events).
+Multi-GPU (torchrun, one process per B200): independent instances need no
+communication; C4, C2 and the single-instance workloads
+run one copy per rank ("weak": replicas only -- one instance's decisions are
+a sequential chain), C5 (the 4,096-instance sweep) is sharded across ranks
+by LPT ("strong").  Time = max over ranks of the device time (CUDA events).
 
 value = decisions/s (served requests, reading R21) over all ranks, inputs
-resident in HBM.  e2e = the same through the public API with the host->device
-upload of every instance and the device->host read of every result inside
-the timed region.  --impl reference times the plain CPU oracle (oracle/) on
-the host cores instead (the reference arm for this tier).
+resident in HBM.  e2e = the same through the public API from the caller's
+host arrays: dts_instance_create (validation + copy), upload, run, the
+device->host read of every result and dts_instance_destroy inside the timed
+region (C5: instances created once, see e2e.scope).  roofline = SURVEY.md
+§8(d)'s algorithmic bytes of the loop kernel (from the kernel's counters,
+DESIGN.md "Roofline") / its device time.  --impl reference times the plain
+CPU oracle (oracle/) on the host cores instead (the reference arm).
 """
 from __future__ import annotations
 
@@ -50,6 +56,8 @@ WORKLOADS = {
     "C3": "3D tiled matmul N=40 (64,000 tasks, 3,200 tiles), K=4, M=142 tiles (500 MiB)",
     "C4a": "Cholesky task set N=181 tiles (1,004,731 tasks, 16,471 tiles), K=8, M=142",
     "C4b": "random shared-input tasks (2^20 tasks x 3 inputs over 2^14 data), K=8, M=1024",
+    "C4": "config 4: Cholesky task set N=181 (C4a, 1,004,731 tasks, M=142) + random shared-input "
+          "tasks (C4b, 2^20 x 3 inputs, M=1024), K=8, one batched launch",
     "C5": "sweep of 4,096 2D instances (N 5..160 x M 4..128 x K 1..8), sharded over ranks",
 }
 
@@ -64,14 +72,25 @@ def _peaks():
 
 
 def _traffic(workload):
-    """Per-launch DRAM bytes of the loop kernel from the committed ncu --set full
-    summary (profiles/ncu_full_<workload>.json), else None."""
+    """Per-launch DRAM bytes (dram__bytes_read.sum + dram__bytes_write.sum) of
+    the loop kernel from the committed ncu --set full summary of this round's
+    build (profiles/ncu_full_<workload>.json, tools/ncu_summary.py), else None."""
     p = os.path.join(ROOT, "profiles", f"ncu_full_{workload}.json")
     try:
         d = json.load(open(p))
         return int(d["dram_bytes_per_launch"])
     except Exception:
         return None
+
+
+def bytes_8d(r, inst):
+    """SURVEY.md §8(d) algorithmic bytes of one instance's decision loop
+    (DESIGN.md "Roofline"): per scan 4 m_avail + 4.125 n, per load / evict of
+    D 12 deg(D), per allocated task 4 K + 8 E/m -- from the kernel's counters
+    (parity-tested against the oracle's)."""
+    abar = inst.E / max(inst.m, 1)
+    return (4.0 * r.sum_avail_at_scans + 4.125 * inst.n * r.n_scans
+            + 12.0 * r.sum_deg_loads_evictions + (4.0 * inst.K + 8.0 * abar) * r.n_allocations)
 
 
 class Clocks:
@@ -142,6 +161,8 @@ class Clocks:
 
 
 def workload_instances(name, rank, world):
+    if name == "C4":
+        return gen.config_instances("C4a") + gen.config_instances("C4b"), "weak"
     if name == "C5":
         from paper_conf_ipps_gonthiermt22_b200.shard import instance_cost, shard
         params = gen.sweep_params()
@@ -196,7 +217,7 @@ def run_reference(args, rank, world):
         return
     insts, scaling = workload_instances(args.workload, 0, 1)
     cores = os.cpu_count() or 1
-    big = args.workload in ("C4a", "C4b")
+    big = args.workload in ("C4a", "C4b", "C4")
     for _ in range(args.warmup):
         if big:
             oracle_prefix_sample(insts[0], 2.0)
@@ -205,8 +226,14 @@ def run_reference(args, rank, world):
     times, decs = [], []
     for _ in range(args.steps):
         if big:
-            rate, dt, nd = oracle_prefix_sample(insts[0], 8.0)
-            sample = f"prefix of {nd} served requests of {insts[0].name}, 1 thread"
+            dt = nd = 0
+            parts = []
+            for inst in insts:  # C4: a prefix of each instance
+                _, dti, ndi = oracle_prefix_sample(inst, 8.0 / len(insts))
+                dt += dti
+                nd += ndi
+                parts.append(f"{ndi} of {inst.name}")
+            sample = "prefix of the served requests (" + ", ".join(parts) + "), 1 thread"
             thr = 1
         else:
             sub = insts if args.workload != "C5" else insts[::16]
@@ -236,7 +263,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="C2", choices=list(WORKLOADS))
+    ap.add_argument("--workload", default="C4", choices=list(WORKLOADS))
     ap.add_argument("--policy", default="darts_luf", choices=["darts_luf", "darts_lru", "eager_lru"],
                     help="DARTS+LUF (the method) or a comparison policy of the paper")
     ap.add_argument("--opti", action="store_true", help="OPTI variant (PAPER.md:2121-2124)")
@@ -329,7 +356,7 @@ def main():
     # ---- device-resident timed region
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
            for _ in range(args.steps)]
-    loop_ms, alg_bytes, launches = [], [], 0
+    loop_ms_steps = []
     barrier()
     with Clocks(dev) as clk:
         l0 = dts.dts_kernel_launches()
@@ -338,22 +365,26 @@ def main():
             evs[i][0].record(stream)
             step()
             evs[i][1].record(stream)
+            # the loop kernel's own launch time (library events on the same
+            # stream); waits for this step, so the next step's enqueue starts
+            # after it -- outside both events
+            loop_ms_steps.append(max(dts.dts_run_times(h)[0] for h in handles))
         barrier()
         launches = dts.dts_kernel_launches() - l0
-        flush_launches = 0
     step_ms = [a.elapsed_time(b) for a, b in evs]
     rs = [dts.dts_result(h) for h in handles]  # last step's results (after the region)
-    loop_ms = max(r.loop_ms for r in rs)
+    loop_ms = sum(loop_ms_steps) / len(loop_ms_steps)
     alg = sum(r.alg_bytes for r in rs)
-    scan_alg = sum(r.scan_alg_bytes for r in rs)
+    # §8(d) bytes of one launch (a task-sharded group counts the instance once)
+    b8d = sum(bytes_8d(r, i) for r, i in zip(rs, insts if not (gsh or xsh) else insts[:1]))
     bytes_loaded = sum(r.bytes_loaded for r in rs)
     n_loads = sum(r.n_loads for r in rs)
     n_scans = sum(r.n_scans for r in rs)
-    # per-step loop time: re-measure the loop kernel's own events over the timed steps
     ms = sum(step_ms) / len(step_ms)
 
-    # ---- e2e: host arrays -> device, run, results -> host, every step
+    # ---- e2e: the public API from the caller's host arrays, every step
     e2e_ms = []
+    create_each_step = args.workload != "C5" and not (gsh or xsh)
     h2d = sum(8 * (i.m + 1) + 4 * i.E + 8 * i.n + (8 * i.m if i.task_ns is not None else 0)
               for i in insts) * (args.shards if gsh else 1)
     d2h = 0
@@ -363,16 +394,31 @@ def main():
         t1 = torch.cuda.Event(enable_timing=True)
         flush.zero_()
         t0.record(stream)
-        for h in handles:
-            dts.dts_instance_upload(h, dev, sptr)
-        step()
-        dts.dts_fetch_results(handles)  # all instances' results to host, two waits
-        out = [dts.dts_result(h, copy=False) for h in handles]  # views of the pinned result buffers
+        if create_each_step:  # create (host validation + copy) .. destroy, all timed
+            hs = [dts.create(x) for x in insts]
+            for h in hs:
+                dts.dts_instance_upload(h, dev, sptr)
+            if single:
+                for h in hs:
+                    dts.dts_run(h, policy, opts)
+            else:
+                dts.dts_sweep_run(hs, policy, opts)
+        else:
+            hs = handles
+            for h in hs:
+                dts.dts_instance_upload(h, dev, sptr)
+            step()
+        dts.dts_fetch_results(hs)  # all instances' results to host, two waits
+        out = [dts.dts_result(h, copy=False) for h in hs]  # views of the pinned result buffers
+        d2h = sum(8 * (r.K + 1) + 4 * r.n_served * 3 + 16 * len(r.task_start) + 32 * len(r.events)
+                  + 128 for r in out)
+        assert sum(r.n_served for r in out) == decisions or xsh or gsh
+        del out
+        if create_each_step:
+            del hs  # dts_instance_destroy (inside the timed region)
         t1.record(stream)
         t1.synchronize()
         e2e_ms.append(t0.elapsed_time(t1))
-        d2h = sum(8 * (r.K + 1) + 4 * r.n_served * 3 + 16 * len(r.task_start) + 32 * len(r.events)
-                  + 128 for r in out)
     e2e_avg = sum(e2e_ms) / len(e2e_ms)
 
     # ---- max over ranks (device times), sum of the work
@@ -382,14 +428,20 @@ def main():
 
     if rank == 0:
         peak, peak_src = _peaks()
-        achieved = (alg / 1e9) / (loop_ms / 1e3) if loop_ms > 0 else 0.0  # GB/s, this rank
+        achieved = (b8d / 1e9) / (loop_ms / 1e3) if loop_ms > 0 else 0.0  # GB/s, this rank's launch
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
             cores = os.cpu_count() or 1
-            if args.workload in ("C4a", "C4b", "C3"):
-                rate, dt, nd = oracle_prefix_sample(insts[0], args.cpu_budget)
-                cpu = {"value": rate, "unit": UNIT, "cores": 1, "kind": "oracle",
-                       "sample": f"prefix of {nd} served requests of {insts[0].name} ({dt:.1f} s, 1 thread)"}
+            if args.workload in ("C4a", "C4b", "C3", "C4"):
+                nd, dt, parts = 0, 0.0, []
+                for inst in insts:
+                    _, dti, ndi = oracle_prefix_sample(inst, args.cpu_budget / len(insts))
+                    nd += ndi
+                    dt += dti
+                    parts.append(f"{ndi} of {inst.name}")
+                cpu = {"value": nd / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+                       "sample": "prefix of the served requests (" + ", ".join(parts)
+                                 + f"; {dt:.1f} s, 1 thread)"}
             else:
                 sub = insts if args.workload != "C5" else insts[::16]
                 rate, dt, nb, nd = oracle_sample(sub, args.cpu_budget, cores)
@@ -397,6 +449,13 @@ def main():
                        "sample": f"{nb} passes over {len(sub)} instances of {args.workload}"
                                  f" ({nd} decisions, {dt:.1f} s, one instance per thread)"}
         clocks = clk.summary()
+        launch = ("one batched loop launch, one CTA per instance" if len(insts) < 296 else
+                  "two concurrent batched loop launches (256-thread CTAs for the long-segment "
+                  "instances, <= 128 for the rest), one CTA per instance") if not single \
+            else (f"one cooperative launch: the instance task-sharded over {args.shards} CTAs"
+                  if gsh else f"one loop launch per rank: the instance task-sharded over "
+                  f"{world} B200s, peer-memory exchanges" if xsh
+                  else "one loop launch (one CTA) per instance")
         line = {
             "metric": METRIC, "value": all_dec / (ms / 1e3), "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
@@ -405,24 +464,24 @@ def main():
             "config": {"workload": f"{args.workload}: {WORKLOADS[args.workload]}",
                        "policy": args.policy + ("+opti" if args.opti else "") + " (3inputs fallback on)",
                        "instances_per_rank": len(insts), "decisions_per_step": int(all_dec),
-                       "l2": "flushed between timed steps (256 MiB write)",
-                       "launch": ("one batched loop launch, one CTA per instance" if len(insts) < 296 else
-                                  "two concurrent batched loop launches (256-thread CTAs for the long-segment "
-                                  "instances, <= 128 for the rest), one CTA per instance") if not single
-                       else (f"one cooperative launch: the instance task-sharded over {args.shards} CTAs"
-                             if gsh else f"one loop launch per rank: the instance task-sharded over "
-                             f"{world} B200s, peer-memory exchanges" if xsh
-                             else "one loop launch (one CTA) per instance")},
+                       "l2": "flushed between timed steps (256 MiB write)", "launch": launch},
             "e2e": {"value": all_dec / (e2e_avg / 1e3), "unit": UNIT,
-                    "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h)},
+                    "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+                    "scope": ("dts_instance_create from host arrays, upload, run, result D2H, destroy"
+                              if create_each_step else
+                              "upload (from the library's pinned copy), run, result D2H; "
+                              "instances created once outside the timed region")},
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": _traffic(args.workload),
                          "kernel": "dts_cta_kernel", "peak_source": peak_src,
-                         "alg_bytes_per_launch": int(alg), "launch_ms": loop_ms},
-            "hbm_gbs": achieved,
+                         "bytes": "SURVEY.md §8(d) algorithmic bytes per launch: 4*sum(m_avail at scans)"
+                                  " + 4.125*n*scans + 12*sum(deg over loads/evictions)"
+                                  " + (4K + 8E/m)*allocations (kernel counters = oracle counters)",
+                         "alg_bytes_per_launch": int(b8d), "launch_ms": loop_ms,
+                         "launch_ms_steps": [round(x, 3) for x in loop_ms_steps],
+                         "kernel_model_bytes_per_launch": int(alg)},
             "bytes_loaded": int(bytes_loaded), "n_loads": int(n_loads), "n_scans": int(n_scans),
-            "scan_alg_bytes_per_launch": int(scan_alg),
             "cpu_baseline": cpu,
             "clocks": clocks,
         }

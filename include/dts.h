@@ -183,10 +183,25 @@ typedef struct {
     int64_t prof_cycles[16];        /* diagnostics: SM cycles of the loop per phase (pop, argmax,
                                       plan, serve-with-loads, LUF, evict, load-update, other,
                                       pop-batch warp-0 phase, pop-batch rank phase, #batches, #pops) */
+    /* Counters of the SURVEY.md §8(d) algorithmic-byte model (DESIGN.md
+     * "Roofline"): bytes = 4 * sum_avail_at_scans + 4.125 * n * n_scans
+     *                    + 12 * sum_deg_loads_evictions
+     *                    + (4 K + 8 E / m) * n_allocations.
+     * The oracle counts the same three quantities (parity-tested). */
+    int64_t sum_avail_at_scans;      /* sum over scans of #unallocated tasks when the scan began */
+    int64_t n_allocations;           /* tasks leaving the shared pool (plans, fallback / EAGER picks) */
+    int64_t sum_deg_loads_evictions; /* sum of deg(D) over every LOAD and EVICT event            */
 } dts_result_view;
 
 /* Synchronise on the run's stream, copy the results to host (once) and fill *out. */
 dts_status dts_result(dts_instance *inst, dts_result_view *out);
+
+/* Device times of the instance's last run (CUDA events on the run's stream):
+ * *loop_ms = the decision-loop kernel launch (for a batched launch: the whole
+ * batch's loop launch), *total_ms = from the first enqueued step (CSR build)
+ * to the end of that launch.  Waits for the loop to finish; copies no result.
+ * DTS_E_STATE before any dts_run. */
+dts_status dts_run_times(dts_instance *inst, float *loop_ms, float *total_ms);
 
 /* Copy the results of insts[0..n) to host in two batched phases -- every
  * instance's scalars, one wait per distinct stream, then every instance's
@@ -196,15 +211,32 @@ dts_status dts_result(dts_instance *inst, dts_result_view *out);
  * instance's status is returned. */
 dts_status dts_fetch_results(dts_instance *const *insts, int32_t n);
 
-/* Sweep (BASELINE config 5) / batch: run every instance of insts[0..n) on
- * ONE device (opts->device) in a single batched launch of the decision loop,
- * one CTA per instance, CTAs pulling instances from a device counter (no
- * communication between instances).  Each instance gets the same options.
- * Results are read per instance with dts_result.  An instance must not
- * appear twice.  Multi-GPU sweeps shard the list across processes (one per
- * GPU, bench.py) -- nothing crosses devices. */
+/* Sweep (BASELINE config 5) / batch of independent instances (SURVEY.md
+ * §8(e): instances share nothing, so they shard over devices with no
+ * communication).
+ *   insts[0..n)  : distinct instances (none of them a task shard); each gets
+ *                  the same policy and options; results are read per
+ *                  instance with dts_result / dts_fetch_results.
+ *   devices      : NULL or n_devices CUDA ordinals (repeats allowed: two
+ *                  entries naming one device give two concurrent launches on
+ *                  it).  NULL / n_devices = 0: everything on opts->device.
+ *                  Otherwise the instances are split over the entries by LPT
+ *                  on a chain-cost estimate (m * mean degree), longest first,
+ *                  each to the least loaded entry.
+ * Per device entry: ONE batched launch of the decision loop (two concurrent
+ * ones for a large batch: wide CTAs for long-segment instances, narrow ones
+ * for the rest), one CTA per instance, CTAs pulling instances from that
+ * launch's own device counter; every launch has its own descriptor buffer,
+ * so concurrent sweeps on different streams or threads do not interfere.
+ * The first entry on opts->device is enqueued on opts->cuda_stream; the
+ * others on library streams of their devices, forked from and joined back
+ * into opts->cuda_stream (so a synchronisation of that stream covers the
+ * whole sweep).  Returns after enqueueing.
+ * Errors: DTS_E_INVAL (NULL / repeated instance, bad device list, a task
+ * shard in the list), DTS_E_CUDA, DTS_E_CAPACITY / DTS_E_UNSUPPORTED as for
+ * dts_run (checked for every instance before anything is enqueued). */
 dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy,
-                         const dts_run_opts *opts);
+                         const dts_run_opts *opts, const int32_t *devices, int32_t n_devices);
 
 /* ---- Task-sharded single instance (second mode) ----------
  * One instance whose tasks are split into G consecutive id ranges with about

@@ -29,6 +29,7 @@ F_FALLBACK2 = 1
 F_OPTI = 8
 F_LRU = 16     # evict by LRU (not LUF): the paper's plain "DARTS" and "EAGER"
 F_EAGER = 32   # EAGER task choice: shared FIFO queue in submission order
+F_COUNT_DEG = 64  # measurement only: count sum of deg(D) over loads/evictions (slow)
 
 POLICY_FLAGS = {"darts_luf": 0, "darts_lru": F_LRU, "eager_lru": F_EAGER | F_LRU}
 DEFAULT_BUS_BPS = 12_000_000_000
@@ -52,7 +53,9 @@ class _Result(C.Structure):
                 ("n_evictions", C.c_int64), ("n_scans", C.c_int64), ("n_fallback2", C.c_int64),
                 ("n_fallback_first", C.c_int64), ("n_belady", C.c_int64),
                 ("n_idle_requests", C.c_int64), ("bytes_loaded", C.c_uint64),
-                ("makespan", C.c_int64), ("n_wakes", C.c_int64)]
+                ("makespan", C.c_int64), ("n_wakes", C.c_int64),
+                ("sum_avail_at_scans", C.c_int64), ("n_allocations", C.c_int64),
+                ("sum_deg", C.c_int64)]
 
 
 _lib = None
@@ -91,6 +94,9 @@ class OracleResult:
     makespan: int
     K: int
     n_wakes: int = 0
+    sum_avail_at_scans: int = 0   # SURVEY §8(d) byte-model counters (measurement only)
+    n_allocations: int = 0
+    sum_deg: int = 0              # only with F_COUNT_DEG
 
     def orders(self):
         """Per-GPU task order sigma(k, .)."""
@@ -124,4 +130,5 @@ def run(inst, W: int = 0, flags: int = F_FALLBACK2, bus_bps: int = DEFAULT_BUS_B
     return OracleResult(sg[:ns].copy(), st[:ns].copy(), ts[:m].copy(), te[:m].copy(),
                         ev[:r.n_events].copy(), ns, r.n_loads, r.n_evictions, r.n_scans,
                         r.n_fallback2, r.n_fallback_first, r.n_belady, r.n_idle_requests,
-                        r.bytes_loaded, r.makespan, int(inst.K), r.n_wakes)
+                        r.bytes_loaded, r.makespan, int(inst.K), r.n_wakes,
+                        r.sum_avail_at_scans, r.n_allocations, r.sum_deg)

@@ -23,6 +23,7 @@ from .dts import (  # noqa: F401
     dts_instance_upload,
     dts_result,
     dts_fetch_results,
+    dts_run_times,
     dts_run,
     dts_run_opts_default,
     dts_sweep_run,

@@ -14,6 +14,7 @@
 #include <new>
 #include <string>
 #include <memory>
+#include <mutex>
 #include <vector>
 
 #include "dts.h"
@@ -108,6 +109,7 @@ struct dts_instance {
     int64_t *d_delta = nullptr;
     dts::Inst *h_pinned = nullptr;   // pinned staging copy of the descriptor (async H2D)
     cudaEvent_t ev_desc = nullptr;   // the last H2D copy out of h_pinned
+    cudaEvent_t ev_up = nullptr;     // the last H2D upload of the inputs
     void *d_csr_scratch = nullptr;
     int *d_work = nullptr;
     dts::Inst h_inst{};
@@ -158,6 +160,7 @@ struct dts_instance {
             for (auto &e : ev)
                 if (e) cudaEventDestroy(e);
             if (ev_desc) cudaEventDestroy(ev_desc);
+            if (ev_up) cudaEventDestroy(ev_up);
             cudaSetDevice(cur);
         }
         if (h_pinned) cudaFreeHost(h_pinned);
@@ -218,6 +221,11 @@ dts_status dts_instance_create(int32_t n_tasks, int32_t n_data, const int64_t *t
     if (!task_ptr) return fail(DTS_E_INVAL, "task_ptr is NULL");
     if (n_data > 0 && !data_size) return fail(DTS_E_INVAL, "data_size is NULL");
     if (task_ptr[0] != 0) return fail(DTS_E_INVAL, "task_ptr[0] != 0");
+    // the whole of task_ptr first: 0 <= task_ptr[T] <= task_ptr[T+1] for every T,
+    // so no row is read past E = task_ptr[m]
+    for (int32_t T = 0; T < n_tasks; T++)
+        if (task_ptr[T + 1] < task_ptr[T])
+            return fail(DTS_E_INVAL, "task_ptr not monotone at " + std::to_string(T));
     const int64_t E = task_ptr[n_tasks];
     if (E > 0 && !task_data) return fail(DTS_E_INVAL, "task_data is NULL");
     if (default_task_ns < 0) return fail(DTS_E_INVAL, "default_task_ns < 0");
@@ -337,7 +345,9 @@ dts_status ensure_device(dts_instance *I, int device) {
         for (auto &e : I->ev)
             if (e) cudaEventDestroy(e);
         if (I->ev_desc) cudaEventDestroy(I->ev_desc);
+        if (I->ev_up) cudaEventDestroy(I->ev_up);
         I->ev_desc = nullptr;
+        I->ev_up = nullptr;
         I->ar = Arena{};
         I->uploaded = false;
     }
@@ -378,6 +388,7 @@ dts_status ensure_device(dts_instance *I, int device) {
     I->device = device;
     for (auto &ev : I->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
     CK(cudaEventCreateWithFlags(&I->ev_desc, cudaEventDisableTiming), "cudaEventCreate");
+    CK(cudaEventCreateWithFlags(&I->ev_up, cudaEventDisableTiming), "cudaEventCreate");
     if (!I->h_pinned) CK(cudaMallocHost(&I->h_pinned, sizeof(dts::Inst)), "cudaMallocHost");
     if (!I->h_pin) {
         size_t hb = 0;
@@ -492,6 +503,7 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
     const char *end = I->has_tau && I->m > 0 ? reinterpret_cast<const char *>(I->d_tau + I->m)
                                              : reinterpret_cast<const char *>(I->d_size + I->n);
     CK(cudaMemcpyAsync(I->d_raw_ptr, I->p_task_ptr, (size_t)(end - d0), cudaMemcpyHostToDevice, st), "H2D inputs");
+    CK(cudaEventRecord(I->ev_up, st), "event");  // a run on another stream waits for it (stage)
     I->uploaded = true;
     return DTS_OK;
 }
@@ -512,9 +524,22 @@ dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_op
     return DTS_OK;
 }
 
-int env_int(const char *name, int dflt) {
+// Tuning knobs: fixed in the product library.  Only the profiling build
+// (lib/libdts_prof.so, -DDTS_PROF) lets an experiment override them from the
+// environment, so the launch shape of a product run never depends on it.
+int tuning(const char *name, int dflt) {
+#ifdef DTS_PROF
     const char *v = std::getenv(name);
     return v ? std::atoi(v) : dflt;
+#else
+    (void)name;
+    return dflt;
+#endif
+}
+
+// Relative cost of an instance's chain (longest-first ordering, LPT over devices).
+double instance_cost(const dts_instance *I) {
+    return (double)I->m * (double)I->E_raw / std::max(1, I->n);
 }
 
 // Shared-memory placement of one instance's state:
@@ -595,6 +620,9 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     I->have_host = false;
     s = upload(I, st);
     if (s != DTS_OK) return s;
+    // inputs uploaded on another stream (dts_instance_upload) are complete
+    // before this run reads them (no-op on the same stream)
+    CK(cudaStreamWaitEvent(st, I->ev_up, 0), "wait upload");
     dts::Inst &h = I->h_inst;
     h.W = (int32_t)o.lookahead_W;
     h.flags = o.flags;
@@ -621,8 +649,8 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     h.ep_base = (unsigned long long)(++I->runs) << 32;
     h.box_bytes = I->box_bytes;
     h.xsys = I->xsys ? 1 : 0;
-    h.pop_batch_min = env_int("DTS_POP_BATCH_MIN", 10);
-    h.poison = env_int("DTS_POISON", 0);
+    h.pop_batch_min = tuning("DTS_POP_BATCH_MIN", 10);
+    h.poison = tuning("DTS_POISON", 0);  // debug (profiling build only)
     // small instances: the loop CTA builds its own CSR and state (one launch)
     const int fs = fused_scratch_bytes(I, block);
     h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
@@ -651,21 +679,167 @@ int budget_of(const dts_run_opts &o) {
     return o.smem_budget == 0 ? mx : std::min(o.smem_budget, mx);
 }
 
-// Per-device buffer of instance descriptors for batched (sweep) launches.
-// Reuse is ordered on the stream: the H2D copy of a later sweep is enqueued
-// after the previous sweep's kernels on the same stream.
-struct SweepBuf {
-    static constexpr int RING = 4;
-    dts::Inst *d_insts = nullptr;        // read by the kernels; reuse is stream-ordered
-    dts::Inst *h_insts[RING] = {};       // pinned staging ring: the host never waits on
-    cudaEvent_t copied[RING] = {};       // the GPU unless it is RING sweeps behind
-    int slot = 0;
-    int *d_work = nullptr;               // [0]: group A's instance counter, [1]: group B's
+// Per-device ring of descriptor buffers for batched (sweep / shard-group)
+// launches.  Every launch gets its own slot: the device copy of its instance
+// descriptors and its own instance counters, so a sweep on one stream never
+// overwrites what a still-running launch on another stream reads.  A slot is
+// reused only after the event recorded behind its last kernel has completed
+// (host wait, only when the ring wraps around a running launch).  The mutex
+// serialises the enqueue of batched launches on one device (slot choice,
+// capacity growth, the shared side stream and its fork/join events).
+struct SweepSlot {
+    dts::Inst *d_insts = nullptr;  // descriptors, then the launch's instance counters
+    dts::Inst *h_insts = nullptr;  // pinned staging copy (async H2D)
+    int *d_work = nullptr;         // [0]: group A's instance counter, [1]: group B's
     size_t cap = 0;
-    cudaStream_t side = nullptr;         // group B of a split batch (forked from / joined into the caller's stream)
-    cudaEvent_t fork = nullptr, join = nullptr;
+    cudaEvent_t done = nullptr;    // recorded after every kernel that reads this slot
 };
-SweepBuf g_sweep[64];
+struct DeviceSweep {
+    static constexpr int RING = 8;
+    std::mutex mu;
+    SweepSlot slot[RING];
+    int next = 0;
+    bool init = false;
+    cudaStream_t side = nullptr;  // group B of a split batch (forked from / joined into the caller's stream)
+    cudaEvent_t fork = nullptr, join = nullptr;
+    std::vector<cudaStream_t> extra;  // library streams for multi-device sweeps (dts_sweep_run devices[])
+};
+DeviceSweep g_dev[64];
+
+// Caller holds D.mu; the device is current.
+dts_status acquire_slot(DeviceSweep &D, size_t n, SweepSlot **out) {
+    if (!D.init) {
+        CK(cudaEventCreateWithFlags(&D.fork, cudaEventDisableTiming), "cudaEventCreate");
+        CK(cudaEventCreateWithFlags(&D.join, cudaEventDisableTiming), "cudaEventCreate");
+        CK(cudaStreamCreateWithFlags(&D.side, cudaStreamNonBlocking), "cudaStreamCreate");
+        D.init = true;
+    }
+    SweepSlot &S = D.slot[D.next];
+    D.next = (D.next + 1) % DeviceSweep::RING;
+    if (S.done) CK(cudaEventSynchronize(S.done), "sweep slot event");  // its last launch has finished
+    else CK(cudaEventCreateWithFlags(&S.done, cudaEventDisableTiming), "cudaEventCreate");
+    if (S.cap < n) {
+        if (S.d_insts) cudaFree(S.d_insts);
+        if (S.h_insts) cudaFreeHost(S.h_insts);
+        S.d_insts = nullptr;
+        S.h_insts = nullptr;
+        S.cap = 0;
+        const size_t cap = std::max<size_t>(n, 64);
+        CK(cudaMalloc(&S.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
+        CK(cudaMallocHost(&S.h_insts, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
+        S.d_work = reinterpret_cast<int *>(S.d_insts + cap);
+        S.cap = cap;
+    }
+    *out = &S;
+    return DTS_OK;
+}
+
+// One batched launch (or two concurrent ones) of insts[0..n) on o.device,
+// enqueued on st.  The instances are validated by the caller.
+dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy policy, const dts_run_opts &o,
+                           cudaStream_t st) {
+    int64_t work = 1;
+    for (int32_t i = 0; i < n; i++)
+        work = std::max<int64_t>(work, std::max<int64_t>(insts[i]->m_pad, (int64_t)insts[i]->n * insts[i]->K));
+    // Each instance is a latency-bound chain: with many more instances than
+    // SMs, run several CTAs per SM (their chains interleave) by default --
+    // a share of the shared memory each; few instances get all of it.
+    int nsm = 0;
+    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
+    const bool many = n >= 2 * nsm;
+    int budget = budget_of(o);
+    const int smem_div = std::max(1, tuning("DTS_SWEEP_SMEM_DIV", 6));
+    if (o.smem_budget == 0 && many) budget = std::min(budget, (max_dyn_smem(o.device) + 1024) / smem_div - 4096);
+    // longest first (cost ~ m * mean degree), so the device counter hands the
+    // long chains out early and the tail of the batch stays short
+    std::vector<int32_t> ord((size_t)n);
+    for (int32_t i = 0; i < n; i++) ord[(size_t)i] = i;
+    std::stable_sort(ord.begin(), ord.end(),
+                     [&](int32_t a, int32_t b) { return instance_cost(insts[a]) > instance_cost(insts[b]); });
+    // CTA size per group: a batch of many instances runs as two concurrent
+    // launches -- the instances whose segments want wide CTAs (auto_block >=
+    // 256) with those, the rest with small CTAs so more chains share an SM.
+    // Few instances, or a forced size: one launch.
+    const int forced = o.block_threads;
+    const int small_max = tuning("DTS_SWEEP_SMALL_BLOCK", 128);
+    int nb = n, block_a = 32, block_b = 32;  // group A = ord[0, nb), group B = ord[nb, n)
+    if (!forced && many && small_max > 0) {
+        nb = 0;
+        for (int32_t i = 0; i < n; i++)
+            if (auto_block(insts[ord[(size_t)i]]) > small_max) nb = i + 1;  // the long ones come first
+        // group B: every instance after the last wide one (cost order ~ width order)
+    }
+    for (int32_t i = 0; i < n; i++) {
+        const int ab = auto_block(insts[ord[(size_t)i]], !many);
+        if (i < nb) block_a = std::max(block_a, ab);
+        else block_b = std::max(block_b, std::min(ab, small_max));
+    }
+    if (forced) block_a = block_b = forced;
+    int smem_a = 0, smem_b = 0;
+    bool any_unfused = false;
+    auto sev = std::make_shared<SweepEvents>();
+    sev->device = o.device;
+    CK(cudaEventCreate(&sev->begin), "cudaEventCreate");
+    CK(cudaEventCreate(&sev->loop_begin), "cudaEventCreate");
+    CK(cudaEventCreate(&sev->loop_end), "cudaEventCreate");
+    CK(cudaEventRecord(sev->begin, st), "event");
+    for (int32_t i = 0; i < n; i++) {
+        dts_instance *I = insts[ord[(size_t)i]];
+        dts_status s = stage(I, policy, o, budget, i < nb ? block_a : block_b, st, false, false);
+        if (s != DTS_OK) return s;
+        (i < nb ? smem_a : smem_b) = std::max(i < nb ? smem_a : smem_b, I->h_inst.smem_bytes);
+        any_unfused |= !I->h_inst.fused;
+    }
+    DeviceSweep &D = g_dev[o.device];
+    std::lock_guard<std::mutex> lock(D.mu);
+    SweepSlot *S = nullptr;
+    dts_status s = acquire_slot(D, (size_t)n, &S);
+    if (s != DTS_OK) return s;
+    for (int32_t i = 0; i < n; i++) S->h_insts[i] = insts[ord[(size_t)i]]->h_inst;
+    CK(cudaMemcpyAsync(S->d_insts, S->h_insts, sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
+       "H2D sweep");
+    CK(cudaMemsetAsync(S->d_work, 0, 2 * sizeof(int), st), "memset");
+    if (any_unfused) CK(dts::launch_init(S->d_insts, n, o.bus_bytes_per_s, work, st), "init");
+    CK(cudaEventRecord(sev->loop_begin, st), "event");
+    const bool two = nb > 0 && nb < n;
+    if (two) {  // group B on the side stream, forked from and joined back into st
+        CK(cudaEventRecord(D.fork, st), "event");
+        CK(cudaStreamWaitEvent(D.side, D.fork, 0), "wait");
+        const int per_b = std::max(1, dts::loop_max_blocks_per_sm(block_b, smem_b));
+        const int grid_b = (int)std::min<int64_t>((int64_t)(n - nb), (int64_t)per_b * nsm);
+        CK(dts::launch_loop(S->d_insts + nb, n - nb, block_b, grid_b, S->d_work + 1, smem_b, D.side), "loop B");
+        CK(cudaEventRecord(D.join, D.side), "event");
+    }
+    const int na = two ? nb : n;
+    const int blk = two ? block_a : std::max(block_a, block_b);
+    const int sm = two ? smem_a : std::max(smem_a, smem_b);
+    const int per = std::max(1, dts::loop_max_blocks_per_sm(blk, sm));
+    const int grid = (int)std::min<int64_t>((int64_t)na, (int64_t)per * nsm);
+    CK(dts::launch_loop(S->d_insts, na, blk, grid, S->d_work, sm, st), "loop");
+    if (two) CK(cudaStreamWaitEvent(st, D.join, 0), "wait");
+    CK(cudaEventRecord(sev->loop_end, st), "event");
+    CK(cudaEventRecord(S->done, st), "event");
+    for (int32_t i = 0; i < n; i++) {
+        insts[i]->sev = sev;
+        insts[i]->ran = true;
+    }
+    return DTS_OK;
+}
+
+// A library stream on `device` for the j-th extra group of a multi-device sweep.
+dts_status extra_stream(int device, size_t j, cudaStream_t *out) {
+    DeviceSweep &D = g_dev[device];
+    std::lock_guard<std::mutex> lock(D.mu);
+    CK(cudaSetDevice(device), "cudaSetDevice");
+    while (D.extra.size() <= j) {
+        cudaStream_t s = nullptr;
+        CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking), "cudaStreamCreate");
+        D.extra.push_back(s);
+    }
+    *out = D.extra[j];
+    return DTS_OK;
+}
 
 }  // namespace
 
@@ -693,7 +867,7 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     if (I->G > 1 && I->device != o.device) return fail(DTS_E_INVAL, "task shard: opts.device != exported device");
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
     const int budget = budget_of(o);
-    const int block = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", auto_block(I, true));
+    const int block = o.block_threads ? o.block_threads : auto_block(I, true);
     s = stage(I, policy, o, budget, block, st);
     if (s != DTS_OK) return s;
     const int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n + 4);
@@ -707,16 +881,18 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     return DTS_OK;
 }
 
-dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy,
-                         const dts_run_opts *opts) {
+dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy policy, const dts_run_opts *opts,
+                         const int32_t *devices, int32_t n_devices) {
     if (n < 0 || (n > 0 && !insts)) return fail(DTS_E_INVAL, "insts");
+    if (n_devices < 0 || (n_devices > 0 && !devices)) return fail(DTS_E_INVAL, "devices");
     if (n == 0) return DTS_OK;
     dts_run_opts o;
     if (opts) o = *opts;
     else dts_run_opts_default(&o);
     dts_status s = check_device(o.device);
     if (s != DTS_OK) return s;
-    int64_t work = 1;
+    for (int32_t g = 0; g < n_devices; g++)
+        if ((s = check_device(devices[g])) != DTS_OK) return s;
     std::vector<dts_instance *> seen(insts, insts + n);
     std::sort(seen.begin(), seen.end());
     if (std::adjacent_find(seen.begin(), seen.end()) != seen.end())
@@ -725,111 +901,71 @@ dts_status dts_sweep_run(dts_instance *const *insts, int32_t n, dts_policy polic
         if (!insts[i]) return fail(DTS_E_INVAL, "instance is NULL");
         s = check_opts(insts[i], policy, &o);
         if (s != DTS_OK) return s;
-        work = std::max<int64_t>(work, std::max<int64_t>(insts[i]->m_pad, (int64_t)insts[i]->n * insts[i]->K));
+        if (insts[i]->G > 1) return fail(DTS_E_INVAL, "a task shard cannot be part of a sweep");
     }
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
-    // Each instance is a latency-bound chain: with many more instances than
-    // SMs, run several CTAs per SM (their chains interleave) by default --
-    // a share of the shared memory each; few instances get all of it.
-    int nsm = 0;
-    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, o.device), "attr SMs");
-    const bool many = n >= 2 * nsm;
-    int budget = budget_of(o);
-    const int smem_div = std::max(1, env_int("DTS_SWEEP_SMEM_DIV", 6));
-    if (o.smem_budget == 0 && many) budget = std::min(budget, (max_dyn_smem(o.device) + 1024) / smem_div - 4096);
-    // longest first (cost ~ m * mean degree), so the device counter hands the
-    // long chains out early and the tail of the batch stays short
+    if (n_devices == 0) return sweep_on_device(insts, n, policy, o, st);
+
+    // Several devices (independent instances, no
+    // communication): LPT over the device list on the chain-cost estimate,
+    // longest first, each to the least loaded entry (lower index on ties).
+    // Entry g runs ONE batched launch on devices[g]; the first entry on
+    // opts->device uses the caller's stream, the others library streams
+    // forked from it and joined back into it (cross-device event waits).
     std::vector<int32_t> ord((size_t)n);
     for (int32_t i = 0; i < n; i++) ord[(size_t)i] = i;
-    auto cost = [&](int32_t i) { return (double)insts[i]->m * (double)insts[i]->E_raw / std::max(1, insts[i]->n); };
-    std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return cost(a) > cost(b); });
-    // CTA size per group: a batch of many instances runs as two concurrent
-    // launches -- the instances whose segments want wide CTAs (auto_block >=
-    // 256) with those, the rest with small CTAs so more chains share an SM.
-    // Few instances, or a forced size: one launch.
-    const int forced = o.block_threads ? o.block_threads : env_int("DTS_BLOCK", 0);
-    const int small_max = env_int("DTS_SWEEP_SMALL_BLOCK", 128);
-    int nb = n, block_a = 32, block_b = 32;  // group A = ord[0, nb), group B = ord[nb, n)
-    if (!forced && many && small_max > 0) {
-        nb = 0;
-        for (int32_t i = 0; i < n; i++)
-            if (auto_block(insts[ord[(size_t)i]]) > small_max) nb = i + 1;  // the long ones come first
-        // group B: every instance after the last wide one (cost order ~ width order)
+    std::stable_sort(ord.begin(), ord.end(),
+                     [&](int32_t a, int32_t b) { return instance_cost(insts[a]) > instance_cost(insts[b]); });
+    std::vector<double> load((size_t)n_devices, 0.0);
+    std::vector<std::vector<dts_instance *>> part((size_t)n_devices);
+    for (int32_t i : ord) {
+        size_t g = 0;
+        for (size_t q = 1; q < load.size(); q++)
+            if (load[q] < load[g]) g = q;
+        load[g] += instance_cost(insts[i]);
+        part[g].push_back(insts[i]);
     }
-    for (int32_t i = 0; i < n; i++) {
-        const int ab = auto_block(insts[ord[(size_t)i]], !many);
-        if (i < nb) block_a = std::max(block_a, ab);
-        else block_b = std::max(block_b, std::min(ab, small_max));
-    }
-    if (forced) block_a = block_b = forced;
-    int smem_a = 0, smem_b = 0;
-    bool any_unfused = false;
-    auto sev = std::make_shared<SweepEvents>();
-    sev->device = o.device;
     CK(cudaSetDevice(o.device), "cudaSetDevice");
-    CK(cudaEventCreate(&sev->begin), "cudaEventCreate");
-    CK(cudaEventCreate(&sev->loop_begin), "cudaEventCreate");
-    CK(cudaEventCreate(&sev->loop_end), "cudaEventCreate");
-    CK(cudaEventRecord(sev->begin, st), "event");
-    for (int32_t i = 0; i < n; i++) {
-        dts_instance *I = insts[ord[(size_t)i]];
-        s = stage(I, policy, o, budget, i < nb ? block_a : block_b, st, false, false);
-        if (s != DTS_OK) return s;
-        (i < nb ? smem_a : smem_b) = std::max(i < nb ? smem_a : smem_b, I->h_inst.smem_bytes);
-        any_unfused |= !I->h_inst.fused;
+    cudaEvent_t fork = nullptr;
+    CK(cudaEventCreateWithFlags(&fork, cudaEventDisableTiming), "cudaEventCreate");
+    CK(cudaEventRecord(fork, st), "event");
+    std::vector<cudaEvent_t> joins;
+    std::vector<int> used((size_t)64, 0);  // library streams taken per device
+    bool caller_taken = false;
+    dts_status rs = DTS_OK;
+    for (int32_t g = 0; g < n_devices && rs == DTS_OK; g++) {
+        if (part[(size_t)g].empty()) continue;
+        const int d = devices[g];
+        dts_run_opts od = o;
+        od.device = d;
+        cudaStream_t sg = st;
+        const bool on_caller = d == o.device && !caller_taken;
+        if (on_caller) {
+            caller_taken = true;
+        } else {
+            if ((rs = extra_stream(d, (size_t)used[(size_t)d]++, &sg)) != DTS_OK) break;
+            CK(cudaSetDevice(d), "cudaSetDevice");
+            CK(cudaStreamWaitEvent(sg, fork, 0), "wait");
+        }
+        od.cuda_stream = sg;
+        rs = sweep_on_device(part[(size_t)g].data(), (int32_t)part[(size_t)g].size(), policy, od, sg);
+        if (rs != DTS_OK) break;
+        if (!on_caller) {
+            cudaEvent_t j = nullptr;
+            CK(cudaSetDevice(d), "cudaSetDevice");
+            CK(cudaEventCreateWithFlags(&j, cudaEventDisableTiming), "cudaEventCreate");
+            CK(cudaEventRecord(j, sg), "event");
+            joins.push_back(j);
+        }
     }
-    SweepBuf &B = g_sweep[o.device];
-    if (!B.copied[0]) {
-        for (auto &e : B.copied) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
-        CK(cudaEventCreateWithFlags(&B.fork, cudaEventDisableTiming), "cudaEventCreate");
-        CK(cudaEventCreateWithFlags(&B.join, cudaEventDisableTiming), "cudaEventCreate");
-        CK(cudaStreamCreateWithFlags(&B.side, cudaStreamNonBlocking), "cudaStreamCreate");
+    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    for (cudaEvent_t j : joins) {
+        CK(cudaStreamWaitEvent(st, j, 0), "wait");
+        cudaEventDestroy(j);  // released once it has completed
     }
-    if (B.cap < (size_t)n) {
-        CK(cudaDeviceSynchronize(), "sync");
-        if (B.d_insts) cudaFree(B.d_insts);
-        for (auto &h : B.h_insts)
-            if (h) cudaFreeHost(h);
-        size_t cap = std::max<size_t>((size_t)n, 64);
-        CK(cudaMalloc(&B.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
-        for (auto &h : B.h_insts) CK(cudaMallocHost(&h, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
-        B.d_work = reinterpret_cast<int *>(B.d_insts + cap);
-        B.cap = cap;
-    }
-    const int sl = B.slot;
-    B.slot = (B.slot + 1) % SweepBuf::RING;
-    CK(cudaEventSynchronize(B.copied[sl]), "sweep event");
-    for (int32_t i = 0; i < n; i++) B.h_insts[sl][i] = insts[ord[(size_t)i]]->h_inst;
-    CK(cudaMemcpyAsync(B.d_insts, B.h_insts[sl], sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
-       "H2D sweep");
-    CK(cudaEventRecord(B.copied[sl], st), "event");
-    CK(cudaMemsetAsync(B.d_work, 0, 2 * sizeof(int), st), "memset");
-    if (any_unfused) CK(dts::launch_init(B.d_insts, n, o.bus_bytes_per_s, work, st), "init");
-    CK(cudaEventRecord(sev->loop_begin, st), "event");
-    const bool two = nb > 0 && nb < n;
-    if (two) {  // group B on the side stream, forked from and joined back into st
-        CK(cudaEventRecord(B.fork, st), "event");
-        CK(cudaStreamWaitEvent(B.side, B.fork, 0), "wait");
-        const int per_b = std::max(1, dts::loop_max_blocks_per_sm(block_b, smem_b));
-        const int grid_b = (int)std::min<int64_t>((int64_t)(n - nb), (int64_t)per_b * nsm);
-        CK(dts::launch_loop(B.d_insts + nb, n - nb, block_b, grid_b, B.d_work + 1, smem_b, B.side), "loop B");
-        CK(cudaEventRecord(B.join, B.side), "event");
-    }
-    const int na = two ? nb : n;
-    const int blk = two ? block_a : std::max(block_a, block_b);
-    const int sm = two ? smem_a : std::max(smem_a, smem_b);
-    const int per = std::max(1, dts::loop_max_blocks_per_sm(blk, sm));
-    const int grid = (int)std::min<int64_t>((int64_t)na, (int64_t)per * nsm);
-    CK(dts::launch_loop(B.d_insts, na, blk, grid, B.d_work, sm, st), "loop");
-    if (two) CK(cudaStreamWaitEvent(st, B.join, 0), "wait");
-    CK(cudaEventRecord(sev->loop_end, st), "event");
-    for (int32_t i = 0; i < n; i++) {
-        insts[i]->sev = sev;
-        insts[i]->ran = true;
-    }
-    return DTS_OK;
+    cudaEventDestroy(fork);
+    return rs;
 }
-
 
 }  // extern "C"
 
@@ -1002,7 +1138,6 @@ dts_status dts_shard_group_run(dts_instance *const *shards, int32_t G, dts_polic
         }
     }
     if (o.block_threads) block = o.block_threads;
-    else block = env_int("DTS_BLOCK", block);
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
     const int budget = budget_of(o);
     // one exchange-number range for the whole group: above every shard's last
@@ -1015,32 +1150,20 @@ dts_status dts_shard_group_run(dts_instance *const *shards, int32_t G, dts_polic
         if (s != DTS_OK) return s;
         smem = std::max(smem, shards[i]->h_inst.smem_bytes);
     }
-    SweepBuf &B = g_sweep[o.device];
-    if (!B.copied[0])
-        for (auto &e : B.copied) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
-    if (B.cap < (size_t)G) {
-        CK(cudaDeviceSynchronize(), "sync");
-        if (B.d_insts) cudaFree(B.d_insts);
-        for (auto &h : B.h_insts)
-            if (h) cudaFreeHost(h);
-        size_t cap = std::max<size_t>((size_t)G, 64);
-        CK(cudaMalloc(&B.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
-        for (auto &h : B.h_insts) CK(cudaMallocHost(&h, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
-        B.d_work = reinterpret_cast<int *>(B.d_insts + cap);
-        B.cap = cap;
-    }
-    const int sl = B.slot;
-    B.slot = (B.slot + 1) % SweepBuf::RING;
-    CK(cudaEventSynchronize(B.copied[sl]), "sweep event");
-    for (int32_t i = 0; i < G; i++) B.h_insts[sl][i] = shards[i]->h_inst;
-    CK(cudaMemcpyAsync(B.d_insts, B.h_insts[sl], sizeof(dts::Inst) * (size_t)G, cudaMemcpyHostToDevice, st),
+    DeviceSweep &D = g_dev[o.device];
+    std::lock_guard<std::mutex> lock(D.mu);
+    SweepSlot *S = nullptr;
+    s = acquire_slot(D, (size_t)G, &S);
+    if (s != DTS_OK) return s;
+    for (int32_t i = 0; i < G; i++) S->h_insts[i] = shards[i]->h_inst;
+    CK(cudaMemcpyAsync(S->d_insts, S->h_insts, sizeof(dts::Inst) * (size_t)G, cudaMemcpyHostToDevice, st),
        "H2D shards");
-    CK(cudaEventRecord(B.copied[sl], st), "event");
-    CK(cudaMemsetAsync(B.d_work, 0, sizeof(int), st), "memset");
-    CK(dts::launch_init(B.d_insts, G, o.bus_bytes_per_s, work, st), "init");
+    CK(cudaMemsetAsync(S->d_work, 0, sizeof(int), st), "memset");
+    CK(dts::launch_init(S->d_insts, G, o.bus_bytes_per_s, work, st), "init");
     for (int32_t i = 0; i < G; i++) CK(cudaEventRecord(shards[i]->ev[1], st), "event");
     // the G shards exchange inside the kernel: they must be co-resident
-    CK(dts::launch_loop_coop(B.d_insts, G, block, B.d_work, smem, st), "loop (cooperative)");
+    CK(dts::launch_loop_coop(S->d_insts, G, block, S->d_work, smem, st), "loop (cooperative)");
+    CK(cudaEventRecord(S->done, st), "event");
     for (int32_t i = 0; i < G; i++) {
         CK(cudaEventRecord(shards[i]->ev[2], st), "event");
         CK(cudaEventRecord(shards[i]->ev[3], st), "event");
@@ -1060,7 +1183,8 @@ static dts_status fetch_out(dts_instance *I) {
 static dts_status fetch_arrays(dts_instance *I) {
     I->out = *I->r_out;
     if (I->out.error == 2) return fail(DTS_E_STATE, "task shards: a peer did not reach an exchange in time");
-    if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim (Belady branch)");
+    if (I->out.error == 3) return fail(DTS_E_STATE, "device loop: plannedTasks inconsistent (internal)");
+    if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim");
     const dts::Inst &h = I->h_inst;
     const size_t ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);
     cudaStream_t st = I->stream;  // the run's stream: the copies follow the run
@@ -1113,6 +1237,18 @@ dts_status dts_fetch_results(dts_instance *const *insts, int32_t n) {
     return DTS_OK;
 }
 
+dts_status dts_run_times(dts_instance *I, float *loop_ms, float *total_ms) {
+    if (!I || !loop_ms || !total_ms) return fail(DTS_E_INVAL, "NULL argument");
+    if (!I->ran) return fail(DTS_E_STATE, "dts_run_times before dts_run");
+    CK(cudaSetDevice(I->device), "cudaSetDevice");
+    cudaEvent_t b = I->sev ? I->sev->loop_begin : I->ev[1], e = I->sev ? I->sev->loop_end : I->ev[2];
+    cudaEvent_t b0 = I->sev ? I->sev->begin : I->ev[0];
+    CK(cudaEventSynchronize(e), "loop event");
+    CK(cudaEventElapsedTime(loop_ms, b, e), "elapsed");
+    CK(cudaEventElapsedTime(total_ms, b0, e), "elapsed");
+    return DTS_OK;
+}
+
 dts_status dts_result(dts_instance *I, dts_result_view *v) {
     if (!I || !v) return fail(DTS_E_INVAL, "NULL argument");
     if (!I->ran) return fail(DTS_E_STATE, "dts_result before dts_run");
@@ -1147,6 +1283,9 @@ dts_status dts_result(dts_instance *I, dts_result_view *v) {
     v->alg_bytes = I->out.alg_bytes;
     v->scan_alg_bytes = I->out.scan_alg_bytes;
     for (int i = 0; i < 16; i++) v->prof_cycles[i] = I->out.prof[i];
+    v->sum_avail_at_scans = I->out.sum_avail;
+    v->n_allocations = I->out.n_alloc;
+    v->sum_deg_loads_evictions = I->out.sum_deg;
     v->loop_ms = I->loop_ms;
     v->total_ms = I->total_ms;
     return DTS_OK;

@@ -57,6 +57,10 @@ struct Out {
     uint64_t bytes_loaded;
     int64_t makespan;
     uint64_t alg_bytes, scan_alg_bytes;
+    // SURVEY.md §8(d) byte model: sum over scans of the
+    // unallocated tasks when the scan started, task allocations, sum of deg(D)
+    // over loads and evictions
+    int64_t sum_avail, n_alloc, sum_deg;
     int32_t error;
     int32_t pad;
     int64_t prof[16];  // SM cycles seen by thread 0 per phase (see PROF_* in dts_loop.cu)

@@ -98,6 +98,8 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
         n_verr;
     uint64_t bytes_loaded, alg_bytes, scan_alg_bytes;
     int64_t makespan;
+    int64_t sum_avail, n_alloc, sum_deg;  // SURVEY §8(d) byte-model counters (Out)
+    int32_t scan_avail;                   // m_avail when the current scan started
     int32_t n_avail, avail_lo;
     int32_t error;
     int32_t cmd, k, T, vslot, row_len;
@@ -616,8 +618,19 @@ __device__ int32_t pop_planned(int k, int64_t *tau) {
     const View &V = SV;
     const int4 *pl = V.plan + (size_t)k * I.plan_cap;
     int h = L.plan_head[k];
+    const int pe = L.plan_end[k];
+    if (h >= pe) {  // internal inconsistency (never expected): end the run with an error
+        L.error = 3;
+        L.row_len = 0;
+        return -1;
+    }
     int4 e = pl[h];
-    while (e.x < 0) e = pl[++h];
+    while (e.x < 0 && h + 1 < pe) e = pl[++h];  // bounded by plan_end (LUF-removed entries)
+    if (e.x < 0) {
+        L.error = 3;
+        L.row_len = 0;
+        return -1;
+    }
     L.plan_head[k] = h + 1;
     L.plan_live[k]--;
     int32_t *npk = V.np + (size_t)k * I.nstr;
@@ -1203,6 +1216,7 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
         int64_t sb, se;
         seg_of(Vd, sb, se);
         L.alg_bytes += 24ull * (uint64_t)(se - sb) + (uint64_t)nret * (8ull * I.K + 40ull) + 32ull;
+        L.sum_deg += se - sb;
     }
     cta_sync();
     if (nret > 0) compact_plan(k);
@@ -1270,6 +1284,7 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
             int64_t sb, se;
             seg_of(D, sb, se);
             L.alg_bytes += 24ull * (uint64_t)(se - sb) + 32ull;
+            L.sum_deg += se - sb;
         }
         // seg_update reads nothing thread 0 just wrote unless a row is longer
         // than its edge record (missing_pair reads the residency bitmap)
@@ -1435,6 +1450,7 @@ __device__ void plan(int k, int32_t Dopt) {
         L.plan_end[k] = base_out;
         L.plan_live[k] = base_out;
         L.n_avail -= base_out;
+        L.n_alloc += base_out;
         L.alg_bytes += 20ull * (uint64_t)(e - b) + (uint64_t)base_out * (8ull * I.K + 40ull);
     }
     cta_sync();
@@ -1746,6 +1762,7 @@ __device__ __noinline__ void plan_shard(int k, int32_t Dopt) {
         L.plan_end[k] = total;
         L.plan_live[k] = total;
         L.n_avail -= total;
+        L.n_alloc += total;
         L.alg_bytes += 20ull * (uint64_t)(e - b) + (uint64_t)total * (8ull * I.K + 40ull);
     }
     cta_sync();
@@ -2153,6 +2170,7 @@ __global__ void __launch_bounds__(512, 1)
             L.n_events = L.n_served = L.n_loads = L.n_evictions = L.n_scans = L.n_fb2 = L.n_fbf =
                 L.n_belady = L.n_idle = L.n_verr = 0;
             L.bytes_loaded = L.alg_bytes = L.scan_alg_bytes = 0;
+            L.sum_avail = L.n_alloc = L.sum_deg = 0;
             L.makespan = 0;
             L.n_avail = I.m;
             L.avail_lo = 0;
@@ -2216,6 +2234,7 @@ __global__ void __launch_bounds__(512, 1)
             int32_t T = -1;
             if (L.cmd == CMD_POP) {
                 T = L.T;
+                if (T < 0) break;  // pop_planned found no entry (L.error set)
             } else if (L.cmd == CMD_EAGER) {
                 // EAGER: the shared FIFO queue in submission
                 // order -- the lowest-id unallocated task
@@ -2226,6 +2245,7 @@ __global__ void __launch_bounds__(512, 1)
                         L.fent = entry_of_task(T);
                         row_from_entry(L.fent);
                         L.n_avail--;
+                        L.n_alloc++;
                     } else {
                         L.idle[k] = 1;
                         L.n_idle++;
@@ -2250,17 +2270,22 @@ __global__ void __launch_bounds__(512, 1)
             if (tid == 0) {
                 L.scan_alg_bytes += 8ull * (uint64_t)n;
                 L.alg_bytes += 8ull * (uint64_t)n;
+                L.scan_avail = L.n_avail;  // before this scan allocates anything
             }
+            if (I.G > 1 && L.xerr) break;  // a peer timed out in the scan exchange (CTA-uniform)
             if (Dopt >= 0) {
                 if (I.G > 1) plan_shard(k, Dopt);
                 else plan(k, Dopt);
+                if (I.G > 1 && L.xerr) break;  // plan exchange failed: no plan to pop from
                 if (tid == 0) {
                     int64_t tau;
                     L.T = pop_planned(k, &tau);
                     L.n_scans++;
+                    L.sum_avail += L.scan_avail;
                 }
                 cta_sync();
                 T = L.T;
+                if (T < 0) break;  // pop_planned found no entry (L.error set)
                 PROF_ADD(L, P_PLAN, p_pl);
             } else {
                 if (I.flags & DTS_F_FALLBACK2) {
@@ -2286,7 +2311,9 @@ __global__ void __launch_bounds__(512, 1)
                         L.fent = entry_of_task(T);
                         row_from_entry(L.fent);
                         L.n_avail--;
+                        L.n_alloc++;
                         L.n_scans++;
+                        L.sum_avail += L.scan_avail;
                     }
                     cta_sync();
                     pool_move_many(&L.fent, 1, -1, -1);
@@ -2296,6 +2323,7 @@ __global__ void __launch_bounds__(512, 1)
                 }
                 cta_sync();
                 PROF_ADD(L, P_OTHER, p_pl);
+                if (I.G > 1 && L.xerr) break;  // a min-exchange failed: T is not trustworthy
                 if (T < 0) continue;
             }
             }  // scan
@@ -2338,6 +2366,9 @@ __global__ void __launch_bounds__(512, 1)
             o->makespan = L.makespan;
             o->alg_bytes = L.alg_bytes;
             o->scan_alg_bytes = L.scan_alg_bytes;
+            o->sum_avail = L.sum_avail;
+            o->n_alloc = L.n_alloc;
+            o->sum_deg = L.sum_deg;
             o->error = L.error;
             for (int i = 0; i < 16; i++) o->prof[i] = L.prof[i];
         }

@@ -43,7 +43,8 @@ EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data",
                         ("task", "<i4"), ("op", "u1"), ("pad", "u1", (3,))])
 
 EXPORTED = ["dts_run_opts_default", "dts_instance_create", "dts_instance_upload", "dts_run",
-            "dts_result", "dts_fetch_results", "dts_sweep_run", "dts_instance_destroy", "dts_status_str",
+            "dts_result", "dts_fetch_results", "dts_run_times", "dts_sweep_run", "dts_instance_destroy",
+            "dts_status_str",
             "dts_last_error", "dts_version", "dts_kernel_launches",
             "dts_shard_set", "dts_shard_range", "dts_shard_export", "dts_shard_connect",
             "dts_shard_group_run"]
@@ -76,7 +77,8 @@ class dts_result_view(C.Structure):
                 ("n_idle_requests", C.c_int64), ("n_verify_err", C.c_int64),
                 ("alg_bytes", C.c_uint64),
                 ("scan_alg_bytes", C.c_uint64), ("loop_ms", C.c_float), ("total_ms", C.c_float),
-                ("prof_cycles", C.c_int64 * 16)]
+                ("prof_cycles", C.c_int64 * 16), ("sum_avail_at_scans", C.c_int64),
+                ("n_allocations", C.c_int64), ("sum_deg_loads_evictions", C.c_int64)]
 
 
 _lib = None
@@ -103,11 +105,13 @@ def load_library(path: str = LIB_PATH):
     lib.dts_result.argtypes = [P, C.POINTER(dts_result_view)]
     lib.dts_result.restype = C.c_int
     lib.dts_sweep_run.argtypes = [C.POINTER(C.c_void_p), C.c_int32, C.c_int,
-                                  C.POINTER(dts_run_opts)]
+                                  C.POINTER(dts_run_opts), C.POINTER(C.c_int32), C.c_int32]
     lib.dts_sweep_run.restype = C.c_int
     if hasattr(lib, "dts_fetch_results"):  # (older builds, tools/lib_ab.py, lack it)
         lib.dts_fetch_results.argtypes = [C.POINTER(C.c_void_p), C.c_int32]
         lib.dts_fetch_results.restype = C.c_int
+    lib.dts_run_times.argtypes = [P, C.POINTER(C.c_float), C.POINTER(C.c_float)]
+    lib.dts_run_times.restype = C.c_int
     lib.dts_instance_destroy.argtypes = [P]
     lib.dts_instance_destroy.restype = None
     lib.dts_status_str.argtypes = [C.c_int]
@@ -187,10 +191,16 @@ def dts_run(inst: Instance, policy: int = DTS_POLICY_DARTS_LUF, opts: Optional[d
     _check(load_library().dts_run(inst.handle, int(policy), None if opts is None else C.byref(opts)))
 
 
-def dts_sweep_run(insts, policy: int = DTS_POLICY_DARTS_LUF, opts: Optional[dts_run_opts] = None):
+def dts_sweep_run(insts, policy: int = DTS_POLICY_DARTS_LUF, opts: Optional[dts_run_opts] = None,
+                  devices=None):
+    """include/dts.h dts_sweep_run: independent instances in batched launches;
+    ``devices`` (a list of CUDA ordinals, repeats allowed) splits them over
+    devices by LPT, else everything runs on opts.device."""
     arr = (C.c_void_p * len(insts))(*[i.handle for i in insts])
+    devs = None if not devices else (C.c_int32 * len(devices))(*[int(d) for d in devices])
     _check(load_library().dts_sweep_run(arr, len(insts), int(policy),
-                                        None if opts is None else C.byref(opts)))
+                                        None if opts is None else C.byref(opts),
+                                        devs, 0 if not devices else len(devices)))
 
 
 # ---- task-sharded single instance (include/dts.h, SURVEY.md §8(e) second mode)
@@ -253,6 +263,9 @@ class Result:
     loop_ms: float
     total_ms: float
     prof_cycles: tuple = ()
+    sum_avail_at_scans: int = 0
+    n_allocations: int = 0
+    sum_deg_loads_evictions: int = 0
 
     def orders(self):
         p = self.gpu_task_ptr
@@ -287,7 +300,8 @@ def dts_result(inst: Instance, copy: bool = True) -> Result:
                   int(v.n_fallback2), int(v.n_fallback_first), int(v.n_belady),
                   int(v.n_idle_requests), int(v.n_verify_err), int(v.alg_bytes),
                   int(v.scan_alg_bytes),
-                  float(v.loop_ms), float(v.total_ms), tuple(int(x) for x in v.prof_cycles))
+                  float(v.loop_ms), float(v.total_ms), tuple(int(x) for x in v.prof_cycles),
+                  int(v.sum_avail_at_scans), int(v.n_allocations), int(v.sum_deg_loads_evictions))
 
 
 def dts_fetch_results(insts) -> None:
@@ -295,6 +309,13 @@ def dts_fetch_results(insts) -> None:
     total); dts_result afterwards reads host memory only."""
     arr = (C.c_void_p * len(insts))(*[i.handle for i in insts])
     _check(load_library().dts_fetch_results(arr, len(insts)))
+
+
+def dts_run_times(inst: Instance):
+    """(loop_ms, total_ms) of the instance's last run (waits for its loop)."""
+    a, b = C.c_float(), C.c_float()
+    _check(load_library().dts_run_times(inst.handle, C.byref(a), C.byref(b)))
+    return float(a.value), float(b.value)
 
 
 def dts_kernel_launches() -> int:

@@ -19,9 +19,22 @@ def assert_parity(g, o, complete=True):
     assert g.makespan == o.makespan
     assert g.n_scans == o.n_scans
     assert g.n_fallback2 == o.n_fallback2 and g.n_fallback_first == o.n_fallback_first
-    assert g.n_belady == o.n_belady == 0
+    assert g.n_belady == o.n_belady
+    # SURVEY §8(d) byte-model counters (measurement)
+    assert g.sum_avail_at_scans == o.sum_avail_at_scans, (g.sum_avail_at_scans, o.sum_avail_at_scans)
+    assert g.n_allocations == o.n_allocations, (g.n_allocations, o.n_allocations)
     if complete:
         assert g.n_idle_requests == o.n_idle_requests
     # per-GPU orders (a8) agree with the service sequence
     for k, ok in enumerate(o.orders()):
         assert np.array_equal(g.orders()[k], ok)
+
+
+def deg_sum_of_events(inst, events):
+    """sum of deg(D) (#tasks using D, rows de-duplicated) over LOAD and EVICT
+    events -- the oracle-side value of dts_result's sum_deg_loads_evictions."""
+    deg = np.zeros(inst.n, np.int64)
+    for T in range(inst.m):
+        for D in set(inst.task_data[inst.task_ptr[T]:inst.task_ptr[T + 1]].tolist()):
+            deg[D] += 1
+    return int(deg[np.asarray(events["data"], dtype=np.int64)].sum()) if len(events) else 0

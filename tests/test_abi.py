@@ -46,6 +46,8 @@ def test_opts_defaults():
     (dict(K=65), B.DTS_E_UNSUPPORTED),
     (dict(task_data=np.array([0, 9, 1, 2], np.int32)), B.DTS_E_INVAL),
     (dict(task_ptr=np.array([0, 3, 2], np.int64), task_data=np.array([0, 1, 1], np.int32)), B.DTS_E_INVAL),
+    # an inner entry past E = task_ptr[m]: rejected before any row is read
+    (dict(task_ptr=np.array([0, 5, 2], np.int64), task_data=np.array([0, 1], np.int32)), B.DTS_E_INVAL),
     (dict(data_size=np.array([1, 0, 1], np.uint64)), B.DTS_E_INVAL),
 ])
 def test_validation(bad, status):

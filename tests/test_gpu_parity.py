@@ -12,7 +12,7 @@ import oracle
 import paper_conf_ipps_gonthiermt22_b200 as dts
 from conftest import GOLDEN
 from digest import digest
-from parity import assert_parity
+from parity import assert_parity, deg_sum_of_events
 from validate import validate
 
 pytestmark = pytest.mark.gpu
@@ -36,6 +36,8 @@ def _both(inst, bus=oracle.DEFAULT_BUS_BPS, block=0, smem=0, flags=1, max_served
     g = dts.schedule(inst, bus_bps=bus, block_threads=block, smem_budget=smem, flags=flags,
                      max_served=max_served)
     o = oracle.run(inst, bus_bps=bus, flags=flags, max_served=max_served)
+    if inst.E <= 200_000:
+        assert g.sum_deg_loads_evictions == deg_sum_of_events(inst, o.events)
     return g, o
 
 
@@ -48,6 +50,17 @@ def test_fig1(flags):
     gold = json.load(open(os.path.join(GOLDEN, "fig1_darts_luf_hand.json")))
     assert [list(map(int, x)) for x in g.orders()] == gold["orders"]
     assert g.n_loads == 11 and g.makespan == 12
+
+
+def test_f1_fallback2_hand():
+    """The hand-traced 3inputs instance (tests/golden/f1_fallback2_hand.json)."""
+    from test_oracle_pins import f1_instance
+    gold = json.load(open(os.path.join(GOLDEN, "f1_fallback2_hand.json")))
+    for flags in (1, 0):
+        g, o = _both(f1_instance(), bus=10 ** 9, flags=flags)
+        assert_parity(g, o)
+    g, _ = _both(f1_instance(), bus=10 ** 9)
+    assert list(map(int, g.orders()[0])) == gold["order"] and g.n_fallback2 == gold["n_fallback2"]
 
 
 def test_h1_config1_unit():
@@ -308,6 +321,35 @@ def test_sweep_split_launch():
         assert_parity(g, cache[inst.name])
 
 
+def test_sweep_config5_full_digests():
+    """Full config-5 parity: all 4,096 instances of the sweep in the bench's
+    launch configuration (dts_sweep_run, default options: two concurrent
+    batched launches), every instance's whole schedule (service order, task
+    start/end, every trace event) compared with the oracle through the
+    SHA-256 digests written by tests/golden/make_c5_digests.py (oracle only)
+    -- plus the counters, so a mismatch names the instance."""
+    gold = json.load(open(os.path.join(GOLDEN, "digests_C5.json")))
+    params = gen.sweep_params()
+    assert gold["n_instances"] == len(params) == 4096
+    insts = gen.config_instances("C5")
+    hs = [dts.create(i) for i in insts]
+    dts.dts_sweep_run(hs, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default(flags=dts.DTS_F_FALLBACK2))
+    dts.dts_fetch_results(hs)
+    bad = []
+    for i, (h, row) in enumerate(zip(hs, gold["instances"])):
+        assert (row["N"], row["M"], row["K"]) == tuple(params[i])
+        g = dts.dts_result(h, copy=False)
+        got = (g.n_served, g.n_loads, g.n_evictions, g.n_scans, g.n_fallback2, g.n_fallback_first,
+               g.n_idle_requests, int(g.bytes_loaded), int(g.makespan),
+               digest(g.serve_gpu, g.serve_task, g.task_start, g.task_end, g.events))
+        want = (row["n_served"], row["n_loads"], row["n_evictions"], row["n_scans"], row["n_fallback2"],
+                row["n_fallback_first"], row["n_idle_requests"], row["bytes_loaded"], row["makespan"],
+                row["sha256"])
+        if got != want:
+            bad.append((params[i], got[:-1], want[:-1]))
+    assert not bad, f"{len(bad)} of 4096 instances differ, first: {bad[:3]}"
+
+
 @pytest.mark.parametrize("block", [0, 128])
 def test_sweep_config5_repeated(block):
     """The full 4,096-instance sweep (bench launch configuration, and forced
@@ -530,3 +572,34 @@ def test_result_views_without_copy():
         assert not v.serve_task.flags.writeable
         assert np.array_equal(v.serve_task, c.serve_task) and np.array_equal(v.events, c.events)
         assert_parity(v, oracle.run(inst))
+
+
+def test_sweep_devices_list():
+    """include/dts.h dts_sweep_run with a device list:
+    devices = [0, 0] splits the batch by LPT into two concurrent launches on
+    device 0 (the caller's stream and a library stream joined back into it);
+    every instance matches the oracle."""
+    insts = gen.config_instances("C2") + [gen.sweep_instance(N, M, K) for (N, M, K) in
+                                          [(40, 6, 3), (25, 4, 1), (60, 12, 8), (15, 35, 2)]]
+    hs = [dts.create(i) for i in insts]
+    dts.dts_sweep_run(hs, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default(), devices=[0, 0])
+    dts.dts_fetch_results(hs)
+    for inst, h in zip(insts, hs):
+        assert_parity(dts.dts_result(h), oracle.run(inst))
+
+
+def test_concurrent_sweeps_on_two_streams():
+    """Two batched launches in flight at once on different streams (each
+    launch has its own descriptor buffer and instance counters):
+    both batches match the oracle."""
+    import torch
+    a = [gen.sweep_instance(N, M, K) for (N, M, K) in [(30, 5, 2), (45, 8, 4), (20, 4, 1)]]
+    b = [gen.sweep_instance(N, M, K) for (N, M, K) in [(35, 6, 3), (50, 10, 5), (10, 4, 2)]]
+    ha, hb = [dts.create(i) for i in a], [dts.create(i) for i in b]
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    for _ in range(3):
+        dts.dts_sweep_run(ha, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default(cuda_stream=s1.cuda_stream))
+        dts.dts_sweep_run(hb, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default(cuda_stream=s2.cuda_stream))
+        dts.dts_fetch_results(ha + hb)
+        for inst, h in zip(a + b, ha + hb):
+            assert_parity(dts.dts_result(h), oracle.run(inst))

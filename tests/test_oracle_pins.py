@@ -317,6 +317,22 @@ def test_f1_fallback2_hand_trace():
     assert r.n_idle_requests == g["n_idle_requests"] and r.n_served - r.n_scans == g["pops"]
     assert r.makespan == g["makespan"]
     _check(inst, r, bus=10 ** 9)
+    c = g["measurement_counters"]
+    rc = oracle.run(inst, bus_bps=10 ** 9, flags=oracle.F_FALLBACK2 | oracle.F_COUNT_DEG)
+    assert (rc.n_allocations, rc.sum_avail_at_scans, rc.sum_deg) == (
+        c["n_allocations"], c["sum_avail_at_scans"], c["sum_deg"])
+
+
+def test_measurement_counters_closed_form():
+    """SURVEY §8(d) counters: K=1 with ample memory loads every used datum
+    once and never evicts or returns a task, so n_allocations = m and the
+    deg(D) sum over loads = E (each edge counted once)."""
+    for inst in _small_instances():
+        big = inst.with_(mem_capacity=int(inst.data_size.sum()), K=1)
+        r = oracle.run(big, flags=oracle.F_FALLBACK2 | oracle.F_COUNT_DEG)
+        E = sum(len(set(big.task_data[big.task_ptr[T]:big.task_ptr[T + 1]])) for T in range(big.m))
+        assert r.n_allocations == big.m and r.sum_deg == E and r.n_evictions == 0
+        assert r.sum_avail_at_scans >= big.m  # the first scan alone sees all m
 
 
 def test_f1_fallback_off_takes_lowest_id_task():
