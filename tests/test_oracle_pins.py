@@ -359,3 +359,64 @@ def test_r18_idle_wake_never_fires(seed):
         for flags in (oracle.F_FALLBACK2, 0, oracle.F_FALLBACK2 | oracle.F_OPTI):
             r = oracle.run(inst, W=W, bus_bps=10 ** 9, flags=flags)
             assert r.n_wakes == 0 and r.n_served == inst.m
+
+
+# -------------------------------------- Belady (Alg. 6 l.6-7) and W >= 2 (R29)
+def belady_instance(g):
+    if "rows" in g:
+        rows = g["rows"]
+        tp = np.zeros(len(rows) + 1, np.int64)
+        tp[1:] = np.cumsum([len(r) for r in rows])
+        td = np.array([d for r in rows for d in r], np.int32)
+        return gen.Instance("belady_rows", tp, td, np.ones(g["data"], np.uint64), None, g["tau"],
+                            g["M"], g["K"])
+    return _unit(gen.matmul2d(g["N"], M=g["M"], K=g["K"]))
+
+
+BELADY_GOLDENS = ["belady_w1_2d_N2.json", "belady_w2_2d_N3.json", "belady_w1_disjoint.json"]
+
+
+@pytest.mark.parametrize("name", BELADY_GOLDENS)
+def test_belady_hand_traces(name):
+    """Alg. 6's Belady branch made reachable by a
+    capacity of max(1, W) tasks' inputs, and a W+1-task taskBuffer
+    (PAPER.md:742-746), under reading R29 -- hand traces."""
+    g = _golden(name)
+    inst = belady_instance(g)
+    r = oracle.run(inst, W=g["W"], bus_bps=10 ** 9)
+    assert list(map(int, r.orders()[0])) == g["order"]
+    ev = [["L" if e["op"] == 0 else "E", int(e["data"]), int(e["task"]), int(e["t"]), int(e["t_end"])]
+          for e in r.events]
+    assert ev == g["events"]
+    assert (r.n_loads, r.n_evictions, r.n_belady) == (g["n_loads"], g["n_evictions"], g["n_belady"])
+    assert (r.n_scans, r.n_fallback2, r.n_idle_requests) == (g["n_scans"], g["n_fallback2"], g["n_idle_requests"])
+    assert r.makespan == g["makespan"]
+    _check(inst, r, W=g["W"], bus=10 ** 9)
+
+
+@pytest.mark.parametrize("W", [1, 2, 3, 5])
+@pytest.mark.parametrize("idx", range(8))
+def test_w_tight_capacity_invariants(W, idx):
+    """Any W with the capacity the library accepts for DARTS+LUF (max(1, W)
+    tasks' inputs): the schedule passes the independent validator (which
+    checks R29's Belady conditions and request times), every task runs."""
+    inst = _small_instances()[idx]
+    row = max(int(inst.data_size[inst.task_data[inst.task_ptr[T]:inst.task_ptr[T + 1]]].sum())
+              for T in range(inst.m))
+    inst = inst.with_(mem_capacity=max(1, W) * row)
+    r = oracle.run(inst, W=W)
+    chk = _check(inst, r, W=W)
+    assert chk["n_loads"] == r.n_loads and chk["makespan"] == r.makespan
+    assert r.n_served == inst.m and r.n_wakes == 0
+
+
+def test_belady_fires_on_random_tight_instances():
+    """The branch is reachable: with W = 2 and 2 tasks' inputs of memory the
+    random shared-input instances trigger it."""
+    tot = 0
+    for seed in range(6):
+        inst = gen.random_shared(400, 64, 3, M=6, K=2, seed=seed)
+        r = oracle.run(inst, W=2)
+        _check(inst, r, W=2)
+        tot += r.n_belady
+    assert tot > 0

@@ -67,12 +67,24 @@ MUTANTS = [
      "* 1000000000u + (s->bw - 1);",
      "* 1000000000u;", "killed"),
     ("W=0 asks for the next task at the start of the current one (R7)",
-     "s->req[k] = (s->W == 0) ? end : start;",
-     "s->req[k] = start;", "killed"),
+     "if (s->W == 0) s->req[k] = end;",
+     "if (s->W == 0) s->req[k] = start;", "killed"),
     ("OPTI takes the best datum instead of the first (R28)",
      "            best = D;\n            break;",
      "            if (best < 0 || better(s->cnt_n[D], s->cnt_u[D], D, s->cnt_n[best], s->cnt_u[best], best)) best = D;\n            continue;",
      "killed"),
+    ("Belady counts the running task's use as a next use (R29)",
+     "const int started = i < nbuf - 1 && s->r->task_start[Tb] <= s->now;",
+     "const int started = 0;", "killed"),
+    ("Belady eviction takes effect at the request, not when the running task ends",
+     "const int64_t te = s->evict_at > t ? s->evict_at : t;",
+     "const int64_t te = t;", "killed"),
+    ("Belady ties to the highest id",
+     "if (pos > far) { far = pos; V = D; }",
+     "if (pos >= far) { far = pos; V = D; }", "killed"),
+    ("W >= 2 asks when its last task starts (as W = 1)",
+     "else if (s->n_on[k] < s->W) s->req[k] = t;",
+     "else if (1) s->req[k] = r->task_start[T];", "killed"),
     ("R18 removed: idle GPUs are not woken when planned tasks return",
      "if (s->idle[j]) { s->idle[j] = 0; s->req[j] = t; s->r->n_wakes++; }",
      "if (0) { s->idle[j] = 0; s->req[j] = t; s->r->n_wakes++; }",
