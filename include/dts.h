@@ -46,7 +46,8 @@ typedef struct dts_instance dts_instance; /* opaque, owned by the library */
 typedef enum {
     DTS_OK = 0,
     DTS_E_INVAL = -1,       /* malformed argument (pointer, range, monotonicity) */
-    DTS_E_CAPACITY = -2,    /* capacity < (W+1) * max_T sum_{D in D(T)} size(D) */
+    DTS_E_CAPACITY = -2,    /* capacity < max(1,W) (DARTS+LUF) or (W+1) (LRU policies)
+                               * max_T sum_{D in D(T)} size(D) */
     DTS_E_NOMEM = -3,       /* host or device allocation failed */
     DTS_E_CUDA = -4,        /* CUDA error, no device, or device is not sm_100 */
     DTS_E_STATE = -5,       /* call out of order (e.g. dts_result before dts_run) */
@@ -90,11 +91,17 @@ enum {
 
 typedef struct {
     uint32_t flags;           /* DTS_F_* ; default DTS_F_FALLBACK2 */
-    uint32_t lookahead_W;     /* taskBuffer depth beyond the served task:
-                                 0 (default, the formal model of §III: a GPU asks for its
-                                 next task when the current one ends) or 1 (StarPU's
-                                 prefetch: it asks when the current one starts, and LUF
-                                 protects both tasks' inputs; reading R7); >1: UNSUPPORTED */
+    uint32_t lookahead_W;     /* taskBuffer depth beyond the running task,
+                                 0..8.  0 (default, the formal model of §III): a GPU asks
+                                 for its next task when the current one ends.  W >= 1
+                                 (StarPU's prefetch, readings R7 / R29): it keeps W tasks
+                                 ahead -- asks when the (j-W+1)-th of its j tasks starts, the
+                                 first W at once; LUF protects the inputs of every task not
+                                 ended.  DARTS+LUF accepts a capacity of max(1, W) tasks'
+                                 inputs: then Alg. 6's Belady branch can fire -- it evicts
+                                 an input of the running task only (no future use), which
+                                 leaves memory when that task ends (the load waits).
+                                 W * (inputs per task) must be <= 128 */
     uint64_t bus_bytes_per_s; /* shared host->GPU bus bandwidth; default 12e9 (reading R9) */
     int32_t device;           /* CUDA device ordinal; default 0 */
     int32_t block_threads;    /* threads of the ONE CTA that runs an instance: a multiple of
@@ -155,7 +162,8 @@ dts_status dts_instance_upload(dts_instance *inst, int32_t device, void *cuda_st
  * resident decision loop -> result assembly.  Returns after enqueueing; the
  * results stay on the device until dts_result (which synchronises).
  * opts may be NULL (defaults).  DTS_E_CAPACITY if the capacity cannot hold
- * (W+1) tasks' inputs (this keeps Alg. 6 l.4's first branch non-empty). */
+ * max(1, W) tasks' inputs for DARTS+LUF (Alg. 6's Belady branch then always
+ * finds a victim, reading R29), (W+1) for the LRU policies. */
 dts_status dts_run(dts_instance *inst, dts_policy policy, const dts_run_opts *opts);
 
 typedef struct {

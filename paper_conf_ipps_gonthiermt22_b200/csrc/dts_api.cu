@@ -513,14 +513,23 @@ dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_op
         return fail(DTS_E_UNSUPPORTED, "policy");
     if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI | DTS_F_PACKED))
         return fail(DTS_E_UNSUPPORTED, "unknown flags");
-    if (o->lookahead_W > 1) return fail(DTS_E_UNSUPPORTED, "lookahead_W > 1");
+    if (o->lookahead_W > (uint32_t)dts::MAX_W) return fail(DTS_E_UNSUPPORTED, "lookahead_W > 8");
+    if ((int64_t)o->lookahead_W * I->max_row_len > dts::MAX_ROW + 1)
+        return fail(DTS_E_UNSUPPORTED, "lookahead_W * (inputs per task) > 128");
     if (o->bus_bytes_per_s == 0) return fail(DTS_E_INVAL, "bus_bytes_per_s == 0");
     if (o->block_threads != 0 && (o->block_threads < 32 || o->block_threads > 512 || o->block_threads % 32))
         return fail(DTS_E_INVAL, "block_threads must be 0 or a multiple of 32 in [32, 512]");
     if (o->smem_budget < -1) return fail(DTS_E_INVAL, "smem_budget < -1");
-    unsigned __int128 need = (unsigned __int128)(o->lookahead_W + 1) * I->max_row_bytes;
+    // DARTS+LUF: max(1, W) tasks' inputs -- with W >= 1 Alg. 6's Belady branch
+    // may fire and always finds a datum only the running task uses (R29);
+    // the LRU policies have no Belady branch: (W+1) tasks' inputs
+    const uint64_t tasks = policy == DTS_POLICY_DARTS_LUF ? std::max<uint64_t>(1, o->lookahead_W)
+                                                          : (uint64_t)o->lookahead_W + 1;
+    unsigned __int128 need = (unsigned __int128)tasks * I->max_row_bytes;
     if ((unsigned __int128)I->cap < need)
-        return fail(DTS_E_CAPACITY, "mem_capacity_bytes < (W+1) * max_T size(D(T))");
+        return fail(DTS_E_CAPACITY, policy == DTS_POLICY_DARTS_LUF
+                                        ? "mem_capacity_bytes < max(1, W) * max_T size(D(T))"
+                                        : "mem_capacity_bytes < (W+1) * max_T size(D(T))");
     return DTS_OK;
 }
 

@@ -48,6 +48,7 @@ constexpr uint32_t CNT_ONE = 1u << 24;
 constexpr uint32_t XOR_MASK = 0x00FFFFFFu;
 constexpr int MAX_K = 64;
 constexpr int MAX_ROW = 127;
+constexpr int MAX_W = 8;  // lookahead_W <= 8: taskBuffer of at most 9 tasks (R7, R29)
 constexpr int ROW_LONG = -2;  // plan entry: |D(T)| > 3, read the row from the CSR
 
 // Scalar results written by the decision loop.

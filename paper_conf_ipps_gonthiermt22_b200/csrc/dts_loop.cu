@@ -89,10 +89,16 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     int32_t plan_head[MAX_K], plan_end[MAX_K], plan_live[MAX_K];
     int32_t res_cnt[MAX_K];
     int32_t idle[MAX_K];
-    int32_t last_task[MAX_K];  // W = 1: the task that may still run when k asks again
-    int64_t last_end[MAX_K];
-    int32_t row2[MAX_ROW + 1];  // its inputs (taskBuffer_k = {running, served}, R7)
+    // W >= 1: the last W tasks served on k (ring by serve count won[k]), the
+    // candidates of taskBuffer_k (R7, R29)
+    int32_t wring[MAX_K][MAX_W];
+    int32_t won[MAX_K];
+    int32_t row2[MAX_ROW + 1];  // inputs of the buffered task running at the request
     int32_t row2_len;
+    int32_t row3[MAX_ROW + 1];  // inputs of the buffered tasks not started yet (W >= 2)
+    int32_t row3_len;
+    int64_t run_end;            // end of the running buffered task (Belady evictions, R29)
+    int64_t mem_ready;          // serve_loads: the freed memory of this serve is available from
     int64_t bus_free;
     int64_t n_events, n_served, n_loads, n_evictions, n_scans, n_fb2, n_fbf, n_belady, n_idle,
         n_verr;
@@ -593,8 +599,22 @@ __device__ __forceinline__ void push_event(uint8_t op, int k, int32_t D, int32_t
     L.n_events = i + 1;
 }
 
+// Thread 0: T (started at `start`) becomes the newest of k's last W served
+// tasks; returns k's next request time (R7 / R29): W = 0 when T ends, W >= 1
+// when the (j-W+1)-th of its j tasks starts -- the first W requests at once
+// (at t).  Task times of earlier tasks are this thread's own writes.
+__device__ __forceinline__ int64_t next_request(int k, int32_t T, int64_t t, int64_t start, int64_t end) {
+    const Inst &I = SI;
+    if (I.W == 0) return end;
+    const int W = I.W;
+    const int j = ++L.won[k];
+    L.wring[k][(j - 1) % W] = T;
+    if (j < W) return t;
+    return W == 1 ? start : __ldcg(&I.tstart[L.wring[k][j % W]]);
+}
+
 // Thread 0: record the service of T on k (time model of PAPER.md:276-342, R7, R9).
-__device__ __forceinline__ void finish_serve(int k, int32_t T, int64_t ready, int64_t tau) {
+__device__ __forceinline__ void finish_serve(int k, int32_t T, int64_t t, int64_t ready, int64_t tau) {
     const Inst &I = SI;
     const int64_t start = ready > L.gpu_free[k] ? ready : L.gpu_free[k];
     const int64_t end = start + tau;
@@ -605,9 +625,7 @@ __device__ __forceinline__ void finish_serve(int k, int32_t T, int64_t ready, in
     I.serve_gpu[L.n_served] = k;
     I.serve_task[L.n_served] = T;
     L.n_served++;
-    L.req[k] = (I.W == 0) ? end : start;  // R7
-    L.last_task[k] = T;
-    L.last_end[k] = end;
+    L.req[k] = next_request(k, T, t, start, end);  // R7, R29
     L.alg_bytes += 24;
 }
 
@@ -735,9 +753,7 @@ __device__ __forceinline__ int pop_run_seq() {
             __stcg(&stk[ns], T);
             ns++;
             pops++;
-            req = (W == 0) ? end : start;  // R7
-            L.last_task[k] = T;
-            L.last_end[k] = end;
+            req = W == 0 ? end : next_request(k, T, req, start, end);  // R7, R29
             if (live == 0 || (maxs >= 0 && ns >= maxs)) break;
             if (k2 >= 0 && (req > t2 || (req == t2 && k2 < k))) break;
         }
@@ -1144,9 +1160,14 @@ __device__ __forceinline__ bool entry_uses(int4 e, int32_t D) {
 // LUF (Alg. 6): among the data in GPU k's memory that the taskBuffer does not
 // use (nb(D) = 0, l.4-5; the taskBuffer = the task being served for W = 0),
 // the one with the fewest uses in plannedTasks_k, lowest id on ties (R1).
-// Block-wide; returns V (or -1: the Belady branch, unreachable, R7) and sets
-// L.vslot to its index in res_list.
-__device__ int32_t luf_victim(int k) {
+// When every resident datum is a buffered input: Belady (l.6-7, reading R29)
+// -- the datum whose next use is the furthest; a datum only the task running
+// at the request uses has no future use, and the capacity check (>= max(1, W)
+// tasks' inputs) guarantees one exists, so the victim is the lowest-id such
+// datum (*belady = 1; it leaves memory when that task ends).  Block-wide;
+// returns V (-1: none -- outside the model) and sets L.vslot to its index in
+// res_list.
+__device__ int32_t luf_victim(int k, int *belady) {
     const Inst &I = SI;
     const View &V = SV;
     const int cnt = L.res_cnt[k];
@@ -1160,14 +1181,35 @@ __device__ int32_t luf_victim(int k) {
         bool in_buf = false;  // nb(D) > 0: an input of a taskBuffer_k task
         for (int r = 0; r < L.row_len; r++) in_buf |= (L.row[r] == D);
         for (int r = 0; r < L.row2_len; r++) in_buf |= (L.row2[r] == D);
+        for (int r = 0; r < L.row3_len; r++) in_buf |= (L.row3[r] == D);
         const unsigned long long key =
             ((unsigned long long)(uint32_t)npk[D] << 32) | (unsigned long long)(uint32_t)D;
         const bool take = !in_buf & (key < best);
         best = take ? key : best;
         bslot = take ? i : bslot;
     }
-    const unsigned long long mine = best;
+    unsigned long long mine = best;
     best = block_min_u64(best);
+    *belady = 0;
+    if (best == ~0ull && I.policy == DTS_POLICY_DARTS_LUF && I.W >= 1) {
+        // Alg. 6 l.6-7: every resident datum is buffered -> one used by the
+        // running task only (no future use), lowest id
+        best = ~0ull;
+        bslot = -1;
+        for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
+            const int32_t D = rl[i];
+            bool run = false, later = false;
+            for (int r = 0; r < L.row2_len; r++) run |= (L.row2[r] == D);
+            for (int r = 0; r < L.row_len; r++) later |= (L.row[r] == D);
+            for (int r = 0; r < L.row3_len; r++) later |= (L.row3[r] == D);
+            const bool take = run & !later & ((unsigned long long)D < best);
+            best = take ? (unsigned long long)D : best;
+            bslot = take ? i : bslot;
+        }
+        mine = best;
+        best = block_min_u64(best);
+        *belady = 1;
+    }
     if (best == ~0ull) return -1;
     if (mine == best) L.vslot = bslot;  // the one thread holding V (ids are unique)
     cta_sync();
@@ -1176,7 +1218,7 @@ __device__ int32_t luf_victim(int k) {
 
 // Alg. 6 l.8-9: planned tasks of k that use V return to the shared pool (R4,
 // idle GPUs wake at t, R18); then V leaves GPU k's memory.  Block-wide.
-__device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
+__device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t, int64_t te) {
     const Inst &I = SI;
     const View &V = SV;
     int4 *pl = V.plan + (size_t)k * I.plan_cap;
@@ -1212,7 +1254,8 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t) {
         V.resb[(size_t)k * I.nw + (Vd >> 5)] &= ~(1u << (Vd & 31));
         L.used[k] -= size_of(Vd);
         L.n_evictions++;
-        push_event(1, k, Vd, Tserved, t, t);
+        push_event(1, k, Vd, Tserved, te, te);  // te > t: a Belady eviction waits for the running task (R29)
+        if (te > L.mem_ready) L.mem_ready = te;
         int64_t sb, se;
         seg_of(Vd, sb, se);
         L.alg_bytes += 24ull * (uint64_t)(se - sb) + (uint64_t)nret * (8ull * I.K + 40ull) + 32ull;
@@ -1235,18 +1278,39 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
     // a taskBuffer task), so the list is fixed up front: one barrier.
     if (threadIdx.x == 0) {
         L.ready = t;
+        L.mem_ready = t;
         L.row2_len = 0;
+        L.row3_len = 0;
         int nm = 0;
         for (int r = 0; r < L.row_len; r++)
             if (!resident(k, L.row[r])) L.miss[nm++] = L.row[r];
         L.nmiss = nm;
     }
-    // W = 1: taskBuffer_k also holds the task still running on k (R7)
-    if (I.W >= 1 && L.last_task[k] >= 0 && L.last_end[k] > t && threadIdx.x < 32) {
-        const int32_t Tr = L.last_task[k];
-        const int64_t rb = __ldg(&I.tptr[Tr]), re = __ldg(&I.tptr[Tr + 1]);
-        for (int r = threadIdx.x; r < (int)(re - rb); r += 32) L.row2[r] = __ldg(&I.tdat[rb + r]);
-        if (threadIdx.x == 0) L.row2_len = (int)(re - rb);
+    // W >= 1: taskBuffer_k also holds the tasks served on k that have not
+    // ended by t (R7, R29): the running one's inputs -> row2, the inputs of
+    // those not started yet -> row3 (warp 0, oldest first)
+    if (I.W >= 1 && threadIdx.x < 32) {
+        const int W = I.W, j = L.won[k];
+        for (int q = j > W ? j - W : 0; q < j; q++) {
+            const int32_t Tq = L.wring[k][q % W];
+            const int64_t st = __ldcg(&I.tstart[Tq]), en = __ldcg(&I.tend[Tq]);
+            if (en <= t) continue;
+            const bool run = st <= t;
+            const int64_t rb = __ldg(&I.tptr[Tq]), re = __ldg(&I.tptr[Tq + 1]);
+            const int base = run ? L.row2_len : L.row3_len;
+            int32_t *dst = run ? L.row2 : L.row3;
+            for (int r = threadIdx.x; r < (int)(re - rb); r += 32) dst[base + r] = __ldg(&I.tdat[rb + r]);
+            __syncwarp();
+            if (threadIdx.x == 0) {
+                if (run) {
+                    L.row2_len = base + (int)(re - rb);
+                    L.run_end = en;
+                } else {
+                    L.row3_len = base + (int)(re - rb);
+                }
+            }
+            __syncwarp();
+        }
     }
     cta_sync();
     const int nmiss = L.nmiss;
@@ -1258,15 +1322,17 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
             cta_sync();
             if (!full) break;
             PROF_T0(p_luf);
-            const int32_t Vd = luf_victim(k);
+            int belady = 0;
+            const int32_t Vd = luf_victim(k, &belady);
             PROF_ADD(L, P_LUF, p_luf);
             if (Vd < 0) {
                 if (threadIdx.x == 0) L.error = 1;
                 cta_sync();
                 return;
             }
+            if (belady && threadIdx.x == 0) L.n_belady++;
             PROF_T0(p_ev);
-            evict(k, Vd, T, t);
+            evict(k, Vd, T, t, belady ? (L.run_end > t ? L.run_end : t) : t);
             PROF_ADD(L, P_EVICT, p_ev);
         }
         if (threadIdx.x == 0) {
@@ -1274,7 +1340,8 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
             rl[L.res_cnt[k]++] = D;
             V.resb[(size_t)k * I.nw + (D >> 5)] |= 1u << (D & 31);
             L.used[k] += sz;
-            const int64_t st = L.bus_free > t ? L.bus_free : t;
+            int64_t st = L.bus_free > t ? L.bus_free : t;
+            if (L.mem_ready > st) st = L.mem_ready;  // its memory is freed then (R29)
             const int64_t en = st + delta_of(D);
             L.bus_free = en;
             if (en > L.ready) L.ready = en;
@@ -1299,7 +1366,7 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
             int32_t *lk = V.lru + (size_t)k * I.nstr;
             for (int r = 0; r < L.row_len; r++) lk[L.row[r]] = (int32_t)L.n_served;
         }
-        finish_serve(k, T, L.ready, tau_of(T));
+        finish_serve(k, T, t, L.ready, tau_of(T));
     }
     cta_sync();
 }
@@ -2163,8 +2230,7 @@ __global__ void __launch_bounds__(512, 1)
                 L.plan_head[k] = L.plan_end[k] = L.plan_live[k] = 0;
                 L.res_cnt[k] = 0;
                 L.idle[k] = 0;
-                L.last_task[k] = -1;
-                L.last_end[k] = 0;
+                L.won[k] = 0;
             }
             L.bus_free = 0;
             L.n_events = L.n_served = L.n_loads = L.n_evictions = L.n_scans = L.n_fb2 = L.n_fbf =

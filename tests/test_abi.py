@@ -88,7 +88,7 @@ def test_unsupported_options():
     i = gen.fig1()
     h = dts.dts_instance_create(i.task_ptr, i.task_data, i.data_size, None, 1, 4, 2)
     with pytest.raises(dts.DtsError) as e:
-        dts.dts_run(h, opts=dts.dts_run_opts_default(lookahead_W=2))
+        dts.dts_run(h, opts=dts.dts_run_opts_default(lookahead_W=9))  # taskBuffer > 9 tasks
     assert e.value.status == B.DTS_E_UNSUPPORTED
 
 

@@ -603,3 +603,78 @@ def test_concurrent_sweeps_on_two_streams():
         dts.dts_fetch_results(ha + hb)
         for inst, h in zip(a + b, ha + hb):
             assert_parity(dts.dts_result(h), oracle.run(inst))
+
+
+# ---------------------------------------- W >= 2 and Alg. 6's Belady branch (R29)
+def _tight(inst, W):
+    """The least capacity the library accepts for DARTS+LUF with window W:
+    max(1, W) tasks' inputs (Belady fires, reading R29)."""
+    row = max(int(inst.data_size[inst.task_data[inst.task_ptr[T]:inst.task_ptr[T + 1]]].sum())
+              for T in range(inst.m))
+    return inst.with_(mem_capacity=max(1, W) * row)
+
+
+@pytest.mark.parametrize("name", ["belady_w1_2d_N2.json", "belady_w2_2d_N3.json", "belady_w1_disjoint.json"])
+def test_belady_hand_traces_gpu(name):
+    from test_oracle_pins import belady_instance
+    gold = json.load(open(os.path.join(GOLDEN, name)))
+    inst = belady_instance(gold)
+    g = dts.schedule(inst, W=gold["W"], bus_bps=10 ** 9)
+    o = oracle.run(inst, W=gold["W"], bus_bps=10 ** 9)
+    assert_parity(g, o)
+    assert g.n_belady == gold["n_belady"] > 0
+    assert list(map(int, g.orders()[0])) == gold["order"]
+
+
+@pytest.mark.parametrize("W", [1, 2, 3, 5, 8])
+@pytest.mark.parametrize("idx", range(12))
+def test_w_tight_shapes(W, idx):
+    inst = _tight(_shapes()[idx], W)
+    if W * max(inst.task_ptr[1:] - inst.task_ptr[:-1]) > 128:
+        pytest.skip("W * inputs per task > 128 (UNSUPPORTED by design)")
+    g, o = dts.schedule(inst, W=W), oracle.run(inst, W=W)
+    assert_parity(g, o)
+    validate(inst, g.serve_gpu, g.serve_task, g.events, g.task_start, g.task_end, W=W)
+
+
+@pytest.mark.parametrize("W", [2, 4])
+@pytest.mark.parametrize("name", ["darts_lru", "eager_lru"])
+def test_w_lru_policies(W, name):
+    """LRU policies with W >= 2 (their capacity check keeps (W+1) tasks)."""
+    for inst in _shapes()[:6]:
+        inst = inst.with_(mem_capacity=int(inst.mem_capacity) + (W + 1) * 3 * int(inst.data_size.max()))
+        pol = _POL[name]
+        g = dts.schedule(inst, policy=pol[0], W=W)
+        o = oracle.run(inst, W=W, flags=1 | pol[1])
+        assert_parity(g, o)
+
+
+def test_w2_configs_tight():
+    """Paper-scale shapes with W = 2 and the tight capacity: C2's largest
+    instances, C3, and a C4a / C4b prefix; Belady fires."""
+    bel = 0
+    for inst in gen.config_instances("C2")[8:10] + gen.config_instances("C3"):
+        inst = _tight(inst, 2)
+        g, o = dts.schedule(inst, W=2), oracle.run(inst, W=2)
+        assert_parity(g, o)
+        bel += g.n_belady
+    for cfg in ("C4a", "C4b"):
+        inst = _tight(gen.config_instances(cfg)[0], 2)
+        g = dts.schedule(inst, W=2, max_served=1500)
+        o = oracle.run(inst, W=2, max_served=1500)
+        assert_parity(g, o, complete=False)
+    assert bel > 0
+
+
+def test_capacity_check_by_policy():
+    """DARTS+LUF accepts max(1, W) tasks' inputs, the LRU policies (W+1)."""
+    inst = _tight(gen.matmul2d(6, M=4, K=1), 2)
+    h = dts.create(inst)
+    dts.dts_run(h, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default(lookahead_W=2))
+    dts.dts_result(h)
+    with pytest.raises(dts.DtsError) as e:
+        dts.dts_run(h, dts.DTS_POLICY_DARTS_LRU, dts.dts_run_opts_default(lookahead_W=2))
+    assert e.value.status == -2
+    with pytest.raises(dts.DtsError) as e:
+        dts.dts_run(h, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default(lookahead_W=9))
+    assert e.value.status == -6
