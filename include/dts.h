@@ -86,13 +86,7 @@ enum {
      * (cnt:7 | xor:24, 4 K m bytes) even when every task has <= 3 inputs
      * (default then: no per-GPU task state, the missing inputs are read off
      * the task's row and the residency bitmaps). */
-    DTS_F_PACKED = 1u << 4,
-    /* Diagnostic: run a large instance on ONE CTA even when it qualifies for
-     * the cluster mode (default for n >= 4096 data: a thread-block cluster --
-     * the CTA running the decision loop plus up to 15 helper CTAs that hold
-     * the scores n_k(D), n2_k(D), u(D) by datum slice in their shared memory
-     * and compute the argmax slices). */
-    DTS_F_NOCLUSTER = 1u << 5
+    DTS_F_PACKED = 1u << 4
 };
 
 typedef struct {

@@ -513,8 +513,7 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
 dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_opts *o) {
     if (policy != DTS_POLICY_DARTS_LUF && policy != DTS_POLICY_DARTS_LRU && policy != DTS_POLICY_EAGER_LRU)
         return fail(DTS_E_UNSUPPORTED, "policy");
-    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI | DTS_F_PACKED |
-                               DTS_F_NOCLUSTER))
+    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI | DTS_F_PACKED))
         return fail(DTS_E_UNSUPPORTED, "unknown flags");
     if (o->lookahead_W > (uint32_t)dts::MAX_W) return fail(DTS_E_UNSUPPORTED, "lookahead_W > 8");
     if ((int64_t)o->lookahead_W * I->max_row_len > dts::MAX_ROW + 1)
@@ -557,14 +556,12 @@ double instance_cost(const dts_instance *I) {
 // Shared-memory placement of one instance's state:
 // greedy, most latency-critical array first, each either fully in the CTA's
 // dynamic shared memory or in its global home.  Returns the bytes used.
-// no_scores: h, h2, u stay out of this CTA's shared memory (task shards: peers
-// read them; cluster mode: they live in the helper CTAs).
-int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool no_scores, bool sl) {
+int place_smem(dts::Inst &h, bool has_tau, int budget, bool lru, bool shard, bool sl) {
     const int64_t K = h.K, n = h.n;
     int used = 0;
     auto put = [&](int32_t &so, int64_t bytes) {
         bytes = (bytes + 15) & ~int64_t(15);
-        const bool peer_read = no_scores && (&so == &h.so_u || &so == &h.so_h || &so == &h.so_h2);
+        const bool peer_read = shard && (&so == &h.so_u || &so == &h.so_h || &so == &h.so_h2);
         if (budget > 0 && !peer_read && used + bytes <= budget) {
             so = used;
             used += (int)bytes;
@@ -619,32 +616,6 @@ int auto_block(const dts_instance *I, bool alone = false) {
 }
 
 
-// Cluster mode: a large instance (n >= 4096 data)
-// whose scores fit the 32-bit argmax keys runs on a thread-block cluster --
-// the leader CTA (the decision loop) plus H <= 15 helper CTAs holding h, h2, u
-// by datum slice of S = 2^csh data, S the largest power of two whose slices
-// ((2K+1) S int32) fit a CTA's shared memory.  Returns H (0: one CTA).
-constexpr int CLUSTER_MIN_N = 4096;
-int cluster_helpers(const dts_instance *I, dts_policy policy, const dts_run_opts &o, bool fused, int *csh,
-                    int *bytes) {
-    *csh = 0;
-    *bytes = 0;
-    if (I->G != 1 || fused || (o.flags & (DTS_F_NOCLUSTER | DTS_F_VERIFY)) || policy == DTS_POLICY_EAGER_LRU)
-        return 0;
-    if (I->n < CLUSTER_MIN_N || I->max_deg_ub >= 32768) return 0;
-    const int64_t budget = max_dyn_smem(o.device);
-    for (int sh = 14; sh >= 8; sh--) {
-        const int64_t S = int64_t(1) << sh, b = (2 * (int64_t)I->K + 1) * S * 4;
-        if (b > budget) continue;
-        const int64_t H = ((int64_t)I->n + S - 1) / S;
-        if (H > dts::MAX_HELPERS) return 0;  // smaller slices would need still more helpers
-        *csh = sh;
-        *bytes = (int)b;
-        return (int)H;
-    }
-    return 0;
-}
-
 // Enqueue everything of one instance up to (not including) the decision loop:
 // upload if needed, CSR build (a1), state init (a2), descriptor H2D.
 // Shared scratch of the fused in-CTA CSR build (dts_loop.cu fused_build).
@@ -680,14 +651,7 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     }
     // row-derived state (no per-(GPU, task) words) when every edge record holds its row
     h.sl = I->G == 1 && I->max_row_len <= 3 && !(o.flags & DTS_F_PACKED) ? 1 : 0;
-    // small instances: the loop CTA builds its own CSR and state (one launch)
-    const int fs = fused_scratch_bytes(I, block);
-    h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
-    int csh = 0, cbytes = 0;
-    h.cl = cluster_helpers(I, policy, o, h.fused != 0, &csh, &cbytes);
-    h.csh = csh;
-    place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF, I->G > 1 || h.cl > 0, h.sl != 0);
-    if (h.cl) h.smem_bytes = std::max(h.smem_bytes, cbytes);  // every CTA of the cluster gets this much
+    place_smem(h, I->has_tau, budget, policy != DTS_POLICY_DARTS_LUF, I->G > 1, h.sl != 0);
     h.G = I->G;
     h.g = I->g;
     h.t_lo = I->G > 1 ? I->t_lo : 0;
@@ -698,6 +662,9 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     h.xsys = I->xsys ? 1 : 0;
     h.pop_batch_min = tuning("DTS_POP_BATCH_MIN", 10);
     h.poison = tuning("DTS_POISON", 0);  // debug (profiling build only)
+    // small instances: the loop CTA builds its own CSR and state (one launch)
+    const int fs = fused_scratch_bytes(I, block);
+    h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
     if (h.fused) h.smem_bytes = std::max(h.smem_bytes, fs);
     h.smem_bytes = std::max(h.smem_bytes, dts::ASSEMBLE_SMEM_BYTES);  // result assembly's scratch
     if (own_events) {
@@ -747,8 +714,6 @@ struct DeviceSweep {
     bool init = false;
     cudaStream_t side = nullptr;  // group B of a split batch (forked from / joined into the caller's stream)
     cudaEvent_t fork = nullptr, join = nullptr;
-    cudaStream_t side_c = nullptr;  // the cluster-mode instances of a mixed batch
-    cudaEvent_t join_c = nullptr;
     std::vector<cudaStream_t> extra;  // library streams for multi-device sweeps (dts_sweep_run devices[])
 };
 DeviceSweep g_dev[64];
@@ -759,8 +724,6 @@ dts_status acquire_slot(DeviceSweep &D, size_t n, SweepSlot **out) {
         CK(cudaEventCreateWithFlags(&D.fork, cudaEventDisableTiming), "cudaEventCreate");
         CK(cudaEventCreateWithFlags(&D.join, cudaEventDisableTiming), "cudaEventCreate");
         CK(cudaStreamCreateWithFlags(&D.side, cudaStreamNonBlocking), "cudaStreamCreate");
-        CK(cudaEventCreateWithFlags(&D.join_c, cudaEventDisableTiming), "cudaEventCreate");
-        CK(cudaStreamCreateWithFlags(&D.side_c, cudaStreamNonBlocking), "cudaStreamCreate");
         D.init = true;
     }
     SweepSlot &S = D.slot[D.next];
@@ -845,61 +808,28 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     SweepSlot *S = nullptr;
     dts_status s = acquire_slot(D, (size_t)n, &S);
     if (s != DTS_OK) return s;
-    // descriptors: the cluster-mode instances first (one cluster each), then
-    // group A, then group B (one CTA each, pulled from the launch's counters)
-    int nc = 0, na = 0, nbb = 0, csize = 1, block_c = 32, smem_c = 0;
-    smem_a = smem_b = 0;
-    for (int32_t i = 0; i < n; i++) {
-        const dts::Inst &h = insts[ord[(size_t)i]]->h_inst;
-        if (h.cl) {
-            S->h_insts[nc++] = h;
-            csize = std::max(csize, h.cl + 1);
-            block_c = std::max(block_c, i < nb ? block_a : block_b);
-            smem_c = std::max(smem_c, h.smem_bytes);
-        }
-    }
-    for (int pass = 0; pass < 2; pass++)
-        for (int32_t i = 0; i < n; i++) {
-            const dts::Inst &h = insts[ord[(size_t)i]]->h_inst;
-            if (h.cl || (pass == 0) != (i < nb)) continue;
-            S->h_insts[nc + na + nbb] = h;
-            (pass == 0 ? na : nbb)++;
-            (pass == 0 ? smem_a : smem_b) = std::max(pass == 0 ? smem_a : smem_b, h.smem_bytes);
-        }
+    for (int32_t i = 0; i < n; i++) S->h_insts[i] = insts[ord[(size_t)i]]->h_inst;
     CK(cudaMemcpyAsync(S->d_insts, S->h_insts, sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
        "H2D sweep");
     CK(cudaMemsetAsync(S->d_work, 0, 2 * sizeof(int), st), "memset");
     if (any_unfused) CK(dts::launch_init(S->d_insts, n, o.bus_bytes_per_s, work, st), "init");
     CK(cudaEventRecord(sev->loop_begin, st), "event");
-    const bool rest = na + nbb > 0;
-    if (nc > 0) {  // the cluster-mode instances: a cluster launch (side stream when others run too)
-        cudaStream_t sc = rest ? D.side_c : st;
-        if (rest) {
-            CK(cudaEventRecord(D.fork, st), "event");
-            CK(cudaStreamWaitEvent(sc, D.fork, 0), "wait");
-        }
-        CK(dts::launch_cluster(S->d_insts, nc, csize, block_c, smem_c, sc), "loop (cluster)");
-        if (rest) CK(cudaEventRecord(D.join_c, sc), "event");
-    }
-    const bool two = na > 0 && nbb > 0;
+    const bool two = nb > 0 && nb < n;
     if (two) {  // group B on the side stream, forked from and joined back into st
         CK(cudaEventRecord(D.fork, st), "event");
         CK(cudaStreamWaitEvent(D.side, D.fork, 0), "wait");
         const int per_b = std::max(1, dts::loop_max_blocks_per_sm(block_b, smem_b));
-        const int grid_b = (int)std::min<int64_t>((int64_t)nbb, (int64_t)per_b * nsm);
-        CK(dts::launch_loop(S->d_insts + nc + na, nbb, block_b, grid_b, S->d_work + 1, smem_b, D.side), "loop B");
+        const int grid_b = (int)std::min<int64_t>((int64_t)(n - nb), (int64_t)per_b * nsm);
+        CK(dts::launch_loop(S->d_insts + nb, n - nb, block_b, grid_b, S->d_work + 1, smem_b, D.side), "loop B");
         CK(cudaEventRecord(D.join, D.side), "event");
     }
-    if (rest) {
-        const int nr = two ? na : na + nbb;
-        const int blk = two ? block_a : (na > 0 ? block_a : block_b);
-        const int sm = two ? smem_a : std::max(smem_a, smem_b);
-        const int per = std::max(1, dts::loop_max_blocks_per_sm(blk, sm));
-        const int grid = (int)std::min<int64_t>((int64_t)nr, (int64_t)per * nsm);
-        CK(dts::launch_loop(S->d_insts + nc, nr, blk, grid, S->d_work, sm, st), "loop");
-    }
+    const int na = two ? nb : n;
+    const int blk = two ? block_a : std::max(block_a, block_b);
+    const int sm = two ? smem_a : std::max(smem_a, smem_b);
+    const int per = std::max(1, dts::loop_max_blocks_per_sm(blk, sm));
+    const int grid = (int)std::min<int64_t>((int64_t)na, (int64_t)per * nsm);
+    CK(dts::launch_loop(S->d_insts, na, blk, grid, S->d_work, sm, st), "loop");
     if (two) CK(cudaStreamWaitEvent(st, D.join, 0), "wait");
-    if (nc > 0 && rest) CK(cudaStreamWaitEvent(st, D.join_c, 0), "wait");
     CK(cudaEventRecord(sev->loop_end, st), "event");
     CK(cudaEventRecord(S->done, st), "event");
     for (int32_t i = 0; i < n; i++) {
@@ -956,10 +886,7 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     if (!I->h_inst.fused) CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
     CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
     CK(cudaEventRecord(I->ev[1], st), "event");
-    if (I->h_inst.cl)
-        CK(dts::launch_cluster(I->d_inst, 1, I->h_inst.cl + 1, block, I->h_inst.smem_bytes, st), "loop (cluster)");
-    else
-        CK(dts::launch_loop(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");
+    CK(dts::launch_loop(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");
     CK(cudaEventRecord(I->ev[2], st), "event");
     CK(cudaEventRecord(I->ev[3], st), "event");
     I->ran = true;

@@ -48,10 +48,9 @@ constexpr uint32_t CNT_ONE = 1u << 24;
 constexpr uint32_t XOR_MASK = 0x00FFFFFFu;
 constexpr int MAX_K = 64;
 constexpr int MAX_ROW = 127;
-constexpr int MAX_W = 8;
-constexpr int MAX_HELPERS = 15;
+constexpr int MAX_W = 8;  // lookahead_W <= 8: taskBuffer of at most 9 tasks (R7, R29)
 // result assembly's scratch in the CTA's dynamic shared memory (after the loop)
-constexpr int ASSEMBLE_SMEM_BYTES = 8 * MAX_K + 4 * MAX_K + 4 * 16 * MAX_K;  // cluster mode: helper CTAs (a cluster of <= 16, non-portable size)  // lookahead_W <= 8: taskBuffer of at most 9 tasks (R7, R29)
+constexpr int ASSEMBLE_SMEM_BYTES = 8 * MAX_K + 4 * MAX_K + 4 * 16 * MAX_K;
 constexpr int ROW_LONG = -2;  // plan entry: |D(T)| > 3, read the row from the CSR
 
 // Scalar results written by the decision loop.
@@ -163,10 +162,6 @@ struct Inst {
     int32_t so_al;            // shared-memory offset of al, -1 = global home
     uint32_t *al;             // [m_pad / 32 + 1] global home
     int32_t poison;  // debug (env DTS_POISON=1): fill the CTA's dynamic shared memory at instance start
-    // cluster mode (large instances, dts_cluster_kernel): the leader CTA runs
-    // the decision loop; cl helper CTAs of its cluster hold the score arrays
-    // h, h2, u by datum slice of 2^csh data and compute the argmax slices
-    int32_t cl, csh;
     int32_t *wring;  // [K][MAX_W] W >= 1: the last W tasks served on each simulated GPU
 };
 

@@ -26,7 +26,6 @@
 // barrier and no global read: a planned task has all its inputs resident
 // (its inputs were resident or Dopt when planned; LUF drops planned tasks whose
 // inputs it evicts, Alg. 6 l.8), so serving it is pure time-model arithmetic.
-#include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
 #include <climits>
@@ -93,10 +92,8 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     // W >= 1: tasks served on k so far; the last W of them (I.wring[k][.], a
     // ring by this count) are the candidates of taskBuffer_k (R7, R29)
     int32_t won[MAX_K];
-    int32_t row2[MAX_ROW + 1];  // inputs of the buffered task running at the request
-    int32_t row2_len;
-    int32_t row3[MAX_ROW + 1];  // inputs of the buffered tasks not started yet (W >= 2)
-    int32_t row3_len;
+    int32_t row2[MAX_ROW + 1];  // inputs of the other buffered tasks: [0, row2_run) those of
+    int32_t row2_len, row2_run; // the task running at the request, then those not started (R29)
     int64_t run_end;            // end of the running buffered task (Belady evictions, R29)
     int64_t mem_ready;          // serve_loads: the freed memory of this serve is available from
     int64_t bus_free;
@@ -126,7 +123,6 @@ struct Lead {  // leader scalars + broadcast slots (static shared memory)
     int64_t xe;      // task shards: exchanges done in this run
     int32_t xerr;    // task shards: a peer did not arrive in time (the run is abandoned)
     int32_t xoff[MAX_G + 1];  // plan exchange: each shard's offset in the merged plan
-    uint32_t cl_seq;          // cluster mode: requests sent to the helpers
 };
 
 // Per-instance views: shared-memory arrays where placed, else global homes.
@@ -140,12 +136,6 @@ struct View {
     int32_t *dptr32;    // shared-memory copy of dptr, or nullptr
     int32_t *lru;       // [K][nstr] last-use stamps (LRU policies)
     uint32_t *al;       // row-derived mode: allocation bitmap (bit set = left the pool)
-    // cluster mode (Inst::cl): h, h2, u live in the helper CTAs of this CTA's
-    // thread-block cluster, datum slice q = [q cS, (q+1) cS) in helper q+1's
-    // shared memory as h[K][cS], h2[K][cS], u[cS] from cb[q] (generic
-    // addresses in the cluster's distributed shared-memory window)
-    int32_t cl, csh, cS;
-    int32_t *cb[MAX_HELPERS];
 };
 
 // Per-CTA state at namespace scope, so the (non-inlined) phase functions
@@ -155,54 +145,6 @@ __shared__ Lead L;
 __shared__ Inst SI;
 __shared__ View SV;
 __shared__ ShardPeer SP[MAX_G];  // task shards: the peer table (copied at instance start)
-
-// The score arrays h_k(D) (n_k, Alg. 5 l.5), h2_k(D) (3inputs) and u(D) (R23):
-// this CTA's view (shared-memory placement or global home) or, in cluster
-// mode, the helper CTA that owns D's datum slice (remote atomics over DSMEM;
-// made visible to the helpers by the cluster barrier of the next argmax).
-__device__ __forceinline__ int32_t *h_at(int k, int32_t D) {
-    if (SV.cl) return SV.cb[D >> SV.csh] + (size_t)k * SV.cS + (D & (SV.cS - 1));
-    return SV.h + (size_t)k * SI.nstr + D;
-}
-__device__ __forceinline__ int32_t *h2_at(int k, int32_t D) {
-    if (SV.cl) return SV.cb[D >> SV.csh] + (size_t)(SI.K + k) * SV.cS + (D & (SV.cS - 1));
-    return SV.h2 + (size_t)k * SI.nstr + D;
-}
-__device__ __forceinline__ int32_t *u_at(int32_t D) {
-    if (SV.cl) return SV.cb[D >> SV.csh] + (size_t)(2 * SI.K) * SV.cS + (D & (SV.cS - 1));
-    return SV.u + D;
-}
-
-struct ClReq {
-    int32_t cmd, k;
-    uint32_t seq;
-    int32_t pad;
-};
-enum : int32_t { CL_SCAN = 1, CL_OPTI = 2, CL_EXIT = 4 };
-__shared__ ClReq CR;                                  // helper: the current request (written by the leader)
-__shared__ unsigned long long CK[MAX_HELPERS][2];     // leader: each helper's (main, 3inputs) slice key
-__shared__ uint32_t CKS[MAX_HELPERS];                 // leader: the request number those keys answer
-
-__device__ __forceinline__ void cl_arrive() {
-    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void cl_wait() {
-    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void cluster_barrier() {
-    cl_arrive();
-    cl_wait();
-}
-__device__ __forceinline__ void st_release_cluster(uint32_t *p, uint32_t v) {
-    asm volatile("st.release.cluster.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ uint32_t ld_acquire_cluster(const uint32_t *p) {
-    uint32_t v;
-    asm volatile("ld.acquire.cluster.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-
-
 
 // Warp reductions with redux.sync (one instruction per 32-bit reduction): a
 // 64-bit max / min is the high words' extremum, then the low words' among the
@@ -362,7 +304,7 @@ __device__ __noinline__ void pool_move_long_row(int32_t T, int sign, int plan_k,
     const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
     for (int64_t i = rb; i < re; i++) {
         const int32_t D = __ldg(&I.tdat[i]);
-        if (own) atomicAdd(u_at(D), sign);
+        if (own) atomicAdd(&V.u[D], sign);
         if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + D], -sign);
     }
 }
@@ -389,10 +331,10 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
             int32_t a, b;
             const int c = missing_of(j, r.r0, r.r1, r.r2, a, b);
             if (c == 1) {
-                atomicAdd(h_at(j, a), sign);
+                atomicAdd(&V.h[(size_t)j * I.nstr + a], sign);
             } else if (c == 2) {
-                atomicAdd(h2_at(j, a), sign);
-                atomicAdd(h2_at(j, b), sign);
+                atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+                atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
             }
         }
     }
@@ -410,12 +352,12 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
             V.s[(size_t)j * I.m_pad + T] = sign < 0 ? (w | ALLOC_BIT) : (w & ~ALLOC_BIT);
             const uint32_t c = (w >> 24) & 0x7fu;
             if (c == 1u) {
-                atomicAdd(h_at(j, (w & XOR_MASK)), sign);
+                atomicAdd(&V.h[(size_t)j * I.nstr + (w & XOR_MASK)], sign);
             } else if (c == 2u) {
                 int32_t a, b;
                 missing_pair(j, T, r, -1, a, b);
-                atomicAdd(h2_at(j, a), sign);
-                atomicAdd(h2_at(j, b), sign);
+                atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+                atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
             }
         }
     }
@@ -427,7 +369,7 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
 #pragma unroll
     for (int i = 0; i < 3; i++) {
         if (c[i] < 0) continue;
-        if (own) atomicAdd(u_at(c[i]), sign);
+        if (own) atomicAdd(&V.u[c[i]], sign);
         if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[i]], -sign);
     }
 }
@@ -443,7 +385,7 @@ __device__ __noinline__ void pool_item_packed(int4 e, int j, int sign) {
     *sp = sign < 0 ? (w | ALLOC_BIT) : (w & ~ALLOC_BIT);
     const uint32_t c = (w >> 24) & 0x7fu;
     if (c == 1u) {
-        atomicAdd(h_at(j, (w & XOR_MASK)), sign);
+        atomicAdd(&V.h[(size_t)j * I.nstr + (w & XOR_MASK)], sign);
     } else if (c == 2u) {
         int32_t a, b;
         const bool lng = e.w == ROW_LONG;
@@ -454,8 +396,8 @@ __device__ __noinline__ void pool_item_packed(int4 e, int j, int sign) {
         } else {
             missing_pair(j, T, Row{e.y, e.z, lng ? -1 : e.w, len}, -1, a, b);
         }
-        atomicAdd(h2_at(j, a), sign);
-        atomicAdd(h2_at(j, b), sign);
+        atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+        atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
     }
 }
 
@@ -479,10 +421,10 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
                 int32_t a, b;
                 const int c = missing_of(j, e.y, e.z, e.w, a, b);
                 if (c == 1) {
-                    atomicAdd(h_at(j, a), sign);
+                    atomicAdd(&V.h[(size_t)j * I.nstr + a], sign);
                 } else if (c == 2) {
-                    atomicAdd(h2_at(j, a), sign);
-                    atomicAdd(h2_at(j, b), sign);
+                    atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
+                    atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
                 }
                 continue;
             }
@@ -501,7 +443,7 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
 #pragma unroll
             for (int q = 0; q < 3; q++) {
                 if (c[q] < 0) continue;
-                if (own) atomicAdd(u_at(c[q]), sign);
+                if (own) atomicAdd(&V.u[c[q]], sign);
                 if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[q]], -sign);
             }
         }
@@ -543,6 +485,8 @@ __device__ __noinline__ void seg_update_packed(int k, int32_t D, bool load) {
     int64_t b, e;
     seg_of(D, b, e);
     uint32_t *sk = V.s + (size_t)k * I.m_pad;
+    int32_t *hk = V.h + (size_t)k * I.nstr;
+    int32_t *h2k = V.h2 + (size_t)k * I.nstr;
     for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
         const int4 ed = __ldg(&I.dedge[i]);
         const int32_t T = ed.x;
@@ -553,30 +497,30 @@ __device__ __noinline__ void seg_update_packed(int k, int32_t D, bool load) {
         const int32_t x = (int32_t)(w & XOR_MASK);
         if (load) {
             if (c == 1u) {  // 1 -> 0: no longer scores for D
-                atomicSub(h_at(k, D), 1);
+                atomicSub(&hk[D], 1);
             } else if (c == 2u) {  // 2 -> 1: now freed by its other missing datum
                 const int32_t o = x ^ D;
-                atomicSub(h2_at(k, D), 1);
-                atomicSub(h2_at(k, o), 1);
-                atomicAdd(h_at(k, o), 1);
+                atomicSub(&h2k[D], 1);
+                atomicSub(&h2k[o], 1);
+                atomicAdd(&hk[o], 1);
             } else if (c == 3u) {  // 3 -> 2: one load away from two data
                 int32_t a2 = ed.y, b2 = ed.z;  // |D(T)| = 3: both others miss
                 if (ed.w > 3) missing_pair(k, T, Row{-1, -1, -1, ed.w}, -1, a2, b2);
-                atomicAdd(h2_at(k, a2), 1);
-                atomicAdd(h2_at(k, b2), 1);
+                atomicAdd(&h2k[a2], 1);
+                atomicAdd(&h2k[b2], 1);
             }
         } else {
             if (c == 0u) {  // 0 -> 1
-                atomicAdd(h_at(k, D), 1);
+                atomicAdd(&hk[D], 1);
             } else if (c == 1u) {  // 1 -> 2: missing {x, D}
-                atomicSub(h_at(k, x), 1);
-                atomicAdd(h2_at(k, x), 1);
-                atomicAdd(h2_at(k, D), 1);
+                atomicSub(&hk[x], 1);
+                atomicAdd(&h2k[x], 1);
+                atomicAdd(&h2k[D], 1);
             } else if (c == 2u) {  // 2 -> 3
                 int32_t a2 = ed.y, b2 = ed.z;  // |D(T)| = 3: both others missed
                 if (ed.w > 3) missing_pair(k, T, Row{-1, -1, -1, ed.w}, D, a2, b2);
-                atomicSub(h2_at(k, a2), 1);
-                atomicSub(h2_at(k, b2), 1);
+                atomicSub(&h2k[a2], 1);
+                atomicSub(&h2k[b2], 1);
             }
         }
     }
@@ -598,6 +542,8 @@ __device__ void seg_update(int k, int32_t D, bool load) {
     }
     int64_t b, e;
     seg_of(D, b, e);
+    int32_t *hk = V.h + (size_t)k * I.nstr;
+    int32_t *h2k = V.h2 + (size_t)k * I.nstr;
     {  // row-derived state: cnt_k(T) before the change from T's other inputs
         for (int64_t i = b + threadIdx.x; i < e; i += blockDim.x) {
             const int4 ed = __ldg(&I.dedge[i]);
@@ -607,25 +553,25 @@ __device__ void seg_update(int k, int32_t D, bool load) {
             const int32_t o = my ? ed.y : ed.z;                 // the other missing one (c == 2 / 1)
             if (load) {
                 if (c == 1) {  // 1 -> 0
-                    atomicSub(h_at(k, D), 1);
+                    atomicSub(&hk[D], 1);
                 } else if (c == 2) {  // 2 -> 1: now freed by o
-                    atomicSub(h2_at(k, D), 1);
-                    atomicSub(h2_at(k, o), 1);
-                    atomicAdd(h_at(k, o), 1);
+                    atomicSub(&h2k[D], 1);
+                    atomicSub(&h2k[o], 1);
+                    atomicAdd(&hk[o], 1);
                 } else if (c == 3) {  // 3 -> 2
-                    atomicAdd(h2_at(k, ed.y), 1);
-                    atomicAdd(h2_at(k, ed.z), 1);
+                    atomicAdd(&h2k[ed.y], 1);
+                    atomicAdd(&h2k[ed.z], 1);
                 }
             } else {
                 if (c == 0) {  // 0 -> 1
-                    atomicAdd(h_at(k, D), 1);
+                    atomicAdd(&hk[D], 1);
                 } else if (c == 1) {  // 1 -> 2: missing {o, D}
-                    atomicSub(h_at(k, o), 1);
-                    atomicAdd(h2_at(k, o), 1);
-                    atomicAdd(h2_at(k, D), 1);
+                    atomicSub(&hk[o], 1);
+                    atomicAdd(&h2k[o], 1);
+                    atomicAdd(&h2k[D], 1);
                 } else if (c == 2) {  // 2 -> 3
-                    atomicSub(h2_at(k, ed.y), 1);
-                    atomicSub(h2_at(k, ed.z), 1);
+                    atomicSub(&h2k[ed.y], 1);
+                    atomicSub(&h2k[ed.z], 1);
                 }
             }
         }
@@ -1211,60 +1157,67 @@ __device__ __forceinline__ bool entry_uses(int4 e, int32_t D) {
 // LUF (Alg. 6): among the data in GPU k's memory that the taskBuffer does not
 // use (nb(D) = 0, l.4-5; the taskBuffer = the task being served for W = 0),
 // the one with the fewest uses in plannedTasks_k, lowest id on ties (R1).
-// When every resident datum is a buffered input: Belady (l.6-7, reading R29)
-// -- the datum whose next use is the furthest; a datum only the task running
-// at the request uses has no future use, and the capacity check (>= max(1, W)
-// tasks' inputs) guarantees one exists, so the victim is the lowest-id such
-// datum (*belady = 1; it leaves memory when that task ends).  Block-wide;
-// returns V (-1: none -- outside the model) and sets L.vslot to its index in
-// res_list.
-__device__ int32_t luf_victim(int k, int *belady) {
+// Block-wide; returns V (-1: every resident datum is a buffered input -- Alg.
+// 6 l.6-7, belady_victim) and sets L.vslot to its index in res_list.
+__device__ int32_t luf_victim(int k) {
     const Inst &I = SI;
     const View &V = SV;
     const int cnt = L.res_cnt[k];
     const int32_t *rl = V.res_list + (size_t)k * I.res_cap;
     // LUF key np_k(D); LRU policies: the serve index of D's last use on k
     const int32_t *npk = (I.policy == DTS_POLICY_DARTS_LUF ? V.np : V.lru) + (size_t)k * I.nstr;
+    const int nr = L.row_len, nr2 = L.row2_len;
     unsigned long long best = ~0ull;
     int bslot = -1;
     for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
         const int32_t D = rl[i];
         bool in_buf = false;  // nb(D) > 0: an input of a taskBuffer_k task
-        for (int r = 0; r < L.row_len; r++) in_buf |= (L.row[r] == D);
-        for (int r = 0; r < L.row2_len; r++) in_buf |= (L.row2[r] == D);
-        for (int r = 0; r < L.row3_len; r++) in_buf |= (L.row3[r] == D);
+        for (int r = 0; r < nr; r++) in_buf |= (L.row[r] == D);
+        for (int r = 0; r < nr2; r++) in_buf |= (L.row2[r] == D);
         const unsigned long long key =
             ((unsigned long long)(uint32_t)npk[D] << 32) | (unsigned long long)(uint32_t)D;
         const bool take = !in_buf & (key < best);
         best = take ? key : best;
         bslot = take ? i : bslot;
     }
-    unsigned long long mine = best;
+    const unsigned long long mine = best;
     best = block_min_u64(best);
-    *belady = 0;
-    if (best == ~0ull && I.policy == DTS_POLICY_DARTS_LUF && I.W >= 1) {
-        // Alg. 6 l.6-7: every resident datum is buffered -> one used by the
-        // running task only (no future use), lowest id
-        best = ~0ull;
-        bslot = -1;
-        for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
-            const int32_t D = rl[i];
-            bool run = false, later = false;
-            for (int r = 0; r < L.row2_len; r++) run |= (L.row2[r] == D);
-            for (int r = 0; r < L.row_len; r++) later |= (L.row[r] == D);
-            for (int r = 0; r < L.row3_len; r++) later |= (L.row3[r] == D);
-            const bool take = run & !later & ((unsigned long long)D < best);
-            best = take ? (unsigned long long)D : best;
-            bslot = take ? i : bslot;
-        }
-        mine = best;
-        best = block_min_u64(best);
-        *belady = 1;
-    }
     if (best == ~0ull) return -1;
     if (mine == best) L.vslot = bslot;  // the one thread holding V (ids are unique)
     cta_sync();
     return (int32_t)(best & 0xffffffffull);
+}
+
+// Alg. 6 l.6-7 (reading R29), when every resident datum of GPU k is an input
+// of a buffered task: Belady -- the datum whose next use in taskBuffer_k is
+// the furthest.  A datum only the task running at the request uses has no
+// future use, and the capacity check (>= max(1, W) tasks' inputs) guarantees
+// one exists, so the victim is the lowest-id such datum; it leaves memory
+// when that task ends (L.run_end).  Block-wide, out of line (W >= 1 only);
+// returns V (-1: none) and sets L.vslot.
+__device__ __noinline__ int32_t belady_victim(int k) {
+    const Inst &I = SI;
+    const View &V = SV;
+    const int cnt = L.res_cnt[k];
+    const int32_t *rl = V.res_list + (size_t)k * I.res_cap;
+    unsigned long long best = ~0ull;
+    int bslot = -1;
+    for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
+        const int32_t D = rl[i];
+        bool run = false, later = false;
+        for (int r = 0; r < L.row2_run; r++) run |= (L.row2[r] == D);
+        for (int r = 0; r < L.row_len; r++) later |= (L.row[r] == D);
+        for (int r = L.row2_run; r < L.row2_len; r++) later |= (L.row2[r] == D);
+        const bool take = run & !later & ((unsigned long long)D < best);
+        best = take ? (unsigned long long)D : best;
+        bslot = take ? i : bslot;
+    }
+    const unsigned long long mine = best;
+    best = block_min_u64(best);
+    if (best == ~0ull) return -1;
+    if (mine == best) L.vslot = bslot;
+    cta_sync();
+    return (int32_t)best;
 }
 
 // Alg. 6 l.8-9: planned tasks of k that use V return to the shared pool (R4,
@@ -1318,6 +1271,35 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t, int64_t te)
     cta_sync();
 }
 
+// Warp 0, W >= 1: the inputs of the other tasks of taskBuffer_k -- those
+// served on k that have not ended by t (R7, R29) -- into L.row2: first the
+// task running at t (at most one), then those not started yet, oldest first.
+__device__ __noinline__ void buffer_rows(int k, int64_t t) {
+    const Inst &I = SI;
+    const int W = I.W, j = L.won[k];
+    __syncwarp();  // thread 0 reset row2_len
+    for (int pass = 0; pass < 2; pass++) {  // 0: the running task, 1: the queued ones
+        for (int q = j > W ? j - W : 0; q < j; q++) {
+            const int32_t Tq = __ldcg(&I.wring[k * MAX_W + q % W]);
+            const int64_t st = __ldcg(&I.tstart[Tq]), en = __ldcg(&I.tend[Tq]);
+            if (en <= t || (st <= t) != (pass == 0)) continue;
+            const int64_t rb = __ldg(&I.tptr[Tq]), re = __ldg(&I.tptr[Tq + 1]);
+            const int base = L.row2_len;
+            __syncwarp();
+            for (int r = threadIdx.x; r < (int)(re - rb); r += 32) L.row2[base + r] = __ldg(&I.tdat[rb + r]);
+            __syncwarp();
+            if (threadIdx.x == 0) {
+                L.row2_len = base + (int)(re - rb);
+                if (pass == 0) {
+                    L.row2_run = L.row2_len;
+                    L.run_end = en;
+                }
+            }
+            __syncwarp();
+        }
+    }
+}
+
 // Serve T on GPU k at time t with loads: evict V(k,i), load the missing inputs
 // in ascending id (R10), process; shared FIFO bus (R9).
 // Block-wide.  L.row holds D(T).
@@ -1331,38 +1313,13 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
         L.ready = t;
         L.mem_ready = t;
         L.row2_len = 0;
-        L.row3_len = 0;
+        L.row2_run = 0;
         int nm = 0;
         for (int r = 0; r < L.row_len; r++)
             if (!resident(k, L.row[r])) L.miss[nm++] = L.row[r];
         L.nmiss = nm;
     }
-    // W >= 1: taskBuffer_k also holds the tasks served on k that have not
-    // ended by t (R7, R29): the running one's inputs -> row2, the inputs of
-    // those not started yet -> row3 (warp 0, oldest first)
-    if (I.W >= 1 && threadIdx.x < 32) {
-        const int W = I.W, j = L.won[k];
-        for (int q = j > W ? j - W : 0; q < j; q++) {
-            const int32_t Tq = __ldcg(&I.wring[k * MAX_W + q % W]);
-            const int64_t st = __ldcg(&I.tstart[Tq]), en = __ldcg(&I.tend[Tq]);
-            if (en <= t) continue;
-            const bool run = st <= t;
-            const int64_t rb = __ldg(&I.tptr[Tq]), re = __ldg(&I.tptr[Tq + 1]);
-            const int base = run ? L.row2_len : L.row3_len;
-            int32_t *dst = run ? L.row2 : L.row3;
-            for (int r = threadIdx.x; r < (int)(re - rb); r += 32) dst[base + r] = __ldg(&I.tdat[rb + r]);
-            __syncwarp();
-            if (threadIdx.x == 0) {
-                if (run) {
-                    L.row2_len = base + (int)(re - rb);
-                    L.run_end = en;
-                } else {
-                    L.row3_len = base + (int)(re - rb);
-                }
-            }
-            __syncwarp();
-        }
-    }
+    if (I.W >= 1 && threadIdx.x < 32) buffer_rows(k, t);
     cta_sync();
     const int nmiss = L.nmiss;
     for (int r = 0; r < nmiss; r++) {
@@ -1373,15 +1330,19 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
             cta_sync();
             if (!full) break;
             PROF_T0(p_luf);
-            int belady = 0;
-            const int32_t Vd = luf_victim(k, &belady);
+            int32_t Vd = luf_victim(k);
+            bool belady = false;
+            if (Vd < 0 && I.policy == DTS_POLICY_DARTS_LUF && I.W >= 1) {
+                Vd = belady_victim(k);
+                belady = true;
+                if (threadIdx.x == 0) L.n_belady++;
+            }
             PROF_ADD(L, P_LUF, p_luf);
             if (Vd < 0) {
                 if (threadIdx.x == 0) L.error = 1;
                 cta_sync();
                 return;
             }
-            if (belady && threadIdx.x == 0) L.n_belady++;
             PROF_T0(p_ev);
             evict(k, Vd, T, t, belady ? (L.run_end > t ? L.run_end : t) : t);
             PROF_ADD(L, P_EVICT, p_ev);
@@ -2205,454 +2166,295 @@ __device__ __noinline__ void fused_init() {
 
 }  // namespace
 
-// Cluster mode (Inst::cl > 0): the leader asks the helper CTAs of its
-// cluster for the argmax of their datum slices (Alg. 5 l.6-9 and the 3inputs
-// key in one pass).  One cluster barrier per scan makes the leader's remote
-// updates of h, h2, u visible to the helpers: the leader ARRIVES (release) as
-// soon as its last update before the scan is issued -- at the end of a serve,
-// DARTS+LUF pops update no score -- and WAITS (acquire) when the scan starts,
-// so the barrier and the draining of its remote atomics overlap the pop
-// phase.  The request (k, mode, sequence number) then goes to each helper's
-// shared memory and the keys come back into the leader's (release stores,
-// acquire polls).  Leader and helpers pass the same number of barriers.
-// Leader, block-wide: publish request cmd for GPU k and pass the scan
-// barrier (the helpers then see it and every earlier update); for a scan,
-// collect the helpers' keys (release stores into CK / CKS, acquire polls).
-// Returns the main key, *kb the 3inputs key.
-__device__ __noinline__ unsigned long long cl_request(int32_t cmd, int k, unsigned long long *kb) {
-    const Inst &I = SI;
-    const uint32_t seq = L.cl_seq + 1;
-    if (threadIdx.x == 0) {
-        CR.cmd = cmd;
-        CR.k = k;
-        CR.seq = seq;
-    }
-    cluster_barrier();
-    unsigned long long a = 0ull, b = 0ull;
-    if (cmd != CL_EXIT && threadIdx.x < 32) {
-        const int lane = threadIdx.x;
-        if (lane < I.cl) {
-            while (ld_acquire_cluster(&CKS[lane]) != seq) {
-            }
-            a = CK[lane][0];
-            b = CK[lane][1];
-        }
-        a = warp_max_u64(a);
-        b = warp_max_u64(b);
-        if (lane == 0) {
-            L.red64b[0] = a;
-            L.red64b[1] = b;
-        }
-    }
-    if (threadIdx.x == 0) L.cl_seq = seq;
-    cta_sync();
-    *kb = L.red64b[1];
-    return L.red64b[0];
-}
-
-// Leader, block-wide: Dopt (returned) and the 3inputs datum *D2 for GPU k.
-__device__ __noinline__ int32_t cl_scan(int k, bool opti, int32_t *D2) {
-    const unsigned long long idmask = (1ull << SI.id_bits) - 1ull;
-    unsigned long long b;
-    const unsigned long long a = cl_request(CL_SCAN | (opti ? CL_OPTI : 0), k, &b);
-    *D2 = b ? (int32_t)(idmask - (b & idmask)) : -1;
-    return a ? (int32_t)(idmask - (a & idmask)) : -1;
-}
-
-// Leader, block-wide, once per instance after the loop: release the helpers.
-__device__ __noinline__ void cl_exit() {
-    unsigned long long b;
-    cl_request(CL_EXIT, 0, &b);
-    cluster_barrier();  // the helpers have read it: nothing reads this CTA's memory any more
-}
-
-// Helper rank r >= 1 of a cluster-mode instance: owns slice q = r - 1 of the
-// data ([q 2^csh, (q+1) 2^csh) ∩ [0, n)) of h, h2 (all K GPUs) and u in its
-// shared memory; the leader updates them with remote atomics; on each request
-// the helper returns its slice's best keys: (n_k(D), u(D), -D) and
-// (n2_k(D), u(D), -D) (Alg. 5 l.6-9, 3inputs, R1/R23/R24), or for OPTI the
-// lowest D with n_k(D) > 0 (R28).
-__device__ __noinline__ void cl_helper(const Inst *__restrict__ insts, int ii, int rank, unsigned char *dsm) {
-    namespace cg = cooperative_groups;
-    if (threadIdx.x == 0) {
-        SI = insts[ii];
-        CR.seq = 0;
-    }
-    cta_sync();
-    const Inst &I = SI;
-    const int K = I.K, S = 1 << I.csh, q = rank - 1;
-    const int lo = q * S, hi = q < I.cl ? min(I.n, lo + S) : lo;
-    int32_t *hs = reinterpret_cast<int32_t *>(dsm);  // h[K][S], h2[K][S], u[S]
-    for (int i = threadIdx.x; i < (2 * K + 1) * S; i += blockDim.x) {
-        const int a = i / S, d = i - a * S, D = lo + d;
-        int32_t v = 0;
-        if (D < hi) v = a < K ? __ldcg(&I.h[(size_t)a * I.nstr + D])
-                              : (a < 2 * K ? __ldcg(&I.h2[(size_t)(a - K) * I.nstr + D]) : __ldcg(&I.u[D]));
-        hs[i] = v;
-    }
-    cta_sync();
-    cluster_barrier();  // init: slices ready before the leader's first update
-    unsigned long long *ck = cg::this_cluster().map_shared_rank(&CK[0][0], 0);
-    const ClReq *lcr = cg::this_cluster().map_shared_rank(&CR, 0);
-    uint32_t *cks = cg::this_cluster().map_shared_rank(&CKS[0], 0);
-    const unsigned ib = (unsigned)I.id_bits;
-    const unsigned long long idmask = (1ull << ib) - 1ull;
-    __shared__ ClReq req;
-    for (uint32_t seq = 1;; seq++) {
-        cluster_barrier();  // the leader's request and every update before it are visible
-        if (threadIdx.x == 0) req = *lcr;
-        cta_sync();
-        const ClReq r = req;
-        if (r.cmd & CL_EXIT) break;
-        const int32_t *hk = hs + (size_t)r.k * S, *h2k = hs + (size_t)(K + r.k) * S, *us = hs + (size_t)2 * K * S;
-        unsigned long long a = 0ull, b = 0ull;
-        for (int d = threadIdx.x; d < hi - lo; d += blockDim.x) {  // increasing D per thread
-            const int32_t h = hk[d], h2 = h2k[d];
-            const uint32_t u = (uint32_t)us[d];
-            const unsigned long long low = idmask - (unsigned long long)(lo + d);
-            unsigned long long ka;
-            if (r.cmd & CL_OPTI) ka = h > 0 ? ((1ull << 40) | low) : 0ull;
-            else ka = h > 0 ? ((((unsigned long long)(uint32_t)h << 16) | u) << ib) | low : 0ull;
-            const unsigned long long kb = h2 > 0 ? ((((unsigned long long)(uint32_t)h2 << 16) | u) << ib) | low : 0ull;
-            a = ka > a ? ka : a;
-            b = kb > b ? kb : b;
-        }
-        a = block_max_u64(a);
-        b = block_max_u64(b);
-        if (threadIdx.x == 0 && q < MAX_HELPERS) {
-            ck[2 * q] = a;
-            ck[2 * q + 1] = b;
-            st_release_cluster(&cks[q], seq);
-        }
-    }
-    cluster_barrier();  // exit
-}
-
-// The whole schedule of instance insts[ii] on this CTA (block-wide): a1/a2
-// initial state, the decision loop (a2-a7), result assembly (a8).
-__device__ __noinline__ void run_instance(const Inst *__restrict__ insts, int ii, unsigned char *dsm) {
-    const int tid = threadIdx.x;
-    if (tid == 0) SI = insts[ii];
-    cta_sync();
-    const Inst &I = SI;
-    if (I.poison) {  // debug: nothing may depend on the previous instance's shared memory
-        for (int i = tid; i < I.smem_bytes / 4; i += blockDim.x) reinterpret_cast<uint32_t *>(dsm)[i] = 0xA5A5A5A5u;
-        if (tid == 0) {
-            uint32_t *l = reinterpret_cast<uint32_t *>(&L);
-            for (size_t i = 0; i < sizeof(Lead) / 4; i++) l[i] = 0x5A5A5A5Au;
-        }
-        cta_sync();
-    }
-    if (tid == 0) {
-        View &W = SV;
-        W.s = I.so_s >= 0 ? (uint32_t *)(dsm + I.so_s) : I.s;
-        W.u = I.so_u >= 0 ? (int32_t *)(dsm + I.so_u) : I.u;
-        W.h = I.so_h >= 0 ? (int32_t *)(dsm + I.so_h) : I.h;
-        W.h2 = I.so_h2 >= 0 ? (int32_t *)(dsm + I.so_h2) : I.h2;
-        W.np = I.so_np >= 0 ? (int32_t *)(dsm + I.so_np) : I.np;
-        W.resb = I.so_resb >= 0 ? (uint32_t *)(dsm + I.so_resb) : I.resb;
-        W.res_list = I.so_res_list >= 0 ? (int32_t *)(dsm + I.so_res_list) : I.res_list;
-        W.plan = I.so_plan >= 0 ? (int4 *)(dsm + I.so_plan) : I.plan;
-        W.plan_cum = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
-        W.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
-        W.lru = I.so_lru >= 0 ? (int32_t *)(dsm + I.so_lru) : I.lru;
-        W.al = I.so_al >= 0 ? (uint32_t *)(dsm + I.so_al) : I.al;
-        W.cl = I.cl;
-        if (I.cl) {  // h, h2, u in the helpers' shared memory (cl_helper)
-            W.csh = I.csh;
-            W.cS = 1 << I.csh;
-            for (int q = 0; q < I.cl; q++)
-                W.cb[q] = cooperative_groups::this_cluster().map_shared_rank(reinterpret_cast<int32_t *>(dsm), q + 1);
-        }
-    }
-    cta_sync();
-    const View &V = SV;
-    if (I.G > 1)
-        for (int p = tid; p < I.G; p += blockDim.x) SP[p] = I.peers[p];
-
-    const int n = I.n, K = I.K;
-    if (I.fused) {  // a1 + a2 inside this CTA (small instances)
-        fused_build(dsm);
-        fused_init();
-    } else {
-    // ---- CTA-local copies of the initial state (global homes were
-    //      initialised by dts_init_kernel)
-    if (I.so_dptr >= 0)
-        for (int D = tid; D <= n; D += blockDim.x) V.dptr32[D] = (int32_t)__ldg(&I.dptr[D]);
-    if (I.so_s >= 0) {
-        const uint4 *src = reinterpret_cast<const uint4 *>(I.s);
-        uint4 *dst = reinterpret_cast<uint4 *>(V.s);
-        for (int i = tid; i < (K * I.m_pad) / 4; i += blockDim.x) dst[i] = __ldcg(&src[i]);
-    }
-    if (I.sl && I.so_al >= 0)
-        for (int i = tid; i <= I.m_pad / 32; i += blockDim.x) V.al[i] = __ldcg(&I.al[i]);
-    if (I.so_u >= 0)
-        for (int D = tid; D < I.nstr; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
-    if (I.so_h >= 0)
-        for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h[i] = __ldcg(&I.h[i]);
-    if (I.so_h2 >= 0)
-        for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h2[i] = __ldcg(&I.h2[i]);
-    if (I.so_np >= 0)
-        for (int i = tid; i < K * I.nstr; i += blockDim.x) V.np[i] = 0;
-    if (I.so_resb >= 0)
-        for (int i = tid; i < K * I.nw; i += blockDim.x) V.resb[i] = 0u;
-    }
-    if (I.cl) {
-        if (tid == 0) {
-            L.cl_seq = 0;
-            for (int q = 0; q < MAX_HELPERS; q++) CKS[q] = 0;
-        }
-        cta_sync();
-        cluster_barrier();  // init: the helpers' slices are loaded (cl_helper)
-    }
-    if (tid == 0) {
-        for (int k = 0; k < MAX_K; k++) {
-            L.req[k] = 0;
-            L.gpu_free[k] = 0;
-            L.used[k] = 0;
-            L.plan_head[k] = L.plan_end[k] = L.plan_live[k] = 0;
-            L.res_cnt[k] = 0;
-            L.idle[k] = 0;
-            L.won[k] = 0;
-        }
-        L.bus_free = 0;
-        L.n_events = L.n_served = L.n_loads = L.n_evictions = L.n_scans = L.n_fb2 = L.n_fbf =
-            L.n_belady = L.n_idle = L.n_verr = 0;
-        L.bytes_loaded = L.alg_bytes = L.scan_alg_bytes = 0;
-        L.sum_avail = L.n_alloc = L.sum_deg = 0;
-        L.makespan = 0;
-        L.n_avail = I.m;
-        L.avail_lo = 0;
-        L.error = 0;
-        L.row_len = 0;
-        L.xe = 0;
-        L.xerr = 0;
-        for (int i = 0; i < 16; i++) L.prof[i] = 0;
-    }
-    cta_sync();
-
-    // ---- the decision loop
-    while (true) {
-        PROF_T0(p_pop);
-        if (I.policy == DTS_POLICY_DARTS_LUF) {
-            int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
-            for (int j = 0; j < K; j++) pending += L.plan_live[j];
-            if (I.max_served < 0 && I.W == 0 && K <= 32 && pending > I.pop_batch_min) {
-                pop_batch();
-            } else {  // few pops (or a prefix run that stops at an exact count): thread 0
-                cta_sync();
-                if (tid == 0)
-                    L.cmd = ((I.max_served < 0 || L.n_served < I.max_served) && pop_run_seq() >= 0)
-                                ? CMD_SCAN
-                                : CMD_DONE;
-            }
-        } else {
-            // LRU policies: an LRU eviction does not drop planned tasks, so a
-            // pop may need loads -- every request is served block-wide
-            cta_sync();
-            if (tid == 0) {
-                int cmd = CMD_DONE;
-                if (I.max_served < 0 || L.n_served < I.max_served) {
-                    int kk = -1;  // next request: smallest (req_k, k), non-idle (R8)
-                    int64_t tb = 0;
-                    for (int j = 0; j < K; j++)
-                        if (!L.idle[j] && (kk < 0 || L.req[j] < tb)) {
-                            kk = j;
-                            tb = L.req[j];
-                        }
-                    if (kk >= 0) {
-                        L.k = kk;
-                        L.t = tb;
-                        if (I.policy == DTS_POLICY_DARTS_LRU && L.plan_live[kk] > 0) {
-                            int64_t tau;
-                            L.T = pop_planned(kk, &tau);
-                            cmd = CMD_POP;
-                        } else {
-                            cmd = I.policy == DTS_POLICY_EAGER_LRU ? CMD_EAGER : CMD_SCAN;
-                        }
-                    }
-                }
-                L.cmd = cmd;
-            }
-        }
-        PROF_ADD(L, P_POP, p_pop);
-        cta_sync();
-        if (L.cmd == CMD_DONE || L.xerr) break;
-        const int k = L.k;
-        const int64_t t = L.t;
-        int32_t T = -1;
-        if (L.cmd == CMD_POP) {
-            T = L.T;
-            if (T < 0) break;  // pop_planned found no entry (L.error set)
-        } else if (L.cmd == CMD_EAGER) {
-            // EAGER: the shared FIFO queue in submission
-            // order -- the lowest-id unallocated task
-            T = L.n_avail > 0 ? any_first_avail() : -1;
-            if (tid == 0) {
-                if (T >= 0) {
-                    L.avail_lo = T;
-                    L.fent = entry_of_task(T);
-                    row_from_entry(L.fent);
-                    L.n_avail--;
-                    L.n_alloc++;
-                } else {
-                    L.idle[k] = 1;
-                    L.n_idle++;
-                }
-            }
-            cta_sync();
-            if (T < 0) continue;
-            pool_move_many(&L.fent, 1, -1, -1);
-            cta_sync();
-        } else {
-        reset_plan(k);
-        if (I.flags & DTS_F_VERIFY) verify_scores(k);
-        // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
-        PROF_T0(p_am);
-        int32_t D2s = -1;  // task shards: the 3inputs argmax comes with the main one
-        const int32_t Dopt = I.G > 1 ? shard_scan(k, (I.flags & DTS_F_FALLBACK2) != 0,
-                                                  (I.flags & DTS_F_OPTI) != 0, &D2s)
-                             : I.cl ? cl_scan(k, (I.flags & DTS_F_OPTI) != 0, &D2s)
-                             : (I.flags & DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
-                                                      : score_argmax(V.h + (size_t)k * I.nstr);
-        PROF_ADD(L, P_ARGMAX, p_am);
-        PROF_T0(p_pl);
-        if (tid == 0) {
-            L.scan_alg_bytes += 8ull * (uint64_t)n;
-            L.alg_bytes += 8ull * (uint64_t)n;
-            L.scan_avail = L.n_avail;  // before this scan allocates anything
-        }
-        if (I.G > 1 && L.xerr) break;  // a peer timed out in the scan exchange (CTA-uniform)
-        if (Dopt >= 0) {
-            if (I.G > 1) plan_shard(k, Dopt);
-            else plan(k, Dopt);
-            if (I.G > 1 && L.xerr) break;  // plan exchange failed: no plan to pop from
-            if (tid == 0) {
-                int64_t tau;
-                L.T = pop_planned(k, &tau);
-                L.n_scans++;
-                L.sum_avail += L.scan_avail;
-            }
-            cta_sync();
-            T = L.T;
-            if (T < 0) break;  // pop_planned found no entry (L.error set)
-            PROF_ADD(L, P_PLAN, p_pl);
-        } else {
-            if (I.flags & DTS_F_FALLBACK2) {
-                const int32_t D2 = (I.G > 1 || I.cl) ? D2s : score_argmax(V.h2 + (size_t)k * I.nstr);
-                if (tid == 0) {
-                    L.scan_alg_bytes += 8ull * (uint64_t)n;
-                    L.alg_bytes += 8ull * (uint64_t)n;
-                }
-                if (D2 >= 0) {
-                    T = any_first_cnt2(k, D2);
-                    if (tid == 0) L.n_fb2++;
-                }
-            }
-            if (T < 0 && L.n_avail > 0) {
-                T = any_first_avail();
-                if (tid == 0) {
-                    L.n_fbf++;
-                    L.avail_lo = T;
-                }
-            }
-            if (T >= 0) {
-                if (tid == 0) {
-                    L.fent = entry_of_task(T);
-                    row_from_entry(L.fent);
-                    L.n_avail--;
-                    L.n_alloc++;
-                    L.n_scans++;
-                    L.sum_avail += L.scan_avail;
-                }
-                cta_sync();
-                pool_move_many(&L.fent, 1, -1, -1);
-            } else if (tid == 0) {
-                L.idle[k] = 1;
-                L.n_idle++;
-            }
-            cta_sync();
-            PROF_ADD(L, P_OTHER, p_pl);
-            if (I.G > 1 && L.xerr) break;  // a min-exchange failed: T is not trustworthy
-            if (T < 0) continue;
-        }
-        }  // scan
-        // serve T with its loads (block-wide); D(T) from the CSR unless cached
-        const bool need_row = L.row_len < 0;
-        cta_sync();
-        if (need_row && tid < 32) {
-            const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
-            for (int r = tid; r < (int)(re - rb); r += 32) L.row[r] = __ldg(&I.tdat[rb + r]);
-            if (tid == 0) L.row_len = (int)(re - rb);
-        }
-        cta_sync();
-        PROF_T0(p_ld);
-        serve_loads(k, T, t);
-        PROF_ADD(L, P_LOADS, p_ld);
-        if (L.error || L.xerr) break;
-    }
-    cta_sync();
-    if (I.G > 1) {  // no shard leaves while a peer may still read its slots
-        xch_sync();
-        if (tid == 0 && L.xerr && !L.error) L.error = 2;
-        cta_sync();
-    }
-
-    // ---- a8: per-GPU orders, scalars
-    cta_sync();  // the loop's shared-memory arrays are dead from here on
-    assemble(L.n_served, dsm);
-    if (tid == 0) {
-        Out *o = I.out;
-        o->n_events = L.n_events;
-        o->n_served = L.n_served;
-        o->n_loads = L.n_loads;
-        o->n_evictions = L.n_evictions;
-        o->n_scans = L.n_scans;
-        o->n_fallback2 = L.n_fb2;
-        o->n_fallback_first = L.n_fbf;
-        o->n_belady = L.n_belady;
-        o->n_idle = L.n_idle;
-        o->n_verify_err = L.n_verr;
-        o->bytes_loaded = L.bytes_loaded;
-        o->makespan = L.makespan;
-        o->alg_bytes = L.alg_bytes;
-        o->scan_alg_bytes = L.scan_alg_bytes;
-        o->sum_avail = L.sum_avail;
-        o->n_alloc = L.n_alloc;
-        o->sum_deg = L.sum_deg;
-        o->error = L.error;
-        for (int i = 0; i < 16; i++) o->prof[i] = L.prof[i];
-    }
-    cta_sync();
-    if (I.cl) cl_exit();
-}
-
 // One CTA per instance; instances pulled from *work_counter.
 __global__ void __launch_bounds__(512, 1)
     dts_cta_kernel(const Inst *__restrict__ insts, int n_inst, int *work_counter) {
     extern __shared__ __align__(16) unsigned char dsm[];
     __shared__ int sh_inst;
+    const int tid = threadIdx.x;
+
     while (true) {
-        if (threadIdx.x == 0) sh_inst = atomicAdd(work_counter, 1);
+        if (tid == 0) sh_inst = atomicAdd(work_counter, 1);
         cta_sync();
         const int ii = sh_inst;
         if (ii >= n_inst) break;
-        run_instance(insts, ii, dsm);
-    }
-}
+        if (tid == 0) SI = insts[ii];
+        cta_sync();
+        const Inst &I = SI;
+        if (I.poison) {  // debug: nothing may depend on the previous instance's shared memory
+            for (int i = tid; i < I.smem_bytes / 4; i += blockDim.x) reinterpret_cast<uint32_t *>(dsm)[i] = 0xA5A5A5A5u;
+            if (tid == 0) {
+                uint32_t *l = reinterpret_cast<uint32_t *>(&L);
+                for (size_t i = 0; i < sizeof(Lead) / 4; i++) l[i] = 0x5A5A5A5Au;
+            }
+            cta_sync();
+        }
+        if (tid == 0) {
+            View &W = SV;
+            W.s = I.so_s >= 0 ? (uint32_t *)(dsm + I.so_s) : I.s;
+            W.u = I.so_u >= 0 ? (int32_t *)(dsm + I.so_u) : I.u;
+            W.h = I.so_h >= 0 ? (int32_t *)(dsm + I.so_h) : I.h;
+            W.h2 = I.so_h2 >= 0 ? (int32_t *)(dsm + I.so_h2) : I.h2;
+            W.np = I.so_np >= 0 ? (int32_t *)(dsm + I.so_np) : I.np;
+            W.resb = I.so_resb >= 0 ? (uint32_t *)(dsm + I.so_resb) : I.resb;
+            W.res_list = I.so_res_list >= 0 ? (int32_t *)(dsm + I.so_res_list) : I.res_list;
+            W.plan = I.so_plan >= 0 ? (int4 *)(dsm + I.so_plan) : I.plan;
+            W.plan_cum = !I.tau ? nullptr : (I.so_plan_tau >= 0 ? (int64_t *)(dsm + I.so_plan_tau) : I.plan_tau);
+            W.dptr32 = I.so_dptr >= 0 ? (int32_t *)(dsm + I.so_dptr) : nullptr;
+            W.lru = I.so_lru >= 0 ? (int32_t *)(dsm + I.so_lru) : I.lru;
+            W.al = I.so_al >= 0 ? (uint32_t *)(dsm + I.so_al) : I.al;
+        }
+        cta_sync();
+        const View &V = SV;
+        if (I.G > 1)
+            for (int p = tid; p < I.G; p += blockDim.x) SP[p] = I.peers[p];
 
-// Cluster mode: cluster c runs instance c; rank 0 is the leader (the whole
-// decision loop), ranks >= 1 hold the score arrays by datum slice and answer
-// the leader's argmax requests (DSMEM, cluster barriers).
-__global__ void __launch_bounds__(512, 1) dts_cluster_kernel(const Inst *__restrict__ insts, int n_inst) {
-    namespace cg = cooperative_groups;
-    extern __shared__ __align__(16) unsigned char dsm[];
-    cg::cluster_group cl = cg::this_cluster();
-    const int rank = (int)cl.block_rank();
-    const int ii = (int)(blockIdx.x / cl.num_blocks());
-    if (ii >= n_inst) return;  // whole clusters only (grid = n_inst clusters)
-    if (rank == 0) run_instance(insts, ii, dsm);
-    else cl_helper(insts, ii, rank, dsm);
+        const int n = I.n, K = I.K;
+        if (I.fused) {  // a1 + a2 inside this CTA (small instances)
+            fused_build(dsm);
+            fused_init();
+        } else {
+        // ---- CTA-local copies of the initial state (global homes were
+        //      initialised by dts_init_kernel)
+        if (I.so_dptr >= 0)
+            for (int D = tid; D <= n; D += blockDim.x) V.dptr32[D] = (int32_t)__ldg(&I.dptr[D]);
+        if (I.so_s >= 0) {
+            const uint4 *src = reinterpret_cast<const uint4 *>(I.s);
+            uint4 *dst = reinterpret_cast<uint4 *>(V.s);
+            for (int i = tid; i < (K * I.m_pad) / 4; i += blockDim.x) dst[i] = __ldcg(&src[i]);
+        }
+        if (I.sl && I.so_al >= 0)
+            for (int i = tid; i <= I.m_pad / 32; i += blockDim.x) V.al[i] = __ldcg(&I.al[i]);
+        if (I.so_u >= 0)
+            for (int D = tid; D < I.nstr; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
+        if (I.so_h >= 0)
+            for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h[i] = __ldcg(&I.h[i]);
+        if (I.so_h2 >= 0)
+            for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h2[i] = __ldcg(&I.h2[i]);
+        if (I.so_np >= 0)
+            for (int i = tid; i < K * I.nstr; i += blockDim.x) V.np[i] = 0;
+        if (I.so_resb >= 0)
+            for (int i = tid; i < K * I.nw; i += blockDim.x) V.resb[i] = 0u;
+        }
+        if (tid == 0) {
+            for (int k = 0; k < MAX_K; k++) {
+                L.req[k] = 0;
+                L.gpu_free[k] = 0;
+                L.used[k] = 0;
+                L.plan_head[k] = L.plan_end[k] = L.plan_live[k] = 0;
+                L.res_cnt[k] = 0;
+                L.idle[k] = 0;
+                L.won[k] = 0;
+            }
+            L.bus_free = 0;
+            L.n_events = L.n_served = L.n_loads = L.n_evictions = L.n_scans = L.n_fb2 = L.n_fbf =
+                L.n_belady = L.n_idle = L.n_verr = 0;
+            L.bytes_loaded = L.alg_bytes = L.scan_alg_bytes = 0;
+            L.sum_avail = L.n_alloc = L.sum_deg = 0;
+            L.makespan = 0;
+            L.n_avail = I.m;
+            L.avail_lo = 0;
+            L.error = 0;
+            L.row_len = 0;
+            L.xe = 0;
+            L.xerr = 0;
+            for (int i = 0; i < 16; i++) L.prof[i] = 0;
+        }
+        cta_sync();
+
+        // ---- the decision loop
+        while (true) {
+            PROF_T0(p_pop);
+            if (I.policy == DTS_POLICY_DARTS_LUF) {
+                int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
+                for (int j = 0; j < K; j++) pending += L.plan_live[j];
+                if (I.max_served < 0 && I.W == 0 && K <= 32 && pending > I.pop_batch_min) {
+                    pop_batch();
+                } else {  // few pops (or a prefix run that stops at an exact count): thread 0
+                    cta_sync();
+                    if (tid == 0)
+                        L.cmd = ((I.max_served < 0 || L.n_served < I.max_served) && pop_run_seq() >= 0)
+                                    ? CMD_SCAN
+                                    : CMD_DONE;
+                }
+            } else {
+                // LRU policies: an LRU eviction does not drop planned tasks, so a
+                // pop may need loads -- every request is served block-wide
+                cta_sync();
+                if (tid == 0) {
+                    int cmd = CMD_DONE;
+                    if (I.max_served < 0 || L.n_served < I.max_served) {
+                        int kk = -1;  // next request: smallest (req_k, k), non-idle (R8)
+                        int64_t tb = 0;
+                        for (int j = 0; j < K; j++)
+                            if (!L.idle[j] && (kk < 0 || L.req[j] < tb)) {
+                                kk = j;
+                                tb = L.req[j];
+                            }
+                        if (kk >= 0) {
+                            L.k = kk;
+                            L.t = tb;
+                            if (I.policy == DTS_POLICY_DARTS_LRU && L.plan_live[kk] > 0) {
+                                int64_t tau;
+                                L.T = pop_planned(kk, &tau);
+                                cmd = CMD_POP;
+                            } else {
+                                cmd = I.policy == DTS_POLICY_EAGER_LRU ? CMD_EAGER : CMD_SCAN;
+                            }
+                        }
+                    }
+                    L.cmd = cmd;
+                }
+            }
+            PROF_ADD(L, P_POP, p_pop);
+            cta_sync();
+            if (L.cmd == CMD_DONE || L.xerr) break;
+            const int k = L.k;
+            const int64_t t = L.t;
+            int32_t T = -1;
+            if (L.cmd == CMD_POP) {
+                T = L.T;
+                if (T < 0) break;  // pop_planned found no entry (L.error set)
+            } else if (L.cmd == CMD_EAGER) {
+                // EAGER: the shared FIFO queue in submission
+                // order -- the lowest-id unallocated task
+                T = L.n_avail > 0 ? any_first_avail() : -1;
+                if (tid == 0) {
+                    if (T >= 0) {
+                        L.avail_lo = T;
+                        L.fent = entry_of_task(T);
+                        row_from_entry(L.fent);
+                        L.n_avail--;
+                        L.n_alloc++;
+                    } else {
+                        L.idle[k] = 1;
+                        L.n_idle++;
+                    }
+                }
+                cta_sync();
+                if (T < 0) continue;
+                pool_move_many(&L.fent, 1, -1, -1);
+                cta_sync();
+            } else {
+            reset_plan(k);
+            if (I.flags & DTS_F_VERIFY) verify_scores(k);
+            // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
+            PROF_T0(p_am);
+            int32_t D2s = -1;  // task shards: the 3inputs argmax comes with the main one
+            const int32_t Dopt = I.G > 1 ? shard_scan(k, (I.flags & DTS_F_FALLBACK2) != 0,
+                                                      (I.flags & DTS_F_OPTI) != 0, &D2s)
+                                 : (I.flags & DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
+                                                          : score_argmax(V.h + (size_t)k * I.nstr);
+            PROF_ADD(L, P_ARGMAX, p_am);
+            PROF_T0(p_pl);
+            if (tid == 0) {
+                L.scan_alg_bytes += 8ull * (uint64_t)n;
+                L.alg_bytes += 8ull * (uint64_t)n;
+                L.scan_avail = L.n_avail;  // before this scan allocates anything
+            }
+            if (I.G > 1 && L.xerr) break;  // a peer timed out in the scan exchange (CTA-uniform)
+            if (Dopt >= 0) {
+                if (I.G > 1) plan_shard(k, Dopt);
+                else plan(k, Dopt);
+                if (I.G > 1 && L.xerr) break;  // plan exchange failed: no plan to pop from
+                if (tid == 0) {
+                    int64_t tau;
+                    L.T = pop_planned(k, &tau);
+                    L.n_scans++;
+                    L.sum_avail += L.scan_avail;
+                }
+                cta_sync();
+                T = L.T;
+                if (T < 0) break;  // pop_planned found no entry (L.error set)
+                PROF_ADD(L, P_PLAN, p_pl);
+            } else {
+                if (I.flags & DTS_F_FALLBACK2) {
+                    const int32_t D2 = I.G > 1 ? D2s : score_argmax(V.h2 + (size_t)k * I.nstr);
+                    if (tid == 0) {
+                        L.scan_alg_bytes += 8ull * (uint64_t)n;
+                        L.alg_bytes += 8ull * (uint64_t)n;
+                    }
+                    if (D2 >= 0) {
+                        T = any_first_cnt2(k, D2);
+                        if (tid == 0) L.n_fb2++;
+                    }
+                }
+                if (T < 0 && L.n_avail > 0) {
+                    T = any_first_avail();
+                    if (tid == 0) {
+                        L.n_fbf++;
+                        L.avail_lo = T;
+                    }
+                }
+                if (T >= 0) {
+                    if (tid == 0) {
+                        L.fent = entry_of_task(T);
+                        row_from_entry(L.fent);
+                        L.n_avail--;
+                        L.n_alloc++;
+                        L.n_scans++;
+                        L.sum_avail += L.scan_avail;
+                    }
+                    cta_sync();
+                    pool_move_many(&L.fent, 1, -1, -1);
+                } else if (tid == 0) {
+                    L.idle[k] = 1;
+                    L.n_idle++;
+                }
+                cta_sync();
+                PROF_ADD(L, P_OTHER, p_pl);
+                if (I.G > 1 && L.xerr) break;  // a min-exchange failed: T is not trustworthy
+                if (T < 0) continue;
+            }
+            }  // scan
+            // serve T with its loads (block-wide); D(T) from the CSR unless cached
+            const bool need_row = L.row_len < 0;
+            cta_sync();
+            if (need_row && tid < 32) {
+                const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
+                for (int r = tid; r < (int)(re - rb); r += 32) L.row[r] = __ldg(&I.tdat[rb + r]);
+                if (tid == 0) L.row_len = (int)(re - rb);
+            }
+            cta_sync();
+            PROF_T0(p_ld);
+            serve_loads(k, T, t);
+            PROF_ADD(L, P_LOADS, p_ld);
+            if (L.error || L.xerr) break;
+        }
+        cta_sync();
+        if (I.G > 1) {  // no shard leaves while a peer may still read its slots
+            xch_sync();
+            if (tid == 0 && L.xerr && !L.error) L.error = 2;
+            cta_sync();
+        }
+
+        // ---- a8: per-GPU orders, scalars
+        cta_sync();  // the loop's shared-memory arrays are dead from here on
+        assemble(L.n_served, dsm);
+        if (tid == 0) {
+            Out *o = I.out;
+            o->n_events = L.n_events;
+            o->n_served = L.n_served;
+            o->n_loads = L.n_loads;
+            o->n_evictions = L.n_evictions;
+            o->n_scans = L.n_scans;
+            o->n_fallback2 = L.n_fb2;
+            o->n_fallback_first = L.n_fbf;
+            o->n_belady = L.n_belady;
+            o->n_idle = L.n_idle;
+            o->n_verify_err = L.n_verr;
+            o->bytes_loaded = L.bytes_loaded;
+            o->makespan = L.makespan;
+            o->alg_bytes = L.alg_bytes;
+            o->scan_alg_bytes = L.scan_alg_bytes;
+            o->sum_avail = L.sum_avail;
+            o->n_alloc = L.n_alloc;
+            o->sum_deg = L.sum_deg;
+            o->error = L.error;
+            for (int i = 0; i < 16; i++) o->prof[i] = L.prof[i];
+        }
+        cta_sync();
+    }
 }
 
 // ---------------------------------------------------------------- init (a2)
@@ -2761,44 +2563,6 @@ cudaError_t launch_loop_coop(const Inst *d_insts, int n_inst, int block, int *wo
                                     (size_t)smem_bytes, st);
     count_launch();
     return e;
-}
-
-// Cluster mode: n_inst clusters of csize CTAs (leader + helpers), one per
-// instance; csize > 8 needs the non-portable cluster size attribute.
-cudaError_t launch_cluster(const Inst *d_insts, int n_inst, int csize, int block, int smem_bytes, cudaStream_t st) {
-    static int cur[64];
-    static bool init = false;
-    if (!init) {
-        for (int &c : cur) c = -1;
-        init = true;
-    }
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (dev < 0 || dev >= 64) dev = 0;
-    cudaError_t e;
-    if (smem_bytes > cur[dev]) {
-        e = cudaFuncSetAttribute(dts_cluster_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-        if (e != cudaSuccess) return e;
-        e = cudaFuncSetAttribute(dts_cluster_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-        if (e != cudaSuccess) return e;
-        cur[dev] = smem_bytes;
-    }
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)(n_inst * csize));
-    cfg.blockDim = dim3((unsigned)block);
-    cfg.dynamicSmemBytes = (size_t)smem_bytes;
-    cfg.stream = st;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = (unsigned)csize;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    e = cudaLaunchKernelEx(&cfg, dts_cluster_kernel, d_insts, n_inst);
-    count_launch();
-    if (e != cudaSuccess) return e;
-    return cudaGetLastError();
 }
 
 int loop_max_blocks_per_sm(int block, int smem_bytes) {

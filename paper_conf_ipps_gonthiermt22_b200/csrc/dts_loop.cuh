@@ -15,9 +15,6 @@ cudaError_t launch_loop(const Inst *d_insts, int n_inst, int block, int grid, in
 // exchange inside the kernel, so a cooperative launch (all co-resident).
 cudaError_t launch_loop_coop(const Inst *d_insts, int n_inst, int block, int *work_counter, int smem_bytes,
                              cudaStream_t st);
-// Cluster mode (large instances): n_inst clusters of csize CTAs each, one
-// instance per cluster (rank 0 leads, ranks >= 1 hold score slices).
-cudaError_t launch_cluster(const Inst *d_insts, int n_inst, int csize, int block, int smem_bytes, cudaStream_t st);
 int loop_max_blocks_per_sm(int block, int smem_bytes);
 int loop_static_smem();
 }  // namespace dts

@@ -680,10 +680,10 @@ def test_capacity_check_by_policy():
     assert e.value.status == -6
 
 
-# ------------------------------------------------ cluster mode
-def _cluster_shapes():
-    """Instances with n >= 4096 data: they run on a thread-block cluster
-    (leader + helpers holding the score slices) by default."""
+# ------------------------------------------------ large-n shapes (n >= 4096 data)
+def _large_n_shapes():
+    """Random shared-input instances with 4,096-16,384 data and K up to 16:
+    the score arrays live in HBM (L2), not shared memory."""
     return [gen.random_shared(20_000, 8192, 3, M=64, K=4, seed=11),
             gen.random_shared(16_000, 4096, 2, M=40, K=8, seed=12),
             gen.random_shared(12_000, 16384, 3, M=96, K=3, seed=13),
@@ -692,40 +692,25 @@ def _cluster_shapes():
 
 @pytest.mark.parametrize("idx", range(4))
 @pytest.mark.parametrize("flags", [dts.DTS_F_FALLBACK2, 0, dts.DTS_F_FALLBACK2 | dts.DTS_F_OPTI])
-def test_cluster_mode_full_parity(idx, flags):
-    inst = _cluster_shapes()[idx]
+def test_large_n_full_parity(idx, flags):
+    inst = _large_n_shapes()[idx]
     g, o = _both(inst, flags=flags)
     assert_parity(g, o)
 
 
-@pytest.mark.parametrize("cfg", ["C4a", "C4b"])
-def test_cluster_vs_single_cta_config4_prefix(cfg):
-    """The cluster path and the single-CTA path (DTS_F_NOCLUSTER) give the
-    oracle's schedule on a C4 prefix."""
-    inst = gen.config_instances(cfg)[0]
-    o = oracle.run(inst, max_served=3000)
-    for fl in (dts.DTS_F_FALLBACK2, dts.DTS_F_FALLBACK2 | dts.DTS_F_NOCLUSTER):
-        g = dts.schedule(inst, flags=fl, max_served=3000)
-        assert_parity(g, o, complete=False)
-
-
-@pytest.mark.parametrize("name", ["darts_lru"])
-def test_cluster_mode_lru_policy(name):
-    inst = _cluster_shapes()[0]
-    g, o = _both_policy(inst, name)
+def test_large_n_lru_policy():
+    g, o = _both_policy(_large_n_shapes()[0], "darts_lru")
     assert_parity(g, o)
 
 
-def test_cluster_mode_in_mixed_sweep():
-    """A batch mixing cluster-mode instances with small ones: the cluster
-    launch runs beside the one-CTA launches; every instance matches."""
-    insts = _cluster_shapes()[:2] + gen.config_instances("C2")[:6]
+def test_large_n_in_mixed_sweep():
+    insts = _large_n_shapes()[:2] + gen.config_instances("C2")[:6]
     gs = dts.schedule_batch(insts)
     for inst, g in zip(insts, gs):
         assert_parity(g, oracle.run(inst))
 
 
-def test_cluster_mode_w1_and_belady():
-    inst = _tight(_cluster_shapes()[1], 1)
+def test_large_n_w1_and_belady():
+    inst = _tight(_large_n_shapes()[1], 1)
     g, o = dts.schedule(inst, W=1), oracle.run(inst, W=1)
     assert_parity(g, o)
