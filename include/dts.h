@@ -109,7 +109,14 @@ typedef struct {
     int32_t smem_budget;      /* bytes of shared memory per CTA for state placement
                                  (DESIGN.md "Data layout"); 0 = automatic (all that fits);
                                  -1 = none (every array in its global home) */
-    int32_t pad;
+    int32_t n_devices;        /* dts_run only: G physical GPUs for ONE instance (SURVEY.md
+                                 §8(e), second mode).  0 or 1 (default): one CTA on `device`.
+                                 G > 1: the instance is task-sharded over G shards in this
+                                 process, shard j on device (device + j) mod #devices (so a
+                                 single-GPU machine runs all G on one device), exchanging
+                                 through peer memory inside the kernel; the result is the
+                                 same schedule.  The instance then owns G-1 shard copies
+                                 (freed by a later run with n_devices <= 1 or destroy). */
     int64_t max_served;       /* stop after this many served tasks (prefix runs); -1 = all */
     void *cuda_stream;        /* cudaStream_t to enqueue on; NULL = the legacy default stream */
 } dts_run_opts;

@@ -149,8 +149,13 @@ struct dts_instance {
     bool connected = false;
     bool xsys = false;                       // peers mapped through CUDA IPC (other processes / GPUs)
     std::vector<void *> ipc_open;            // peers' arenas mapped through CUDA IPC
+    // dts_run with opts.n_devices = G > 1: this instance is shard 0 of G and
+    // owns the other G-1 shards (same inputs), shard j on device (device+j) mod #devices
+    std::vector<dts_instance *> xs;
+    int32_t xs_dev0 = -1;
 
     ~dts_instance() {
+        for (dts_instance *x : xs) delete x;
         if (device >= 0) {
             int cur = 0;
             cudaGetDevice(&cur);
@@ -206,7 +211,7 @@ const char *dts_status_str(dts_status s) {
 
 const char *dts_last_error(void) { return g_err.c_str(); }
 
-uint32_t dts_version(void) { return (1u << 16) | 1u; }
+uint32_t dts_version(void) { return (1u << 16) | 2u; }
 
 dts_status dts_instance_create(int32_t n_tasks, int32_t n_data, const int64_t *task_ptr,
                                const int32_t *task_data, const uint64_t *data_size,
@@ -865,6 +870,9 @@ dts_status dts_instance_upload(dts_instance *I, int32_t device, void *cuda_strea
     return upload(I, st, true);
 }
 
+static dts_status run_multi_device(dts_instance *I, dts_policy policy, const dts_run_opts &o);
+static dts_status run_one(dts_instance *I, dts_policy policy, const dts_run_opts &o);
+
 dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts) {
     if (!I) return fail(DTS_E_INVAL, "instance is NULL");
     dts_run_opts o;
@@ -874,6 +882,20 @@ dts_status dts_run(dts_instance *I, dts_policy policy, const dts_run_opts *opts)
     if (s != DTS_OK) return s;
     s = check_device(o.device);
     if (s != DTS_OK) return s;
+    if (o.n_devices < 0 || o.n_devices > dts::MAX_G) return fail(DTS_E_INVAL, "n_devices must be in [0, 64]");
+    if (o.n_devices > 1) return run_multi_device(I, policy, o);
+    if (!I->xs.empty()) {  // back to one device: drop the owned shards
+        for (dts_instance *x : I->xs) delete x;
+        I->xs.clear();
+        I->xs_dev0 = -1;
+        dts_shard_set(I, 1, 0);
+    }
+    return run_one(I, policy, o);
+}
+
+// One instance (or one task shard) on o.device, enqueued on o.cuda_stream.
+static dts_status run_one(dts_instance *I, dts_policy policy, const dts_run_opts &o) {
+    dts_status s;
     if (I->G > 1 && !I->connected)
         return fail(DTS_E_STATE, "task shard not connected (dts_shard_connect) -- or use dts_shard_group_run");
     if (I->G > 1 && I->device != o.device) return fail(DTS_E_INVAL, "task shard: opts.device != exported device");
@@ -1184,6 +1206,104 @@ dts_status dts_shard_group_run(dts_instance *const *shards, int32_t G, dts_polic
     return DTS_OK;
 }
 
+
+// dts_run with opts.n_devices = G > 1: the instance is
+// task-sharded over G shards in this process -- shard 0 is the instance
+// itself, shards 1..G-1 are copies it owns -- shard j on device
+// (opts.device + j) mod #devices, each ONE CTA that exchanges with its peers
+// through their memory (peer access / UVA; system-scope release/acquire when
+// the shards span devices), launched on its device's library stream forked
+// from and joined back into opts.cuda_stream.  Every shard computes the whole
+// schedule; dts_result(inst) reads shard 0's.
+static dts_status run_multi_device(dts_instance *I, dts_policy policy, const dts_run_opts &o) {
+    const int32_t G = o.n_devices;
+    int ndev = 0;
+    CK(cudaGetDeviceCount(&ndev), "cudaGetDeviceCount");
+    if (I->G > 1 && I->xs.empty()) return fail(DTS_E_INVAL, "an exported task shard cannot run with n_devices");
+    auto dev_of = [&](int32_t j) { return (o.device + j) % ndev; };
+    dts_status s;
+    if ((int32_t)I->xs.size() != G - 1 || I->xs_dev0 != o.device) {
+        for (dts_instance *x : I->xs) delete x;
+        I->xs.clear();
+        for (int32_t j = 1; j < G; j++) {
+            dts_instance *x = new (std::nothrow) dts_instance();
+            if (!x) return fail(DTS_E_NOMEM, "host allocation");
+            x->m = I->m; x->n = I->n; x->K = I->K; x->E_raw = I->E_raw; x->cap = I->cap;
+            x->default_ns = I->default_ns; x->task_ptr = I->task_ptr; x->task_data = I->task_data;
+            x->size = I->size; x->task_ns = I->task_ns; x->has_tau = I->has_tau;
+            x->max_deg_ub = I->max_deg_ub; x->max_row_len = I->max_row_len; x->uniform_size = I->uniform_size;
+            x->max_row_bytes = I->max_row_bytes; x->min_size = I->min_size; x->res_cap = I->res_cap;
+            x->m_pad = I->m_pad;
+            I->xs.push_back(x);
+        }
+        std::vector<dts_instance *> sh((size_t)G);
+        sh[0] = I;
+        for (int32_t j = 1; j < G; j++) sh[(size_t)j] = I->xs[(size_t)j - 1];
+        bool cross = false;
+        for (int32_t j = 0; j < G; j++) {
+            if ((s = dts_shard_set(sh[(size_t)j], G, j)) != DTS_OK) return s;
+            if ((s = ensure_device(sh[(size_t)j], dev_of(j))) != DTS_OK) return s;
+            cross |= dev_of(j) != o.device;
+        }
+        for (int32_t a = 0; a < G && cross; a++)  // every pair of distinct devices maps each other
+            for (int32_t b = 0; b < G; b++) {
+                if (dev_of(a) == dev_of(b)) continue;
+                CK(cudaSetDevice(dev_of(a)), "cudaSetDevice");
+                const cudaError_t e = cudaDeviceEnablePeerAccess(dev_of(b), 0);
+                if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+                    return cuda_fail(e, "cudaDeviceEnablePeerAccess");
+                cudaGetLastError();
+            }
+        std::vector<dts::ShardPeer> tab((size_t)G);
+        for (int32_t j = 0; j < G; j++) tab[(size_t)j] = own_peer(sh[(size_t)j]);
+        for (int32_t j = 0; j < G; j++) {  // a new group: exchange numbers from 0 on every shard
+            dts_instance *x = sh[(size_t)j];
+            CK(cudaSetDevice(x->device), "cudaSetDevice");
+            CK(cudaDeviceSynchronize(), "sync");
+            CK(cudaMemset(x->d_epoch, 0, 256), "memset epoch");
+            CK(cudaDeviceSynchronize(), "sync");
+            x->runs = 0;
+            if ((s = write_peers(x, tab)) != DTS_OK) return s;
+            x->xsys = cross;
+        }
+        I->xs_dev0 = o.device;
+    }
+    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    cudaStream_t st = (cudaStream_t)o.cuda_stream;
+    cudaEvent_t fork = nullptr;
+    CK(cudaEventCreateWithFlags(&fork, cudaEventDisableTiming), "cudaEventCreate");
+    CK(cudaEventRecord(fork, st), "event");
+    std::vector<std::pair<int, cudaEvent_t>> joins;
+    s = DTS_OK;
+    for (int32_t j = 0; j < G && s == DTS_OK; j++) {
+        dts_instance *x = j == 0 ? I : I->xs[(size_t)j - 1];
+        dts_run_opts oj = o;
+        oj.device = dev_of(j);
+        oj.n_devices = 1;
+        cudaStream_t sj = st;
+        if (j > 0) {  // shards must run concurrently: one library stream each
+            if ((s = extra_stream(oj.device, (size_t)j, &sj)) != DTS_OK) break;
+            CK(cudaSetDevice(oj.device), "cudaSetDevice");
+            CK(cudaStreamWaitEvent(sj, fork, 0), "wait");
+        }
+        oj.cuda_stream = sj;
+        if ((s = run_one(x, policy, oj)) != DTS_OK) break;
+        if (j > 0) {
+            cudaEvent_t e = nullptr;
+            CK(cudaSetDevice(oj.device), "cudaSetDevice");
+            CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "cudaEventCreate");
+            CK(cudaEventRecord(e, sj), "event");
+            joins.emplace_back(oj.device, e);
+        }
+    }
+    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    for (auto &je : joins) {
+        CK(cudaStreamWaitEvent(st, je.second, 0), "wait");
+        cudaEventDestroy(je.second);
+    }
+    cudaEventDestroy(fork);
+    return s;
+}
 
 // Result copies in two phases so that many instances share the waits
 // (dts_fetch_results): the scalars first (they size the rest), then the arrays.

@@ -60,7 +60,7 @@ class DtsError(RuntimeError):
 class dts_run_opts(C.Structure):
     _fields_ = [("flags", C.c_uint32), ("lookahead_W", C.c_uint32),
                 ("bus_bytes_per_s", C.c_uint64), ("device", C.c_int32),
-                ("block_threads", C.c_int32), ("smem_budget", C.c_int32), ("pad", C.c_int32),
+                ("block_threads", C.c_int32), ("smem_budget", C.c_int32), ("n_devices", C.c_int32),
                 ("max_served", C.c_int64), ("cuda_stream", C.c_void_p)]
 
 
@@ -329,14 +329,14 @@ def dts_version() -> int:
 def schedule(inst, *, policy: int = DTS_POLICY_DARTS_LUF, W: int = 0, flags: int = DTS_F_FALLBACK2,
              bus_bps: int = 12_000_000_000,
              device: int = 0, block_threads: int = 0, smem_budget: int = 0,
-             max_served: int = -1, stream: int = 0) -> Result:
+             max_served: int = -1, stream: int = 0, n_devices: int = 0) -> Result:
     """One call: create the instance from host arrays (a ``gen.Instance``-like
     object), run DARTS+LUF on the GPU, return the host result."""
     h = dts_instance_create(inst.task_ptr, inst.task_data, inst.data_size, inst.task_ns,
                             inst.default_task_ns, inst.mem_capacity, inst.K)
     o = dts_run_opts_default(flags=flags, lookahead_W=W, bus_bytes_per_s=bus_bps, device=device,
                              block_threads=block_threads, smem_budget=smem_budget,
-                             max_served=max_served, cuda_stream=stream or None)
+                             max_served=max_served, cuda_stream=stream or None, n_devices=n_devices)
     dts_run(h, policy, o)
     return dts_result(h)
 

@@ -172,3 +172,24 @@ def test_shard_ipc_two_processes():
     for p, out in zip(procs, outs):
         assert p.returncode == 0, out
         assert "PARITY OK" in out, out
+
+
+# ------------------------------------------- dts_run_opts.n_devices
+@pytest.mark.parametrize("G", [2, 3, 4])
+def test_run_n_devices_matches_oracle(G):
+    """dts_run with n_devices = G: the instance task-sharded over G shards in
+    this process (on a one-GPU machine all on device 0, separate launches
+    exchanging through each other's memory) gives the oracle's schedule."""
+    for inst in (gen.matmul2d(30, M=8, K=3), gen.random_shared(5000, 512, 3, M=20, K=4, seed=G),
+                 gen.matmul3d(8, M=12, K=2)):
+        g = dts.schedule(inst, n_devices=G)
+        assert_parity(g, oracle.run(inst))
+
+
+def test_run_n_devices_then_one_device_again():
+    inst = gen.config_instances("C2")[5]
+    h = dts.create(inst)
+    o = oracle.run(inst)
+    for G in (2, 1, 3, 3, 0):
+        dts.dts_run(h, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default(n_devices=G))
+        assert_parity(dts.dts_result(h), o)
