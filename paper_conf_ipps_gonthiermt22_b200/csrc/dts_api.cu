@@ -63,6 +63,91 @@ struct Arena {
 
 }  // namespace
 
+// ---------------------------------------------------------------- allocator
+// Caching allocator for instance memory (device arenas, pinned host buffers).
+// cudaMalloc / cudaMallocHost / cudaFree cost milliseconds (cudaFree also
+// synchronises the device), so creating and destroying instances per request
+// -- the public API's end-to-end path -- would be dominated by them.  A freed
+// block goes to a per-process pool with an event recorded on the stream of
+// its instance's last work; a later allocation takes the smallest pooled block
+// of at least the size (and at most twice it, plus 1 MiB) on the same device,
+// waiting for that event first.  Bounded: beyond POOL_CAP bytes per kind,
+// blocks are freed.  Arenas exported through CUDA IPC are never pooled.
+namespace {
+struct PoolBlock {
+    void *p;
+    size_t bytes;
+    int device;        // -1: pinned host memory
+    cudaEvent_t done;  // the last work using it (nullptr: none)
+};
+std::mutex g_pool_mu;
+std::vector<PoolBlock> g_pool;
+size_t g_pool_bytes[2] = {0, 0};  // [0] device, [1] host
+constexpr size_t POOL_CAP[2] = {size_t(16) << 30, size_t(4) << 30};
+
+void *pool_take(int device, size_t bytes, size_t *got) {
+    PoolBlock b{nullptr, 0, 0, nullptr};
+    {
+        std::lock_guard<std::mutex> lk(g_pool_mu);
+        size_t bi = SIZE_MAX;
+        for (size_t i = 0; i < g_pool.size(); i++) {
+            const PoolBlock &c = g_pool[i];
+            if (c.device != device || c.bytes < bytes || c.bytes > 2 * bytes + (size_t(1) << 20)) continue;
+            if (bi == SIZE_MAX || c.bytes < g_pool[bi].bytes) bi = i;
+        }
+        if (bi == SIZE_MAX) return nullptr;
+        b = g_pool[bi];
+        g_pool.erase(g_pool.begin() + (std::ptrdiff_t)bi);
+        g_pool_bytes[device < 0] -= b.bytes;
+    }
+    if (b.done) {
+        cudaEventSynchronize(b.done);
+        cudaEventDestroy(b.done);
+    }
+    *got = b.bytes;
+    return b.p;
+}
+
+// `last`: the stream of the block's last work (nullptr: none pending).
+void pool_give(int device, void *p, size_t bytes, cudaStream_t last, bool has_last) {
+    if (!p) return;
+    cudaEvent_t done = nullptr;
+    if (has_last && cudaEventCreateWithFlags(&done, cudaEventDisableTiming) == cudaSuccess &&
+        cudaEventRecord(done, last) != cudaSuccess) {
+        cudaEventDestroy(done);
+        done = nullptr;
+        cudaStreamSynchronize(last);
+    }
+    {
+        std::lock_guard<std::mutex> lk(g_pool_mu);
+        if (g_pool_bytes[device < 0] + bytes <= POOL_CAP[device < 0]) {
+            g_pool.push_back(PoolBlock{p, bytes, device, done});
+            g_pool_bytes[device < 0] += bytes;
+            return;
+        }
+    }
+    if (done) {
+        cudaEventSynchronize(done);
+        cudaEventDestroy(done);
+    }
+    if (device < 0) cudaFreeHost(p);
+    else cudaFree(p);
+}
+
+cudaError_t dev_alloc(int device, size_t bytes, void **p, size_t *got) {
+    *p = pool_take(device, bytes, got);
+    if (*p) return cudaSuccess;
+    *got = bytes;
+    return cudaMalloc(p, bytes);
+}
+cudaError_t host_alloc(size_t bytes, void **p, size_t *got) {
+    *p = pool_take(-1, bytes, got);
+    if (*p) return cudaSuccess;
+    *got = bytes;
+    return cudaMallocHost(p, bytes);
+}
+}  // namespace
+
 // The events of one batched launch, shared by all its instances: recording
 // two events per instance after a long launch fills the device work queue and
 // blocks the host until the launch ends (4,096 instances: the whole sweep).
@@ -110,6 +195,7 @@ struct dts_instance {
     dts::Inst *h_pinned = nullptr;   // pinned staging copy of the descriptor (async H2D)
     cudaEvent_t ev_desc = nullptr;   // the last H2D copy out of h_pinned
     cudaEvent_t ev_up = nullptr;     // the last H2D upload of the inputs
+    cudaStream_t up_stream = nullptr; // ... and the stream it was enqueued on
     void *d_csr_scratch = nullptr;
     int *d_work = nullptr;
     dts::Inst h_inst{};
@@ -125,6 +211,8 @@ struct dts_instance {
     // pinned host memory (allocated with the device arena): a mirror of the
     // inputs for the H2D upload and the result buffers for the D2H read-back
     char *h_pin = nullptr;
+    size_t h_pin_cap = 0, h_pinned_cap = 0, h_res_cap = 0;  // pooled block sizes
+    bool exported = false;                   // arena shared through CUDA IPC: never pooled
     int64_t *p_task_ptr = nullptr, *p_task_ns = nullptr;
     int32_t *p_task_data = nullptr;
     uint64_t *p_size = nullptr;
@@ -156,21 +244,31 @@ struct dts_instance {
 
     ~dts_instance() {
         for (dts_instance *x : xs) delete x;
+        // memory back to the pool behind an event on the last stream that used it
+        // (the default stream when it was never used on another)
+        const bool used = device >= 0;
         if (device >= 0) {
             int cur = 0;
             cudaGetDevice(&cur);
             cudaSetDevice(device);
             for (void *p : ipc_open) cudaIpcCloseMemHandle(p);
-            if (ar.base) cudaFree(ar.base);
+            if (ar.base) {
+                if (exported) cudaFree(ar.base);
+                else pool_give(device, ar.base, ar.size, stream, true);
+            }
             for (auto &e : ev)
                 if (e) cudaEventDestroy(e);
             if (ev_desc) cudaEventDestroy(ev_desc);
             if (ev_up) cudaEventDestroy(ev_up);
+            if (h_pinned) pool_give(-1, h_pinned, h_pinned_cap, stream, true);
+            if (h_pin) pool_give(-1, h_pin, h_pin_cap, stream, true);
+            if (h_res) pool_give(-1, h_res, h_res_cap, stream, true);
             cudaSetDevice(cur);
+        } else {
+            if (h_pinned) pool_give(-1, h_pinned, h_pinned_cap, nullptr, used);
+            if (h_pin) pool_give(-1, h_pin, h_pin_cap, nullptr, used);
+            if (h_res) pool_give(-1, h_res, h_res_cap, nullptr, used);
         }
-        if (h_pinned) cudaFreeHost(h_pinned);
-        if (h_pin) cudaFreeHost(h_pin);
-        if (h_res) cudaFreeHost(h_res);
     }
 };
 
@@ -346,7 +444,8 @@ dts_status ensure_device(dts_instance *I, int device) {
         if (I->connected && I->G > 1)
             return fail(DTS_E_STATE, "a connected task shard cannot move to another device");
         cudaSetDevice(I->device);
-        cudaFree(I->ar.base);
+        if (I->exported) cudaFree(I->ar.base);
+        else pool_give(I->device, I->ar.base, I->ar.size, I->stream, true);
         for (auto &e : I->ev)
             if (e) cudaEventDestroy(e);
         if (I->ev_desc) cudaEventDestroy(I->ev_desc);
@@ -386,16 +485,18 @@ dts_status ensure_device(dts_instance *I, int device) {
     const int64_t box_bytes = (int64_t)sizeof(dts::ShardSlot) + 16 * (int64_t)plan_cap;
     add(256); add(2 * (size_t)box_bytes); add(sizeof(dts::ShardPeer) * dts::MAX_G);  // shard exchange
     char *base = nullptr;
-    cudaError_t e = cudaMalloc(&base, need);
+    size_t got = 0;
+    cudaError_t e = dev_alloc(device, need, reinterpret_cast<void **>(&base), &got);
     if (e != cudaSuccess) return fail(DTS_E_NOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
     I->ar.base = base;
-    I->ar.size = need;
+    I->ar.size = got;
     I->ar.used = 0;
     I->device = device;
     for (auto &ev : I->ev) CK(cudaEventCreate(&ev), "cudaEventCreate");
     CK(cudaEventCreateWithFlags(&I->ev_desc, cudaEventDisableTiming), "cudaEventCreate");
     CK(cudaEventCreateWithFlags(&I->ev_up, cudaEventDisableTiming), "cudaEventCreate");
-    if (!I->h_pinned) CK(cudaMallocHost(&I->h_pinned, sizeof(dts::Inst)), "cudaMallocHost");
+    if (!I->h_pinned)
+        CK(host_alloc(sizeof(dts::Inst), reinterpret_cast<void **>(&I->h_pinned), &I->h_pinned_cap), "cudaMallocHost");
     if (!I->h_pin) {
         size_t hb = 0;
         // the input mirror has the device arena's layout (256-byte rounding, same
@@ -403,7 +504,7 @@ dts_status ensure_device(dts_instance *I, int device) {
         auto hadd = [&](size_t bytes) { size_t o = hb; hb += (bytes + 255) & ~size_t(255); return o; };
         const size_t o_tp = hadd(8 * (m + 1)), o_td = hadd(4 * (E + 1)), o_sz = hadd(8 * (n + 1)),
                      o_tn = hadd(8 * (m + 1)), o_out = hadd(sizeof(dts::Out));
-        CK(cudaMallocHost(&I->h_pin, hb), "cudaMallocHost");
+        CK(host_alloc(hb, reinterpret_cast<void **>(&I->h_pin), &I->h_pin_cap), "cudaMallocHost");
         I->p_task_ptr = (int64_t *)(I->h_pin + o_tp);
         I->p_task_data = (int32_t *)(I->h_pin + o_td);
         I->p_size = (uint64_t *)(I->h_pin + o_sz);
@@ -461,11 +562,11 @@ dts_status ensure_device(dts_instance *I, int device) {
     {  // host mirror of the result region, same relative layout
         char *r0 = reinterpret_cast<char *>(h.gpu_task_ptr);
         const size_t bytes = (size_t)(reinterpret_cast<char *>(h.events) - r0) + sizeof(dts_event) * ev_cap;
-        if (I->h_res && I->res_bytes != bytes) {
-            cudaFreeHost(I->h_res);
+        if (I->h_res && I->h_res_cap < bytes) {
+            pool_give(-1, I->h_res, I->h_res_cap, I->stream, true);
             I->h_res = nullptr;
         }
-        if (!I->h_res) CK(cudaMallocHost(&I->h_res, bytes), "cudaMallocHost");
+        if (!I->h_res) CK(host_alloc(bytes, reinterpret_cast<void **>(&I->h_res), &I->h_res_cap), "cudaMallocHost");
         I->res_bytes = bytes;
         auto at = [&](const void *d) { return I->h_res + (reinterpret_cast<const char *>(d) - r0); };
         I->r_gpu_ptr = reinterpret_cast<int64_t *>(at(h.gpu_task_ptr));
@@ -511,6 +612,7 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
                                              : reinterpret_cast<const char *>(I->d_size + I->n);
     CK(cudaMemcpyAsync(I->d_raw_ptr, I->p_task_ptr, (size_t)(end - d0), cudaMemcpyHostToDevice, st), "H2D inputs");
     CK(cudaEventRecord(I->ev_up, st), "event");  // a run on another stream waits for it (stage)
+    I->up_stream = st;
     I->uploaded = true;
     return DTS_OK;
 }
@@ -637,8 +739,11 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     s = upload(I, st);
     if (s != DTS_OK) return s;
     // inputs uploaded on another stream (dts_instance_upload) are complete
-    // before this run reads them (no-op on the same stream)
-    CK(cudaStreamWaitEvent(st, I->ev_up, 0), "wait upload");
+    // before this run reads them (the same stream orders them already)
+    if (I->up_stream != st) {
+        CK(cudaStreamWaitEvent(st, I->ev_up, 0), "wait upload");
+        I->up_stream = st;
+    }
     dts::Inst &h = I->h_inst;
     h.W = (int32_t)o.lookahead_W;
     h.flags = o.flags;
@@ -1082,6 +1187,7 @@ dts_status dts_shard_export(dts_instance *I, int32_t device, void *handle) {
     ShardHandle hd;
     std::memset(&hd, 0, sizeof hd);
     CK(cudaIpcGetMemHandle(&hd.mem, I->ar.base), "cudaIpcGetMemHandle");
+    I->exported = true;
     const char *b = I->ar.base;
     hd.off_epoch = (const char *)I->d_epoch - b;
     hd.off_box = (const char *)I->d_box - b;
