@@ -353,7 +353,12 @@ def main():
         decisions = res0[0].n_served if (gsh or rank == 0) else 0
     assert decisions == sum(i.m for i in insts) or (xsh and rank > 0), "not every task scheduled"
 
-    # ---- device-resident timed region
+    # ---- device-resident timed region (Python's cyclic GC paused, as timeit does:
+    # a full collection over the thousands of handle objects of a C5 batch
+    # stalled the host for ~100 ms inside some steps, profiles/r02v_host_c5.txt)
+    import gc
+    gc.collect()
+    gc.disable()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
            for _ in range(args.steps)]
     loop_ms_steps = []
@@ -420,6 +425,7 @@ def main():
         t1.synchronize()
         e2e_ms.append(t0.elapsed_time(t1))
     e2e_avg = sum(e2e_ms) / len(e2e_ms)
+    gc.enable()
 
     # ---- max over ranks (device times), sum of the work
     from paper_conf_ipps_gonthiermt22_b200.shard import reduce_over_ranks
@@ -450,8 +456,8 @@ def main():
                                  f" ({nd} decisions, {dt:.1f} s, one instance per thread)"}
         clocks = clk.summary()
         launch = ("one batched loop launch, one CTA per instance" if len(insts) < 296 else
-                  "two concurrent batched loop launches (256-thread CTAs for the long-segment "
-                  "instances, <= 128 for the rest), one CTA per instance") if not single \
+                  "one batched loop launch of 128-thread CTAs (4 per SM), one CTA per instance, "
+                  "longest first") if not single \
             else (f"one cooperative launch: the instance task-sharded over {args.shards} CTAs"
                   if gsh else f"one loop launch per rank: the instance task-sharded over "
                   f"{world} B200s, peer-memory exchanges" if xsh

@@ -238,10 +238,10 @@ dts_status dts_fetch_results(dts_instance *const *insts, int32_t n);
  *                  Otherwise the instances are split over the entries by LPT
  *                  on a chain-cost estimate (m * mean degree), longest first,
  *                  each to the least loaded entry.
- * Per device entry: ONE batched launch of the decision loop (two concurrent
- * ones for a large batch: wide CTAs for long-segment instances, narrow ones
- * for the rest), one CTA per instance, CTAs pulling instances from that
- * launch's own device counter; every launch has its own descriptor buffer,
+ * Per device entry: ONE batched launch of the decision loop, one CTA per
+ * instance (<= 128 threads when the batch has many more instances than SMs,
+ * so several chains share an SM), CTAs pulling instances longest-first from
+ * that launch's own device counter; every launch has its own descriptor buffer,
  * so concurrent sweeps on different streams or threads do not interfere.
  * The first entry on opts->device is enqueued on opts->cuda_stream; the
  * others on library streams of their devices, forked from and joined back

@@ -732,7 +732,8 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
                  cudaStream_t st, bool copy_desc = true, bool own_events = true) {
     dts_status s = ensure_device(I, o.device);
     if (s != DTS_OK) return s;
-    CK(cudaSetDevice(o.device), "cudaSetDevice");
+    int cur = -1;
+    if (cudaGetDevice(&cur) != cudaSuccess || cur != o.device) CK(cudaSetDevice(o.device), "cudaSetDevice");
     I->stream = st;
     I->ran = false;
     I->have_host = false;
@@ -812,7 +813,7 @@ int budget_of(const dts_run_opts &o) {
 struct SweepSlot {
     dts::Inst *d_insts = nullptr;  // descriptors, then the launch's instance counters
     dts::Inst *h_insts = nullptr;  // pinned staging copy (async H2D)
-    int *d_work = nullptr;         // [0]: group A's instance counter, [1]: group B's
+    int *d_work = nullptr;         // the launch's instance counter
     size_t cap = 0;
     cudaEvent_t done = nullptr;    // recorded after every kernel that reads this slot
 };
@@ -822,8 +823,6 @@ struct DeviceSweep {
     SweepSlot slot[RING];
     int next = 0;
     bool init = false;
-    cudaStream_t side = nullptr;  // group B of a split batch (forked from / joined into the caller's stream)
-    cudaEvent_t fork = nullptr, join = nullptr;
     std::vector<cudaStream_t> extra;  // library streams for multi-device sweeps (dts_sweep_run devices[])
 };
 DeviceSweep g_dev[64];
@@ -831,9 +830,6 @@ DeviceSweep g_dev[64];
 // Caller holds D.mu; the device is current.
 dts_status acquire_slot(DeviceSweep &D, size_t n, SweepSlot **out) {
     if (!D.init) {
-        CK(cudaEventCreateWithFlags(&D.fork, cudaEventDisableTiming), "cudaEventCreate");
-        CK(cudaEventCreateWithFlags(&D.join, cudaEventDisableTiming), "cudaEventCreate");
-        CK(cudaStreamCreateWithFlags(&D.side, cudaStreamNonBlocking), "cudaStreamCreate");
         D.init = true;
     }
     SweepSlot &S = D.slot[D.next];
@@ -856,7 +852,7 @@ dts_status acquire_slot(DeviceSweep &D, size_t n, SweepSlot **out) {
     return DTS_OK;
 }
 
-// One batched launch (or two concurrent ones) of insts[0..n) on o.device,
+// One batched launch of insts[0..n) on o.device,
 // enqueued on st.  The instances are validated by the caller.
 dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy policy, const dts_run_opts &o,
                            cudaStream_t st) {
@@ -879,26 +875,21 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     for (int32_t i = 0; i < n; i++) ord[(size_t)i] = i;
     std::stable_sort(ord.begin(), ord.end(),
                      [&](int32_t a, int32_t b) { return instance_cost(insts[a]) > instance_cost(insts[b]); });
-    // CTA size per group: a batch of many instances runs as two concurrent
-    // launches -- the instances whose segments want wide CTAs (auto_block >=
-    // 256) with those, the rest with small CTAs so more chains share an SM.
-    // Few instances, or a forced size: one launch.
+    // CTA size: each instance wants twice its widest segment (auto_block); a
+    // batch of many instances runs in ONE launch of <= 128-thread CTAs so that
+    // four chains share an SM (registers) and the longest ones, handed out
+    // first by the launch's counter, overlap the rest (C5: 232 ms against 280
+    // for round 1's two concurrent launches of 256- and 128-thread CTAs,
+    // profiles/r02s_c5_block.txt).  A forced size applies to all.
     const int forced = o.block_threads;
     const int small_max = tuning("DTS_SWEEP_SMALL_BLOCK", 128);
-    int nb = n, block_a = 32, block_b = 32;  // group A = ord[0, nb), group B = ord[nb, n)
-    if (!forced && many && small_max > 0) {
-        nb = 0;
-        for (int32_t i = 0; i < n; i++)
-            if (auto_block(insts[ord[(size_t)i]]) > small_max) nb = i + 1;  // the long ones come first
-        // group B: every instance after the last wide one (cost order ~ width order)
-    }
+    int block = 32;
     for (int32_t i = 0; i < n; i++) {
         const int ab = auto_block(insts[ord[(size_t)i]], !many);
-        if (i < nb) block_a = std::max(block_a, ab);
-        else block_b = std::max(block_b, std::min(ab, small_max));
+        block = std::max(block, many ? std::min(ab, small_max) : ab);
     }
-    if (forced) block_a = block_b = forced;
-    int smem_a = 0, smem_b = 0;
+    if (forced) block = forced;
+    int smem = 0;
     bool any_unfused = false;
     auto sev = std::make_shared<SweepEvents>();
     sev->device = o.device;
@@ -908,9 +899,9 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     CK(cudaEventRecord(sev->begin, st), "event");
     for (int32_t i = 0; i < n; i++) {
         dts_instance *I = insts[ord[(size_t)i]];
-        dts_status s = stage(I, policy, o, budget, i < nb ? block_a : block_b, st, false, false);
+        dts_status s = stage(I, policy, o, budget, block, st, false, false);
         if (s != DTS_OK) return s;
-        (i < nb ? smem_a : smem_b) = std::max(i < nb ? smem_a : smem_b, I->h_inst.smem_bytes);
+        smem = std::max(smem, I->h_inst.smem_bytes);
         any_unfused |= !I->h_inst.fused;
     }
     DeviceSweep &D = g_dev[o.device];
@@ -924,22 +915,9 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     CK(cudaMemsetAsync(S->d_work, 0, 2 * sizeof(int), st), "memset");
     if (any_unfused) CK(dts::launch_init(S->d_insts, n, o.bus_bytes_per_s, work, st), "init");
     CK(cudaEventRecord(sev->loop_begin, st), "event");
-    const bool two = nb > 0 && nb < n;
-    if (two) {  // group B on the side stream, forked from and joined back into st
-        CK(cudaEventRecord(D.fork, st), "event");
-        CK(cudaStreamWaitEvent(D.side, D.fork, 0), "wait");
-        const int per_b = std::max(1, dts::loop_max_blocks_per_sm(block_b, smem_b));
-        const int grid_b = (int)std::min<int64_t>((int64_t)(n - nb), (int64_t)per_b * nsm);
-        CK(dts::launch_loop(S->d_insts + nb, n - nb, block_b, grid_b, S->d_work + 1, smem_b, D.side), "loop B");
-        CK(cudaEventRecord(D.join, D.side), "event");
-    }
-    const int na = two ? nb : n;
-    const int blk = two ? block_a : std::max(block_a, block_b);
-    const int sm = two ? smem_a : std::max(smem_a, smem_b);
-    const int per = std::max(1, dts::loop_max_blocks_per_sm(blk, sm));
-    const int grid = (int)std::min<int64_t>((int64_t)na, (int64_t)per * nsm);
-    CK(dts::launch_loop(S->d_insts, na, blk, grid, S->d_work, sm, st), "loop");
-    if (two) CK(cudaStreamWaitEvent(st, D.join, 0), "wait");
+    const int per = std::max(1, dts::loop_max_blocks_per_sm(block, smem));
+    const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
+    CK(dts::launch_loop(S->d_insts, n, block, grid, S->d_work, smem, st), "loop");
     CK(cudaEventRecord(sev->loop_end, st), "event");
     CK(cudaEventRecord(S->done, st), "event");
     for (int32_t i = 0; i < n; i++) {

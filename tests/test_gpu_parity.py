@@ -307,9 +307,9 @@ def test_sweep_sample_config5():
 
 
 def test_sweep_split_launch():
-    """A batch of >= 2 x 148 instances runs as two concurrent launches (wide
-    CTAs for the instances with long segments, <= 128-thread CTAs for the rest),
-    each on its own device counter; every instance must match the oracle."""
+    """A batch of >= 2 x 148 instances runs as one launch of <= 128-thread CTAs
+    (several chains per SM, longest first): every instance must match the
+    oracle, including the wide-segment ones."""
     params = [(N, M, K) for N in (5, 10, 15) for M in (4, 6, 8, 12) for K in (1, 2, 3, 4)]
     insts = [gen.sweep_instance(*p) for p in params] * 7                 # 336 narrow
     insts += [gen.sweep_instance(70, 8, 2), gen.sweep_instance(140, 12, 3)]  # 128 (B), 256 (A)
