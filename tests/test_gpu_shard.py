@@ -193,3 +193,22 @@ def test_run_n_devices_then_one_device_again():
     for G in (2, 1, 3, 3, 0):
         dts.dts_run(h, dts.DTS_POLICY_DARTS_LUF, dts.dts_run_opts_default(n_devices=G))
         assert_parity(dts.dts_result(h), o)
+
+
+@pytest.mark.parametrize("policy,flag", [(dts.DTS_POLICY_DARTS_LRU, oracle.F_LRU),
+                                         (dts.DTS_POLICY_EAGER_LRU, oracle.F_EAGER | oracle.F_LRU)])
+def test_run_n_devices_lru_policies(policy, flag):
+    inst = gen.matmul2d(24, M=10, K=3)
+    g = dts.schedule(inst, policy=policy, n_devices=2)
+    assert_parity(g, oracle.run(inst, flags=1 | flag))
+
+
+@pytest.mark.parametrize("W", [1, 2])
+def test_run_n_devices_window(W):
+    """Task-sharded runs with a prefetch window and the tight capacity (Belady, R29)."""
+    inst = gen.random_shared(3000, 256, 3, M=8, K=3, seed=W)
+    row = 3 * int(inst.data_size[0])
+    inst = inst.with_(mem_capacity=max(1, W) * row)
+    g = dts.schedule(inst, W=W, n_devices=3)
+    o = oracle.run(inst, W=W)
+    assert_parity(g, o)
