@@ -86,7 +86,11 @@ enum {
      * (cnt:7 | xor:24, 4 K m bytes) even when every task has <= 3 inputs
      * (default then: no per-GPU task state, the missing inputs are read off
      * the task's row and the residency bitmaps). */
-    DTS_F_PACKED = 1u << 4
+    DTS_F_PACKED = 1u << 4,
+    /* Diagnostic: run the generic decision loop even when the one compiled for
+     * the default mode applies (row-derived state, one shard, W = 0,
+     * DARTS+LUF: every BASELINE config). */
+    DTS_F_GENERIC = 1u << 5
 };
 
 typedef struct {

@@ -10,6 +10,7 @@ from .dts import (  # noqa: F401
     DTS_F_NOFUSE,
     DTS_F_OPTI,
     DTS_F_PACKED,
+    DTS_F_GENERIC,
     DTS_POLICY_DARTS_LUF,
     DTS_POLICY_DARTS_LRU,
     DTS_POLICY_EAGER_LRU,

@@ -620,7 +620,8 @@ dts_status upload(dts_instance *I, cudaStream_t st, bool force = false) {
 dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_opts *o) {
     if (policy != DTS_POLICY_DARTS_LUF && policy != DTS_POLICY_DARTS_LRU && policy != DTS_POLICY_EAGER_LRU)
         return fail(DTS_E_UNSUPPORTED, "policy");
-    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI | DTS_F_PACKED))
+    if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI | DTS_F_PACKED |
+                               DTS_F_GENERIC))
         return fail(DTS_E_UNSUPPORTED, "unknown flags");
     if (o->lookahead_W > (uint32_t)dts::MAX_W) return fail(DTS_E_UNSUPPORTED, "lookahead_W > 8");
     if ((int64_t)o->lookahead_W * I->max_row_len > dts::MAX_ROW + 1)
@@ -658,6 +659,13 @@ int tuning(const char *name, int dflt) {
 // Relative cost of an instance's chain (longest-first ordering, LPT over devices).
 double instance_cost(const dts_instance *I) {
     return (double)I->m * (double)I->E_raw / std::max(1, I->n);
+}
+
+// The compile-time specialised loop (dts_loop_fast.cu) applies: row-derived
+// state, one shard, W = 0, DARTS+LUF, no self-check, not forced generic.
+bool fast_mode(const dts::Inst &h) {
+    return h.sl && h.G == 1 && h.W == 0 && h.policy == DTS_POLICY_DARTS_LUF &&
+           !(h.flags & (DTS_F_VERIFY | DTS_F_GENERIC));
 }
 
 // Shared-memory placement of one instance's state:
@@ -703,7 +711,7 @@ int max_dyn_smem(int device) {
     if (device >= 0 && device < 64 && cache[device] > 0) return cache[device];
     int optin = 0;
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
-    int st = dts::loop_static_smem();
+    int st = std::max(dts::loop_static_smem(), dts::loop_static_smem_fast());
     if (st < 0) st = 16384;
     const int r = std::max(0, optin - st - 1024);
     if (device >= 0 && device < 64) cache[device] = r;
@@ -915,9 +923,13 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     CK(cudaMemsetAsync(S->d_work, 0, 2 * sizeof(int), st), "memset");
     if (any_unfused) CK(dts::launch_init(S->d_insts, n, o.bus_bytes_per_s, work, st), "init");
     CK(cudaEventRecord(sev->loop_begin, st), "event");
-    const int per = std::max(1, dts::loop_max_blocks_per_sm(block, smem));
+    bool fast = true;
+    for (int32_t i = 0; i < n; i++) fast &= fast_mode(insts[i]->h_inst);
+    const int per = std::max(1, fast ? dts::loop_max_blocks_per_sm_fast(block, smem)
+                                     : dts::loop_max_blocks_per_sm(block, smem));
     const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
-    CK(dts::launch_loop(S->d_insts, n, block, grid, S->d_work, smem, st), "loop");
+    if (fast) CK(dts::launch_loop_fast(S->d_insts, n, block, grid, S->d_work, smem, st), "loop");
+    else CK(dts::launch_loop(S->d_insts, n, block, grid, S->d_work, smem, st), "loop");
     CK(cudaEventRecord(sev->loop_end, st), "event");
     CK(cudaEventRecord(S->done, st), "event");
     for (int32_t i = 0; i < n; i++) {
@@ -991,7 +1003,10 @@ static dts_status run_one(dts_instance *I, dts_policy policy, const dts_run_opts
     if (!I->h_inst.fused) CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
     CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
     CK(cudaEventRecord(I->ev[1], st), "event");
-    CK(dts::launch_loop(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");
+    if (fast_mode(I->h_inst))
+        CK(dts::launch_loop_fast(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");
+    else
+        CK(dts::launch_loop(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");
     CK(cudaEventRecord(I->ev[2], st), "event");
     CK(cudaEventRecord(I->ev[3], st), "event");
     I->ran = true;

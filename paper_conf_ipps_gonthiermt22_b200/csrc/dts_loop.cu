@@ -34,6 +34,27 @@
 #include "dts_internal.cuh"
 #include "dts_loop.cuh"
 
+// Mode predicates.  This file is compiled twice: as the generic loop (every
+// mode, chosen at run time from the descriptor) and, from dts_loop_fast.cu
+// with DTS_FAST = 1, specialised at compile time to the mode every BASELINE
+// config runs in -- row-derived state (rows of <= 3 inputs), one shard, W = 0,
+// DARTS+LUF -- so the other modes' code is compiled out of the hot loop (the
+// loop is instruction-cache bound: DESIGN.md §6).
+#ifndef DTS_FAST
+#define DTS_FAST 0
+#endif
+#define M_SL(I) (DTS_FAST || (I).sl)                           // row-derived state
+#define M_SHARD(I) (!DTS_FAST && (I).G > 1)                    // task shards
+#define M_W(I) (DTS_FAST ? 0 : (I).W)                          // prefetch window
+#define M_LUF(I) (DTS_FAST || (I).policy == DTS_POLICY_DARTS_LUF)
+#define M_POL(I, p) (!DTS_FAST && (I).policy == (p))            // an LRU policy
+#define M_LONG(c) (!DTS_FAST && (c))                           // rows of > 3 inputs
+#if DTS_FAST
+#define DTS_KNAME(x) x##_fast
+#else
+#define DTS_KNAME(x) x
+#endif
+
 namespace dts {
 
 namespace {
@@ -281,7 +302,7 @@ __device__ __noinline__ void missing_pair_long(int k, int32_t T, int32_t skip, i
 
 // The (first two) inputs of T not resident on GPU k, skipping `skip`.
 __device__ __forceinline__ void missing_pair(int k, int32_t T, Row r, int32_t skip, int32_t &a, int32_t &b) {
-    if (r.len > 3) {
+    if (M_LONG(r.len > 3)) {
         missing_pair_long(k, T, skip, a, b);
         return;
     }
@@ -323,8 +344,8 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
     const Inst &I = SI;
     const View &V = SV;
     const int K = I.K;
-    const bool own = T >= I.t_lo && T < I.t_hi;
-    if (I.sl) {  // row-derived state: the allocation bit, then each GPU's buckets
+    const bool own = DTS_FAST || (T >= I.t_lo && T < I.t_hi);
+    if (M_SL(I)) {  // row-derived state: the allocation bit, then each GPU's buckets
         set_alloc(T, sign);
 #pragma unroll 1
         for (int j = 0; j < K; j++) {
@@ -338,7 +359,7 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
             }
         }
     }
-    for (int j0 = 0; own && !I.sl && j0 < K; j0 += 4) {
+    for (int j0 = 0; own && !M_SL(I) && j0 < K; j0 += 4) {
         uint32_t w0 = 0, w1 = 0, w2 = 0, w3 = 0;
         w0 = V.s[(size_t)j0 * I.m_pad + T];
         if (j0 + 1 < K) w1 = V.s[(size_t)(j0 + 1) * I.m_pad + T];
@@ -361,7 +382,7 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
             }
         }
     }
-    if (r.len > 3) {
+    if (M_LONG(r.len > 3)) {
         pool_move_long_row(T, sign, plan_k, own);
         return;
     }
@@ -388,7 +409,7 @@ __device__ __noinline__ void pool_item_packed(int4 e, int j, int sign) {
         atomicAdd(&V.h[(size_t)j * I.nstr + (w & XOR_MASK)], sign);
     } else if (c == 2u) {
         int32_t a, b;
-        const bool lng = e.w == ROW_LONG;
+        const bool lng = M_LONG(e.w == ROW_LONG);
         const int len = lng ? 4 : (e.y >= 0) + (e.z >= 0) + (e.w >= 0);
         if (len == 2) {  // both inputs miss: no residency lookups
             a = e.y;
@@ -417,7 +438,7 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
             const int p = idx / K, j = idx - p * K;
             const int4 e = ents[p];
             const int32_t T = e.x;
-            if (I.sl) {  // row-derived state: T's missing inputs on GPU j from its row
+            if (M_SL(I)) {  // row-derived state: T's missing inputs on GPU j from its row
                 int32_t a, b;
                 const int c = missing_of(j, e.y, e.z, e.w, a, b);
                 if (c == 1) {
@@ -433,9 +454,9 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
         } else {
             const int4 e = ents[idx - n_state];
             const int32_t T = e.x;
-            const bool own = T >= I.t_lo && T < I.t_hi;
-            if (I.sl) set_alloc(T, sign);
-            if (e.w == ROW_LONG) {
+            const bool own = DTS_FAST || (T >= I.t_lo && T < I.t_hi);
+            if (M_SL(I)) set_alloc(T, sign);
+            if (M_LONG(e.w == ROW_LONG)) {
                 pool_move_long_row(T, sign, plan_k, own);
                 continue;
             }
@@ -466,7 +487,7 @@ __device__ __forceinline__ int4 entry_of_task(int32_t T) {
 // entry (rows are sorted, so the entry lists them ascending, R10) -- no second
 // CSR read; a longer row is read by the serve path (row_len = -1).
 __device__ __forceinline__ void row_from_entry(int4 e) {
-    if (e.w == ROW_LONG) {
+    if (M_LONG(e.w == ROW_LONG)) {
         L.row_len = -1;
         return;
     }
@@ -505,7 +526,7 @@ __device__ __noinline__ void seg_update_packed(int k, int32_t D, bool load) {
                 atomicAdd(&hk[o], 1);
             } else if (c == 3u) {  // 3 -> 2: one load away from two data
                 int32_t a2 = ed.y, b2 = ed.z;  // |D(T)| = 3: both others miss
-                if (ed.w > 3) missing_pair(k, T, Row{-1, -1, -1, ed.w}, -1, a2, b2);
+                if (M_LONG(ed.w > 3)) missing_pair(k, T, Row{-1, -1, -1, ed.w}, -1, a2, b2);
                 atomicAdd(&h2k[a2], 1);
                 atomicAdd(&h2k[b2], 1);
             }
@@ -518,7 +539,7 @@ __device__ __noinline__ void seg_update_packed(int k, int32_t D, bool load) {
                 atomicAdd(&h2k[D], 1);
             } else if (c == 2u) {  // 2 -> 3
                 int32_t a2 = ed.y, b2 = ed.z;  // |D(T)| = 3: both others missed
-                if (ed.w > 3) missing_pair(k, T, Row{-1, -1, -1, ed.w}, D, a2, b2);
+                if (M_LONG(ed.w > 3)) missing_pair(k, T, Row{-1, -1, -1, ed.w}, D, a2, b2);
                 atomicSub(&h2k[a2], 1);
                 atomicSub(&h2k[b2], 1);
             }
@@ -536,7 +557,7 @@ __device__ __noinline__ void seg_update_packed(int k, int32_t D, bool load) {
 __device__ void seg_update(int k, int32_t D, bool load) {
     const Inst &I = SI;
     const View &V = SV;
-    if (!I.sl) {
+    if (!M_SL(I)) {
         seg_update_packed(k, D, load);
         return;
     }
@@ -602,12 +623,17 @@ __device__ __forceinline__ void push_event(uint8_t op, int k, int32_t D, int32_t
 // (at t).  Task times of earlier tasks are this thread's own writes.
 __device__ __forceinline__ int64_t next_request(int k, int32_t T, int64_t t, int64_t start, int64_t end) {
     const Inst &I = SI;
+#if DTS_FAST
+    (void)I, (void)k, (void)T, (void)t, (void)start;
+    return end;
+#else
     if (I.W == 0) return end;
     const int W = I.W;
     const int j = ++L.won[k];
     I.wring[k * MAX_W + (j - 1) % W] = T;
     if (j < W) return t;
     return W == 1 ? start : __ldcg(&I.tstart[I.wring[k * MAX_W + j % W]]);
+#endif
 }
 
 // Thread 0: record the service of T on k (time model of PAPER.md:276-342, R7, R9).
@@ -649,7 +675,7 @@ __device__ int32_t pop_planned(int k, int64_t *tau) {
     L.plan_head[k] = h + 1;
     L.plan_live[k]--;
     int32_t *npk = V.np + (size_t)k * I.nstr;
-    if (e.w != ROW_LONG) {
+    if (!M_LONG(e.w == ROW_LONG)) {
         if (e.y >= 0) atomicSub(&npk[e.y], 1);
         if (e.z >= 0) atomicSub(&npk[e.z], 1);
         if (e.w >= 0) atomicSub(&npk[e.w], 1);
@@ -664,7 +690,7 @@ __device__ int32_t pop_planned(int k, int64_t *tau) {
         *tau = I.default_tau;
     }
     // D(T) for serve_loads, ascending (R10), straight from the entry when cached
-    if (e.w != ROW_LONG) {
+    if (!M_LONG(e.w == ROW_LONG)) {
         int32_t a = e.y, b = e.z, c = e.w;  // -1 = absent; sort descending, count
         if (a < b) { const int32_t t = a; a = b; b = t; }
         if (b < c) { const int32_t t = b; b = c; c = t; }
@@ -690,7 +716,7 @@ __device__ int32_t pop_planned(int k, int64_t *tau) {
 __device__ __forceinline__ int pop_run_seq() {
     const Inst &I = SI;
     const View &V = SV;
-    const int K = I.K, W = I.W, pcap = I.plan_cap;
+    const int K = I.K, W = M_W(I), pcap = I.plan_cap;
     const int64_t maxs = I.max_served, dtau = I.default_tau;
     int32_t *const sg = I.serve_gpu;
     int32_t *const stk = I.serve_task;
@@ -1118,7 +1144,7 @@ __device__ void reset_plan(int k) {
     const int pe = L.plan_end[k];
     for (int i = threadIdx.x; i < pe; i += blockDim.x) {
         const int4 e = pl[i];
-        if (e.w != ROW_LONG) {
+        if (!M_LONG(e.w == ROW_LONG)) {
             if (e.y >= 0) npk[e.y] = 0;
             if (e.z >= 0) npk[e.z] = 0;
             if (e.w >= 0) npk[e.w] = 0;
@@ -1140,14 +1166,14 @@ __device__ void reset_plan(int k) {
 }
 
 __device__ __forceinline__ Row row_of_entry(int4 e) {
-    if (e.w == ROW_LONG) return Row{-1, -1, -1, 4};
+    if (M_LONG(e.w == ROW_LONG)) return Row{-1, -1, -1, 4};
     return Row{e.y, e.z, e.w, (e.y >= 0) + (e.z >= 0) + (e.w >= 0)};
 }
 
 __device__ __forceinline__ bool entry_uses(int4 e, int32_t D) {
     const Inst &I = SI;
     if (e.y == D || e.z == D) return true;
-    if (e.w != ROW_LONG) return e.w == D;
+    if (!M_LONG(e.w == ROW_LONG)) return e.w == D;
     const int64_t rb = __ldg(&I.tptr[e.x]), re = __ldg(&I.tptr[e.x + 1]);
     for (int64_t i = rb; i < re; i++)
         if (__ldg(&I.tdat[i]) == D) return true;
@@ -1165,7 +1191,7 @@ __device__ int32_t luf_victim(int k) {
     const int cnt = L.res_cnt[k];
     const int32_t *rl = V.res_list + (size_t)k * I.res_cap;
     // LUF key np_k(D); LRU policies: the serve index of D's last use on k
-    const int32_t *npk = (I.policy == DTS_POLICY_DARTS_LUF ? V.np : V.lru) + (size_t)k * I.nstr;
+    const int32_t *npk = (M_LUF(I) ? V.np : V.lru) + (size_t)k * I.nstr;
     const int nr = L.row_len, nr2 = L.row2_len;
     unsigned long long best = ~0ull;
     int bslot = -1;
@@ -1229,7 +1255,7 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t, int64_t te)
     int nret = 0;
     unsigned tmin = 0xffffffffu;
     // Alg. 6 l.8 is LUF's; an LRU eviction leaves plannedTasks_k alone
-    const int ph = L.plan_head[k], pe = I.policy == DTS_POLICY_DARTS_LUF ? L.plan_end[k] : ph;
+    const int ph = L.plan_head[k], pe = M_LUF(I) ? L.plan_end[k] : ph;
     for (int i = ph + threadIdx.x; i < pe; i += blockDim.x) {
         const int4 e = pl[i];
         if (e.x >= 0 && entry_uses(e, Vd)) {
@@ -1319,7 +1345,7 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
             if (!resident(k, L.row[r])) L.miss[nm++] = L.row[r];
         L.nmiss = nm;
     }
-    if (I.W >= 1 && threadIdx.x < 32) buffer_rows(k, t);
+    if (M_W(I) >= 1 && threadIdx.x < 32) buffer_rows(k, t);
     cta_sync();
     const int nmiss = L.nmiss;
     for (int r = 0; r < nmiss; r++) {
@@ -1332,7 +1358,7 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
             PROF_T0(p_luf);
             int32_t Vd = luf_victim(k);
             bool belady = false;
-            if (Vd < 0 && I.policy == DTS_POLICY_DARTS_LUF && I.W >= 1) {
+            if (Vd < 0 && M_LUF(I) && M_W(I) >= 1) {
                 Vd = belady_victim(k);
                 belady = true;
                 if (threadIdx.x == 0) L.n_belady++;
@@ -1367,14 +1393,14 @@ __device__ void serve_loads(int k, int32_t T, int64_t t) {
         }
         // seg_update reads nothing thread 0 just wrote unless a row is longer
         // than its edge record (missing_pair reads the residency bitmap)
-        if (I.max_row > 3) cta_sync();
+        if (M_LONG(I.max_row > 3)) cta_sync();
         PROF_T0(p_seg);
         seg_update(k, D, true);
         cta_sync();
         PROF_ADD(L, P_SEG, p_seg);
     }
     if (threadIdx.x == 0) {
-        if (I.policy != DTS_POLICY_DARTS_LUF) {  // LRU: D(T) used by the n_served-th task
+        if (!M_LUF(I)) {  // LRU: D(T) used by the n_served-th task
             int32_t *lk = V.lru + (size_t)k * I.nstr;
             for (int r = 0; r < L.row_len; r++) lk[L.row[r]] = (int32_t)L.n_served;
         }
@@ -1497,7 +1523,7 @@ __device__ void plan(int k, int32_t Dopt) {
         if (i < e) {
             ed = __ldg(&I.dedge[i]);
             T = ed.x;
-            sel = I.sl ? !allocated(T) && (ed.y < 0 || resident(k, ed.y)) && (ed.z < 0 || resident(k, ed.z))
+            sel = M_SL(I) ? !allocated(T) && (ed.y < 0 || resident(k, ed.y)) && (ed.z < 0 || resident(k, ed.z))
                        : (sk[T] >> 24) == 1u;
         }
         const unsigned msk = __ballot_sync(FULL, sel);
@@ -1511,7 +1537,7 @@ __device__ void plan(int k, int32_t Dopt) {
         }
         if (sel) {
             const int pos = off + __popc(msk & lt);
-            pl[pos] = make_int4(T, Dopt, ed.y, ed.w > 3 ? ROW_LONG : ed.z);
+            pl[pos] = make_int4(T, Dopt, ed.y, M_LONG(ed.w > 3) ? ROW_LONG : ed.z);
             if (pt) pt[pos] = tau_of(T);
         }
         base_out += tot;
@@ -1547,7 +1573,7 @@ __device__ __noinline__ int32_t first_cnt2(int k, int32_t D2) {
         const int64_t i = base + threadIdx.x;
         unsigned long long c = ~0ull;
         if (i < e) {
-            if (I.sl) {  // D2 misses (n2(D2) > 0): exactly one other input misses
+            if (M_SL(I)) {  // D2 misses (n2(D2) > 0): exactly one other input misses
                 const int4 ed = __ldg(&I.dedge[i]);
                 const int mo = (int)(ed.y >= 0 && !resident(k, ed.y)) + (int)(ed.z >= 0 && !resident(k, ed.z));
                 if (!allocated(ed.x) && mo == 1) c = (unsigned long long)ed.x;
@@ -1567,7 +1593,7 @@ __device__ __noinline__ int32_t first_cnt2(int k, int32_t D2) {
 __device__ __noinline__ int32_t first_avail() {
     const Inst &I = SI;
     const View &V = SV;
-    if (I.sl) {  // the allocation bitmap, a word per thread (bits past m are set)
+    if (M_SL(I)) {  // the allocation bitmap, a word per thread (bits past m are set)
         const int lo = L.avail_lo;
         const int nwd = (I.m + 31) >> 5;
         for (int w0 = lo >> 5; w0 < nwd; w0 += blockDim.x) {
@@ -1583,6 +1609,7 @@ __device__ __noinline__ int32_t first_avail() {
         }
         return -1;
     }
+#if !DTS_FAST
     for (int64_t base = L.avail_lo > I.t_lo ? L.avail_lo : I.t_lo; base < I.t_hi; base += blockDim.x) {
         const int64_t T = base + threadIdx.x;
         unsigned long long c = ~0ull;
@@ -1590,6 +1617,7 @@ __device__ __noinline__ int32_t first_avail() {
         c = block_min_u64(c);
         if (c != ~0ull) return (int32_t)c;
     }
+#endif
     return -1;
 }
 
@@ -1802,7 +1830,7 @@ __device__ __noinline__ void plan_shard(int k, int32_t Dopt) {
             if (j < w) off += c;
             tot += c;
         }
-        if (sel) ents[off + __popc(msk & lt)] = make_int4(ed.x, Dopt, ed.y, ed.w > 3 ? ROW_LONG : ed.z);
+        if (sel) ents[off + __popc(msk & lt)] = make_int4(ed.x, Dopt, ed.y, M_LONG(ed.w > 3) ? ROW_LONG : ed.z);
         base_out += tot;
         cta_sync();
     }
@@ -1851,7 +1879,7 @@ __device__ __noinline__ void plan_shard(int k, int32_t Dopt) {
 // candidate, then the minimum.
 __device__ __noinline__ int32_t any_first_avail() {
     int32_t T = first_avail();
-    if (SI.G > 1) {
+    if (M_SHARD(SI)) {
         const unsigned long long r = xch_min(T < 0 ? ~0ull : (unsigned long long)T);
         T = r == ~0ull ? -1 : (int32_t)r;
     }
@@ -1859,7 +1887,7 @@ __device__ __noinline__ int32_t any_first_avail() {
 }
 __device__ __noinline__ int32_t any_first_cnt2(int k, int32_t D2) {
     int32_t T = first_cnt2(k, D2);
-    if (SI.G > 1) {
+    if (M_SHARD(SI)) {
         const unsigned long long r = xch_min(T < 0 ? ~0ull : (unsigned long long)T);
         T = r == ~0ull ? -1 : (int32_t)r;
     }
@@ -1878,7 +1906,7 @@ __device__ __noinline__ void verify_scores(int k) {
     const uint32_t *sk = V.s + (size_t)k * I.m_pad;
     int bad = 0;
     for (int T = I.t_lo + threadIdx.x; T < I.t_hi; T += blockDim.x) {  // owned tasks
-        const uint32_t w = I.sl ? 0u : sk[T];
+        const uint32_t w = M_SL(I) ? 0u : sk[T];
         const int64_t rb = __ldg(&I.tptr[T]), re = __ldg(&I.tptr[T + 1]);
         int c = 0;
         uint32_t x = 0;
@@ -1886,7 +1914,7 @@ __device__ __noinline__ void verify_scores(int k) {
             const int32_t D = __ldg(&I.tdat[i]);
             if (!resident(k, D)) c++, x ^= (uint32_t)D;
         }
-        if (I.sl) {
+        if (M_SL(I)) {
             if (allocated(T)) continue;
         } else {
             bad += (c != (int)((w >> 24) & 0x7fu)) || (x != (w & XOR_MASK));
@@ -2128,10 +2156,10 @@ __device__ __noinline__ void fused_init() {
             I.tstart[T] = -1;
             I.tend[T] = -1;
         }
-        if (!I.sl)
+        if (!M_SL(I))
             for (int k = 0; k < K; k++) V.s[(size_t)k * I.m_pad + T] = w;
     }
-    if (I.sl)  // nothing allocated; bits past m set
+    if (M_SL(I))  // nothing allocated; bits past m set
         for (int wd = threadIdx.x; wd <= I.m_pad / 32; wd += blockDim.x) {
             const int t0 = 32 * wd;
             V.al[wd] = t0 >= m ? ~0u : (m - t0 >= 32 ? 0u : ~((1u << (m - t0)) - 1u));
@@ -2168,7 +2196,7 @@ __device__ __noinline__ void fused_init() {
 
 // One CTA per instance; instances pulled from *work_counter.
 __global__ void __launch_bounds__(512, 1)
-    dts_cta_kernel(const Inst *__restrict__ insts, int n_inst, int *work_counter) {
+    DTS_KNAME(dts_cta_kernel)(const Inst *__restrict__ insts, int n_inst, int *work_counter) {
     extern __shared__ __align__(16) unsigned char dsm[];
     __shared__ int sh_inst;
     const int tid = threadIdx.x;
@@ -2206,7 +2234,7 @@ __global__ void __launch_bounds__(512, 1)
         }
         cta_sync();
         const View &V = SV;
-        if (I.G > 1)
+        if (M_SHARD(I))
             for (int p = tid; p < I.G; p += blockDim.x) SP[p] = I.peers[p];
 
         const int n = I.n, K = I.K;
@@ -2223,7 +2251,7 @@ __global__ void __launch_bounds__(512, 1)
             uint4 *dst = reinterpret_cast<uint4 *>(V.s);
             for (int i = tid; i < (K * I.m_pad) / 4; i += blockDim.x) dst[i] = __ldcg(&src[i]);
         }
-        if (I.sl && I.so_al >= 0)
+        if (M_SL(I) && I.so_al >= 0)
             for (int i = tid; i <= I.m_pad / 32; i += blockDim.x) V.al[i] = __ldcg(&I.al[i]);
         if (I.so_u >= 0)
             for (int D = tid; D < I.nstr; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
@@ -2265,10 +2293,10 @@ __global__ void __launch_bounds__(512, 1)
         // ---- the decision loop
         while (true) {
             PROF_T0(p_pop);
-            if (I.policy == DTS_POLICY_DARTS_LUF) {
+            if (M_LUF(I)) {
                 int pending = 0;  // planned tasks left on all GPUs (uniform: every thread sums)
                 for (int j = 0; j < K; j++) pending += L.plan_live[j];
-                if (I.max_served < 0 && I.W == 0 && K <= 32 && pending > I.pop_batch_min) {
+                if (I.max_served < 0 && M_W(I) == 0 && K <= 32 && pending > I.pop_batch_min) {
                     pop_batch();
                 } else {  // few pops (or a prefix run that stops at an exact count): thread 0
                     cta_sync();
@@ -2294,12 +2322,12 @@ __global__ void __launch_bounds__(512, 1)
                         if (kk >= 0) {
                             L.k = kk;
                             L.t = tb;
-                            if (I.policy == DTS_POLICY_DARTS_LRU && L.plan_live[kk] > 0) {
+                            if (M_POL(I, DTS_POLICY_DARTS_LRU) && L.plan_live[kk] > 0) {
                                 int64_t tau;
                                 L.T = pop_planned(kk, &tau);
                                 cmd = CMD_POP;
                             } else {
-                                cmd = I.policy == DTS_POLICY_EAGER_LRU ? CMD_EAGER : CMD_SCAN;
+                                cmd = M_POL(I, DTS_POLICY_EAGER_LRU) ? CMD_EAGER : CMD_SCAN;
                             }
                         }
                     }
@@ -2341,7 +2369,7 @@ __global__ void __launch_bounds__(512, 1)
             // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
             PROF_T0(p_am);
             int32_t D2s = -1;  // task shards: the 3inputs argmax comes with the main one
-            const int32_t Dopt = I.G > 1 ? shard_scan(k, (I.flags & DTS_F_FALLBACK2) != 0,
+            const int32_t Dopt = M_SHARD(I) ? shard_scan(k, (I.flags & DTS_F_FALLBACK2) != 0,
                                                       (I.flags & DTS_F_OPTI) != 0, &D2s)
                                  : (I.flags & DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
                                                           : score_argmax(V.h + (size_t)k * I.nstr);
@@ -2352,11 +2380,11 @@ __global__ void __launch_bounds__(512, 1)
                 L.alg_bytes += 8ull * (uint64_t)n;
                 L.scan_avail = L.n_avail;  // before this scan allocates anything
             }
-            if (I.G > 1 && L.xerr) break;  // a peer timed out in the scan exchange (CTA-uniform)
+            if (M_SHARD(I) && L.xerr) break;  // a peer timed out in the scan exchange (CTA-uniform)
             if (Dopt >= 0) {
-                if (I.G > 1) plan_shard(k, Dopt);
+                if (M_SHARD(I)) plan_shard(k, Dopt);
                 else plan(k, Dopt);
-                if (I.G > 1 && L.xerr) break;  // plan exchange failed: no plan to pop from
+                if (M_SHARD(I) && L.xerr) break;  // plan exchange failed: no plan to pop from
                 if (tid == 0) {
                     int64_t tau;
                     L.T = pop_planned(k, &tau);
@@ -2369,7 +2397,7 @@ __global__ void __launch_bounds__(512, 1)
                 PROF_ADD(L, P_PLAN, p_pl);
             } else {
                 if (I.flags & DTS_F_FALLBACK2) {
-                    const int32_t D2 = I.G > 1 ? D2s : score_argmax(V.h2 + (size_t)k * I.nstr);
+                    const int32_t D2 = M_SHARD(I) ? D2s : score_argmax(V.h2 + (size_t)k * I.nstr);
                     if (tid == 0) {
                         L.scan_alg_bytes += 8ull * (uint64_t)n;
                         L.alg_bytes += 8ull * (uint64_t)n;
@@ -2403,7 +2431,7 @@ __global__ void __launch_bounds__(512, 1)
                 }
                 cta_sync();
                 PROF_ADD(L, P_OTHER, p_pl);
-                if (I.G > 1 && L.xerr) break;  // a min-exchange failed: T is not trustworthy
+                if (M_SHARD(I) && L.xerr) break;  // a min-exchange failed: T is not trustworthy
                 if (T < 0) continue;
             }
             }  // scan
@@ -2422,7 +2450,7 @@ __global__ void __launch_bounds__(512, 1)
             if (L.error || L.xerr) break;
         }
         cta_sync();
-        if (I.G > 1) {  // no shard leaves while a peer may still read its slots
+        if (M_SHARD(I)) {  // no shard leaves while a peer may still read its slots
             xch_sync();
             if (tid == 0 && L.xerr && !L.error) L.error = 2;
             cta_sync();
@@ -2457,6 +2485,7 @@ __global__ void __launch_bounds__(512, 1)
     }
 }
 
+#if !DTS_FAST
 // ---------------------------------------------------------------- init (a2)
 // Global homes: s_k(T) = (|D(T)| << 24) | XOR D(T) for every k (nothing
 // resident), pad words allocated; u(D) = deg(D); h_k(D) / h2_k(D) = the tasks
@@ -2479,10 +2508,10 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
                 I.tstart[T] = -1;
                 I.tend[T] = -1;
             }
-            if (!I.sl)
+            if (!M_SL(I))
                 for (int k = 0; k < I.K; k++) I.s[(size_t)k * I.m_pad + T] = w;
         }
-        if (I.sl)  // allocation bitmap: nothing allocated, bits past m set
+        if (M_SL(I))  // allocation bitmap: nothing allocated, bits past m set
             for (int64_t wd = tid; wd <= I.m_pad / 32; wd += str) {
                 const int64_t t0 = 32 * wd;
                 I.al[wd] = t0 >= I.m ? ~0u : (I.m - t0 >= 32 ? 0u : ~((1u << (I.m - t0)) - 1u));
@@ -2517,7 +2546,10 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
     }
 }
 
+#endif  // !DTS_FAST
+
 // ---------------------------------------------------------------- launchers
+#if !DTS_FAST
 cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t work, cudaStream_t st) {
     int64_t blocks = (work + 255) / 256;
     if (blocks < 1) blocks = 1;
@@ -2526,6 +2558,7 @@ cudaError_t launch_init(const Inst *d_insts, int n_inst, uint64_t bw, int64_t wo
     count_launch();
     return cudaGetLastError();
 }
+#endif
 
 // cudaFuncSetAttribute is a driver call worth avoiding per launch: raise the
 // kernel's dynamic shared-memory limit only when a launch needs more.
@@ -2540,20 +2573,22 @@ static cudaError_t ensure_smem_attr(int smem_bytes) {
     cudaGetDevice(&dev);
     if (dev < 0 || dev >= 64) dev = 0;
     if (smem_bytes <= cur[dev]) return cudaSuccess;
-    cudaError_t e = cudaFuncSetAttribute(dts_cta_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+    cudaError_t e =
+        cudaFuncSetAttribute(DTS_KNAME(dts_cta_kernel), cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
     if (e == cudaSuccess) cur[dev] = smem_bytes;
     return e;
 }
 
-cudaError_t launch_loop(const Inst *d_insts, int n_inst, int block, int grid, int *work_counter,
-                        int smem_bytes, cudaStream_t st) {
+cudaError_t DTS_KNAME(launch_loop)(const Inst *d_insts, int n_inst, int block, int grid, int *work_counter,
+                                   int smem_bytes, cudaStream_t st) {
     cudaError_t e = ensure_smem_attr(smem_bytes);
     if (e != cudaSuccess) return e;
-    dts_cta_kernel<<<grid, block, smem_bytes, st>>>(d_insts, n_inst, work_counter);
+    DTS_KNAME(dts_cta_kernel)<<<grid, block, smem_bytes, st>>>(d_insts, n_inst, work_counter);
     count_launch();
     return cudaGetLastError();
 }
 
+#if !DTS_FAST
 cudaError_t launch_loop_coop(const Inst *d_insts, int n_inst, int block, int *work_counter, int smem_bytes,
                              cudaStream_t st) {
     cudaError_t e = ensure_smem_attr(smem_bytes);
@@ -2564,18 +2599,20 @@ cudaError_t launch_loop_coop(const Inst *d_insts, int n_inst, int block, int *wo
     count_launch();
     return e;
 }
+#endif
 
-int loop_max_blocks_per_sm(int block, int smem_bytes) {
+int DTS_KNAME(loop_max_blocks_per_sm)(int block, int smem_bytes) {
     int nb = 0;
     if (ensure_smem_attr(smem_bytes) != cudaSuccess) return 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, dts_cta_kernel, block, smem_bytes) != cudaSuccess)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, DTS_KNAME(dts_cta_kernel), block, smem_bytes) !=
+        cudaSuccess)
         return 0;
     return nb;
 }
 
-int loop_static_smem() {
+int DTS_KNAME(loop_static_smem)() {
     cudaFuncAttributes a;
-    if (cudaFuncGetAttributes(&a, dts_cta_kernel) != cudaSuccess) return -1;
+    if (cudaFuncGetAttributes(&a, DTS_KNAME(dts_cta_kernel)) != cudaSuccess) return -1;
     return (int)a.sharedSizeBytes;
 }
 

@@ -17,4 +17,10 @@ cudaError_t launch_loop_coop(const Inst *d_insts, int n_inst, int block, int *wo
                              cudaStream_t st);
 int loop_max_blocks_per_sm(int block, int smem_bytes);
 int loop_static_smem();
+// The same loop specialised at compile time (dts_loop_fast.cu) to row-derived
+// state, one shard, W = 0 and DARTS+LUF (Inst::sl, G = 1, W = 0, policy LUF).
+cudaError_t launch_loop_fast(const Inst *d_insts, int n_inst, int block, int grid, int *work_counter,
+                             int smem_bytes, cudaStream_t st);
+int loop_max_blocks_per_sm_fast(int block, int smem_bytes);
+int loop_static_smem_fast();
 }  // namespace dts

@@ -38,6 +38,7 @@ DTS_F_VERIFY = 2
 DTS_F_NOFUSE = 4
 DTS_F_OPTI = 8
 DTS_F_PACKED = 16
+DTS_F_GENERIC = 32
 
 EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data", "<i4"),
                         ("task", "<i4"), ("op", "u1"), ("pad", "u1", (3,))])

@@ -714,3 +714,27 @@ def test_large_n_w1_and_belady():
     inst = _tight(_large_n_shapes()[1], 1)
     g, o = dts.schedule(inst, W=1), oracle.run(inst, W=1)
     assert_parity(g, o)
+
+
+# ------------------------------- the generic loop vs the specialised one
+@pytest.mark.parametrize("idx", range(12))
+def test_generic_loop_on_shapes(idx):
+    """DTS_F_GENERIC forces the run-time-moded loop where the compile-time
+    specialised one (row-derived, one shard, W = 0, DARTS+LUF) would run; both
+    must give the oracle's schedule."""
+    inst = _shapes()[idx]
+    for fl in (dts.DTS_F_FALLBACK2 | dts.DTS_F_GENERIC, dts.DTS_F_FALLBACK2):
+        g = dts.schedule(inst, flags=fl)
+        assert_parity(g, oracle.run(inst))
+
+
+def test_generic_loop_batch_and_config4_prefix():
+    insts = gen.config_instances("C2")[::4] + [gen.sweep_instance(N, M, K) for (N, M, K) in
+                                               [(60, 5, 3), (35, 12, 8), (100, 6, 1)]]
+    gs = dts.schedule_batch(insts, flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_GENERIC)
+    for inst, g in zip(insts, gs):
+        assert_parity(g, oracle.run(inst))
+    for cfg in ("C4a", "C4b"):
+        inst = gen.config_instances(cfg)[0]
+        g = dts.schedule(inst, flags=dts.DTS_F_FALLBACK2 | dts.DTS_F_GENERIC, max_served=1500)
+        assert_parity(g, oracle.run(inst, max_served=1500), complete=False)
