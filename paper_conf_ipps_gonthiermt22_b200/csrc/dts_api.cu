@@ -662,10 +662,11 @@ double instance_cost(const dts_instance *I) {
 }
 
 // The compile-time specialised loop (dts_loop_fast.cu) applies: row-derived
-// state, one shard, W = 0, DARTS+LUF, no self-check, not forced generic.
+// state, one shard, W = 0, DARTS+LUF, 32-bit argmax keys, uniform data sizes,
+// no OPTI, no self-check, not forced generic.
 bool fast_mode(const dts::Inst &h) {
-    return h.sl && h.G == 1 && h.W == 0 && h.policy == DTS_POLICY_DARTS_LUF &&
-           !(h.flags & (DTS_F_VERIFY | DTS_F_GENERIC));
+    return h.sl && h.G == 1 && h.W == 0 && h.policy == DTS_POLICY_DARTS_LUF && h.key32 && h.size0 &&
+           !(h.flags & (DTS_F_VERIFY | DTS_F_OPTI | DTS_F_GENERIC));
 }
 
 // Shared-memory placement of one instance's state:

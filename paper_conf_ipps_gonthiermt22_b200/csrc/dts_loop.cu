@@ -38,8 +38,9 @@
 // mode, chosen at run time from the descriptor) and, from dts_loop_fast.cu
 // with DTS_FAST = 1, specialised at compile time to the mode every BASELINE
 // config runs in -- row-derived state (rows of <= 3 inputs), one shard, W = 0,
-// DARTS+LUF -- so the other modes' code is compiled out of the hot loop (the
-// loop is instruction-cache bound: DESIGN.md §6).
+// DARTS+LUF, 32-bit argmax keys, uniform data sizes, no OPTI / VERIFY -- so the
+// other modes' code is compiled out of the hot loop (it is instruction-cache
+// bound: DESIGN.md §6).
 #ifndef DTS_FAST
 #define DTS_FAST 0
 #endif
@@ -49,6 +50,8 @@
 #define M_LUF(I) (DTS_FAST || (I).policy == DTS_POLICY_DARTS_LUF)
 #define M_POL(I, p) (!DTS_FAST && (I).policy == (p))            // an LRU policy
 #define M_LONG(c) (!DTS_FAST && (c))                           // rows of > 3 inputs
+#define M_KEY32(I) (DTS_FAST || (I).key32)                     // scores and u(D) < 2^15
+#define M_FLAG(I, f) (!DTS_FAST && ((I).flags & (f)))          // OPTI, VERIFY: generic only
 #if DTS_FAST
 #define DTS_KNAME(x) x##_fast
 #else
@@ -266,11 +269,11 @@ __device__ __forceinline__ void seg_of(int32_t D, int64_t &b, int64_t &e) {
 // Size and bus time of D: scalars when all sizes are equal (the paper's model).
 __device__ __forceinline__ uint64_t size_of(int32_t D) {
     const Inst &I = SI;
-    return I.size0 ? I.size0 : __ldg(&I.size[D]);
+    return (DTS_FAST || I.size0) ? I.size0 : __ldg(&I.size[D]);
 }
 __device__ __forceinline__ int64_t delta_of(int32_t D) {
     const Inst &I = SI;
-    return I.size0 ? I.delta0 : __ldg(&I.delta[D]);
+    return (DTS_FAST || I.size0) ? I.delta0 : __ldg(&I.delta[D]);
 }
 
 __device__ __forceinline__ int64_t tau_of(int32_t T) {
@@ -1443,7 +1446,7 @@ __device__ int32_t score_argmax(const int32_t *score) {
     const unsigned ib = (unsigned)I.id_bits;
     const unsigned long long idmask = (1ull << ib) - 1ull;
     unsigned long long best = 0ull;
-    if (I.key32) {
+    if (M_KEY32(I)) {
         const int4 *h4 = reinterpret_cast<const int4 *>(score);
         const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
         const int nv = I.nstr >> 2;
@@ -2365,13 +2368,13 @@ __global__ void __launch_bounds__(512, 1)
                 cta_sync();
             } else {
             reset_plan(k);
-            if (I.flags & DTS_F_VERIFY) verify_scores(k);
+            if (M_FLAG(I, DTS_F_VERIFY)) verify_scores(k);
             // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
             PROF_T0(p_am);
             int32_t D2s = -1;  // task shards: the 3inputs argmax comes with the main one
             const int32_t Dopt = M_SHARD(I) ? shard_scan(k, (I.flags & DTS_F_FALLBACK2) != 0,
-                                                      (I.flags & DTS_F_OPTI) != 0, &D2s)
-                                 : (I.flags & DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
+                                                      M_FLAG(I, DTS_F_OPTI) != 0, &D2s)
+                                 : M_FLAG(I, DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
                                                           : score_argmax(V.h + (size_t)k * I.nstr);
             PROF_ADD(L, P_ARGMAX, p_am);
             PROF_T0(p_pl);
