@@ -90,7 +90,12 @@ enum {
     /* Diagnostic: run the generic decision loop even when the one compiled for
      * the default mode applies (row-derived state, one shard, W = 0,
      * DARTS+LUF: every BASELINE config). */
-    DTS_F_GENERIC = 1u << 5
+    DTS_F_GENERIC = 1u << 5,
+    /* Diagnostic: run a small instance on a CTA of the decision loop even
+     * where the one-warp-per-instance loop applies (the default for instances
+     * of <= 2 inputs per task in the mode above whose state fits a warp's
+     * share of shared memory: C1, C2, the C5 sweep). */
+    DTS_F_CTA = 1u << 6
 };
 
 typedef struct {

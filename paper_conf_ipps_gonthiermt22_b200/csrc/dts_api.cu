@@ -621,7 +621,7 @@ dts_status check_opts(const dts_instance *I, dts_policy policy, const dts_run_op
     if (policy != DTS_POLICY_DARTS_LUF && policy != DTS_POLICY_DARTS_LRU && policy != DTS_POLICY_EAGER_LRU)
         return fail(DTS_E_UNSUPPORTED, "policy");
     if (o->flags & ~(uint32_t)(DTS_F_FALLBACK2 | DTS_F_VERIFY | DTS_F_NOFUSE | DTS_F_OPTI | DTS_F_PACKED |
-                               DTS_F_GENERIC))
+                               DTS_F_GENERIC | DTS_F_CTA))
         return fail(DTS_E_UNSUPPORTED, "unknown flags");
     if (o->lookahead_W > (uint32_t)dts::MAX_W) return fail(DTS_E_UNSUPPORTED, "lookahead_W > 8");
     if ((int64_t)o->lookahead_W * I->max_row_len > dts::MAX_ROW + 1)
@@ -668,6 +668,36 @@ bool fast_mode(const dts::Inst &h) {
     return h.sl && h.G == 1 && h.W == 0 && h.policy == DTS_POLICY_DARTS_LUF && h.key32 && h.size0 &&
            !(h.flags & (DTS_F_VERIFY | DTS_F_OPTI | DTS_F_GENERIC));
 }
+
+// The one-warp-per-instance loop (dts_warp.cu) applies: the fast mode's
+// conditions, <= 2 inputs per task, 16-bit task and data ids in the edge
+// words, K <= 32 (a lane per simulated GPU), 16-bit scores, automatic launch
+// shape and placement, and a state slice that fits in shared memory.
+int64_t warp_slot_bytes(const dts_instance *I) {
+    return dts::warp_layout(I->m, I->n, I->K, I->max_deg_ub + 1, I->res_cap + 1).total;
+}
+int max_dyn_smem_warp(int device) {
+    int optin = 0;
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
+    return std::max(0, optin - 1024);
+}
+bool warp_eligible(const dts_instance *I, dts_policy policy, const dts_run_opts &o) {
+    if (policy != DTS_POLICY_DARTS_LUF || o.lookahead_W != 0 || o.block_threads != 0 || o.smem_budget < 0 ||
+        (o.flags & (DTS_F_VERIFY | DTS_F_OPTI | DTS_F_GENERIC | DTS_F_CTA | DTS_F_PACKED | DTS_F_NOFUSE)) ||
+        I->G != 1)
+        return false;
+    if (I->max_row_len > 2 || I->m > 65535 || I->n > 65534 || I->K > 32 || !I->uniform_size ||
+        I->max_deg_ub >= 32768)
+        return false;
+    const int64_t slot = warp_slot_bytes(I);
+    const int64_t lim = o.smem_budget > 0 ? std::min<int64_t>(o.smem_budget, max_dyn_smem_warp(o.device))
+                                          : max_dyn_smem_warp(o.device);
+    return slot <= lim;
+}
+// A lone instance runs on one warp only while its per-decision scans are
+// short (n data, the widest segment): a wider instance wants a whole CTA.
+constexpr int WARP_SOLO_MAX = 2048;
+bool warp_solo(const dts_instance *I) { return I->n <= WARP_SOLO_MAX && I->max_deg_ub <= WARP_SOLO_MAX; }
 
 // Shared-memory placement of one instance's state:
 // greedy, most latency-critical array first, each either fully in the CTA's
@@ -738,7 +768,7 @@ int auto_block(const dts_instance *I, bool alone = false) {
 int fused_scratch_bytes(const dts_instance *I, int block) { return (2 * (block / 32) + 1) * 4 * (I->n + 1); }
 
 dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int budget, int block,
-                 cudaStream_t st, bool copy_desc = true, bool own_events = true) {
+                 cudaStream_t st, bool copy_desc = true, bool own_events = true, bool warp = false) {
     dts_status s = ensure_device(I, o.device);
     if (s != DTS_OK) return s;
     int cur = -1;
@@ -787,6 +817,10 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     h.fused = I->G == 1 && !(o.flags & DTS_F_NOFUSE) && I->max_row_len <= 8 && fs <= max_dyn_smem(o.device) ? 1 : 0;
     if (h.fused) h.smem_bytes = std::max(h.smem_bytes, fs);
     h.smem_bytes = std::max(h.smem_bytes, dts::ASSEMBLE_SMEM_BYTES);  // result assembly's scratch
+    if (warp) {  // dts_warp.cu: the warp builds its CSR and state in its own slice
+        h.fused = 1;
+        h.smem_bytes = (int32_t)warp_slot_bytes(I);
+    }
     if (own_events) {
         I->sev.reset();
         CK(cudaEventRecord(I->ev[0], st), "event");
@@ -890,6 +924,9 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     // first by the launch's counter, overlap the rest (C5: 232 ms against 280
     // for round 1's two concurrent launches of 256- and 128-thread CTAs,
     // profiles/r02s_c5_block.txt).  A forced size applies to all.
+    bool warp = true;  // every instance on one warp (dts_warp.cu)
+    for (int32_t i = 0; i < n && warp; i++) warp = warp_eligible(insts[i], policy, o);
+    if (n == 1) warp = warp && warp_solo(insts[0]);
     const int forced = o.block_threads;
     const int small_max = tuning("DTS_SWEEP_SMALL_BLOCK", 128);
     int block = 32;
@@ -908,7 +945,7 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     CK(cudaEventRecord(sev->begin, st), "event");
     for (int32_t i = 0; i < n; i++) {
         dts_instance *I = insts[ord[(size_t)i]];
-        dts_status s = stage(I, policy, o, budget, block, st, false, false);
+        dts_status s = stage(I, policy, o, budget, block, st, false, false, warp);
         if (s != DTS_OK) return s;
         smem = std::max(smem, I->h_inst.smem_bytes);
         any_unfused |= !I->h_inst.fused;
@@ -926,11 +963,17 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     CK(cudaEventRecord(sev->loop_begin, st), "event");
     bool fast = true;
     for (int32_t i = 0; i < n; i++) fast &= fast_mode(insts[i]->h_inst);
-    const int per = std::max(1, fast ? dts::loop_max_blocks_per_sm_fast(block, smem)
-                                     : dts::loop_max_blocks_per_sm(block, smem));
-    const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
-    if (fast) CK(dts::launch_loop_fast(S->d_insts, n, block, grid, S->d_work, smem, st), "loop");
-    else CK(dts::launch_loop(S->d_insts, n, block, grid, S->d_work, smem, st), "loop");
+    if (warp) {
+        const int per = std::max(1, dts::warp_max_blocks_per_sm(smem));
+        const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
+        CK(dts::launch_warp(S->d_insts, n, grid, S->d_work, smem, st), "loop (warp)");
+    } else {
+        const int per = std::max(1, fast ? dts::loop_max_blocks_per_sm_fast(block, smem)
+                                         : dts::loop_max_blocks_per_sm(block, smem));
+        const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
+        if (fast) CK(dts::launch_loop_fast(S->d_insts, n, block, grid, S->d_work, smem, st), "loop");
+        else CK(dts::launch_loop(S->d_insts, n, block, grid, S->d_work, smem, st), "loop");
+    }
     CK(cudaEventRecord(sev->loop_end, st), "event");
     CK(cudaEventRecord(S->done, st), "event");
     for (int32_t i = 0; i < n; i++) {
@@ -998,13 +1041,16 @@ static dts_status run_one(dts_instance *I, dts_policy policy, const dts_run_opts
     cudaStream_t st = (cudaStream_t)o.cuda_stream;
     const int budget = budget_of(o);
     const int block = o.block_threads ? o.block_threads : auto_block(I, true);
-    s = stage(I, policy, o, budget, block, st);
+    const bool warp = warp_eligible(I, policy, o) && warp_solo(I);
+    s = stage(I, policy, o, budget, block, st, true, true, warp);
     if (s != DTS_OK) return s;
     const int64_t work = std::max<int64_t>((int64_t)I->m_pad, (int64_t)I->n + 4);
     if (!I->h_inst.fused) CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
     CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
     CK(cudaEventRecord(I->ev[1], st), "event");
-    if (fast_mode(I->h_inst))
+    if (warp)
+        CK(dts::launch_warp(I->d_inst, 1, 1, I->d_work, I->h_inst.smem_bytes, st), "loop (warp)");
+    else if (fast_mode(I->h_inst))
         CK(dts::launch_loop_fast(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");
     else
         CK(dts::launch_loop(I->d_inst, 1, block, 1, I->d_work, I->h_inst.smem_bytes, st), "loop");

@@ -39,6 +39,7 @@ DTS_F_NOFUSE = 4
 DTS_F_OPTI = 8
 DTS_F_PACKED = 16
 DTS_F_GENERIC = 32
+DTS_F_CTA = 64  # force the per-CTA loop where the one-warp loop applies (diagnostic)
 
 EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data", "<i4"),
                         ("task", "<i4"), ("op", "u1"), ("pad", "u1", (3,))])
