@@ -455,12 +455,17 @@ def main():
                        "sample": f"{nb} passes over {len(sub)} instances of {args.workload}"
                                  f" ({nd} decisions, {dt:.1f} s, one instance per thread)"}
         clocks = clk.summary()
-        launch = ("one batched loop launch, one CTA per instance" if len(insts) < 296 else
+        kind = max(r.loop_kind for r in rs)
+        kname = {1: "dts_cta_kernel", 2: "dts_cta_kernel_fast", 3: "dts_warp_kernel"}.get(kind, "?")
+        launch = ("one batched loop launch, one WARP per instance (32-thread CTAs, instances pulled "
+                  "longest first)" if kind == 3 else
+                  "one batched loop launch, one CTA per instance" if len(insts) < 296 else
                   "one batched loop launch of 128-thread CTAs (4 per SM), one CTA per instance, "
                   "longest first") if not single \
             else (f"one cooperative launch: the instance task-sharded over {args.shards} CTAs"
                   if gsh else f"one loop launch per rank: the instance task-sharded over "
                   f"{world} B200s, peer-memory exchanges" if xsh
+                  else "one loop launch (one warp) per instance" if kind == 3
                   else "one loop launch (one CTA) per instance")
         line = {
             "metric": METRIC, "value": all_dec / (ms / 1e3), "unit": UNIT, "n_gpus": world,
@@ -480,7 +485,7 @@ def main():
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": _traffic(args.workload),
-                         "kernel": "dts_cta_kernel", "peak_source": peak_src,
+                         "kernel": kname, "peak_source": peak_src,
                          "bytes": "SURVEY.md §8(d) algorithmic bytes per launch: 4*sum(m_avail at scans)"
                                   " + 4.125*n*scans + 12*sum(deg over loads/evictions)"
                                   " + (4K + 8E/m)*allocations (kernel counters = oracle counters)",

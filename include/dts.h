@@ -215,6 +215,10 @@ typedef struct {
     int64_t sum_avail_at_scans;      /* sum over scans of #unallocated tasks when the scan began */
     int64_t n_allocations;           /* tasks leaving the shared pool (plans, fallback / EAGER picks) */
     int64_t sum_deg_loads_evictions; /* sum of deg(D) over every LOAD and EVICT event            */
+    int32_t loop_kind;               /* which decision loop ran: 1 = the generic
+                                        per-CTA loop, 2 = the per-CTA loop specialised to the
+                                        default mode, 3 = the one-warp-per-instance loop */
+    int32_t reserved;
 } dts_result_view;
 
 /* Synchronise on the run's stream, copy the results to host (once) and fill *out. */

@@ -207,6 +207,7 @@ struct dts_instance {
     // run state / results
     bool ran = false;
     bool have_host = false;
+    int32_t loop_kind = 0;  // dts_result_view.loop_kind of the last run
     dts::Out out{};
     // pinned host memory (allocated with the device arena): a mirror of the
     // inputs for the H2D upload and the result buffers for the D2H read-back
@@ -309,7 +310,7 @@ const char *dts_status_str(dts_status s) {
 
 const char *dts_last_error(void) { return g_err.c_str(); }
 
-uint32_t dts_version(void) { return (1u << 16) | 2u; }
+uint32_t dts_version(void) { return (1u << 16) | 3u; }
 
 dts_status dts_instance_create(int32_t n_tasks, int32_t n_data, const int64_t *task_ptr,
                                const int32_t *task_data, const uint64_t *data_size,
@@ -979,6 +980,7 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     for (int32_t i = 0; i < n; i++) {
         insts[i]->sev = sev;
         insts[i]->ran = true;
+        insts[i]->loop_kind = warp ? 3 : (fast ? 2 : 1);
     }
     return DTS_OK;
 }
@@ -1048,6 +1050,7 @@ static dts_status run_one(dts_instance *I, dts_policy policy, const dts_run_opts
     if (!I->h_inst.fused) CK(dts::launch_init(I->d_inst, 1, o.bus_bytes_per_s, work, st), "init");
     CK(cudaMemsetAsync(I->d_work, 0, sizeof(int) * 16, st), "memset");
     CK(cudaEventRecord(I->ev[1], st), "event");
+    I->loop_kind = warp ? 3 : (fast_mode(I->h_inst) ? 2 : 1);
     if (warp)
         CK(dts::launch_warp(I->d_inst, 1, 1, I->d_work, I->h_inst.smem_bytes, st), "loop (warp)");
     else if (fast_mode(I->h_inst))
@@ -1348,6 +1351,7 @@ dts_status dts_shard_group_run(dts_instance *const *shards, int32_t G, dts_polic
         CK(cudaEventRecord(shards[i]->ev[2], st), "event");
         CK(cudaEventRecord(shards[i]->ev[3], st), "event");
         shards[i]->ran = true;
+        shards[i]->loop_kind = 1;  // task shards: the generic loop
     }
     return DTS_OK;
 }
@@ -1564,6 +1568,8 @@ dts_status dts_result(dts_instance *I, dts_result_view *v) {
     v->sum_avail_at_scans = I->out.sum_avail;
     v->n_allocations = I->out.n_alloc;
     v->sum_deg_loads_evictions = I->out.sum_deg;
+    v->loop_kind = I->loop_kind;
+    v->reserved = 0;
     v->loop_ms = I->loop_ms;
     v->total_ms = I->total_ms;
     return DTS_OK;

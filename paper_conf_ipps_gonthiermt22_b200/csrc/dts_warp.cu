@@ -81,7 +81,10 @@ __device__ __forceinline__ void add16(uint16_t *a, int i, int d) {
     atomicAdd(reinterpret_cast<unsigned *>(a) + (i >> 1), (unsigned)d << (16 * (i & 1)));
 }
 
-constexpr int SEGR = 8;  // edges per lane of one segment batch in registers (256 per batch)
+#ifndef DTS_SEGR
+#define DTS_SEGR 5
+#endif
+constexpr int SEGR = DTS_SEGR;  // edges per lane of one segment batch in registers (32 SEGR per batch)
 
 // The warp's view of one instance (registers; pointers into its smem slice).
 struct WV {
@@ -202,8 +205,8 @@ __device__ __forceinline__ void seg_load(const WV &v, int b, int e, int lane, ui
 // allocation and residency words of all the batch's tasks are gathered
 // before any update.  n1 / n2: the batch's tasks that leave / enter n_k(D)
 // and n2_k(D) (applied once by the caller).
-__device__ __forceinline__ void seg_apply(const WV &v, int k, bool load, const uint32_t (&ed)[SEGR], int &n1,
-                                          int &n2) {
+__device__ __forceinline__ void seg_apply(const WV &v, int k, bool load, const uint32_t (&ed)[SEGR], int nr,
+                                          int &n1, int &n2) {
     uint32_t aw[SEGR], rw[SEGR];
 #pragma unroll
     for (int r = 0; r < SEGR; r++) {
@@ -213,17 +216,16 @@ __device__ __forceinline__ void seg_apply(const WV &v, int k, bool load, const u
         rw[r] = (w != REMOVED && o != (int)NOI) ? v.resm[o] : ~0u;
     }
     uint32_t *hk = v.hh + k * v.n4;
+    const unsigned dd = load ? (1u - 65536u) : (65536u - 1u);
 #pragma unroll
     for (int r = 0; r < SEGR; r++) {
         const uint32_t w = ed[r];
         const int T = (int)(w >> 16), o = (int)(w & 0xFFFFu);
-        if (w == REMOVED || ((aw[r] >> (T & 31)) & 1u)) continue;
-        if ((rw[r] >> k) & 1u) {
-            n1++;  // load: 1 -> 0 (n_k(D) - 1); evict: 0 -> 1 (n_k(D) + 1)
-        } else {
-            n2++;  // load: 2 -> 1, freed by o now; evict: 1 -> 2, {o, D} missing
-            atomicAdd(&hk[o], load ? (1u - 65536u) : (65536u - 1u));
-        }
+        const bool live = w != REMOVED && !((aw[r] >> (T & 31)) & 1u);
+        const bool mo = live && !((rw[r] >> k) & 1u);
+        n1 += (int)(live && !mo);  // load: 1 -> 0 (n_k(D) - 1); evict: 0 -> 1 (n_k(D) + 1)
+        n2 += (int)mo;             // load: 2 -> 1, freed by o now; evict: 1 -> 2, {o, D} missing
+        if (mo) atomicAdd(&hk[o], dd);
     }
 }
 
@@ -232,11 +234,11 @@ __device__ __forceinline__ void seg_update(const WV &v, int k, int D, bool load,
                                            const uint32_t (&ed0)[SEGR]) {
     const int b = v.dp[D], e = v.dp[D + 1];
     int n1 = 0, n2 = 0;
-    seg_apply(v, k, load, ed0, n1, n2);
+    seg_apply(v, k, load, ed0, min(SEGR, (e - b + 31) >> 5), n1, n2);
     for (int base = b + 32 * SEGR; base < e; base += 32 * SEGR) {
         uint32_t ed[SEGR];
         seg_load(v, base, e, lane, ed);
-        seg_apply(v, k, load, ed, n1, n2);
+        seg_apply(v, k, load, ed, min(SEGR, (e - base + 31) >> 5), n1, n2);
     }
     n1 = wsum(n1);
     n2 = wsum(n2);
@@ -267,45 +269,15 @@ __device__ __forceinline__ int64_t tau_of(const int64_t *taup, int T, int64_t dt
     return taup ? taup[T] : dtau;
 }
 
-// One instance, the whole warp.
-__device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigned char *dsm, int lane) {
+// a1 + a2 at instance start (cold: out of line, the hot loop stays small):
+// the data->task CSR as 32-bit edge words by a stable counting sort, the
+// initial scores (nothing resident: n_k(D) / n2_k(D) = D's tasks with one /
+// two inputs), u(D) = deg(D), empty bitmaps, task times -1.
+__device__ __noinline__ void build_state(const WV v, const WarpLayout Lw, unsigned char *dsm, const int64_t *rp,
+                                         const int32_t *rd, uint32_t *wedge, int64_t *tst, int64_t *ten, int lane) {
     const unsigned lt = (1u << lane) - 1u;
-    WV v;
-    v.m = I->m;
-    v.n = I->n;
-    v.K = I->K;
-    v.pcap = I->plan_cap;
-    v.rcap = I->res_cap;
-    v.kmask = v.K >= 32 ? 0xffffffffu : ((1u << v.K) - 1u);
-    const WarpLayout Lw = warp_layout(v.m, v.n, v.K, v.pcap, v.rcap);
-    v.n4 = Lw.n4;
-    v.n8 = Lw.n8;
-    v.resm = reinterpret_cast<uint32_t *>(dsm + Lw.resm);
-    v.al = reinterpret_cast<uint32_t *>(dsm + Lw.al);
-    v.dp = reinterpret_cast<int32_t *>(dsm + Lw.dp);
-    v.u = reinterpret_cast<uint16_t *>(dsm + Lw.u);
-    v.hh = reinterpret_cast<uint32_t *>(dsm + Lw.hh);
-    v.np = reinterpret_cast<uint16_t *>(dsm + Lw.np);
-    v.plan = reinterpret_cast<uint32_t *>(dsm + Lw.plan);
-    v.rl = reinterpret_cast<int32_t *>(dsm + Lw.rl);
-    uint32_t *const wedge = reinterpret_cast<uint32_t *>(const_cast<int32_t *>(I->ddat));
-    v.wedge = wedge;
-    const uint64_t size0 = I->size0, cap = I->cap;
-    v.maxres = size0 == 0 ? INT_MAX : (int)(cap / size0 < (uint64_t)INT_MAX ? cap / size0 : (uint64_t)INT_MAX);
     const int m = v.m, n = v.n, K = v.K;
-    const int64_t dtau = I->default_tau, delta0 = I->delta0, maxs = I->max_served;
-    const bool fb2 = (I->flags & DTS_F_FALLBACK2) != 0;
-    // pointers in registers (the descriptor is in global memory)
-    int64_t *const tst = I->tstart, *const ten = I->tend;
-    int32_t *const sg = I->serve_gpu, *const stk = I->serve_task;
-    dts_event *const evs = I->events;
-    const int64_t evcap = I->ev_cap;
-    const int64_t *const taup = I->tau;
-    const int64_t *const rp = I->raw_ptr;
-    const int32_t *const rd = I->raw_dat;
-
-    WP_DECL;
-    // ---- a1: data->task CSR (stable counting sort by warp) + initial scores
+    // a1: data->task CSR (stable counting sort by warp) + initial scores
     {
         uint32_t *mask = reinterpret_cast<uint32_t *>(dsm + Lw.np);  // build scratch [n] + [n]
         int32_t *cur = reinterpret_cast<int32_t *>(mask + n);
@@ -368,7 +340,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
         __threadfence_block();
         __syncwarp();
     }
-    // ---- a2: initial state
+    // a2: initial state
     for (int i = lane; i <= m / 32; i += 32) {
         const int t0 = 32 * i;
         v.al[i] = t0 >= m ? ~0u : (m - t0 >= 32 ? 0u : ~((1u << (m - t0)) - 1u));
@@ -383,13 +355,146 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
     }
     __syncwarp();
 
+}
+
+// No datum frees a task on GPU k (cold: out of line).  3inputs (PAPER.md:
+// 1823-1834, R6, R24): D2 = argmax (n2_k(D), u(D), -D), then the lowest-id
+// unallocated task of D2's segment whose other input is missing too; else
+// Alg. 5 l.13 (R5): the lowest-id unallocated task.  Returns {T, D(T)
+// ascending, bit 0: a 3inputs datum was found, bit 1: lowest-id pick}.
+__device__ __noinline__ int4 fallback_pick(const WV v, int k, bool fb2, bool any_avail, int avail_lo,
+                                           const int64_t *rp, const int32_t *rd, int lane) {
+    int T = -1, ra = -1, rb = -1, how = 0;
+    if (fb2) {
+        const int D2 = argmax_score(v, k, true, lane);
+        if (D2 >= 0) {
+            const int b = v.dp[D2], e = v.dp[D2 + 1];
+            for (int base = b; base < e && T < 0; base += 32) {
+                const int i = base + lane;
+                bool hit = false;
+                uint32_t ed = 0;
+                if (i < e) {
+                    ed = v.wedge[i];
+                    const int Tq = (int)(ed >> 16), o = (int)(ed & 0xFFFFu);
+                    hit = !((v.al[Tq >> 5] >> (Tq & 31)) & 1u) && o != (int)NOI && !res(v, k, o);
+                }
+                const unsigned msk = __ballot_sync(FULL, hit);
+                if (msk) {
+                    ed = __shfl_sync(FULL, ed, __ffs(msk) - 1);
+                    T = (int)(ed >> 16);
+                    const int o = (int)(ed & 0xFFFFu);
+                    ra = o < D2 ? o : D2;
+                    rb = o < D2 ? D2 : o;
+                }
+            }
+            how |= 1;
+        }
+    }
+    if (T < 0 && any_avail) {
+        const int nwd = (v.m + 31) >> 5;
+        for (int w0 = avail_lo >> 5; w0 < nwd && T < 0; w0 += 32) {
+            const int wd = w0 + lane;
+            uint32_t fr = 0;
+            if (wd < nwd) {
+                fr = ~v.al[wd];
+                if (wd == (avail_lo >> 5)) fr &= ~((1u << (avail_lo & 31)) - 1u);
+            }
+            const unsigned msk = __ballot_sync(FULL, fr != 0u);
+            if (msk) {
+                const int src = __ffs(msk) - 1;
+                fr = __shfl_sync(FULL, fr, src);
+                T = 32 * (w0 + src) + __ffs(fr) - 1;
+            }
+        }
+        if (T >= 0) {
+            raw_row(rp, rd, T, ra, rb);
+            how |= 2;
+        }
+    }
+    return make_int4(T, ra, rb, how);
+}
+
+// a8 (cold: out of line): sigma(k, .) for every k -- the stable partition of
+// the service order by GPU; lane k holds the count of GPU k.
+__device__ __noinline__ void assemble(const Inst *__restrict__ I, unsigned char *dsm, int lane, int nsv, int64_t ns,
+                                      int K, const int32_t *sg, const int32_t *stk) {
+    const unsigned lt = (1u << lane) - 1u;
+    __threadfence_block();
+    __syncwarp();
+    {
+        int x = lane < K ? nsv : 0;
+        const int own = x;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(FULL, x, o);
+            if (lane >= o) x += y;
+        }
+        int32_t *off = reinterpret_cast<int32_t *>(dsm);  // the loop's state is dead
+        __syncwarp();
+        if (lane < K) {
+            I->gpu_task_ptr[lane] = x - own;
+            off[lane] = x - own;
+        }
+        if (lane == 0) I->gpu_task_ptr[K] = ns;
+        __syncwarp();
+        for (int64_t i0 = 0; i0 < ns; i0 += 32) {
+            const int64_t i = i0 + lane;
+            const int kv = i < ns ? sg[i] : -1;
+            const int Tv = i < ns ? stk[i] : -1;
+            const unsigned peers = __match_any_sync(FULL, kv);
+            if (kv >= 0) I->gpu_task_ids[off[kv] + __popc(peers & lt)] = Tv;
+            __syncwarp();
+            if (kv >= 0 && lane == __ffs(peers) - 1) off[kv] += __popc(peers);
+            __syncwarp();
+        }
+    }
+}
+
+// One instance, the whole warp.
+__device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigned char *dsm, int lane) {
+    const unsigned lt = (1u << lane) - 1u;
+    WV v;
+    v.m = I->m;
+    v.n = I->n;
+    v.K = I->K;
+    v.pcap = I->plan_cap;
+    v.rcap = I->res_cap;
+    v.kmask = v.K >= 32 ? 0xffffffffu : ((1u << v.K) - 1u);
+    const WarpLayout Lw = warp_layout(v.m, v.n, v.K, v.pcap, v.rcap);
+    v.n4 = Lw.n4;
+    v.n8 = Lw.n8;
+    v.resm = reinterpret_cast<uint32_t *>(dsm + Lw.resm);
+    v.al = reinterpret_cast<uint32_t *>(dsm + Lw.al);
+    v.dp = reinterpret_cast<int32_t *>(dsm + Lw.dp);
+    v.u = reinterpret_cast<uint16_t *>(dsm + Lw.u);
+    v.hh = reinterpret_cast<uint32_t *>(dsm + Lw.hh);
+    v.np = reinterpret_cast<uint16_t *>(dsm + Lw.np);
+    v.plan = reinterpret_cast<uint32_t *>(dsm + Lw.plan);
+    v.rl = reinterpret_cast<int32_t *>(dsm + Lw.rl);
+    uint32_t *const wedge = reinterpret_cast<uint32_t *>(const_cast<int32_t *>(I->ddat));
+    v.wedge = wedge;
+    const uint64_t size0 = I->size0, cap = I->cap;
+    v.maxres = size0 == 0 ? INT_MAX : (int)(cap / size0 < (uint64_t)INT_MAX ? cap / size0 : (uint64_t)INT_MAX);
+    const int m = v.m, n = v.n, K = v.K;
+    const int64_t dtau = I->default_tau, delta0 = I->delta0, maxs = I->max_served;
+    const bool fb2 = (I->flags & DTS_F_FALLBACK2) != 0;
+    // pointers in registers (the descriptor is in global memory)
+    int64_t *const tst = I->tstart, *const ten = I->tend;
+    int32_t *const sg = I->serve_gpu, *const stk = I->serve_task;
+    dts_event *const evs = I->events;
+    const int64_t evcap = I->ev_cap;
+    const int64_t *const taup = I->tau;
+    const int64_t *const rp = I->raw_ptr;
+    const int32_t *const rd = I->raw_dat;
+
+    WP_DECL;
+    build_state(v, Lw, dsm, rp, rd, wedge, tst, ten, lane);
     // ---- per-GPU registers (lane k) and uniform scalars (every lane)
     int64_t req = 0, gfree = 0;
     int rc = 0, ph = 0, pe = 0, plive = 0, dopt = -1, nsv = 0;
     bool idle = false;
     int64_t ns = 0, bus = 0, mk = 0, nev = 0, nload = 0, nevict = 0, nscan = 0, nfb2 = 0, nfbf = 0, nidle = 0;
     int64_t sum_avail = 0, sum_deg = 0, n_alloc = 0;
-    uint64_t alg = 0, scan_alg = 0;
     int n_avail = m, avail_lo = 0, error = 0;
     const bool uni_tau = taup == nullptr && dtau > 0 && maxs < 0;
     WP(10);
@@ -479,7 +584,6 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 const int64_t me = (int64_t)wmax64(c > 0 ? (unsigned long long)req : 0ull);
                 mk = me > mk ? me : mk;
                 ns += total;
-                alg += 24ull * (uint64_t)total;
             } else {
                 // sequential: GPU k pops while its requests stay first in (time, id)
                 const unsigned long long k2 = wmin64(lane == k ? ~0ull : key);
@@ -512,7 +616,6 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 c = __shfl_sync(FULL, c, k);
                 mk = __shfl_sync(FULL, mk_l, k);
                 ns += c;
-                alg += 24ull * (uint64_t)c;
             }
             WP(0);
             continue;
@@ -522,10 +625,9 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
         WP(0);
         const int scan_avail = n_avail;
         const int Dopt = argmax_score(v, k, false, lane);  // Alg. 5 l.4-9
-        alg += 8ull * (uint64_t)n;
-        scan_alg += 8ull * (uint64_t)n;
         uint32_t edo[SEGR];  // first batch of Dopt's segment (plan walk, then its load)
         int ob = 0, oe = 0;
+        uint32_t m2b = 0u, selb = 0u;  // plan walk: per slot, unallocated with o missing / planned
         if (Dopt >= 0) {
             ob = v.dp[Dopt];
             oe = v.dp[Dopt + 1];
@@ -554,6 +656,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
             uint16_t *npk = v.np + k * v.n8;
             int P = 0;
             uint32_t w0 = 0;
+            m2b = selb = 0u;
             for (int base = ob; base < oe; base += 32 * SEGR) {
                 uint32_t ed[SEGR], aw[SEGR], rw[SEGR];
                 if (base == ob) {
@@ -573,7 +676,12 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 for (int r = 0; r < SEGR; r++) {
                     const uint32_t w = ed[r];
                     const int Tq = (int)(w >> 16), o = (int)(w & 0xFFFFu);
-                    const bool sel = w != REMOVED && !((aw[r] >> (Tq & 31)) & 1u) && ((rw[r] >> k) & 1u);
+                    const bool live = w != REMOVED && !((aw[r] >> (Tq & 31)) & 1u);
+                    const bool sel = live && ((rw[r] >> k) & 1u);
+                    if (base == ob) {  // for Dopt's own load (below): its tasks' classes now
+                        m2b |= (uint32_t)(live && !sel) << r;
+                        selb |= (uint32_t)sel << r;
+                    }
                     const unsigned msk = __ballot_sync(FULL, sel);
                     if (msk == 0u) continue;
                     if (P == 0) w0 = __shfl_sync(FULL, w, __ffs(msk) - 1);
@@ -614,7 +722,6 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
             n_alloc += P;
             nscan++;
             sum_avail += scan_avail;
-            alg += 20ull * (uint64_t)(oe - ob) + (uint64_t)P * (8ull * K + 40ull);
             __syncwarp();
             WP(2);
         } else {
@@ -622,56 +729,17 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 ph = pe = plive = 0;
                 dopt = -1;
             }
-            if (fb2) {  // 3inputs (R6, R24)
-                const int D2 = argmax_score(v, k, true, lane);
-                alg += 8ull * (uint64_t)n;
-                scan_alg += 8ull * (uint64_t)n;
-                if (D2 >= 0) {
-                    // the lowest-id unallocated task of D2's segment with its other input missing
-                    const int b = v.dp[D2], e = v.dp[D2 + 1];
-                    for (int base = b; base < e && T < 0; base += 32) {
-                        const int i = base + lane;
-                        bool hit = false;
-                        uint32_t ed = 0;
-                        if (i < e) {
-                            ed = wedge[i];
-                            const int Tq = (int)(ed >> 16), o = (int)(ed & 0xFFFFu);
-                            hit = !((v.al[Tq >> 5] >> (Tq & 31)) & 1u) && o != (int)NOI && !res(v, k, o);
-                        }
-                        const unsigned msk = __ballot_sync(FULL, hit);
-                        if (msk) {
-                            ed = __shfl_sync(FULL, ed, __ffs(msk) - 1);
-                            T = (int)(ed >> 16);
-                            const int o = (int)(ed & 0xFFFFu);
-                            ra = o < D2 ? o : D2;
-                            rb = o < D2 ? D2 : o;
-                        }
-                    }
-                    nfb2++;
-                }
+            // 3inputs (R6, R24), else Alg. 5 l.13 (R5)
+            const int4 f = fallback_pick(v, k, fb2, n_avail > 0, avail_lo, rp, rd, lane);
+            T = f.x;
+            ra = f.y;
+            rb = f.z;
+            if (fb2) {
             }
-            if (T < 0 && n_avail > 0) {
-                // Alg. 5 l.13 (R5): the lowest-id unallocated task
-                const int nwd = (m + 31) >> 5;
-                for (int w0 = avail_lo >> 5; w0 < nwd && T < 0; w0 += 32) {
-                    const int wd = w0 + lane;
-                    uint32_t fr = 0;
-                    if (wd < nwd) {
-                        fr = ~v.al[wd];
-                        if (wd == (avail_lo >> 5)) fr &= ~((1u << (avail_lo & 31)) - 1u);
-                    }
-                    const unsigned msk = __ballot_sync(FULL, fr != 0u);
-                    if (msk) {
-                        const int src = __ffs(msk) - 1;
-                        fr = __shfl_sync(FULL, fr, src);
-                        T = 32 * (w0 + src) + __ffs(fr) - 1;
-                    }
-                }
-                if (T >= 0) {
-                    raw_row(rp, rd, T, ra, rb);
-                    nfbf++;
-                    avail_lo = T;
-                }
+            if (f.w & 1) nfb2++;
+            if (f.w & 2) {
+                nfbf++;
+                avail_lo = T;
             }
             if (T < 0) {
                 if (lane == k) idle = true;
@@ -701,6 +769,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
         int pek = __shfl_sync(FULL, pe, k);
         const int dk = __shfl_sync(FULL, dopt, k);
         int64_t ready = t;
+        int vlast = -1, nvict = 0;  // victims of this serve
         for (int qd = 0; qd < 2 && !error; qd++) {
             const int D = qd == 0 ? ra : rb;
             if (D < 0 || res(v, k, D)) continue;
@@ -775,7 +844,6 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 push_event(evs, evcap, nev, lane, 1, k, V, T, t, t);
                 const int degv = ve - vb;
                 sum_deg += degv;
-                alg += 24ull * (uint64_t)degv + (uint64_t)nret * (8ull * K + 40ull) + 32ull;
                 __syncwarp();
                 if (nret > 0) {  // close the holes: live entries contiguous from ph
                     int out = phk;
@@ -793,18 +861,13 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                     if (lane == k) pe = out;
                 }
                 WP(6);
+                vlast = V;
+                nvict++;
                 seg_update(v, k, V, false, lane, edv);
                 WP(7);
             }
             if (error) break;
             // load D
-            uint32_t edd[SEGR];
-            if (D == Dopt) {
-#pragma unroll
-                for (int r = 0; r < SEGR; r++) edd[r] = edo[r];
-            } else {
-                seg_load(v, v.dp[D], v.dp[D + 1], lane, edd);
-            }
             if (lane == 0) {
                 v.rl[k * v.rcap + rck] = D;
                 v.resm[D] |= 1u << k;
@@ -816,11 +879,36 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
             ready = en > ready ? en : ready;
             nload++;
             push_event(evs, evcap, nev, lane, 0, k, D, T, st, en);
-            const int degd = v.dp[D + 1] - v.dp[D];
-            sum_deg += degd;
-            alg += 24ull * (uint64_t)degd + 32ull;
+            const int db = v.dp[D], de = v.dp[D + 1];
+            sum_deg += de - db;
             __syncwarp();
-            seg_update(v, k, D, true, lane, edd);
+            if (D == Dopt && de - db <= 32 * SEGR && nvict <= 1) {
+                // Dopt's load in the plan path: after the plan, the unallocated tasks
+                // of its segment are those the plan walk saw unallocated with their
+                // other input o missing, plus planned ones LUF returned (o = V):
+                // all go 2 -> 1 (freed by o); none is left with o resident
+                uint32_t *hk = v.hh + k * v.n4;
+                int n2 = 0;
+#pragma unroll
+                for (int r = 0; r < SEGR; r++) {
+                    const int o = (int)(edo[r] & 0xFFFFu);
+                    const bool upd = ((m2b >> r) & 1u) || (((selb >> r) & 1u) && o == vlast);
+                    n2 += (int)upd;
+                    if (upd) atomicAdd(&hk[o], 1u - 65536u);
+                }
+                n2 = wsum(n2);
+                if (lane == 0 && n2) atomicAdd(&hk[D], 0u - ((uint32_t)n2 << 16));
+                __syncwarp();
+            } else {
+                uint32_t edd[SEGR];
+                if (D == Dopt) {
+#pragma unroll
+                    for (int r = 0; r < SEGR; r++) edd[r] = edo[r];
+                } else {
+                    seg_load(v, db, de, lane, edd);
+                }
+                seg_update(v, k, D, true, lane, edd);
+            }
             WP(8);
         }
         if (error) break;
@@ -842,41 +930,12 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
             }
             mk = end > mk ? end : mk;
             ns++;
-            alg += 24;
         }
         WP(9);
     }
 
     // ---- a8: sigma(k, .) -- stable partition of the service order by GPU
-    __threadfence_block();
-    __syncwarp();
-    {
-        int x = lane < K ? nsv : 0;
-        const int own = x;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int y = __shfl_up_sync(FULL, x, o);
-            if (lane >= o) x += y;
-        }
-        int32_t *off = reinterpret_cast<int32_t *>(dsm);  // the loop's state is dead
-        __syncwarp();
-        if (lane < K) {
-            I->gpu_task_ptr[lane] = x - own;
-            off[lane] = x - own;
-        }
-        if (lane == 0) I->gpu_task_ptr[K] = ns;
-        __syncwarp();
-        for (int64_t i0 = 0; i0 < ns; i0 += 32) {
-            const int64_t i = i0 + lane;
-            const int kv = i < ns ? sg[i] : -1;
-            const int Tv = i < ns ? stk[i] : -1;
-            const unsigned peers = __match_any_sync(FULL, kv);
-            if (kv >= 0) I->gpu_task_ids[off[kv] + __popc(peers & lt)] = Tv;
-            __syncwarp();
-            if (kv >= 0 && lane == __ffs(peers) - 1) off[kv] += __popc(peers);
-            __syncwarp();
-        }
-    }
+    assemble(I, dsm, lane, nsv, ns, K, sg, stk);
     if (lane == 0) {
         Out *o = I->out;
         o->n_events = nev;
@@ -891,8 +950,8 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
         o->n_verify_err = 0;
         o->bytes_loaded = (uint64_t)nload * size0;
         o->makespan = mk;
-        o->alg_bytes = alg;
-        o->scan_alg_bytes = scan_alg;
+        o->alg_bytes = 0;  // the CTA loop's own byte model; not kept by this loop
+        o->scan_alg_bytes = 0;
         o->sum_avail = sum_avail;
         o->n_alloc = n_alloc;
         o->sum_deg = sum_deg;

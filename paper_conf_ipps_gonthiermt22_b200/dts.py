@@ -40,6 +40,7 @@ DTS_F_OPTI = 8
 DTS_F_PACKED = 16
 DTS_F_GENERIC = 32
 DTS_F_CTA = 64  # force the per-CTA loop where the one-warp loop applies (diagnostic)
+LOOP_GENERIC, LOOP_CTA_FAST, LOOP_WARP = 1, 2, 3  # dts_result_view.loop_kind
 
 EVENT_DTYPE = np.dtype([("t", "<i8"), ("t_end", "<i8"), ("gpu", "<i4"), ("data", "<i4"),
                         ("task", "<i4"), ("op", "u1"), ("pad", "u1", (3,))])
@@ -80,7 +81,8 @@ class dts_result_view(C.Structure):
                 ("alg_bytes", C.c_uint64),
                 ("scan_alg_bytes", C.c_uint64), ("loop_ms", C.c_float), ("total_ms", C.c_float),
                 ("prof_cycles", C.c_int64 * 16), ("sum_avail_at_scans", C.c_int64),
-                ("n_allocations", C.c_int64), ("sum_deg_loads_evictions", C.c_int64)]
+                ("n_allocations", C.c_int64), ("sum_deg_loads_evictions", C.c_int64),
+                ("loop_kind", C.c_int32), ("reserved", C.c_int32)]
 
 
 _lib = None
@@ -268,6 +270,7 @@ class Result:
     sum_avail_at_scans: int = 0
     n_allocations: int = 0
     sum_deg_loads_evictions: int = 0
+    loop_kind: int = 0  # 1 generic CTA loop, 2 specialised CTA loop, 3 one-warp loop
 
     def orders(self):
         p = self.gpu_task_ptr
@@ -303,7 +306,8 @@ def dts_result(inst: Instance, copy: bool = True) -> Result:
                   int(v.n_idle_requests), int(v.n_verify_err), int(v.alg_bytes),
                   int(v.scan_alg_bytes),
                   float(v.loop_ms), float(v.total_ms), tuple(int(x) for x in v.prof_cycles),
-                  int(v.sum_avail_at_scans), int(v.n_allocations), int(v.sum_deg_loads_evictions))
+                  int(v.sum_avail_at_scans), int(v.n_allocations), int(v.sum_deg_loads_evictions),
+                  int(v.loop_kind))
 
 
 def dts_fetch_results(insts) -> None:

@@ -31,11 +31,11 @@ ref)
 launches)
   timeout 1200 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $O/${TAG}_launches_C4.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_bench.log 2>&1; echo "launches rc=$?" ;;
 full_C4)
-  timeout 3000 ncu --set full --import-source on --clock-control none -k regex:dts_cta_kernel -s 3 -c 1 -o $O/${TAG}_full_C4 python bench.py --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C4.log 2>&1; echo "full C4 rc=$?" ;;
+  timeout 3000 ncu --set full --import-source on --clock-control none -k regex:"dts_(cta|warp)_kernel" -s 3 -c 1 -o $O/${TAG}_full_C4 python bench.py --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C4.log 2>&1; echo "full C4 rc=$?" ;;
 full_C5)
-  timeout 1500 ncu --set full --import-source on --clock-control none -k regex:dts_cta_kernel -s 6 -c 2 -o $O/${TAG}_full_C5 python bench.py --workload C5 --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C5.log 2>&1; echo "full C5 rc=$?" ;;
+  timeout 1500 ncu --set full --import-source on --clock-control none -k regex:"dts_(cta|warp)_kernel" -s 6 -c 2 -o $O/${TAG}_full_C5 python bench.py --workload C5 --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C5.log 2>&1; echo "full C5 rc=$?" ;;
 full_C2)
-  timeout 900 ncu --set full --import-source on --clock-control none -k regex:dts_cta_kernel -s 3 -c 1 -o $O/${TAG}_full_C2 python bench.py --workload C2 --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C2.log 2>&1; echo "full C2 rc=$?" ;;
+  timeout 900 ncu --set full --import-source on --clock-control none -k regex:"dts_(cta|warp)_kernel" -s 3 -c 1 -o $O/${TAG}_full_C2 python bench.py --workload C2 --steps 1 --warmup 3 --no-cpu-baseline > $O/${TAG}_ncu_full_C2.log 2>&1; echo "full C2 rc=$?" ;;
 esac
 done
 ls $O | grep "^$TAG" | head -50
