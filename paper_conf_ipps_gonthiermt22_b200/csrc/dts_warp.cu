@@ -81,10 +81,15 @@ __device__ __forceinline__ void add16(uint16_t *a, int i, int d) {
     atomicAdd(reinterpret_cast<unsigned *>(a) + (i >> 1), (unsigned)d << (16 * (i & 1)));
 }
 
+// Segment walks hold SEGR edges per lane in registers (32 SEGR = 160 per
+// batch: C5's widest segment).  Every unrolled slot costs instructions: 8
+// and 6 were slower, and one copy of the loop per width (2, 4, 5, 8 chosen
+// per instance) made the C5 sweep 33 % slower (registers, instruction cache;
+// profiles/r03/r03_warp_var.txt).
 #ifndef DTS_SEGR
 #define DTS_SEGR 5
 #endif
-constexpr int SEGR = DTS_SEGR;  // edges per lane of one segment batch in registers (32 SEGR per batch)
+constexpr int SEGR = DTS_SEGR;
 
 // The warp's view of one instance (registers; pointers into its smem slice).
 struct WV {
@@ -153,12 +158,14 @@ __device__ __forceinline__ void pool_buckets(const WV &v, int a, int b, int sign
 // (Alg. 5 l.6-9 with hi = 0; the 3inputs key with hi = 1; R1, R23, R24).  A
 // datum with a positive score is never resident.  -1 if none.  Four vectors
 // of four data per lane are loaded before any compare.
+__device__ __forceinline__ unsigned long long max64(unsigned long long a, unsigned long long b) {
+    return a > b ? a : b;
+}
 __device__ __forceinline__ int argmax_score(const WV &v, int k, bool hi, int lane) {
     const uint4 *h4 = reinterpret_cast<const uint4 *>(v.hh + k * v.n4);
     const uint2 *u2 = reinterpret_cast<const uint2 *>(v.u);
     const int nv = v.n4 >> 2;
-    uint32_t bk = 0;
-    int bd = 0;
+    unsigned long long best = 0ull;  // (score << 16 | u) << 32 | (2^32 - 1 - D): ties -> lowest D
     for (int q0 = lane; q0 < nv; q0 += 128) {
         uint4 x[4];
         uint2 y[4];
@@ -168,23 +175,23 @@ __device__ __forceinline__ int argmax_score(const WV &v, int k, bool hi, int lan
             x[r] = q < nv ? h4[q] : make_uint4(0, 0, 0, 0);
             y[r] = q < nv ? u2[q] : make_uint2(0, 0);
         }
+        unsigned long long c[4];
 #pragma unroll
-        for (int r = 0; r < 4; r++) {
-            const int D = 4 * (q0 + 32 * r);
+        for (int r = 0; r < 4; r++) {  // a max tree per vector, then over the vectors
+            const uint32_t D = 4u * (uint32_t)(q0 + 32 * r);
             const uint32_t s0 = hi ? (x[r].x & 0xFFFF0000u) : (x[r].x << 16);
             const uint32_t s1 = hi ? (x[r].y & 0xFFFF0000u) : (x[r].y << 16);
             const uint32_t s2 = hi ? (x[r].z & 0xFFFF0000u) : (x[r].z << 16);
             const uint32_t s3 = hi ? (x[r].w & 0xFFFF0000u) : (x[r].w << 16);
-            const uint32_t k0 = s0 | (y[r].x & 0xFFFFu), k1 = s1 | (y[r].x >> 16);
-            const uint32_t k2 = s2 | (y[r].y & 0xFFFFu), k3 = s3 | (y[r].y >> 16);
-            if (k0 > bk) { bk = k0; bd = D; }
-            if (k1 > bk) { bk = k1; bd = D + 1; }
-            if (k2 > bk) { bk = k2; bd = D + 2; }
-            if (k3 > bk) { bk = k3; bd = D + 3; }
+            const unsigned long long c0 = ((unsigned long long)(s0 | (y[r].x & 0xFFFFu)) << 32) | (0xFFFFFFFFu - D);
+            const unsigned long long c1 = ((unsigned long long)(s1 | (y[r].x >> 16)) << 32) | (0xFFFFFFFEu - D);
+            const unsigned long long c2 = ((unsigned long long)(s2 | (y[r].y & 0xFFFFu)) << 32) | (0xFFFFFFFDu - D);
+            const unsigned long long c3 = ((unsigned long long)(s3 | (y[r].y >> 16)) << 32) | (0xFFFFFFFCu - D);
+            c[r] = max64(max64(c0, c1), max64(c2, c3));
         }
+        best = max64(best, max64(max64(c[0], c[1]), max64(c[2], c[3])));
     }
-    const unsigned long long best =
-        bk >= 65536u ? (((unsigned long long)bk << 32) | (0xFFFFFFFFu - (uint32_t)bd)) : 0ull;
+    if ((best >> 32) < 65536u) best = 0ull;  // no positive score
     const unsigned long long w = wmax64(best);
     return w ? (int)(0xFFFFFFFFu - (uint32_t)w) : -1;
 }
@@ -263,6 +270,23 @@ __device__ __forceinline__ void push_event(dts_event *evs, int64_t evcap, int64_
         evs[nev] = ev;
     }
     nev++;
+}
+
+// x / tau and x mod tau for 0 <= x < 2^52 (times in ns): a double-precision
+// estimate corrected by one step (exact; no 64-bit integer division).
+__device__ __forceinline__ int64_t div_tau(int64_t x, int64_t tau, double inv, int64_t &rem) {
+    int64_t q = (int64_t)((double)x * inv);
+    int64_t r = x - q * tau;
+    while (r < 0) {
+        q--;
+        r += tau;
+    }
+    while (r >= tau) {
+        q++;
+        r -= tau;
+    }
+    rem = r;
+    return q;
 }
 
 __device__ __forceinline__ int64_t tau_of(const int64_t *taup, int T, int64_t dtau) {
@@ -497,6 +521,9 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
     int64_t sum_avail = 0, sum_deg = 0, n_alloc = 0;
     int n_avail = m, avail_lo = 0, error = 0;
     const bool uni_tau = taup == nullptr && dtau > 0 && maxs < 0;
+    const double inv_tau = dtau > 0 ? 1.0 / (double)dtau : 0.0;
+    // (task, GPU) item lane + 32 i of a plan's pool move: task p0 + i q32 (+ carries), GPU j0 + i r32
+    const int p0 = lane / K, j0 = lane % K, q32 = 32 / K, r32 = 32 % K;
     WP(10);
 
     // ---- the decision loop
@@ -526,12 +553,12 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                     const int64_t d = St - req;
                     int64_t cnt = 0;
                     if (d >= 0) {
-                        const int64_t qd = d / dtau, rr = d - qd * dtau;
+                        int64_t rr;
+                        const int64_t qd = div_tau(d, dtau, inv_tau, rr);
                         cnt = qd + (rr != 0 ? 1 : 0) + ((rr == 0 && lane < Sj) ? 1 : 0);
                     }
                     c = (int)(cnt < plive ? cnt : plive);
-                    q = req / dtau;
-                    rho = req - q * dtau;
+                    q = div_tau(req, dtau, inv_tau, rho);
                 }
                 const unsigned pm = __ballot_sync(FULL, c > 0);
                 const uint32_t *pl = v.plan + lane * v.pcap;
@@ -655,7 +682,6 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
             uint32_t *pl = v.plan + k * v.pcap;
             uint16_t *npk = v.np + k * v.n8;
             int P = 0;
-            uint32_t w0 = 0;
             m2b = selb = 0u;
             for (int base = ob; base < oe; base += 32 * SEGR) {
                 uint32_t ed[SEGR], aw[SEGR], rw[SEGR];
@@ -684,7 +710,6 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                     }
                     const unsigned msk = __ballot_sync(FULL, sel);
                     if (msk == 0u) continue;
-                    if (P == 0) w0 = __shfl_sync(FULL, w, __ffs(msk) - 1);
                     if (sel) {
                         const int pos = P + __popc(msk & lt);
                         pl[pos] = w;
@@ -693,9 +718,35 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                             add16(v.u, o, -1);
                             if (pos > 0) add16(npk, o, 1);
                         }
-                        pool_buckets(v, Dopt, o == (int)NOI ? -1 : o, -1, 1u << k);
                     }
                     P += __popc(msk);
+                }
+            }
+            if (K > 1) {
+                // the planned tasks' buckets on the other GPUs j: (task, GPU) items
+                // spread over the lanes (item lane + 32 i = task p, GPU j)
+                __syncwarp();
+                const uint32_t mD = ~v.resm[Dopt] & v.kmask;  // GPUs missing Dopt
+                int p = p0, j = j0;
+                for (int idx = lane; idx < P * K; idx += 32) {
+                    if (j != k) {
+                        const int o = (int)(pl[p] & 0xFFFFu);
+                        const bool md = (mD >> j) & 1u;
+                        const bool mo = o != (int)NOI && !((v.resm[o] >> j) & 1u);
+                        uint32_t *hj = v.hh + j * v.n4;
+                        if (md && mo) {
+                            atomicAdd(&hj[Dopt], 0u - 65536u);
+                            atomicAdd(&hj[o], 0u - 65536u);
+                        } else if (md || mo) {
+                            atomicAdd(&hj[md ? Dopt : o], 0xFFFFFFFFu);
+                        }
+                    }
+                    p += q32;
+                    j += r32;
+                    if (j >= K) {
+                        j -= K;
+                        p++;
+                    }
                 }
             }
             if (lane == 0) {  // the shared parts: u(Dopt), np_k(Dopt), n_k(Dopt) (every task has
@@ -704,6 +755,8 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 if (P > 1) add16(npk, Dopt, P - 1);
                 atomicAdd(&v.hh[k * v.n4 + Dopt], (unsigned)(-P));
             }
+            __syncwarp();
+            const uint32_t w0 = pl[0];  // Alg. 5 l.11: the plan's first task is served now
             T = (int)(w0 >> 16);
             const int o0 = (int)(w0 & 0xFFFFu);
             if (o0 == (int)NOI) {
@@ -778,22 +831,22 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 // the fewest uses in plannedTasks_k, lowest id on ties (R1)
                 const int32_t *rlk = v.rl + k * v.rcap;
                 const uint16_t *npk = v.np + k * v.n8;
-                unsigned long long best = ~0ull;
+                uint32_t best = 0xFFFFFFFFu;  // np_k(D) << 16 | D (both < 2^16)
                 int bslot = -1;
                 for (int i = lane; i < rck; i += 32) {
                     const int Dv = rlk[i];
-                    const unsigned long long kk = ((unsigned long long)npk[Dv] << 32) | (unsigned)Dv;
+                    const uint32_t kk = ((uint32_t)npk[Dv] << 16) | (uint32_t)Dv;
                     const bool take = Dv != ra && Dv != rb && kk < best;
                     best = take ? kk : best;
                     bslot = take ? i : bslot;
                 }
-                const unsigned long long mine = best;
-                best = wmin64(best);
-                if (best == ~0ull) {
+                const uint32_t mine = best;
+                best = __reduce_min_sync(FULL, best);
+                if (best == 0xFFFFFFFFu) {
                     error = 1;
                     break;
                 }
-                const int V = (int)(uint32_t)best;
+                const int V = (int)(best & 0xFFFFu);
                 uint32_t edv[SEGR];  // V's segment, fetched while the plan is updated
                 const int vb = v.dp[V], ve = v.dp[V + 1];
                 seg_load(v, vb, ve, lane, edv);

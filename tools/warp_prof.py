@@ -10,7 +10,7 @@ import paper_conf_ipps_gonthiermt22_b200 as dts  # noqa: E402
 
 NAMES = ["pop", "argmax", "planwalk", "planpool", "fallback", "luf", "evict", "seg_ev", "load", "finish",
          "build", "assemble"]
-for inst in (gen.sweep_instance(160, 4, 1), gen.sweep_instance(160, 128, 8), gen.config_instances("C2")[19],
+for inst in (gen.sweep_instance(160, 4, 1), gen.sweep_instance(160, 4, 7), gen.sweep_instance(160, 128, 8), gen.config_instances("C2")[19],
              gen.matmul2d(10, M=6, K=1)):
     dts.schedule(inst)
     g = dts.schedule(inst)
