@@ -65,7 +65,7 @@ def _load():
     global _lib
     if _lib is None:
         # DTS_ORACLE_LIB: a deliberately mutated build of dts_oracle.c
-        # (tools/oracle_mutants.py checks that the pins reject it)
+        # (tests/oracle_mutants.py checks that the pins reject it)
         _lib = C.CDLL(os.environ.get("DTS_ORACLE_LIB") or build())
         _lib.or_run.restype = C.c_int
         _lib.or_run.argtypes = [C.c_int32, C.c_int32, C.c_void_p, C.c_void_p, C.c_void_p,

@@ -831,6 +831,7 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
                           (int32_t *)h.tdat, (int64_t *)h.dptr, (int32_t *)h.ddat, (int4 *)h.dedge,
                           I->d_csr_scratch, st, h.t_lo, h.t_hi),
            "build_csr");
+    h.hh = fast_mode(h) ? 1 : 0;  // the specialised loop keeps packed score rows (dts_loop.cu M_HH)
     if (!copy_desc) return DTS_OK;
     // descriptor H2D from pinned memory (a pageable copy would serialise the host)
     CK(cudaEventSynchronize(I->ev_desc), "desc event");
@@ -956,14 +957,17 @@ dts_status sweep_on_device(dts_instance *const *insts, int32_t n, dts_policy pol
     SweepSlot *S = nullptr;
     dts_status s = acquire_slot(D, (size_t)n, &S);
     if (s != DTS_OK) return s;
-    for (int32_t i = 0; i < n; i++) S->h_insts[i] = insts[ord[(size_t)i]]->h_inst;
+    bool fast = true;  // the specialised loop applies to every instance (packed score rows)
+    for (int32_t i = 0; i < n; i++) fast &= fast_mode(insts[i]->h_inst);
+    for (int32_t i = 0; i < n; i++) {
+        S->h_insts[i] = insts[ord[(size_t)i]]->h_inst;
+        S->h_insts[i].hh = fast && !warp ? 1 : 0;
+    }
     CK(cudaMemcpyAsync(S->d_insts, S->h_insts, sizeof(dts::Inst) * (size_t)n, cudaMemcpyHostToDevice, st),
        "H2D sweep");
     CK(cudaMemsetAsync(S->d_work, 0, 2 * sizeof(int), st), "memset");
     if (any_unfused) CK(dts::launch_init(S->d_insts, n, o.bus_bytes_per_s, work, st), "init");
     CK(cudaEventRecord(sev->loop_begin, st), "event");
-    bool fast = true;
-    for (int32_t i = 0; i < n; i++) fast &= fast_mode(insts[i]->h_inst);
     if (warp) {
         const int per = std::max(1, dts::warp_max_blocks_per_sm(smem));
         const int grid = (int)std::min<int64_t>((int64_t)n, (int64_t)per * nsm);
@@ -1466,6 +1470,7 @@ static dts_status fetch_arrays(dts_instance *I) {
     I->out = *I->r_out;
     if (I->out.error == 2) return fail(DTS_E_STATE, "task shards: a peer did not reach an exchange in time");
     if (I->out.error == 3) return fail(DTS_E_STATE, "device loop: plannedTasks inconsistent (internal)");
+    if (I->out.error == 9) return fail(DTS_E_STATE, "device loop: a bounds check failed (profiling build)");
     if (I->out.error) return fail(DTS_E_STATE, "device loop: LUF found no victim");
     const dts::Inst &h = I->h_inst;
     const size_t ne = (size_t)std::min<int64_t>(I->out.n_events, h.ev_cap);

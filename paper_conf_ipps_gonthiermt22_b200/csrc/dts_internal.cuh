@@ -163,6 +163,10 @@ struct Inst {
     uint32_t *al;             // [m_pad / 32 + 1] global home
     int32_t poison;  // debug (env DTS_POISON=1): fill the CTA's dynamic shared memory at instance start
     int32_t *wring;  // [K][MAX_W] W >= 1: the last W tasks served on each simulated GPU
+    // 1: the launch runs the specialised loop (dts_loop_fast.cu), whose score rows are
+    // packed: h[k][D] = n_k(D) | n2_k(D) << 16 (h2 unused); dts_init_kernel writes them so
+    int32_t hh;
+    int32_t pad3;
 };
 
 }  // namespace dts

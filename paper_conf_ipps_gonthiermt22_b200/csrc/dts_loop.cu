@@ -52,6 +52,7 @@
 #define M_LONG(c) (!DTS_FAST && (c))                           // rows of > 3 inputs
 #define M_KEY32(I) (DTS_FAST || (I).key32)                     // scores and u(D) < 2^15
 #define M_FLAG(I, f) (!DTS_FAST && ((I).flags & (f)))          // OPTI, VERIFY: generic only
+#define M_HH (DTS_FAST)  // packed scores: h[k][D] = n_k(D) | n2_k(D) << 16, one argmax pass for both
 #if DTS_FAST
 #define DTS_KNAME(x) x##_fast
 #else
@@ -239,6 +240,13 @@ __device__ __forceinline__ bool resident(int k, int32_t D) {
     return (V.resb[(size_t)k * I.nw + (D >> 5)] >> (D & 31)) & 1u;
 }
 
+// n_k(D) += d and n2_k(D) += d (packed rows in the specialised loop: n2 is the high half).
+__device__ __forceinline__ void add_n(int k, int32_t D, int d) { atomicAdd(&SV.h[(size_t)k * SI.nstr + D], d); }
+__device__ __forceinline__ void add_n2(int k, int32_t D, int d) {
+    if (M_HH) atomicAdd(&SV.h[(size_t)k * SI.nstr + D], d * 65536);
+    else atomicAdd(&SV.h2[(size_t)k * SI.nstr + D], d);
+}
+
 // Row-derived mode (Inst::sl): T has left the shared pool (R2).
 __device__ __forceinline__ bool allocated(int32_t T) { return (SV.al[T >> 5] >> (T & 31)) & 1u; }
 __device__ __forceinline__ void set_alloc(int32_t T, int sign) {
@@ -355,10 +363,10 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
             int32_t a, b;
             const int c = missing_of(j, r.r0, r.r1, r.r2, a, b);
             if (c == 1) {
-                atomicAdd(&V.h[(size_t)j * I.nstr + a], sign);
+                add_n(j, a, sign);
             } else if (c == 2) {
-                atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
-                atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
+                add_n2(j, a, sign);
+                add_n2(j, b, sign);
             }
         }
     }
@@ -445,10 +453,10 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
                 int32_t a, b;
                 const int c = missing_of(j, e.y, e.z, e.w, a, b);
                 if (c == 1) {
-                    atomicAdd(&V.h[(size_t)j * I.nstr + a], sign);
+                    add_n(j, a, sign);
                 } else if (c == 2) {
-                    atomicAdd(&V.h2[(size_t)j * I.nstr + a], sign);
-                    atomicAdd(&V.h2[(size_t)j * I.nstr + b], sign);
+                    add_n2(j, a, sign);
+                    add_n2(j, b, sign);
                 }
                 continue;
             }
@@ -575,6 +583,31 @@ __device__ void seg_update(int k, int32_t D, bool load) {
             const bool my = ed.y >= 0 && !resident(k, ed.y), mz = ed.z >= 0 && !resident(k, ed.z);
             const int c = (int)my + (int)mz + (load ? 1 : 0);  // missing inputs before
             const int32_t o = my ? ed.y : ed.z;                 // the other missing one (c == 2 / 1)
+            if (M_HH) {  // packed rows: n in the low half, n2 in the high half
+                constexpr int U2 = 65536;
+                if (load) {
+                    if (c == 1) {  // 1 -> 0
+                        atomicSub(&hk[D], 1);
+                    } else if (c == 2) {  // 2 -> 1: now freed by o
+                        atomicSub(&hk[D], U2);
+                        atomicAdd(&hk[o], 1 - U2);
+                    } else if (c == 3) {  // 3 -> 2
+                        atomicAdd(&hk[ed.y], U2);
+                        atomicAdd(&hk[ed.z], U2);
+                    }
+                } else {
+                    if (c == 0) {  // 0 -> 1
+                        atomicAdd(&hk[D], 1);
+                    } else if (c == 1) {  // 1 -> 2: missing {o, D}
+                        atomicAdd(&hk[o], U2 - 1);
+                        atomicAdd(&hk[D], U2);
+                    } else if (c == 2) {  // 2 -> 3
+                        atomicSub(&hk[ed.y], U2);
+                        atomicSub(&hk[ed.z], U2);
+                    }
+                }
+                continue;
+            }
             if (load) {
                 if (c == 1) {  // 1 -> 0
                     atomicSub(&hk[D], 1);
@@ -1440,7 +1473,9 @@ __device__ __noinline__ unsigned long long score_best64(const int32_t *score) {
     return best;
 }
 
-__device__ int32_t score_argmax(const int32_t *score) {
+// sh = 16: the key is score << 16 | u; sh = 0 on packed rows (M_HH): the high
+// half (n2) is the score, the 3inputs key.
+__device__ int32_t score_argmax(const int32_t *score, int sh = 16) {
     const Inst &I = SI;
     const View &V = SV;
     const unsigned ib = (unsigned)I.id_bits;
@@ -1464,10 +1499,10 @@ __device__ int32_t score_argmax(const int32_t *score) {
 #pragma unroll
             for (int q = 0; q < UN; q++) {
                 const int D = 4 * (v0 + q * blockDim.x);
-                const uint32_t k0 = ((uint32_t)hv[q].x << 16) | (uint32_t)uv[q].x;
-                const uint32_t k1 = ((uint32_t)hv[q].y << 16) | (uint32_t)uv[q].y;
-                const uint32_t k2 = ((uint32_t)hv[q].z << 16) | (uint32_t)uv[q].z;
-                const uint32_t k3 = ((uint32_t)hv[q].w << 16) | (uint32_t)uv[q].w;
+                const uint32_t k0 = (((uint32_t)hv[q].x << sh) & 0xFFFF0000u) | (uint32_t)uv[q].x;
+                const uint32_t k1 = (((uint32_t)hv[q].y << sh) & 0xFFFF0000u) | (uint32_t)uv[q].y;
+                const uint32_t k2 = (((uint32_t)hv[q].z << sh) & 0xFFFF0000u) | (uint32_t)uv[q].z;
+                const uint32_t k3 = (((uint32_t)hv[q].w << sh) & 0xFFFF0000u) | (uint32_t)uv[q].w;
                 if (k0 > bk) { bk = k0; bd = D; }
                 if (k1 > bk) { bk = k1; bd = D + 1; }
                 if (k2 > bk) { bk = k2; bd = D + 2; }
@@ -1480,6 +1515,64 @@ __device__ int32_t score_argmax(const int32_t *score) {
         best = score_best64(score);
     }
     best = block_max_u64(best);
+    return best ? (int32_t)(idmask - (best & idmask)) : -1;
+}
+
+// Both keys in ONE pass over the packed rows of the specialised loop (M_HH):
+// the main argmax of (n_k(D), u(D), -D) (returned) and the 3inputs argmax of
+// (n2_k(D), u(D), -D) (*d2), in a single block exchange -- the fallback no
+// longer re-reads the rows (it serves 59-68 % of C4's scans).
+__device__ void block_max2_u64(unsigned long long &a, unsigned long long &b) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    a = warp_max_u64(a);
+    b = warp_max_u64(b);
+    if (nw == 1) return;
+    cta_sync();
+    if (lane == 0) {
+        L.red64[w] = a;
+        L.red64b[w] = b;
+    }
+    cta_sync();
+    a = warp_max_u64(lane < nw ? L.red64[lane] : 0ull);
+    b = warp_max_u64(lane < nw ? L.red64b[lane] : 0ull);
+}
+__device__ int32_t score_argmax_hh(const int32_t *score, int32_t *d2) {
+    const Inst &I = SI;
+    const View &V = SV;
+    const unsigned ib = (unsigned)I.id_bits;
+    const unsigned long long idmask = (1ull << ib) - 1ull;
+    const int4 *h4 = reinterpret_cast<const int4 *>(score);
+    const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
+    const int nv = I.nstr >> 2;
+    constexpr int UN = 2;
+    uint32_t bk = 0u, bk2 = 0u;
+    int32_t bd = 0, bd2 = 0;
+    for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
+        int4 hv[UN], uv[UN];
+#pragma unroll
+        for (int q = 0; q < UN; q++) {
+            const int v = v0 + q * blockDim.x;
+            hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
+            uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
+        }
+#pragma unroll
+        for (int q = 0; q < UN; q++) {
+            const int D = 4 * (v0 + q * blockDim.x);
+            const uint32_t hx[4] = {(uint32_t)hv[q].x, (uint32_t)hv[q].y, (uint32_t)hv[q].z, (uint32_t)hv[q].w};
+            const uint32_t ux[4] = {(uint32_t)uv[q].x, (uint32_t)uv[q].y, (uint32_t)uv[q].z, (uint32_t)uv[q].w};
+#pragma unroll
+            for (int c = 0; c < 4; c++) {
+                const uint32_t k1 = (hx[c] << 16) | ux[c], k2 = (hx[c] & 0xFFFF0000u) | ux[c];
+                if (k1 > bk) { bk = k1; bd = D + c; }
+                if (k2 > bk2) { bk2 = k2; bd2 = D + c; }
+            }
+        }
+    }
+    unsigned long long best = bk >= 65536u ? (((unsigned long long)bk << ib) | (idmask - (unsigned long long)bd)) : 0ull;
+    unsigned long long best2 =
+        bk2 >= 65536u ? (((unsigned long long)bk2 << ib) | (idmask - (unsigned long long)bd2)) : 0ull;
+    block_max2_u64(best, best2);
+    *d2 = best2 ? (int32_t)(idmask - (best2 & idmask)) : -1;
     return best ? (int32_t)(idmask - (best & idmask)) : -1;
 }
 
@@ -2185,8 +2278,8 @@ __device__ __noinline__ void fused_init() {
         }
         V.u[D] = dg;
         for (int k = 0; k < K; k++) {
-            V.h[(size_t)k * I.nstr + D] = c1;
-            V.h2[(size_t)k * I.nstr + D] = c2;
+            V.h[(size_t)k * I.nstr + D] = M_HH ? (c1 | (c2 << 16)) : c1;
+            if (!M_HH) V.h2[(size_t)k * I.nstr + D] = c2;
             V.np[(size_t)k * I.nstr + D] = 0;
         }
     }
@@ -2260,7 +2353,7 @@ __global__ void __launch_bounds__(512, 1)
             for (int D = tid; D < I.nstr; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
         if (I.so_h >= 0)
             for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h[i] = __ldcg(&I.h[i]);
-        if (I.so_h2 >= 0)
+        if (I.so_h2 >= 0 && !M_HH)
             for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h2[i] = __ldcg(&I.h2[i]);
         if (I.so_np >= 0)
             for (int i = tid; i < K * I.nstr; i += blockDim.x) V.np[i] = 0;
@@ -2371,11 +2464,14 @@ __global__ void __launch_bounds__(512, 1)
             if (M_FLAG(I, DTS_F_VERIFY)) verify_scores(k);
             // Alg. 5 l.4-9: Dopt = argmax (n_k(D), u(D), -D) over dataNotInMem_k
             PROF_T0(p_am);
-            int32_t D2s = -1;  // task shards: the 3inputs argmax comes with the main one
+            int32_t D2s = -1;  // task shards, packed rows: the 3inputs argmax comes with the main one
             const int32_t Dopt = M_SHARD(I) ? shard_scan(k, (I.flags & DTS_F_FALLBACK2) != 0,
                                                       M_FLAG(I, DTS_F_OPTI) != 0, &D2s)
                                  : M_FLAG(I, DTS_F_OPTI) ? score_first(V.h + (size_t)k * I.nstr)
-                                                          : score_argmax(V.h + (size_t)k * I.nstr);
+                                 // packed rows in HBM/L2 (C4): both keys in one pass; in
+                                 // shared memory (ALU-bound): the 3inputs pass only when needed
+                                 : (M_HH && I.so_h < 0) ? score_argmax_hh(V.h + (size_t)k * I.nstr, &D2s)
+                                                        : score_argmax(V.h + (size_t)k * I.nstr);
             PROF_ADD(L, P_ARGMAX, p_am);
             PROF_T0(p_pl);
             if (tid == 0) {
@@ -2400,7 +2496,9 @@ __global__ void __launch_bounds__(512, 1)
                 PROF_ADD(L, P_PLAN, p_pl);
             } else {
                 if (I.flags & DTS_F_FALLBACK2) {
-                    const int32_t D2 = M_SHARD(I) ? D2s : score_argmax(V.h2 + (size_t)k * I.nstr);
+                    const int32_t D2 = (M_SHARD(I) || (M_HH && I.so_h < 0)) ? D2s
+                                       : M_HH ? score_argmax(V.h + (size_t)k * I.nstr, 0)
+                                              : score_argmax(V.h2 + (size_t)k * I.nstr);
                     if (tid == 0) {
                         L.scan_alg_bytes += 8ull * (uint64_t)n;
                         L.alg_bytes += 8ull * (uint64_t)n;
@@ -2540,7 +2638,7 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
             unsigned __int128 num = (unsigned __int128)I.size[D] * 1000000000ull + (bw - 1);
             delta[D] = (int64_t)(num / bw);
             for (int k = 0; k < I.K; k++) {
-                I.h[(size_t)k * I.nstr + D] = c1;
+                I.h[(size_t)k * I.nstr + D] = I.hh ? (c1 | (c2 << 16)) : c1;
                 I.h2[(size_t)k * I.nstr + D] = c2;
                 I.np[(size_t)k * I.nstr + D] = 0;
             }

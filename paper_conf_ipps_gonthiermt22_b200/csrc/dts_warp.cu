@@ -65,12 +65,16 @@ __device__ __forceinline__ unsigned long long wmin64(unsigned long long v) {
         pt_ = t1_;                       \
     } while (0)
 #define WP_OUT(i) prof_[i]
+// bounds checks of the profiling build (compute-sanitizer is not available on
+// the GPU pool): a failed check sets the instance's error (Out::error = 9)
+#define WCHK(c) (chk_ |= !(c))
 #else
 #define WP_DECL
 #define WP(slot) \
     do {         \
     } while (0)
 #define WP_OUT(i) 0
+#define WCHK(c) ((void)0)
 #endif
 
 __device__ __forceinline__ int wsum(int v) { return (int)__reduce_add_sync(FULL, (unsigned)v); }
@@ -512,6 +516,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
     const int32_t *const rd = I->raw_dat;
 
     WP_DECL;
+    [[maybe_unused]] bool chk_ = false;  // WCHK: a bounds check failed (profiling build)
     build_state(v, Lw, dsm, rp, rd, wedge, tst, ten, lane);
     // ---- per-GPU registers (lane k) and uniform scalars (every lane)
     int64_t req = 0, gfree = 0;
@@ -571,6 +576,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                             tst[T] = st;
                             ten[T] = st + dtau;
                             sg[ns + i] = lane;
+                            WCHK(ns + i < m && T < m);
                             stk[ns + i] = T;
                         }
                     }
@@ -594,6 +600,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                             const int64_t st = req + (int64_t)i * dtau;
                             tst[T] = st;
                             ten[T] = st + dtau;
+                            WCHK(pos < m && T < m);
                             sg[pos] = lane;
                             stk[pos] = T;
                         }
@@ -712,6 +719,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                     if (msk == 0u) continue;
                     if (sel) {
                         const int pos = P + __popc(msk & lt);
+                        WCHK(pos < v.pcap && Tq < m && (o == (int)NOI || o < n));
                         pl[pos] = w;
                         atomicOr(&v.al[Tq >> 5], 1u << (Tq & 31));
                         if (o != (int)NOI) {
@@ -889,6 +897,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 // l.9: V leaves GPU k's memory
                 if (lane == 0) {
                     int32_t *rlw = v.rl + k * v.rcap;
+                    WCHK(vslot >= 0 && vslot < rck && rck <= v.rcap && V < n);
                     rlw[vslot] = rlw[rck - 1];
                     v.resm[V] &= ~(1u << k);
                 }
@@ -922,6 +931,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
             if (error) break;
             // load D
             if (lane == 0) {
+                WCHK(rck < v.rcap && D < n);
                 v.rl[k * v.rcap + rck] = D;
                 v.resm[D] |= 1u << k;
             }
@@ -979,6 +989,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
                 tst[T] = start;
                 ten[T] = end;
                 sg[ns] = k;
+                WCHK(ns < m && T >= 0 && T < m);
                 stk[ns] = T;
             }
             mk = end > mk ? end : mk;
@@ -989,6 +1000,12 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
 
     // ---- a8: sigma(k, .) -- stable partition of the service order by GPU
     assemble(I, dsm, lane, nsv, ns, K, sg, stk);
+#ifdef DTS_PROF
+    const bool bad_ = __any_sync(FULL, chk_);
+#else
+    (void)chk_;
+    (void)n;
+#endif
     if (lane == 0) {
         Out *o = I->out;
         o->n_events = nev;
@@ -1009,6 +1026,9 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
         o->n_alloc = n_alloc;
         o->sum_deg = sum_deg;
         o->error = error;
+#ifdef DTS_PROF
+        if (bad_) o->error = 9;
+#endif
         WP(11);
         for (int i = 0; i < 16; i++) o->prof[i] = WP_OUT(i);
     }

@@ -7,7 +7,7 @@ against it through DTS_ORACLE_LIB.  A mutant is KILLED when at least one pin
 fails.  A mutant listed as `equivalent` cannot be killed: its change is
 unreachable under the model (the reason is given; DESIGN.md restates it).
 
-usage: python tools/oracle_mutants.py [--out profiles/r02_oracle_mutants.txt]
+usage: python tests/oracle_mutants.py [--out profiles/r02_oracle_mutants.txt]
 """
 import argparse
 import os

@@ -5,7 +5,7 @@ blobs), dts_shard_connect, then dts_run on every rank at once -- the kernels
 exchange through each other's memory (NVLink peer memory on an 8xB200 box;
 the same B200 when the ranks share one device, as in tests/test_gpu_shard.py).
 
-    RANK=r WORLD_SIZE=G MASTER_ADDR=127.0.0.1 MASTER_PORT=p python tools/shard_ipc_worker.py
+    RANK=r WORLD_SIZE=G MASTER_ADDR=127.0.0.1 MASTER_PORT=p python tests/shard_ipc_worker.py
 
 Each rank checks its (replicated) schedule against the CPU oracle and prints
 "PARITY OK".

@@ -156,7 +156,7 @@ def test_shard_config4_full_digest(cfg):
 def test_shard_ipc_two_processes():
     """The multi-GPU path (dts_shard_export / connect, CUDA IPC, one process
     per shard) with both processes on this one B200."""
-    script = os.path.join(ROOT, "tools", "shard_ipc_worker.py")
+    script = os.path.join(ROOT, "tests", "shard_ipc_worker.py")
     env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT="29731", WORLD_SIZE="2")
     procs = [subprocess.Popen([sys.executable, script], env=dict(env, RANK=str(r)),
                               stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)

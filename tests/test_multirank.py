@@ -93,7 +93,7 @@ def _shard_worker(rank, world, port, q):
     rng = dts.dts_shard_range(h)
     got = [None] * world
     dist.all_gather_object(got, rng)
-    # the handle exchange the multi-GPU path uses (tools/shard_ipc_worker.py):
+    # the handle exchange the multi-GPU path uses (tests/shard_ipc_worker.py):
     # fixed-size blobs gathered in rank order; without a GPU export must fail loudly
     try:
         blob = dts.dts_shard_export(h, 0)
