@@ -811,7 +811,9 @@ dts_status stage(dts_instance *I, dts_policy policy, const dts_run_opts &o, int 
     h.ep_base = (unsigned long long)(++I->runs) << 32;
     h.box_bytes = I->box_bytes;
     h.xsys = I->xsys ? 1 : 0;
-    h.pop_batch_min = tuning("DTS_POP_BATCH_MIN", 10);
+    // batched pops pay off from ~2.5 planned tasks per simulated GPU (C3, K = 4: 10; C4, K = 8:
+    // 20, where a threshold of 10 made C4a 2.3 % slower, profiles/r03/r03l_pop_batch_min.txt)
+    h.pop_batch_min = tuning("DTS_POP_BATCH_MIN", h.K >= 8 ? 20 : 10);
     h.poison = tuning("DTS_POISON", 0);  // debug (profiling build only)
     // small instances: the loop CTA builds its own CSR and state (one launch)
     const int fs = fused_scratch_bytes(I, block);

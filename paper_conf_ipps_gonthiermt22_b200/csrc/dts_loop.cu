@@ -52,6 +52,9 @@
 #define M_LONG(c) (!DTS_FAST && (c))                           // rows of > 3 inputs
 #define M_KEY32(I) (DTS_FAST || (I).key32)                     // scores and u(D) < 2^15
 #define M_FLAG(I, f) (!DTS_FAST && ((I).flags & (f)))          // OPTI, VERIFY: generic only
+#ifndef DTS_HH_UN
+#define DTS_HH_UN 4
+#endif
 #define M_HH (DTS_FAST)  // packed scores: h[k][D] = n_k(D) | n2_k(D) << 16, one argmax pass for both
 #if DTS_FAST
 #define DTS_KNAME(x) x##_fast
@@ -1544,7 +1547,7 @@ __device__ int32_t score_argmax_hh(const int32_t *score, int32_t *d2) {
     const int4 *h4 = reinterpret_cast<const int4 *>(score);
     const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
     const int nv = I.nstr >> 2;
-    constexpr int UN = 2;
+    constexpr int UN = DTS_HH_UN;
     uint32_t bk = 0u, bk2 = 0u;
     int32_t bd = 0, bd2 = 0;
     for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {

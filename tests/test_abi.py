@@ -35,6 +35,29 @@ def test_struct_layouts():
     assert dts.dts_version() >> 16 == 1
 
 
+def test_struct_layouts_match_the_header(tmp_path):
+    """The binding's ctypes mirrors against the C compiler's view of include/dts.h:
+    size of every struct and the offset of every field (gcc, no GPU)."""
+    import subprocess
+    structs = {"dts_run_opts": B.dts_run_opts, "dts_result_view": B.dts_result_view}
+    lines = ["#include <stdio.h>", "#include <stddef.h>", '#include "dts.h"', "int main(void) {"]
+    for name, cls in structs.items():
+        lines.append(f'printf("{name} %zu\\n", sizeof({name}));')
+        for f, _ in cls._fields_:
+            lines.append(f'printf("{name}.{f} %zu\\n", offsetof({name}, {f}));')
+    lines.append('printf("dts_event %zu\\n", sizeof(dts_event)); return 0; }')
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)])
+    got = dict(l.split() for l in subprocess.check_output([str(exe)], text=True).splitlines())
+    for name, cls in structs.items():
+        assert int(got[name]) == C.sizeof(cls), name
+        for f, _ in cls._fields_:
+            assert int(got[f"{name}.{f}"]) == getattr(cls, f).offset, f"{name}.{f}"
+    assert int(got["dts_event"]) == dts.EVENT_DTYPE.itemsize
+
+
 def test_opts_defaults():
     o = dts.dts_run_opts_default()
     assert o.flags == dts.DTS_F_FALLBACK2 and o.lookahead_W == 0
