@@ -250,6 +250,22 @@ __device__ __forceinline__ void add_n2(int k, int32_t D, int d) {
     else atomicAdd(&SV.h2[(size_t)k * SI.nstr + D], d);
 }
 
+// u(D) += d; the specialised loop keeps u as 16-bit halves (< 2^15 in that mode):
+// the argmax then pulls 2 bytes per datum for it instead of 4.
+__device__ __forceinline__ void add_u(int32_t D, int d) {
+    if (M_HH) atomicAdd(reinterpret_cast<unsigned *>(SV.u) + (D >> 1), (unsigned)d << (16 * (D & 1)));
+    else atomicAdd(&SV.u[D], d);
+}
+// u(D) for the four data 4v .. 4v+3
+__device__ __forceinline__ uint4 u_vec4(int v) {
+    if (M_HH) {
+        const uint2 w = reinterpret_cast<const uint2 *>(SV.u)[v];
+        return make_uint4(w.x & 0xFFFFu, w.x >> 16, w.y & 0xFFFFu, w.y >> 16);
+    }
+    const int4 w = reinterpret_cast<const int4 *>(SV.u)[v];
+    return make_uint4((uint32_t)w.x, (uint32_t)w.y, (uint32_t)w.z, (uint32_t)w.w);
+}
+
 // Row-derived mode (Inst::sl): T has left the shared pool (R2).
 __device__ __forceinline__ bool allocated(int32_t T) { return (SV.al[T >> 5] >> (T & 31)) & 1u; }
 __device__ __forceinline__ void set_alloc(int32_t T, int sign) {
@@ -404,7 +420,7 @@ __device__ void pool_move(int32_t T, Row r, int sign, int plan_k) {
 #pragma unroll
     for (int i = 0; i < 3; i++) {
         if (c[i] < 0) continue;
-        if (own) atomicAdd(&V.u[c[i]], sign);
+        if (own) add_u(c[i], sign);
         if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[i]], -sign);
     }
 }
@@ -478,7 +494,7 @@ __device__ __noinline__ void pool_move_many(const int4 *ents, int P, int sign, i
 #pragma unroll
             for (int q = 0; q < 3; q++) {
                 if (c[q] < 0) continue;
-                if (own) atomicAdd(&V.u[c[q]], sign);
+                if (own) add_u(c[q], sign);
                 if (plan_k >= 0) atomicAdd(&V.np[(size_t)plan_k * I.nstr + c[q]], -sign);
             }
         }
@@ -1234,6 +1250,31 @@ __device__ int32_t luf_victim(int k) {
     const int nr = L.row_len, nr2 = L.row2_len;
     unsigned long long best = ~0ull;
     int bslot = -1;
+#if DTS_FAST
+    // two entries per thread and pass, both loads issued before either key is
+    // formed (C4b: 1,024 resident data, resident list and np_k in L2)
+    for (int i0 = threadIdx.x; i0 < cnt; i0 += 2 * blockDim.x) {
+        const int i1 = i0 + blockDim.x;
+        const int32_t D0 = rl[i0];
+        const int32_t D1 = i1 < cnt ? rl[i1] : -1;
+        const uint32_t p0 = (uint32_t)npk[D0];
+        const uint32_t p1 = D1 >= 0 ? (uint32_t)npk[D1] : 0xffffffffu;
+        bool b0 = false, b1 = D1 < 0;  // W = 0: taskBuffer_k = the task being served
+        for (int r = 0; r < nr; r++) {
+            b0 |= (L.row[r] == D0);
+            b1 |= (L.row[r] == D1);
+        }
+        const unsigned long long k0 = ((unsigned long long)p0 << 32) | (unsigned long long)(uint32_t)D0;
+        const unsigned long long k1 = ((unsigned long long)p1 << 32) | (unsigned long long)(uint32_t)D1;
+        const bool t0 = !b0 & (k0 < best);
+        best = t0 ? k0 : best;
+        bslot = t0 ? i0 : bslot;
+        const bool t1 = !b1 & (k1 < best);
+        best = t1 ? k1 : best;
+        bslot = t1 ? i1 : bslot;
+    }
+    (void)nr2;
+#else
     for (int i = threadIdx.x; i < cnt; i += blockDim.x) {
         const int32_t D = rl[i];
         bool in_buf = false;  // nb(D) > 0: an input of a taskBuffer_k task
@@ -1245,6 +1286,7 @@ __device__ int32_t luf_victim(int k) {
         best = take ? key : best;
         bslot = take ? i : bslot;
     }
+#endif
     const unsigned long long mine = best;
     best = block_min_u64(best);
     if (best == ~0ull) return -1;
@@ -1486,26 +1528,26 @@ __device__ int32_t score_argmax(const int32_t *score, int sh = 16) {
     unsigned long long best = 0ull;
     if (M_KEY32(I)) {
         const int4 *h4 = reinterpret_cast<const int4 *>(score);
-        const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
         const int nv = I.nstr >> 2;
         constexpr int UN = 2;
         uint32_t bk = 0u;
         int32_t bd = 0;
         for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
-            int4 hv[UN], uv[UN];
+            int4 hv[UN];
+            uint4 uv[UN];
 #pragma unroll
             for (int q = 0; q < UN; q++) {
                 const int v = v0 + q * blockDim.x;
                 hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
-                uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
+                uv[q] = v < nv ? u_vec4(v) : make_uint4(0, 0, 0, 0);
             }
 #pragma unroll
             for (int q = 0; q < UN; q++) {
                 const int D = 4 * (v0 + q * blockDim.x);
-                const uint32_t k0 = (((uint32_t)hv[q].x << sh) & 0xFFFF0000u) | (uint32_t)uv[q].x;
-                const uint32_t k1 = (((uint32_t)hv[q].y << sh) & 0xFFFF0000u) | (uint32_t)uv[q].y;
-                const uint32_t k2 = (((uint32_t)hv[q].z << sh) & 0xFFFF0000u) | (uint32_t)uv[q].z;
-                const uint32_t k3 = (((uint32_t)hv[q].w << sh) & 0xFFFF0000u) | (uint32_t)uv[q].w;
+                const uint32_t k0 = (((uint32_t)hv[q].x << sh) & 0xFFFF0000u) | uv[q].x;
+                const uint32_t k1 = (((uint32_t)hv[q].y << sh) & 0xFFFF0000u) | uv[q].y;
+                const uint32_t k2 = (((uint32_t)hv[q].z << sh) & 0xFFFF0000u) | uv[q].z;
+                const uint32_t k3 = (((uint32_t)hv[q].w << sh) & 0xFFFF0000u) | uv[q].w;
                 if (k0 > bk) { bk = k0; bd = D; }
                 if (k1 > bk) { bk = k1; bd = D + 1; }
                 if (k2 > bk) { bk = k2; bd = D + 2; }
@@ -1545,24 +1587,25 @@ __device__ int32_t score_argmax_hh(const int32_t *score, int32_t *d2) {
     const unsigned ib = (unsigned)I.id_bits;
     const unsigned long long idmask = (1ull << ib) - 1ull;
     const int4 *h4 = reinterpret_cast<const int4 *>(score);
-    const int4 *u4 = reinterpret_cast<const int4 *>(V.u);
     const int nv = I.nstr >> 2;
     constexpr int UN = DTS_HH_UN;
     uint32_t bk = 0u, bk2 = 0u;
     int32_t bd = 0, bd2 = 0;
+    (void)V;
     for (int v0 = threadIdx.x; v0 < nv; v0 += UN * blockDim.x) {
-        int4 hv[UN], uv[UN];
+        int4 hv[UN];
+        uint4 uv[UN];
 #pragma unroll
         for (int q = 0; q < UN; q++) {
             const int v = v0 + q * blockDim.x;
             hv[q] = v < nv ? h4[v] : make_int4(0, 0, 0, 0);
-            uv[q] = v < nv ? u4[v] : make_int4(0, 0, 0, 0);
+            uv[q] = v < nv ? u_vec4(v) : make_uint4(0, 0, 0, 0);
         }
 #pragma unroll
         for (int q = 0; q < UN; q++) {
             const int D = 4 * (v0 + q * blockDim.x);
             const uint32_t hx[4] = {(uint32_t)hv[q].x, (uint32_t)hv[q].y, (uint32_t)hv[q].z, (uint32_t)hv[q].w};
-            const uint32_t ux[4] = {(uint32_t)uv[q].x, (uint32_t)uv[q].y, (uint32_t)uv[q].z, (uint32_t)uv[q].w};
+            const uint32_t ux[4] = {uv[q].x, uv[q].y, uv[q].z, uv[q].w};
 #pragma unroll
             for (int c = 0; c < 4; c++) {
                 const uint32_t k1 = (hx[c] << 16) | ux[c], k2 = (hx[c] & 0xFFFF0000u) | ux[c];
@@ -2279,7 +2322,8 @@ __device__ __noinline__ void fused_init() {
             }
             if (V.dptr32) V.dptr32[D] = (int32_t)b;
         }
-        V.u[D] = dg;
+        if (M_HH) reinterpret_cast<uint16_t *>(V.u)[D] = (uint16_t)dg;
+        else V.u[D] = dg;
         for (int k = 0; k < K; k++) {
             V.h[(size_t)k * I.nstr + D] = M_HH ? (c1 | (c2 << 16)) : c1;
             if (!M_HH) V.h2[(size_t)k * I.nstr + D] = c2;
@@ -2352,8 +2396,8 @@ __global__ void __launch_bounds__(512, 1)
         }
         if (M_SL(I) && I.so_al >= 0)
             for (int i = tid; i <= I.m_pad / 32; i += blockDim.x) V.al[i] = __ldcg(&I.al[i]);
-        if (I.so_u >= 0)
-            for (int D = tid; D < I.nstr; D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
+        if (I.so_u >= 0)  // packed rows: u as 16-bit halves, nstr / 2 words
+            for (int D = tid; D < (M_HH ? I.nstr / 2 : I.nstr); D += blockDim.x) V.u[D] = __ldcg(&I.u[D]);
         if (I.so_h >= 0)
             for (int i = tid; i < K * I.nstr; i += blockDim.x) V.h[i] = __ldcg(&I.h[i]);
         if (I.so_h2 >= 0 && !M_HH)
@@ -2621,7 +2665,8 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
                 I.al[wd] = t0 >= I.m ? ~0u : (I.m - t0 >= 32 ? 0u : ~((1u << (I.m - t0)) - 1u));
             }
         for (int64_t D = I.n + tid; D < I.nstr; D += str) {  // row padding: never scores
-            I.u[D] = 0;
+            if (I.hh) reinterpret_cast<uint16_t *>(I.u)[D] = 0;
+            else I.u[D] = 0;
             for (int k = 0; k < I.K; k++) {
                 I.h[(size_t)k * I.nstr + D] = 0;
                 I.h2[(size_t)k * I.nstr + D] = 0;
@@ -2637,7 +2682,8 @@ __global__ void dts_init_kernel(const Inst *__restrict__ insts, int n_inst, uint
                 c1 += (len == 1);
                 c2 += (len == 2);
             }
-            I.u[D] = (int32_t)(e - b);
+            if (I.hh) reinterpret_cast<uint16_t *>(I.u)[D] = (uint16_t)(e - b);
+            else I.u[D] = (int32_t)(e - b);
             unsigned __int128 num = (unsigned __int128)I.size[D] * 1000000000ull + (bw - 1);
             delta[D] = (int64_t)(num / bw);
             for (int k = 0; k < I.K; k++) {
