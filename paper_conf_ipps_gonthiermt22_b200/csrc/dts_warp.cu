@@ -315,17 +315,50 @@ __device__ __noinline__ void build_state(const WV v, const WarpLayout Lw, unsign
         }
         for (int i = lane; i < v.n4; i += 32) v.hh[i] = 0u;
         __syncwarp();
-        for (int T0 = 0; T0 < m; T0 += 32) {  // degrees; n_0(D) / n2_0(D) with nothing resident
-            const int T = T0 + lane;
-            int a = -1, b = -1;
-            if (T < m) raw_row(rp, rd, T, a, b);
-            if (a >= 0) {
-                atomicAdd(&cur[a], 1);
-                atomicAdd(&v.hh[a], b >= 0 ? 65536u : 1u);
+        // degrees; n_0(D) / n2_0(D) with nothing resident.  Four tasks per lane and
+        // pass with their row loads in flight together; each task's D(T) is left as
+        // one word a | b << 16 (0xFFFF: absent) in the task-start array (overwritten
+        // by a2 below) for the scatter pass
+        uint32_t *rows = reinterpret_cast<uint32_t *>(tst);
+        for (int T0 = 0; T0 < m; T0 += 128) {
+            int64_t rb[4], re[4];
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const int T = T0 + 32 * q + lane;
+                rb[q] = T < m ? rp[T] : 0;
+                re[q] = T < m ? rp[T + 1] : 0;
             }
-            if (b >= 0) {
-                atomicAdd(&cur[b], 1);
-                atomicAdd(&v.hh[b], 65536u);
+            int x0[4], x1[4];
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                x0[q] = re[q] > rb[q] ? rd[rb[q]] : -1;
+                x1[q] = re[q] > rb[q] + 1 ? rd[rb[q] + 1] : -1;
+            }
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const int T = T0 + 32 * q + lane;
+                if (T >= m) continue;
+                int a, b;
+                if (re[q] - rb[q] > 2) {  // duplicates in a longer raw row (R27)
+                    raw_row(rp, rd, T, a, b);
+                } else {
+                    a = x0[q];
+                    b = x1[q] != x0[q] ? x1[q] : -1;
+                    if (b >= 0 && b < a) {
+                        const int t = a;
+                        a = b;
+                        b = t;
+                    }
+                }
+                rows[T] = (uint32_t)(a & 0xFFFF) | ((uint32_t)(b & 0xFFFF) << 16);
+                if (a >= 0) {
+                    atomicAdd(&cur[a], 1);
+                    atomicAdd(&v.hh[a], b >= 0 ? 65536u : 1u);
+                }
+                if (b >= 0) {
+                    atomicAdd(&cur[b], 1);
+                    atomicAdd(&v.hh[b], 65536u);
+                }
             }
         }
         __syncwarp();
@@ -347,10 +380,15 @@ __device__ __noinline__ void build_state(const WV v, const WarpLayout Lw, unsign
         }
         if (lane == 0) v.dp[n] = carry;
         __syncwarp();
+        __threadfence_block();
         for (int T0 = 0; T0 < m; T0 += 32) {  // stable scatter: segments in ascending task id
             const int T = T0 + lane;
             int a = -1, b = -1;
-            if (T < m) raw_row(rp, rd, T, a, b);
+            if (T < m) {
+                const uint32_t w = rows[T];
+                a = (w & 0xFFFFu) == 0xFFFFu ? -1 : (int)(w & 0xFFFFu);
+                b = (w >> 16) == 0xFFFFu ? -1 : (int)(w >> 16);
+            }
             if (a >= 0) atomicOr(&mask[a], 1u << lane);
             if (b >= 0) atomicOr(&mask[b], 1u << lane);
             __syncwarp();
