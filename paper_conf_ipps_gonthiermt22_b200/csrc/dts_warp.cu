@@ -705,8 +705,7 @@ __device__ __forceinline__ void run_instance(const Inst *__restrict__ I, unsigne
             oe = v.dp[Dopt + 1];
             seg_load(v, ob, oe, lane, edo);
         }
-        if (__shfl_sync(FULL, pe, k) > 1) {  // np_k counts exactly the plan this scan creates
-            // (Alg. 6 l.3): clear the last one's (a one-task plan never added to np_k)
+        {  // np_k counts exactly the plan this scan creates (Alg. 6 l.3): clear the last one's
             const int pe_k = __shfl_sync(FULL, pe, k), dk = __shfl_sync(FULL, dopt, k);
             uint16_t *npk = v.np + k * v.n8;
             const uint32_t *pl = v.plan + k * v.pcap;
