@@ -1211,13 +1211,14 @@ __device__ void reset_plan(int k) {
             }
         }
     }
-    cta_sync();
+    cta_sync();  // every thread has read plan_end before thread 0 clears it
     if (threadIdx.x == 0) {
         L.plan_head[k] = 0;
         L.plan_end[k] = 0;
         L.plan_live[k] = 0;
     }
-    cta_sync();
+    // no second barrier: nothing reads plannedTasks_k's bounds before the scan's next
+    // barrier (the argmax's block reduction or, on a one-warp CTA, the fallback's)
 }
 
 __device__ __forceinline__ Row row_of_entry(int4 e) {
@@ -1346,7 +1347,9 @@ __device__ void evict(int k, int32_t Vd, int32_t Tserved, int64_t t, int64_t te)
             tmin = (unsigned)e.x < tmin ? (unsigned)e.x : tmin;
         }
     }
-    block_sum_min(nret, tmin);
+    // no planned task left behind the one being served (most of C4's plans): nothing
+    // can return, skip the reduction's two barriers (ph, pe are CTA-uniform)
+    if (ph < pe) block_sum_min(nret, tmin);
     if (threadIdx.x == 0) {
         if (nret > 0) {
             L.plan_live[k] -= nret;
