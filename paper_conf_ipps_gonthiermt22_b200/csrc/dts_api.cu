@@ -695,10 +695,15 @@ bool warp_eligible(const dts_instance *I, dts_policy policy, const dts_run_opts 
                                           : max_dyn_smem_warp(o.device);
     return slot <= lim;
 }
-// A lone instance runs on one warp only while its per-decision scans are
-// short (n data, the widest segment): a wider instance wants a whole CTA.
-constexpr int WARP_SOLO_MAX = 2048;
-bool warp_solo(const dts_instance *I) { return I->n <= WARP_SOLO_MAX && I->max_deg_ub <= WARP_SOLO_MAX; }
+// A lone instance runs on one warp while its segments stay short (the widest
+// segment walk is 2,048 / 160 register batches at most); the warp loop beat the
+// CTA loop on every lone instance whose slice fits (C3 1.64x, n up to 4,096:
+// 1.4-1.8x, profiles/r03/r03q_solo_cross.txt).
+#ifndef DTS_WARP_SOLO_MAX
+#define DTS_WARP_SOLO_MAX 2048
+#endif
+constexpr int WARP_SOLO_MAX = DTS_WARP_SOLO_MAX;
+bool warp_solo(const dts_instance *I) { return I->max_deg_ub <= WARP_SOLO_MAX; }
 
 // Shared-memory placement of one instance's state:
 // greedy, most latency-critical array first, each either fully in the CTA's

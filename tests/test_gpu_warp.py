@@ -77,7 +77,11 @@ def test_loop_kind_selection():
     assert dts.schedule(c1, flags=F | dts.DTS_F_OPTI).loop_kind == dts.LOOP_GENERIC
     three = gen.random_shared(300, 64, 3, M=8, K=3, seed=7)                   # 3-input rows
     assert dts.schedule(three).loop_kind == dts.LOOP_CTA_FAST
-    assert dts.schedule(gen.matmul3d(40, M=142, K=4), max_served=50).loop_kind == dts.LOOP_CTA_FAST  # n > 2048
+    assert dts.schedule(gen.matmul3d(40, M=142, K=4), max_served=50).loop_kind == dts.LOOP_WARP  # C3
+    wide = gen.random_shared(20000, 8, 2, M=3, K=2, seed=3)                   # segments of ~5,000 tasks
+    assert dts.schedule(wide, max_served=20).loop_kind == dts.LOOP_CTA_FAST
+    big = gen.random_shared(60000, 8192, 2, M=128, K=4, seed=1)               # slice > shared memory
+    assert dts.schedule(big, max_served=20).loop_kind == dts.LOOP_CTA_FAST
     k33 = gen.matmul2d(8, M=4, K=33)                                          # K > 32
     assert dts.schedule(k33).loop_kind == dts.LOOP_CTA_FAST
     for g in dts.schedule_batch(gen.config_instances("C2")):
@@ -150,6 +154,13 @@ def test_wide_segments_several_batches():
     several register batches (and Dopt's load the general walk)."""
     _check(gen.random_shared(20000, 32, 2, M=6, K=3, seed=5))
     _check(gen.matmul2d(200, M=10, K=2), max_served=3000)
+
+
+def test_config3_on_the_warp_loop():
+    """C3 (one 64,000-task instance, n = 3,200) runs on one warp: full parity."""
+    inst = gen.config_instances("C3")[0]
+    _check(inst)
+    _check(inst, flags=CTA, kind=dts.LOOP_CTA_FAST)
 
 
 def test_batch_of_mixed_warp_instances():
