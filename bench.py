@@ -365,10 +365,13 @@ def main():
     barrier()
     with Clocks(dev) as clk:
         l0 = dts.dts_kernel_launches()
+        enq = []
         for i in range(args.steps):
             flush.zero_()  # L2 flush between timed steps (outside the events)
             evs[i][0].record(stream)
+            t_enq = time.perf_counter()
             step()
+            enq.append(time.perf_counter() - t_enq)
             evs[i][1].record(stream)
             # the loop kernel's own launch time (library events on the same
             # stream); waits for this step, so the next step's enqueue starts
@@ -377,6 +380,9 @@ def main():
         barrier()
         launches = dts.dts_kernel_launches() - l0
     step_ms = [a.elapsed_time(b) for a, b in evs]
+    if os.environ.get("DTS_BENCH_DEBUG"):
+        print("host enqueue ms", [round(1e3 * x, 2) for x in enq], "step ms", [round(x, 2) for x in step_ms],
+              "loop ms", [round(x, 2) for x in loop_ms_steps], file=sys.stderr, flush=True)
     rs = [dts.dts_result(h) for h in handles]  # last step's results (after the region)
     loop_ms = sum(loop_ms_steps) / len(loop_ms_steps)
     alg = sum(r.alg_bytes for r in rs)

@@ -889,16 +889,24 @@ dts_status acquire_slot(DeviceSweep &D, size_t n, SweepSlot **out) {
     if (S.done) CK(cudaEventSynchronize(S.done), "sweep slot event");  // its last launch has finished
     else CK(cudaEventCreateWithFlags(&S.done, cudaEventDisableTiming), "cudaEventCreate");
     if (S.cap < n) {
-        if (S.d_insts) cudaFree(S.d_insts);
-        if (S.h_insts) cudaFreeHost(S.h_insts);
-        S.d_insts = nullptr;
-        S.h_insts = nullptr;
-        S.cap = 0;
+        // grow EVERY slot of the ring now (each waits for its last launch first): a
+        // batch size seen once is then served without cudaMalloc / cudaMallocHost --
+        // slots first used inside a timed loop cost up to 30 ms of host time each
         const size_t cap = std::max<size_t>(n, 64);
-        CK(cudaMalloc(&S.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
-        CK(cudaMallocHost(&S.h_insts, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
-        S.d_work = reinterpret_cast<int *>(S.d_insts + cap);
-        S.cap = cap;
+        for (SweepSlot &X : D.slot) {
+            if (X.cap >= cap) continue;
+            if (X.done) CK(cudaEventSynchronize(X.done), "sweep slot event");
+            else CK(cudaEventCreateWithFlags(&X.done, cudaEventDisableTiming), "cudaEventCreate");
+            if (X.d_insts) cudaFree(X.d_insts);
+            if (X.h_insts) cudaFreeHost(X.h_insts);
+            X.d_insts = nullptr;
+            X.h_insts = nullptr;
+            X.cap = 0;
+            CK(cudaMalloc(&X.d_insts, sizeof(dts::Inst) * cap + 256), "cudaMalloc sweep");
+            CK(cudaMallocHost(&X.h_insts, sizeof(dts::Inst) * cap), "cudaMallocHost sweep");
+            X.d_work = reinterpret_cast<int *>(X.d_insts + cap);
+            X.cap = cap;
+        }
     }
     *out = &S;
     return DTS_OK;
