@@ -400,7 +400,8 @@ def main():
               for i in insts) * (args.shards if gsh else 1)
     d2h = 0
     barrier()
-    for i in range(max(2, args.steps // 2)):
+    n_e2e = max(2, args.steps // 2)
+    for i in range(n_e2e + 1):  # the first pass is an untimed warm-up (the library's pools)
         t0 = torch.cuda.Event(enable_timing=True)
         t1 = torch.cuda.Event(enable_timing=True)
         flush.zero_()
@@ -429,8 +430,11 @@ def main():
             del hs  # dts_instance_destroy (inside the timed region)
         t1.record(stream)
         t1.synchronize()
-        e2e_ms.append(t0.elapsed_time(t1))
+        if i > 0:
+            e2e_ms.append(t0.elapsed_time(t1))
     e2e_avg = sum(e2e_ms) / len(e2e_ms)
+    if os.environ.get("DTS_BENCH_DEBUG"):
+        print("e2e ms", [round(x, 2) for x in e2e_ms], file=sys.stderr, flush=True)
     gc.enable()
 
     # ---- max over ranks (device times), sum of the work
@@ -487,7 +491,8 @@ def main():
                     "scope": ("dts_instance_create from host arrays, upload, run, result D2H, destroy"
                               if create_each_step else
                               "upload (from the library's pinned copy), run, result D2H; "
-                              "instances created once outside the timed region")},
+                              "instances created once outside the timed region")
+                             + f"; mean of {n_e2e} passes after one untimed warm-up pass"},
             "gpu_launches": int(launches),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": _traffic(args.workload),
