@@ -1525,7 +1525,6 @@ __device__ __noinline__ unsigned long long score_best64(const int32_t *score) {
 // half (n2) is the score, the 3inputs key.
 __device__ int32_t score_argmax(const int32_t *score, int sh = 16) {
     const Inst &I = SI;
-    const View &V = SV;
     const unsigned ib = (unsigned)I.id_bits;
     const unsigned long long idmask = (1ull << ib) - 1ull;
     unsigned long long best = 0ull;
