@@ -1,6 +1,6 @@
 """Same-box A/B of library builds on the single large instances:
 python tools/lib_ab_c4.py LIB.so [flags...]  (loop ms of C4b, C4a, C3, C2[19];
-best of 2; flags are extra DTS_F_* bits, e.g. 32 = DTS_F_NOCLUSTER)."""
+best of 2; flags are extra DTS_F_* bits, e.g. 32 = DTS_F_GENERIC)."""
 import os
 import sys
 
