@@ -678,9 +678,13 @@ int64_t warp_slot_bytes(const dts_instance *I) {
     return dts::warp_layout(I->m, I->n, I->K, I->max_deg_ub + 1, I->res_cap + 1).total;
 }
 int max_dyn_smem_warp(int device) {
+    static std::atomic<int> cache[64];  // 0 = not queried yet
+    if (device >= 0 && device < 64 && cache[device].load() > 0) return cache[device].load();
     int optin = 0;
     cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device);
-    return std::max(0, optin - 1024);
+    const int r = std::max(0, optin - 1024);
+    if (device >= 0 && device < 64 && r > 0) cache[device].store(r);
+    return r;
 }
 bool warp_eligible(const dts_instance *I, dts_policy policy, const dts_run_opts &o) {
     if (policy != DTS_POLICY_DARTS_LUF || o.lookahead_W != 0 || o.block_threads != 0 || o.smem_budget < 0 ||

@@ -30,6 +30,7 @@
 
 #include <climits>
 #include <cstdint>
+#include <mutex>
 
 #include "dts_internal.cuh"
 #include "dts_loop.cuh"
@@ -1089,15 +1090,27 @@ __global__ void __launch_bounds__(32, 1) dts_warp_kernel(const Inst *__restrict_
     }
 }
 
+// The kernel's dynamic shared-memory limit, raised per device (the attribute
+// belongs to the current device's context) and only ever upwards; host
+// threads may launch concurrently.
+static cudaError_t warp_smem_attr(int smem_bytes) {
+    static std::mutex mu;
+    static int cur[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    std::lock_guard<std::mutex> lock(mu);
+    if (smem_bytes <= 48 * 1024 || smem_bytes <= cur[dev]) return cudaSuccess;
+    const cudaError_t e =
+        cudaFuncSetAttribute(dts_warp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+    if (e == cudaSuccess) cur[dev] = smem_bytes;
+    return e;
+}
+
 cudaError_t launch_warp(const Inst *d_insts, int n_inst, int grid, int *work_counter, int smem_bytes,
                         cudaStream_t st) {
-    static int attr_set = 0;
-    if (smem_bytes > 48 * 1024 && smem_bytes > attr_set) {
-        const cudaError_t e =
-            cudaFuncSetAttribute(dts_warp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-        if (e != cudaSuccess) return e;
-        attr_set = smem_bytes;
-    }
+    const cudaError_t e = warp_smem_attr(smem_bytes);
+    if (e != cudaSuccess) return e;
     count_launch();
     dts_warp_kernel<<<grid, 32, smem_bytes, st>>>(d_insts, n_inst, work_counter);
     return cudaGetLastError();
@@ -1105,8 +1118,7 @@ cudaError_t launch_warp(const Inst *d_insts, int n_inst, int grid, int *work_cou
 
 int warp_max_blocks_per_sm(int smem_bytes) {
     int nb = 0;
-    if (smem_bytes > 48 * 1024)
-        cudaFuncSetAttribute(dts_warp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+    if (warp_smem_attr(smem_bytes) != cudaSuccess) return 1;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, dts_warp_kernel, 32, smem_bytes) != cudaSuccess) return 1;
     return nb;
 }
